@@ -1,0 +1,194 @@
+/*
+ * frugal.h -- C ABI of the B200-native Frugal training-step hot path.
+ *
+ * Frugal (Xie et al., ASPLOS '25; /root/reference/PAPER.md) trains embedding
+ * models on several GPUs that share one parameter table in pinned host memory.
+ * Each GPU keeps a private cache of hot rows; rows updated on one GPU are
+ * *proactively flushed* to host memory before any GPU reads them again
+ * (§3.1), scheduled by a priority = next access step (Eq. (1),
+ * L902-911) held in a two-level priority queue (§3.4).
+ *
+ * One process per GPU, one context per process.  Every call returns a
+ * frugal_status (0 = ok, < 0 = error; the text is in frugal_last_error()); no
+ * call throws, aborts or exits.  Device work is enqueued asynchronously on the
+ * caller's stream `stream` (plus one library-owned low-priority side stream);
+ * calls on one context are not thread-safe.
+ *
+ * Row ids are GLOBAL ids in [0, n_rows) (table offset + local id; slot f of a
+ * sample reads table f).  Position i of a rank's step is i = b*slots + f.
+ * Rank g owns row k iff k mod world == g (reading R12 in DESIGN.md): the owner
+ * caches it if hot and applies its optimizer update (R6).
+ *
+ * Per-step call order (after frugal_prefetch(t) for t = 0 .. L-2):
+ *     frugal_step(s) -> frugal_lookup(s) -> [model] -> frugal_backward_update(s)
+ * and frugal_flush(FRUGAL_FLUSH_ALL) at the end of training.  Any other order
+ * returns FRUGAL_ESTATE.
+ */
+#ifndef FRUGAL_H
+#define FRUGAL_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct frugal_ctx frugal_ctx;
+typedef void* frugal_stream; /* a cudaStream_t (NULL = legacy default stream) */
+
+typedef enum {
+    FRUGAL_OK = 0,
+    FRUGAL_EINVAL = -1,   /* bad argument / config, or an id >= n_rows seen by a kernel */
+    FRUGAL_ENOMEM = -2,   /* device or pinned-host allocation failed */
+    FRUGAL_ECUDA = -3,    /* a CUDA runtime/driver call failed */
+    FRUGAL_ESTATE = -4,   /* out-of-order call (e.g. lookup(s) before step(s)) */
+    FRUGAL_ETIMEOUT = -5, /* a peer rank never published a flag */
+    FRUGAL_ESHM = -6      /* shared-memory host table could not be created/attached */
+} frugal_status;
+
+typedef enum { FRUGAL_SGD = 0, FRUGAL_ADAGRAD = 1 } frugal_opt;
+
+typedef enum {
+    FRUGAL_MODE_P2F = 0,          /* priority-based proactive flushing (§3.3) */
+    FRUGAL_MODE_WRITE_THROUGH = 1 /* Frugal-Sync baseline: every update flushed on the
+                                     critical path of the next step (§4.1) */
+} frugal_mode;
+
+enum {
+    FRUGAL_F_RECORD = 1, /* keep per-step schedule artefacts for frugal_get_schedule */
+    FRUGAL_F_TIMERS = 2  /* record CUDA events around every phase (frugal_get_timers) */
+};
+
+enum { FRUGAL_FLUSH_ALL = 0 };
+
+typedef struct {
+    int32_t world;      /* n ranks (GPUs), 1..32                                          */
+    int32_t rank;       /* this rank, 0..world-1 (== torch.distributed rank)               */
+    int32_t device;     /* CUDA ordinal this context runs on                               */
+    int32_t dim;        /* d: embedding dimension, multiple of 4, 4..1024                 */
+    int64_t n_rows;     /* N: rows over all tables, 1 .. 2^31-1                            */
+    int32_t slots;      /* F: lookups per sample                                           */
+    int32_t batch;      /* B: max samples per rank per step                               */
+    int32_t lookahead;  /* L: sample-queue depth, 2..31 (paper default 10, L783-784)      */
+    int32_t age_out;    /* D >= 1: cold dirty rows with no read in sight are flushed D
+                           steps after their update (reading R9)                          */
+    int32_t opt;        /* frugal_opt                                                      */
+    float lr, eps;      /* SGD: w -= lr*g; Adagrad: G += g*g; w -= (lr*g)/(sqrt(G)+eps)    */
+    float init_accum;   /* Adagrad G0                                                      */
+    float init_scale;   /* w0[k][j] = init_scale*(2u-1), u = top24(splitmix64(seed ^ (k*d+j)))/2^24 */
+    uint64_t init_seed;
+    const int64_t* hot_ids; /* host array: the static hot (cached) set, global ids, any
+                               order; each owner caches its share (reading R10/R11)       */
+    int64_t n_hot;
+    const char* shm_name;   /* POSIX shm name of the shared host table ("/frugal_x");
+                               rank 0 creates + initialises, others attach.  NULL:
+                               private pinned table (world must be 1)                     */
+    int32_t mode;           /* frugal_mode                                                 */
+    int32_t flags;          /* FRUGAL_F_*                                                  */
+} frugal_config;
+
+/* Create the context of this rank: validates cfg, maps (and for rank 0 creates and
+   initialises) the host table w[N][d] (+ G[N][d] for Adagrad), registers it with
+   CUDA (mapped, portable), allocates the HBM cache of the owned hot rows, per-row
+   metadata, sample-queue ring, dirty-row pool and scratch.  Ranks > 0 wait (bounded)
+   for rank 0's table.  On error *out is NULL. */
+frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out);
+
+/* Sample queue (§3.2, §3.3): enqueue the ids of step t of ALL
+   ranks.  ids_all: int64 [world][batch*slots], host (pinned) or device pointer,
+   copied before return to the stream's order (caller may reuse it after the stream
+   reaches this point).  counts: host int32[world], samples of each rank (0..batch).
+   Only used for t = 0..L-2 before step 0. */
+frugal_status frugal_prefetch(frugal_ctx* ctx, int64_t t, const int64_t* ids_all,
+                              const int32_t* counts, frugal_stream stream);
+
+/* Begin step s: enqueue step t = s+L-1 (ids_next_all/counts_next as in prefetch; NULL
+   past the end of the stream), run the P2F scheduler for the rows updated at s-1
+   (priority buckets, AdjustPriority inf->t, age-out), flush the urgent bucket on
+   `stream`, hand the deferred buckets to the side stream, and enqueue the gate
+   (PQ front > s, §3.3) on `stream`.  Returns once enqueued. */
+frugal_status frugal_step(frugal_ctx* ctx, int64_t s, const int64_t* ids_next_all,
+                          const int32_t* counts_next, frugal_stream stream);
+
+/* Forward query (§3.2): d_out[i] = current value of row ids[rank][i], for
+   i < counts[rank]*slots, row-major fp32 [count*slots][dim] in device memory.  Owned
+   hot rows come from the HBM cache, all others from the host table by zero-copy
+   loads (CPU bypass, §3.1). */
+frugal_status frugal_lookup(frugal_ctx* ctx, int64_t s, float* d_out, frugal_stream stream);
+
+/* Backward update (§3.2, §3.3): d_grad has d_out's shape.
+   Segment-reduces the gradients per distinct row (positions ascending), routes
+   partials of rows owned by other ranks through the host mailbox (the update
+   staging queue), merges per owned row in ascending rank order and applies the
+   fused optimizer; marks rows dirty and removes s from their read sets. */
+frugal_status frugal_backward_update(frugal_ctx* ctx, int64_t s, const float* d_grad,
+                                     frugal_stream stream);
+
+/* End of training (L1082-1083): every dirty owned row (w and G) and the G of every
+   hot row to the host table; waits for the side stream.  Afterwards the host table
+   is authoritative. */
+frugal_status frugal_flush(frugal_ctx* ctx, int32_t what, frugal_stream stream);
+
+frugal_status frugal_destroy(frugal_ctx* ctx);
+const char* frugal_last_error(void);
+
+/* ---- model glue (not the library proper) ----------------------
+   Frozen-dense dot-interaction BCE for the synthetic REC workload (R15):
+   per sample b: S = sum_f e_f (f ascending, fp32), z = 0.5(|S|^2 - sum_f |e_f|^2)
+   + <x_b,S> (fp64), p = sigmoid(z); loss += softplus(z) - y z (fp64, into *d_loss);
+   grad_f = c*((S - e_f) + x_b), c = (float)((p - y)/nb), nb = samples of step s over
+   all ranks.  d_emb/d_grad: [count*slots][dim]; x: [count][dim]; y: [count] (device). */
+frugal_status frugal_dot_model(frugal_ctx* ctx, int64_t s, const float* d_emb, const float* d_x,
+                               const float* d_y, float* d_grad, double* d_loss,
+                               frugal_stream stream);
+
+/* ---- introspection (tests / bench only; synchronise and copy to caller-owned host
+   buffers) ---------------------------------------------------------------------- */
+/* dedup of this rank's ids at step t (t within the sample queue): uniq ascending
+   (int64), inv[i] = index of ids[i] in uniq. *n_uniq receives the count; uniq/inv may
+   be NULL to query sizes. */
+frugal_status frugal_get_dedup(frugal_ctx* ctx, int64_t t, int64_t* uniq, int32_t* inv,
+                               int64_t* n_uniq);
+
+/* schedule artefacts of the last frugal_step (needs FRUGAL_F_RECORD): rows (global ids)
+   flushed urgently, deferred rows and their deadlines, aged-out rows; gate_wait = 1 iff
+   the urgent bucket was non-empty. Arrays may be NULL to query sizes (cap ignored). */
+typedef struct {
+    int64_t n_urgent, n_deferred, n_ageout;
+    int32_t gate_wait;
+} frugal_schedule_info;
+frugal_status frugal_get_schedule(frugal_ctx* ctx, frugal_schedule_info* info, int64_t* urgent,
+                                  int64_t* deferred, int32_t* deferred_p, int64_t* ageout);
+
+/* rows flushed by the last frugal_flush(FRUGAL_FLUSH_ALL) (global ids, any order) */
+frugal_status frugal_get_final_flush(frugal_ctx* ctx, int64_t* rows, int64_t* n);
+
+/* authoritative current values of rows owned by this rank (cache, dirty pool or
+   host).  ids: host int64[n]; w, G: host float[n][dim] (G may be NULL). */
+frugal_status frugal_read_rows(frugal_ctx* ctx, const int64_t* ids, int64_t n, float* w, float* G);
+
+/* raw host-table contents (any row). */
+frugal_status frugal_read_host(frugal_ctx* ctx, const int64_t* ids, int64_t n, float* w, float* G);
+
+/* per-phase device time (ms) summed over the steps since the last call, plus launch
+   counts (needs FRUGAL_F_TIMERS).  Phases, in order: ingest (a1+a2), schedule (a9),
+   urgent (a10), gate (a3), gather (a4, unique rows), expand (a4, per position),
+   model (a5), segred (a6), exchange (a7), optimizer (a8), side (a11, side stream). */
+#define FRUGAL_N_PHASES 11
+typedef struct {
+    double ms[FRUGAL_N_PHASES];
+    int64_t steps;
+    int64_t kernel_launches;       /* library kernels launched since init               */
+    int64_t rows_urgent, rows_deferred, rows_ageout; /* cumulative (FRUGAL_F_RECORD)    */
+    int64_t host_read_rows;        /* cumulative rows gathered from host (RECORD)        */
+} frugal_stats;
+frugal_status frugal_get_stats(frugal_ctx* ctx, frugal_stats* out);
+
+/* number of owned rows / hot slots of this rank */
+int64_t frugal_owned_rows(frugal_ctx* ctx);
+int64_t frugal_hot_slots(frugal_ctx* ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FRUGAL_H */

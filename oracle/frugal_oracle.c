@@ -15,7 +15,8 @@
  *     e_f = W[id_f];  S = sum_f e_f;  z = sum_{f<f'} <e_f,e_f'> + sum_f <x,e_f>
  *     p = sigmoid(z); loss = BCE(p, y); dL/de_f = c (S - e_f + x), c = (p-y)/nb
  *  then per rank: partial P_g[k] = sum over positions i ascending of grad[i]
- *  (fp32, sequential), per row: g_k = sum over ranks ascending of P_g[k], then
+ *  (fp32, fixed order: sequential within chunks of 64 occurrences, chunk sums
+ *  added sequentially -- reading R23), per row: g_k = sum over ranks ascending of P_g[k], then
  *  SGD  w -= lr*g   or   Adagrad  G += g*g; w -= (lr*g)/(sqrt(G)+eps)
  *  (elementwise fp32, each operation rounded separately; built with
  *  -ffp-contract=off, no fast-math).
@@ -46,6 +47,7 @@
 #include <string.h>
 
 #define OR_INF INT32_MAX
+#define OR_CHUNK 64 /* R23: segment-reduce chunk length */
 enum { OR_SGD = 0, OR_ADAGRAD = 1 };
 enum { OR_MODEL_DOT = 0, OR_MODEL_CONST = 1, OR_MODEL_L2 = 2 };
 enum { OR_CLEAN = 0, OR_UPDATED = 1, OR_INFP = 2, OR_EXEMPT = 3 };
@@ -414,16 +416,29 @@ static void train(oracle* o, int64_t s) {
         o->pk[g] = malloc((m ? m : 1) * sizeof(int64_t));
         o->pv[g] = malloc((m ? m : 1) * d * sizeof(float));
         const float* gr = o->grad + (int64_t)g * B * F * d;
-        for (int64_t i = 0; i < m; i++) {
-            if (i == 0 || a[i].v != a[i - 1].v) {
-                o->pk[g][u] = a[i].v;
-                memcpy(o->pv[g] + u * d, gr + a[i].p * d, d * sizeof(float));
-                u++;
-            } else {
-                float* P = o->pv[g] + (u - 1) * d;
-                for (int64_t j = 0; j < d; j++) P[j] = P[j] + gr[a[i].p * d + j];
+        /* canonical fixed order (reading R23): occurrences of a row, positions
+           ascending, are cut into chunks of OR_CHUNK; each chunk is summed
+           sequentially and the chunk sums are added sequentially in order.
+           (For <= OR_CHUNK occurrences this is the plain sequential sum.) */
+        float* chunk = malloc(d * sizeof(float));
+        int64_t i = 0;
+        while (i < m) {
+            int64_t e = i;
+            while (e < m && a[e].v == a[i].v) e++;
+            o->pk[g][u] = a[i].v;
+            float* P = o->pv[g] + u * d;
+            for (int64_t c0 = i; c0 < e; c0 += OR_CHUNK) {
+                int64_t c1 = c0 + OR_CHUNK < e ? c0 + OR_CHUNK : e;
+                memcpy(chunk, gr + a[c0].p * d, d * sizeof(float));
+                for (int64_t q = c0 + 1; q < c1; q++)
+                    for (int64_t j = 0; j < d; j++) chunk[j] = chunk[j] + gr[a[q].p * d + j];
+                if (c0 == i) memcpy(P, chunk, d * sizeof(float));
+                else for (int64_t j = 0; j < d; j++) P[j] = P[j] + chunk[j];
             }
+            u++;
+            i = e;
         }
+        free(chunk);
         o->pn[g] = u;
         free(a);
     }

@@ -1,0 +1,202 @@
+// frugal_internal.cuh -- shared device/host declarations of libfrugal (CUDA path only).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "frugal.h"
+
+namespace frugal {
+
+constexpr int kSMs = 148;              // B200
+constexpr int kThreads = 256;          // default block size
+constexpr int kTile = 256;             // radix/scan tile (elements per block iteration)
+constexpr int32_t kInfP = 0x7fffffff;  // priority "infinity" (Eq. (1) second case)
+
+// per-owned-row state (the g-entry, made dense)
+enum RowState : int32_t {
+    ST_CLEAN = 0,    // no pending update (W set empty) or flush already scheduled
+    ST_UPDATED = 1,  // updated at last_upd, not yet prioritised
+    ST_INF = 2,      // dirty, no read within the lookahead window (priority inf)
+    ST_EXEMPT = 3    // dirty hot row whose next reader is only its owner (cache hit)
+};
+
+// ---------------------------------------------------------------- radix sort
+// Stable LSD radix sort of (uint32 key, int32 val) pairs, device-resident count.
+struct SortScratch {
+    uint32_t* k[2] = {nullptr, nullptr};
+    int32_t* v[2] = {nullptr, nullptr};
+    int32_t* hist = nullptr;  // [256][nblk]
+    int nblk = 0;
+    int64_t cap = 0;
+};
+void sort_alloc(SortScratch& s, int64_t cap);
+void sort_free(SortScratch& s);
+// Sorts keys/vals of length *d_n (<= cap) held in s.k[0]/s.v[0]; returns index of
+// the buffer holding the result (0 or 1).  Only bits [0, bits) of the keys matter.
+int sort_pairs(SortScratch& s, const int32_t* d_n, int bits, cudaStream_t st, int64_t* launches);
+
+// ---------------------------------------------------------------- scan
+struct ScanScratch {
+    int32_t* part = nullptr;
+    int nblk = 0;
+};
+void scan_alloc(ScanScratch& s, int64_t cap);
+void scan_free(ScanScratch& s);
+
+// ---------------------------------------------------------------- sample-queue slot
+struct QueueSlot {
+    int64_t step = -1;      // which step this slot holds
+    int32_t* ids = nullptr;     // [world][M] int32 (converted, validated)
+    int32_t* counts = nullptr;  // [world] device
+    int32_t* m = nullptr;       // device scalar: counts[g] * slots
+    std::vector<int32_t> h_counts;
+    // own dedup (rank g)
+    int32_t* uniq = nullptr;  // [M] ascending
+    int32_t* inv = nullptr;   // [M]
+    int32_t* off = nullptr;   // [M+1] CSR offsets
+    int32_t* pos = nullptr;   // [M] positions grouped by uniq, ascending within
+    int32_t* n_uniq = nullptr;  // device scalar
+    // owner side: T = owned rows read at this step by any rank, ascending
+    int32_t* T = nullptr;      // [capT] local row index lk = k / world
+    uint32_t* Tmask = nullptr; // [capT] rank mask
+    int32_t* Tidx = nullptr;   // [world][capT] index of T[j] in rank r's owner segment
+    int32_t* nT = nullptr;     // device scalar
+    // sender side grouping (world > 1): uniq positions grouped by owner
+    int32_t* gl = nullptr;     // [M] grouped position -> uniq index
+    int32_t* goff = nullptr;   // [world+1]
+};
+
+struct PhaseEv {
+    int phase;
+    cudaEvent_t a, b;
+};
+
+struct HostShared;  // shm segment layout (runtime.cu)
+
+}  // namespace frugal
+
+struct frugal_ctx {
+    frugal_config cfg;
+    int n, g, d, F, B, L, D, M;  // world, rank, dim, slots, batch, lookahead, age_out, B*F
+    int64_t N, No;               // rows, owned rows
+    int P;                       // pool segments = D + 2
+    int64_t capT;                // max owned rows touched per step
+    int key_bits, lk_bits;       // bits of global ids / local ids
+
+    // host table (pinned/registered) and its device aliases
+    void* shm_base = nullptr;
+    size_t shm_bytes = 0;
+    int shm_fd = -1;
+    bool shm_owner = false;
+    float* h_w = nullptr;  // host pointers
+    float* h_G = nullptr;
+    float* dh_w = nullptr;  // device-side aliases (mapped)
+    float* dh_G = nullptr;
+    // cross-rank flags and mailboxes (world > 1), host memory
+    volatile uint32_t* h_flags = nullptr;
+    uint32_t* dh_flags = nullptr;
+    char* h_mail = nullptr;
+    char* dh_mail = nullptr;
+    size_t mail_stride = 0;  // bytes per (parity, sender) mailbox region
+
+    // per-owned-row metadata (HBM)
+    int32_t* slot = nullptr;      // [No] cache slot or -1
+    int32_t* state = nullptr;     // [No]
+    int32_t* last_upd = nullptr;  // [No]
+    int32_t* pool_idx = nullptr;  // [No]
+    uint64_t* rbits = nullptr;    // [No] low 32: any-reader ring, high 32: host-reader ring
+
+    // HBM cache of owned hot rows
+    int64_t cap_hot = 0;
+    float* cw = nullptr;
+    float* cG = nullptr;
+    int32_t* hot_lk = nullptr;  // [cap_hot] local index of each slot
+
+    // dirty-row pool for cold owned rows: P segments x capT rows
+    float* pw = nullptr;
+    float* pG = nullptr;
+    int32_t* pkey = nullptr;   // [P][capT] local index
+    int32_t* pcount = nullptr; // [P]
+
+    // sample queue
+    std::vector<frugal::QueueSlot> q;
+
+    // per-step scratch
+    float* rows = nullptr;  // [M][d] gathered unique rows
+    float* Pp = nullptr;    // [M][d] partials (grouped order for world > 1)
+    float* chunk_scratch = nullptr;  // [M][d] chunk sums of long segments
+    int32_t* long_q = nullptr;       // [M] long segments of the current step
+    int32_t* long_cnt = nullptr;
+    int32_t* owned_cnt = nullptr;  // scalar
+    // schedule lists (double buffered by step parity)
+    int32_t* nb_rows = nullptr;  // newly bucketed rows [capT + capT]
+    int32_t* nb_p = nullptr;
+    int32_t* nb_cnt = nullptr;   // scalar
+    int32_t* bk_rows[2] = {nullptr, nullptr};  // bucket-sorted rows
+    int32_t* bk_p[2] = {nullptr, nullptr};
+    int32_t* bk_off[2] = {nullptr, nullptr};   // [L+1]
+    int32_t* age_rows[2] = {nullptr, nullptr};
+    int32_t* age_cnt[2] = {nullptr, nullptr};
+    int32_t* err = nullptr;   // device alias of the error word (mapped pinned host memory)
+    int32_t* herr = nullptr;  // host pointer of the same word
+    int32_t* sched_info = nullptr;  // device [4]
+    int32_t* ff_rows = nullptr;  // final flush list
+    int32_t* ff_cnt = nullptr;
+    int64_t* ids_stage = nullptr;  // device int64 staging for incoming ids [world][M]
+    int32_t* counts_pin = nullptr;  // pinned [L+1][world] staging of per-step counts
+    std::vector<cudaEvent_t> ev_counts;  // one per queue slot: staging reusable
+
+    frugal::SortScratch sort;
+    frugal::ScanScratch scan;
+
+    cudaStream_t side = nullptr;
+    cudaEvent_t ev_sched = nullptr;
+    cudaEvent_t ev_side[2] = {nullptr, nullptr};
+    bool side_pending[2] = {false, false};
+
+    // call-order state
+    int64_t next_prefetch = 0;  // next t expected by prefetch/step
+    int64_t cur_step = -1;
+    int phase_in_step = 0;  // 0 = need step, 1 = need lookup, 2 = need backward
+    bool ids_exhausted = false;
+
+    // instrumentation
+    int64_t launches = 0;
+    std::vector<frugal::PhaseEv> evs;
+    std::vector<cudaEvent_t> ev_pool;
+    size_t ev_used = 0;
+    double phase_ms[FRUGAL_N_PHASES] = {0};
+    int64_t timed_steps = 0;
+    int64_t rows_urgent = 0, rows_deferred = 0, rows_ageout = 0, host_read_rows = 0;
+    // recorded schedule artefacts (FRUGAL_F_RECORD)
+    std::vector<int32_t> rec_urgent, rec_deferred, rec_deferred_p, rec_ageout, rec_final;
+    int rec_gate_wait = 0;
+};
+
+namespace frugal {
+// kernels' host launchers (kernels.cu)
+void launch_convert_ids(frugal_ctx* c, QueueSlot& q, cudaStream_t st);
+void launch_dedup(frugal_ctx* c, QueueSlot& q, cudaStream_t st);
+void launch_owner_side(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st);
+void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, cudaStream_t st);
+void launch_bucket(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStream_t st);
+void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begin, const int32_t* d_end,
+                       int with_hot_g, cudaStream_t st);
+void launch_gather(frugal_ctx* c, QueueSlot& q, float* out, cudaStream_t st);
+void launch_expand(frugal_ctx* c, QueueSlot& q, float* out, cudaStream_t st);
+void launch_mail_header(frugal_ctx* c, QueueSlot& q, int par, cudaStream_t st);
+void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const float* x, const float* y,
+                      float* grad, double* loss, int64_t nb, cudaStream_t st);
+void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, cudaStream_t st);
+void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, cudaStream_t st);
+void launch_final_flush(frugal_ctx* c, cudaStream_t st);
+void launch_init_table(frugal_ctx* c, cudaStream_t st);
+void launch_init_meta(frugal_ctx* c, const int64_t* d_hot_global, int64_t n_hot, cudaStream_t st);
+void launch_wait_flags(frugal_ctx* c, int which, uint32_t value, cudaStream_t st);
+void launch_set_flag(frugal_ctx* c, int which, uint32_t value, cudaStream_t st);
+void launch_read_rows(frugal_ctx* c, const int32_t* d_lk, int64_t n, float* d_w, float* d_G, cudaStream_t st);
+void launch_read_host(frugal_ctx* c, const int64_t* d_k, int64_t n, float* d_w, float* d_G, cudaStream_t st);
+}  // namespace frugal

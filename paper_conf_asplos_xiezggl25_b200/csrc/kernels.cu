@@ -1,0 +1,796 @@
+// kernels.cu -- sm_100a kernels of the Frugal step (CUDA path; shares nothing with oracle/).
+//
+// Every kernel here is HBM- or host-link-bound integer / fp32 copy work; nothing is a
+// dense contraction, so there are no tensor-core paths.  Rows are
+// moved as float4 by "row groups" of GS lanes (GS = pow2 >= d/4, capped at 32) so a
+// 128-byte d=32 row is one coalesced 8-lane access; host-table rows are read/written
+// with zero-copy loads/stores through the mapped alias of the pinned shm table
+// (§3.1: "fuses the local GPU cache access and host memory access
+// into one GPU kernel ... zero-copy").
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "frugal_internal.cuh"
+#include "kutil.cuh"
+
+namespace frugal {
+
+// ============================================================================ block scan helpers
+// exclusive scan of one int per thread over a 256-thread block; returns total in *tot
+__device__ __forceinline__ int block_excl_scan(int v, int* sm_w /*[8]*/, int* tot) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        int y = __shfl_up_sync(FULL, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) sm_w[w] = x;
+    __syncthreads();
+    int base = 0, all = 0;
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+        int c = sm_w[i];
+        if (i < w) base += c;
+        all += c;
+    }
+    __syncthreads();
+    *tot = all;
+    return base + x - v;
+}
+
+// single-block exclusive scan of a small int array in place; writes the total
+__global__ void k_scan_small(int32_t* a, int len, int32_t* total) {
+    __shared__ int sm[32];
+    const int t = threadIdx.x, nt = blockDim.x;
+    int per = (len + nt - 1) / nt, lo = min(len, t * per), hi = min(len, lo + per);
+    int s = 0;
+    for (int i = lo; i < hi; i++) s += a[i];
+    // block exclusive scan (1024 threads)
+    const int lane = t & 31, w = t >> 5;
+    int x = s;
+    for (int o = 1; o < 32; o <<= 1) {
+        int y = __shfl_up_sync(FULL, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) sm[w] = x;
+    __syncthreads();
+    if (w == 0) {
+        int v = (lane < (nt >> 5)) ? sm[lane] : 0;
+        int z = v;
+        for (int o = 1; o < 32; o <<= 1) {
+            int y = __shfl_up_sync(FULL, z, o);
+            if (lane >= o) z += y;
+        }
+        sm[lane] = z - v;
+        if (lane == 31 && total) *total = z;
+    }
+    __syncthreads();
+    int run = sm[w] + x - s;
+    for (int i = lo; i < hi; i++) {
+        int c = a[i];
+        a[i] = run;
+        run += c;
+    }
+}
+
+// ============================================================================ radix sort
+__global__ void k_radix_hist(const uint32_t* __restrict__ keys, const int32_t* d_n, int shift,
+                             int32_t* hist, int nblk) {
+    __shared__ int h[256];
+    h[threadIdx.x] = 0;
+    __syncthreads();
+    int lo, hi;
+    chunk_range(*d_n, nblk, blockIdx.x, lo, hi);
+    for (int i = lo + threadIdx.x; i < hi; i += blockDim.x) atomicAdd(&h[(keys[i] >> shift) & 255], 1);
+    __syncthreads();
+    hist[threadIdx.x * nblk + blockIdx.x] = h[threadIdx.x];
+}
+
+__global__ void k_radix_scatter(const uint32_t* __restrict__ kin, const int32_t* __restrict__ vin,
+                                uint32_t* __restrict__ kout, int32_t* __restrict__ vout, const int32_t* d_n,
+                                int shift, const int32_t* __restrict__ hist, int nblk) {
+    __shared__ int run[256];
+    __shared__ int wcnt[8][256];
+    __shared__ int tot[256];
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    run[tid] = hist[tid * nblk + blockIdx.x];
+    int lo, hi;
+    chunk_range(*d_n, nblk, blockIdx.x, lo, hi);
+    for (int base = lo; base < hi; base += kTile) {
+#pragma unroll
+        for (int i = 0; i < 8; i++) wcnt[i][tid] = 0;
+        __syncthreads();
+        const int i = base + tid;
+        const bool valid = i < hi;
+        uint32_t key = valid ? kin[i] : 0u;
+        int32_t val = valid ? vin[i] : 0;
+        int dg = valid ? (int)((key >> shift) & 255u) : -1;
+        unsigned peers = __match_any_sync(FULL, dg);
+        int rank = __popc(peers & lanemask_lt());
+        if (valid && rank == 0) wcnt[w][dg] = __popc(peers);
+        __syncthreads();
+        {
+            int acc = 0;
+#pragma unroll
+            for (int q = 0; q < 8; q++) {
+                int c = wcnt[q][tid];
+                wcnt[q][tid] = acc;
+                acc += c;
+            }
+            tot[tid] = acc;
+        }
+        __syncthreads();
+        if (valid) {
+            int dst = run[dg] + wcnt[w][dg] + rank;
+            kout[dst] = key;
+            vout[dst] = val;
+        }
+        __syncthreads();
+        run[tid] += tot[tid];
+    }
+}
+
+void sort_alloc(SortScratch& s, int64_t cap) {
+    s.cap = cap < 1 ? 1 : cap;
+    for (int i = 0; i < 2; i++) {
+        cudaMalloc(&s.k[i], s.cap * sizeof(uint32_t));
+        cudaMalloc(&s.v[i], s.cap * sizeof(int32_t));
+    }
+    s.nblk = grid_for(s.cap, kTile * 4, 2);
+    cudaMalloc(&s.hist, 256 * (size_t)s.nblk * sizeof(int32_t));
+}
+void sort_free(SortScratch& s) {
+    for (int i = 0; i < 2; i++) {
+        cudaFree(s.k[i]);
+        cudaFree(s.v[i]);
+    }
+    cudaFree(s.hist);
+    s = SortScratch();
+}
+
+int sort_pairs(SortScratch& s, const int32_t* d_n, int bits, cudaStream_t st, int64_t* launches) {
+    int cur = 0;
+    for (int shift = 0; shift < bits; shift += 8) {
+        k_radix_hist<<<s.nblk, 256, 0, st>>>(s.k[cur], d_n, shift, s.hist, s.nblk);
+        k_scan_small<<<1, 1024, 0, st>>>(s.hist, 256 * s.nblk, nullptr);
+        k_radix_scatter<<<s.nblk, 256, 0, st>>>(s.k[cur], s.v[cur], s.k[cur ^ 1], s.v[cur ^ 1], d_n, shift,
+                                                s.hist, s.nblk);
+        *launches += 3;
+        cur ^= 1;
+    }
+    return cur;
+}
+
+void scan_alloc(ScanScratch& s, int64_t cap) {
+    s.nblk = grid_for(cap < 1 ? 1 : cap, kTile * 4, 2);
+    cudaMalloc(&s.part, ((size_t)s.nblk * 33 + 1) * sizeof(int32_t));
+}
+void scan_free(ScanScratch& s) {
+    cudaFree(s.part);
+    s = ScanScratch();
+}
+
+// ============================================================================ ingest: ids
+// int64 ids of all ranks -> int32 ring copy (validated) + this rank's sort input
+__global__ void k_convert_ids(const int64_t* __restrict__ ids64, int32_t* __restrict__ ids32,
+                              const int32_t* __restrict__ counts, int world, int M, int F, int64_t N,
+                              int g, uint32_t* __restrict__ sk, int32_t* __restrict__ sv,
+                              int32_t* __restrict__ d_m, int32_t* err) {
+    // err lives in mapped pinned host memory: the host sees a bad id without a sync
+    const int64_t total = (int64_t)world * M;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total;
+         e += (int64_t)gridDim.x * blockDim.x) {
+        int r = (int)(e / M), i = (int)(e - (int64_t)r * M);
+        if (i >= counts[r] * F) continue;
+        int64_t k = ids64[e];
+        if (k < 0 || k >= N) {
+            atomicExch(err, 1);
+            k = 0;
+        }
+        ids32[e] = (int32_t)k;
+        if (r == g) {
+            sk[i] = (uint32_t)k;
+            sv[i] = i;
+        }
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) *d_m = counts[g] * F;
+}
+
+// ============================================================================ dedup emit
+// sorted (key, pos) -> uniq ascending, CSR (off, pos), inv
+__global__ void k_head_count(const uint32_t* __restrict__ ks, const int32_t* d_n, int32_t* part, int nblk) {
+    __shared__ int sm[8];
+    int lo, hi;
+    chunk_range(*d_n, nblk, blockIdx.x, lo, hi);
+    int c = 0;
+    for (int i = lo + threadIdx.x; i < hi; i += blockDim.x) c += (i == 0 || ks[i] != ks[i - 1]);
+    for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(FULL, c, o);
+    if ((threadIdx.x & 31) == 0) sm[threadIdx.x >> 5] = c;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int t = 0;
+        for (int i = 0; i < 8; i++) t += sm[i];
+        part[blockIdx.x] = t;
+    }
+}
+
+__global__ void k_dedup_emit(const uint32_t* __restrict__ ks, const int32_t* __restrict__ vs, const int32_t* d_n,
+                             const int32_t* __restrict__ part, int nblk, int32_t* __restrict__ uniq,
+                             int32_t* __restrict__ off, int32_t* __restrict__ inv, int32_t* __restrict__ pos,
+                             int32_t* d_nuniq) {
+    __shared__ int smw[8];
+    const int n = *d_n;
+    int lo, hi;
+    chunk_range(n, nblk, blockIdx.x, lo, hi);
+    int run = part[blockIdx.x];
+    for (int base = lo; base < hi; base += kTile) {
+        const int i = base + threadIdx.x;
+        const bool valid = i < hi;
+        uint32_t key = valid ? ks[i] : 0u;
+        int head = valid && (i == 0 || ks[i - 1] != key);
+        int tot;
+        int ex = block_excl_scan(head, smw, &tot);
+        if (valid) {
+            int seg = run + ex + head - 1;
+            if (head) {
+                uniq[seg] = (int32_t)key;
+                off[seg] = i;
+            }
+            int p = vs[i];
+            pos[i] = p;
+            inv[p] = seg;
+            if (i == n - 1) {
+                off[seg + 1] = n;
+                *d_nuniq = seg + 1;
+            }
+        }
+        run += tot;
+    }
+    if (n == 0 && blockIdx.x == 0 && threadIdx.x == 0) {
+        off[0] = 0;
+        *d_nuniq = 0;
+    }
+}
+
+void launch_convert_ids(frugal_ctx* c, QueueSlot& q, cudaStream_t st) {
+    int64_t total = (int64_t)c->n * c->M;
+    k_convert_ids<<<grid_for(total, 256), 256, 0, st>>>(c->ids_stage, q.ids, q.counts, c->n, c->M, c->F, c->N,
+                                                         c->g, c->sort.k[0], c->sort.v[0], q.m, c->err);
+    c->launches++;
+}
+
+// own-rank dedup of the sample-queue slot: keys were staged by k_convert_ids, count in owned_cnt
+void launch_dedup(frugal_ctx* c, QueueSlot& q, cudaStream_t st) {
+    int r = sort_pairs(c->sort, q.m, c->key_bits, st, &c->launches);
+    int nb = c->scan.nblk;
+    k_head_count<<<nb, 256, 0, st>>>(c->sort.k[r], q.m, c->scan.part, nb);
+    k_scan_small<<<1, 1024, 0, st>>>(c->scan.part, nb, nullptr);
+    k_dedup_emit<<<nb, 256, 0, st>>>(c->sort.k[r], c->sort.v[r], q.m, c->scan.part, nb, q.uniq, q.off,
+                                     q.inv, q.pos, q.n_uniq);
+    c->launches += 3;
+}
+
+// ============================================================================ owner side (world > 1)
+// owned entries of all ranks -> composite key (lk * world + r), stable compaction
+__global__ void k_owned_count(const int32_t* __restrict__ ids32, const int32_t* __restrict__ counts, int world,
+                              int M, int F, int g, int32_t* part, int nblk) {
+    __shared__ int sm[8];
+    int total = world * M, lo, hi;
+    chunk_range(total, nblk, blockIdx.x, lo, hi);
+    int cnt = 0;
+    for (int e = lo + threadIdx.x; e < hi; e += blockDim.x) {
+        int r = e / M, i = e - r * M;
+        cnt += (i < counts[r] * F) && (ids32[e] % world == g);
+    }
+    for (int o = 16; o; o >>= 1) cnt += __shfl_xor_sync(FULL, cnt, o);
+    if ((threadIdx.x & 31) == 0) sm[threadIdx.x >> 5] = cnt;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int t = 0;
+        for (int i = 0; i < 8; i++) t += sm[i];
+        part[blockIdx.x] = t;
+    }
+}
+
+__global__ void k_owned_emit(const int32_t* __restrict__ ids32, const int32_t* __restrict__ counts, int world,
+                             int M, int F, int g, const int32_t* __restrict__ part, int nblk,
+                             uint32_t* __restrict__ sk, int32_t* __restrict__ sv, int32_t* d_cnt) {
+    __shared__ int smw[8];
+    int total = world * M, lo, hi;
+    chunk_range(total, nblk, blockIdx.x, lo, hi);
+    int run = part[blockIdx.x];
+    for (int base = lo; base < hi; base += kTile) {
+        int e = base + threadIdx.x;
+        int own = 0, r = 0, k = 0;
+        if (e < hi) {
+            r = e / M;
+            int i = e - r * M;
+            if (i < counts[r] * F) {
+                k = ids32[e];
+                own = (k % world == g);
+            }
+        }
+        int tot;
+        int ex = block_excl_scan(own, smw, &tot);
+        if (own) {
+            sk[run + ex] = (uint32_t)(k / world) * (uint32_t)world + (uint32_t)r;
+            sv[run + ex] = r;
+        }
+        run += tot;
+    }
+    if (blockIdx.x == nblk - 1 && threadIdx.x == 0) *d_cnt = run;
+}
+
+// unique (lk, r) pairs sorted by (lk, r) -> per-block counts of (lk heads, rank r pairs)
+__global__ void k_pairs_count(const uint32_t* __restrict__ ks, const int32_t* d_n, int world, int32_t* part,
+                              int nblk) {
+    // part layout: [(world+1)][nblk], counter 0 = lk heads, 1+r = pairs of rank r
+    __shared__ int sm[33];
+    if (threadIdx.x < 33) sm[threadIdx.x] = 0;
+    __syncthreads();
+    int lo, hi;
+    chunk_range(*d_n, nblk, blockIdx.x, lo, hi);
+    for (int i = lo + threadIdx.x; i < hi; i += blockDim.x) {
+        uint32_t key = ks[i];
+        bool pair_head = (i == 0 || ks[i - 1] != key);
+        if (!pair_head) continue;
+        uint32_t lk = key / world;
+        bool lk_head = (i == 0 || ks[i - 1] / world != lk);
+        if (lk_head) atomicAdd(&sm[0], 1);
+        atomicAdd(&sm[1 + key % world], 1);
+    }
+    __syncthreads();
+    if (threadIdx.x <= world) part[threadIdx.x * nblk + blockIdx.x] = sm[threadIdx.x];
+}
+
+__global__ void k_pairs_emit(const uint32_t* __restrict__ ks, const int32_t* d_n, int world, const int32_t* part,
+                             int nblk, int capT, int32_t* __restrict__ T, uint32_t* __restrict__ Tmask,
+                             int32_t* __restrict__ Tidx, int32_t* d_nT) {
+    __shared__ int smw[8];
+    __shared__ int run[33];
+    const int n = *d_n;
+    if (threadIdx.x <= world) run[threadIdx.x] = part[threadIdx.x * nblk + blockIdx.x];
+    __syncthreads();
+    int lo, hi;
+    chunk_range(n, nblk, blockIdx.x, lo, hi);
+    for (int base = lo; base < hi; base += kTile) {
+        int i = base + threadIdx.x;
+        bool valid = i < hi;
+        uint32_t key = valid ? ks[i] : 0u;
+        bool ph = valid && (i == 0 || ks[i - 1] != key);
+        uint32_t lk = key / world;
+        int r = (int)(key % world);
+        bool lh = ph && (i == 0 || ks[i - 1] / world != lk);
+        int tot;
+        int ex = block_excl_scan(lh ? 1 : 0, smw, &tot);
+        int j = run[0] + ex + (lh ? 1 : 0) - 1;  // T index of this pair
+        // rank-local index: exclusive count of earlier pairs of rank r
+        int ridx = 0;
+        for (int q = 0; q < world; q++) {
+            int t2;
+            int e2 = block_excl_scan((ph && r == q) ? 1 : 0, smw, &t2);
+            if (q == r) ridx = run[1 + q] + e2;
+            __syncthreads();
+            if (threadIdx.x == 0) run[1 + q] += t2;
+        }
+        if (ph) {
+            if (lh) T[j] = (int32_t)lk;
+            atomicOr(&Tmask[j], 1u << r);
+            Tidx[(int64_t)r * capT + j] = ridx;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) run[0] += tot;
+        __syncthreads();
+    }
+    if (blockIdx.x == nblk - 1 && threadIdx.x == 0) *d_nT = run[0];
+}
+
+// grouping of this rank's uniq by owner: owner keys for a 1-pass stable sort
+__global__ void k_owner_keys(const int32_t* __restrict__ uniq, const int32_t* d_nu, int world,
+                             uint32_t* __restrict__ sk, int32_t* __restrict__ sv) {
+    int n = *d_nu;
+    for (int u = blockIdx.x * blockDim.x + threadIdx.x; u < n; u += gridDim.x * blockDim.x) {
+        sk[u] = (uint32_t)(uniq[u] % world);
+        sv[u] = u;
+    }
+}
+__global__ void k_goff(const uint32_t* __restrict__ sk, const int32_t* d_nu, int world, int32_t* goff) {
+    int o = threadIdx.x;
+    if (o > world) return;
+    int n = *d_nu, lo = 0, hi = n;
+    while (lo < hi) {  // lower_bound of o
+        int mid = (lo + hi) >> 1;
+        if ((int)sk[mid] < o) lo = mid + 1;
+        else hi = mid;
+    }
+    goff[o] = lo;
+}
+__global__ void k_copy_i32(const int32_t* __restrict__ a, int32_t* __restrict__ b, const int32_t* d_n) {
+    int n = *d_n;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) b[i] = a[i];
+}
+
+void launch_owner_side(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st) {
+    (void)t;
+    const int n = c->n;
+    const int nb = c->scan.nblk;
+    // (1) owned entries of all ranks, composite key (lk, r)
+    cudaMemsetAsync(q.Tmask, 0, c->capT * sizeof(uint32_t), st);
+    k_owned_count<<<nb, 256, 0, st>>>(q.ids, q.counts, n, c->M, c->F, c->g, c->scan.part, nb);
+    k_scan_small<<<1, 1024, 0, st>>>(c->scan.part, nb, nullptr);
+    k_owned_emit<<<nb, 256, 0, st>>>(q.ids, q.counts, n, c->M, c->F, c->g, c->scan.part, nb, c->sort.k[0],
+                                     c->sort.v[0], c->owned_cnt);
+    c->launches += 3;
+    int bits = 1;
+    while ((((int64_t)1) << bits) < ((c->No + 1) * (int64_t)n)) bits++;
+    int r = sort_pairs(c->sort, c->owned_cnt, bits, st, &c->launches);
+    // (2) unique pairs -> T, masks, per-rank indices
+    k_pairs_count<<<nb, 256, 0, st>>>(c->sort.k[r], c->owned_cnt, n, c->scan.part, nb);
+    for (int qq = 0; qq <= n; qq++) {
+        k_scan_small<<<1, 1024, 0, st>>>(c->scan.part + (size_t)qq * nb, nb, nullptr);
+        c->launches++;
+    }
+    k_pairs_emit<<<nb, 256, 0, st>>>(c->sort.k[r], c->owned_cnt, n, c->scan.part, nb, (int)c->capT, q.T, q.Tmask,
+                                     q.Tidx, q.nT);
+    c->launches += 2;
+    // (3) this rank's uniq grouped by owner (stable 1-pass partition)
+    k_owner_keys<<<grid_for(c->M, 256), 256, 0, st>>>(q.uniq, q.n_uniq, n, c->sort.k[0], c->sort.v[0]);
+    int obits = 1;
+    while ((1 << obits) < n) obits++;
+    int r2 = sort_pairs(c->sort, q.n_uniq, obits, st, &c->launches);
+    k_copy_i32<<<grid_for(c->M, 256), 256, 0, st>>>(c->sort.v[r2], q.gl, q.n_uniq);
+    k_goff<<<1, 64, 0, st>>>(c->sort.k[r2], q.n_uniq, n, q.goff);
+    c->launches += 3;
+}
+
+// ============================================================================ scheduler (P2F)
+// warp-aggregated append of (row, p) to the newly-bucketed list
+__device__ __forceinline__ void nb_append(int32_t* rows, int32_t* ps, int32_t* cnt, bool pred, int32_t lk,
+                                          int32_t p) {
+    unsigned m = __ballot_sync(__activemask(), pred);
+    if (!pred) return;
+    int leader = __ffs(m) - 1, lane = threadIdx.x & 31;
+    int base = 0;
+    if (lane == leader) base = atomicAdd(cnt, __popc(m));
+    base = __shfl_sync(m, base, leader);
+    int at = base + __popc(m & lanemask_lt());
+    rows[at] = lk;
+    ps[at] = p;
+}
+
+// a1: set read-ring bits of step t for the owned rows read at t; AdjustPriority inf -> t
+__global__ void k_ingest_bits(const int32_t* __restrict__ T, const uint32_t* __restrict__ Tmask,
+                              const int32_t* d_nT, int world, int g, int bit, int32_t t, int adjust,
+                              const int32_t* __restrict__ slot, uint64_t* __restrict__ rbits,
+                              int32_t* __restrict__ state, int32_t* nb_rows, int32_t* nb_p, int32_t* nb_cnt) {
+    int n = *d_nT;
+    int nloop = (n + blockDim.x * gridDim.x - 1) / (blockDim.x * gridDim.x) * (blockDim.x * gridDim.x);
+    for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < nloop; j += gridDim.x * blockDim.x) {
+        bool valid = j < n;
+        bool app = false;
+        int32_t lk = 0;
+        if (valid) {
+            lk = T[j];
+            uint32_t mask = (world > 1) ? Tmask[j] : 1u;
+            bool host = (mask & ~(1u << g)) != 0u || slot[lk] < 0;
+            uint64_t b = (1ull << bit) | (host ? (1ull << (32 + bit)) : 0ull);
+            rbits[lk] |= b;
+            if (adjust && state[lk] == ST_INF) {
+                if (host) {
+                    state[lk] = ST_CLEAN;
+                    app = true;
+                } else {
+                    state[lk] = ST_EXEMPT;
+                }
+            }
+        }
+        nb_append(nb_rows, nb_p, nb_cnt, app, lk, t);
+    }
+}
+
+// a9: priority of the rows updated at s-1 = next access step within [s, s+L-1] (Eq. 1)
+__global__ void k_bucket_prev(const int32_t* __restrict__ T, const int32_t* d_nT, int32_t s, int write_through,
+                              const uint64_t* __restrict__ rbits, int32_t* __restrict__ state, int32_t* nb_rows,
+                              int32_t* nb_p, int32_t* nb_cnt) {
+    int n = *d_nT;
+    int nloop = (n + blockDim.x * gridDim.x - 1) / (blockDim.x * gridDim.x) * (blockDim.x * gridDim.x);
+    const int rot = s & 31;
+    for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < nloop; j += gridDim.x * blockDim.x) {
+        bool app = false;
+        int32_t lk = 0, p = s;
+        if (j < n) {
+            lk = T[j];
+            uint64_t b = rbits[lk];
+            uint32_t any = (uint32_t)b, hst = (uint32_t)(b >> 32);
+            if (write_through) {
+                state[lk] = ST_CLEAN;
+                app = true;
+            } else {
+                uint32_t r = (any >> rot) | (rot ? (any << (32 - rot)) : 0u);
+                if (r == 0u) {
+                    state[lk] = ST_INF;
+                } else {
+                    int off = __ffs(r) - 1;
+                    p = s + off;
+                    if ((hst >> ((rot + off) & 31)) & 1u) {
+                        state[lk] = ST_CLEAN;  // flush scheduled before gate p
+                        app = true;
+                    } else {
+                        state[lk] = ST_EXEMPT;
+                    }
+                }
+            }
+        }
+        nb_append(nb_rows, nb_p, nb_cnt, app, lk, p);
+    }
+}
+
+// two-level PQ level 1: counting sort of the newly bucketed rows by deadline p - s in [0, L)
+__global__ void k_bucket_hist(const int32_t* __restrict__ nb_p, const int32_t* nb_cnt, int32_t s, int L,
+                              int32_t* bk_off /*[L+1], zeroed*/) {
+    __shared__ int h[32];
+    if (threadIdx.x < 32) h[threadIdx.x] = 0;
+    __syncthreads();
+    int n = *nb_cnt;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
+        atomicAdd(&h[nb_p[i] - s], 1);
+    __syncthreads();
+    if (threadIdx.x < L && h[threadIdx.x]) atomicAdd(&bk_off[threadIdx.x + 1], h[threadIdx.x]);
+}
+__global__ void k_bucket_scan(int32_t* bk_off, int L, int32_t* cursor) {
+    if (threadIdx.x == 0) {
+        bk_off[0] = 0;
+        for (int i = 1; i <= L; i++) bk_off[i] += bk_off[i - 1];
+        for (int i = 0; i < L; i++) cursor[i] = bk_off[i];
+    }
+}
+__global__ void k_bucket_scatter(const int32_t* __restrict__ nb_rows, const int32_t* __restrict__ nb_p,
+                                 const int32_t* nb_cnt, int32_t s, int32_t* cursor, int32_t* __restrict__ bk_rows,
+                                 int32_t* __restrict__ bk_p) {
+    int n = *nb_cnt;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+        int p = nb_p[i];
+        int at = atomicAdd(&cursor[p - s], 1);
+        bk_rows[at] = nb_rows[i];
+        bk_p[at] = p;
+    }
+}
+
+// a11 age-out: cold rows of pool segment u still dirty with priority inf
+__global__ void k_ageout(const int32_t* __restrict__ pkey, const int32_t* pcount_seg, int32_t u,
+                         const int32_t* __restrict__ last_upd, int32_t* __restrict__ state, int32_t* age_rows,
+                         int32_t* age_cnt) {
+    int n = *pcount_seg;
+    int nloop = (n + blockDim.x * gridDim.x - 1) / (blockDim.x * gridDim.x) * (blockDim.x * gridDim.x);
+    for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < nloop; j += gridDim.x * blockDim.x) {
+        bool app = false;
+        int32_t lk = 0;
+        if (j < n) {
+            lk = pkey[j];
+            if (lk >= 0 && state[lk] == ST_INF && last_upd[lk] == u) {
+                state[lk] = ST_CLEAN;
+                app = true;
+            }
+        }
+        unsigned m = __ballot_sync(FULL, app);
+        if (app) {
+            int leader = __ffs(m) - 1, lane = threadIdx.x & 31, base = 0;
+            if (lane == leader) base = atomicAdd(age_cnt, __popc(m));
+            base = __shfl_sync(m, base, leader);
+            age_rows[base + __popc(m & lanemask_lt())] = lk;
+        }
+    }
+}
+
+void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, cudaStream_t st) {
+    k_ingest_bits<<<grid_for(c->capT, 256), 256, 0, st>>>(q.T, q.Tmask, q.nT, c->n, c->g, (int)(t & 31), (int32_t)t,
+                                                           adjust, c->slot, c->rbits, c->state, c->nb_rows,
+                                                           c->nb_p, c->nb_cnt);
+    c->launches++;
+}
+
+void launch_bucket(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStream_t st) {
+    const int L = c->L;
+    if (prev) {
+        k_bucket_prev<<<grid_for(c->capT, 256), 256, 0, st>>>(prev->T, prev->nT, (int32_t)s,
+                                                               c->cfg.mode == FRUGAL_MODE_WRITE_THROUGH, c->rbits,
+                                                               c->state, c->nb_rows, c->nb_p, c->nb_cnt);
+        c->launches++;
+    }
+    cudaMemsetAsync(c->bk_off[par], 0, (L + 1) * sizeof(int32_t), st);
+    int32_t* cursor = c->sched_info + 8;  // [L] scratch
+    k_bucket_hist<<<grid_for(2 * c->capT, 256, 2), 256, 0, st>>>(c->nb_p, c->nb_cnt, (int32_t)s, L, c->bk_off[par]);
+    k_bucket_scan<<<1, 32, 0, st>>>(c->bk_off[par], L, cursor);
+    k_bucket_scatter<<<grid_for(2 * c->capT, 256, 2), 256, 0, st>>>(c->nb_rows, c->nb_p, c->nb_cnt, (int32_t)s,
+                                                                     cursor, c->bk_rows[par], c->bk_p[par]);
+    c->launches += 3;
+    // age-out of cold rows updated at u = s-1-D
+    cudaMemsetAsync(c->age_cnt[par], 0, sizeof(int32_t), st);
+    int64_t u = s - 1 - c->D;
+    if (u >= 0) {
+        int seg = (int)(u % c->P);
+        k_ageout<<<grid_for(c->capT, 256), 256, 0, st>>>(c->pkey + (size_t)seg * c->capT, c->pcount + seg,
+                                                          (int32_t)u, c->last_upd, c->state, c->age_rows[par],
+                                                          c->age_cnt[par]);
+        c->launches++;
+    }
+}
+
+// ============================================================================ row movers
+// a10/a11/a12: flush rows (local ids) to the host table.  hot: w (and G if with_hot_g)
+// from the HBM cache; cold: w and G from the dirty pool.  Zero-copy stores to host.
+template <int GS>
+__global__ void k_flush_rows(const int32_t* __restrict__ rows, const int32_t* d_begin, const int32_t* d_end,
+                             int world, int g, int d4, int with_hot_g, int adagrad,
+                             const int32_t* __restrict__ slot, const int32_t* __restrict__ last_upd,
+                             const int32_t* __restrict__ pool_idx, int P, int64_t capT,
+                             const float4* __restrict__ cw, const float4* __restrict__ cG,
+                             const float4* __restrict__ pw, const float4* __restrict__ pG, float4* hw, float4* hG) {
+    int64_t gid, gs;
+    int l;
+    RowGroup<GS>::ids(gid, gs, l);
+    const int b = d_begin ? *d_begin : 0, e = *d_end;
+    for (int64_t a = b + gid; a < e; a += gs) {
+        int32_t lk = rows[a];
+        int64_t k = (int64_t)lk * world + g;
+        int sl = slot[lk];
+        if (sl >= 0) {
+            const float4* sw = cw + (int64_t)sl * d4;
+            for (int v = l; v < d4; v += GS) hw[k * d4 + v] = sw[v];
+            if (with_hot_g && adagrad) {
+                const float4* sg = cG + (int64_t)sl * d4;
+                for (int v = l; v < d4; v += GS) hG[k * d4 + v] = sg[v];
+            }
+        } else {
+            int64_t pr = (int64_t)(last_upd[lk] % P) * capT + pool_idx[lk];
+            const float4* sw = pw + pr * d4;
+            for (int v = l; v < d4; v += GS) hw[k * d4 + v] = sw[v];
+            if (adagrad) {
+                const float4* sg = pG + pr * d4;
+                for (int v = l; v < d4; v += GS) hG[k * d4 + v] = sg[v];
+            }
+        }
+    }
+    __threadfence_system();
+}
+
+void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begin, const int32_t* d_end,
+                       int with_hot_g, cudaStream_t st) {
+    const int d4 = c->d / 4, gs = group_size(d4);
+    int grid = grid_for(c->capT * (int64_t)gs, 256, 4);
+    DISPATCH_GS(gs, (k_flush_rows<GS><<<grid, 256, 0, st>>>(
+                        rows, d_begin, d_end, c->n, c->g, d4, with_hot_g, c->cfg.opt == FRUGAL_ADAGRAD, c->slot,
+                        c->last_upd, c->pool_idx, c->P, c->capT, (const float4*)c->cw, (const float4*)c->cG,
+                        (const float4*)c->pw, (const float4*)c->pG, (float4*)c->dh_w, (float4*)c->dh_G)));
+    c->launches++;
+}
+
+// a4 gather: unique rows -> staging (owned hot: HBM cache; else host, zero-copy)
+template <int GS>
+__global__ void k_gather_uniq(const int32_t* __restrict__ uniq, const int32_t* d_nu, int world, int g, int d4,
+                              const int32_t* __restrict__ slot, const float4* __restrict__ cw,
+                              const float4* hw, float4* __restrict__ rows) {
+    int64_t gid, gs;
+    int l;
+    RowGroup<GS>::ids(gid, gs, l);
+    const int n = *d_nu;
+    for (int64_t u = gid; u < n; u += gs) {
+        int32_t k = uniq[u];
+        const float4* src = hw + (int64_t)k * d4;
+        if (k % world == g) {
+            int sl = slot[k / world];
+            if (sl >= 0) src = cw + (int64_t)sl * d4;
+        }
+        for (int v = l; v < d4; v += GS) rows[u * d4 + v] = src[v];
+    }
+}
+// a4 expand: out[i] = rows[inv[i]]
+template <int GS>
+__global__ void k_expand(const int32_t* __restrict__ inv, const int32_t* d_m, int d4, const float4* __restrict__ rows,
+                         float4* __restrict__ out) {
+    int64_t gid, gs;
+    int l;
+    RowGroup<GS>::ids(gid, gs, l);
+    const int m = *d_m;
+    for (int64_t i = gid; i < m; i += gs) {
+        const float4* src = rows + (int64_t)inv[i] * d4;
+        for (int v = l; v < d4; v += GS) out[i * d4 + v] = src[v];
+    }
+}
+
+void launch_gather(frugal_ctx* c, QueueSlot& q, float* out, cudaStream_t st) {
+    const int d4 = c->d / 4, gs = group_size(d4);
+    int grid = grid_for((int64_t)c->M * gs, 256, 8);
+    DISPATCH_GS(gs, (k_gather_uniq<GS><<<grid, 256, 0, st>>>(q.uniq, q.n_uniq, c->n, c->g, d4, c->slot,
+                                                             (const float4*)c->cw, (const float4*)c->dh_w,
+                                                             (float4*)c->rows)));
+    c->launches++;
+}
+void launch_expand(frugal_ctx* c, QueueSlot& q, float* out, cudaStream_t st) {
+    const int d4 = c->d / 4, gs = group_size(d4);
+    int grid = grid_for((int64_t)c->M * gs, 256, 8);
+    DISPATCH_GS(gs, (k_expand<GS><<<grid, 256, 0, st>>>(q.inv, q.m, d4, (const float4*)c->rows,
+                                                        (float4*)out)));
+    c->launches++;
+}
+
+// ============================================================================ model glue
+template <int J>
+__global__ void k_dot_model(const float* __restrict__ emb, const float* __restrict__ x, const float* __restrict__ y,
+                            float* __restrict__ grad, double* loss, int count, int F, int d, double nb) {
+    const int lane = threadIdx.x & 31;
+    const int wid = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int nw = (gridDim.x * blockDim.x) >> 5;
+    double lsum = 0.0;
+    for (int b = wid; b < count; b += nw) {
+        const float* e0 = emb + (int64_t)b * F * d;
+        float S[J];
+#pragma unroll
+        for (int q = 0; q < J; q++) S[q] = 0.0f;
+        double ee = 0.0;
+        for (int f = 0; f < F; f++) {
+#pragma unroll
+            for (int q = 0; q < J; q++) {
+                int j = lane + 32 * q;
+                if (j < d) {
+                    float v = e0[f * d + j];
+                    S[q] = __fadd_rn(S[q], v);
+                    ee += (double)v * (double)v;
+                }
+            }
+        }
+        double sq = 0.0, xs = 0.0;
+        const float* xb = x + (int64_t)b * d;
+#pragma unroll
+        for (int q = 0; q < J; q++) {
+            int j = lane + 32 * q;
+            if (j < d) {
+                sq += (double)S[q] * (double)S[q];
+                xs += (double)xb[j] * (double)S[q];
+            }
+        }
+        for (int o = 16; o; o >>= 1) {
+            sq += __shfl_xor_sync(FULL, sq, o);
+            ee += __shfl_xor_sync(FULL, ee, o);
+            xs += __shfl_xor_sync(FULL, xs, o);
+        }
+        double z = 0.5 * (sq - ee) + xs;
+        double p = 1.0 / (1.0 + exp(-z));
+        double yb = (double)y[b];
+        if (lane == 0) lsum += (z > 0 ? z + log1p(exp(-z)) : log1p(exp(z))) - yb * z;
+        float cc = (float)((p - yb) / nb);  // same rounding as the definition
+        float* g0 = grad + (int64_t)b * F * d;
+        for (int f = 0; f < F; f++) {
+#pragma unroll
+            for (int q = 0; q < J; q++) {
+                int j = lane + 32 * q;
+                if (j < d) {
+                    float t = __fadd_rn(__fsub_rn(S[q], e0[f * d + j]), xb[j]);
+                    g0[f * d + j] = __fmul_rn(cc, t);
+                }
+            }
+        }
+    }
+    if (lane == 0 && lsum != 0.0) atomicAdd(loss, lsum / nb);  // mean over the global batch (R17)
+}
+
+void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const float* x, const float* y, float* grad,
+                      double* loss, int64_t nb, cudaStream_t st) {
+    int count = q.h_counts[c->g];
+    if (count <= 0) return;
+    int J = (c->d + 31) / 32;
+    int grid = grid_for((int64_t)count * 32, 256, 8);
+    const double nbd = (double)nb;
+#define DM(JJ) k_dot_model<JJ><<<grid, 256, 0, st>>>(emb, x, y, grad, loss, count, c->F, c->d, nbd)
+    if (J <= 1) DM(1);
+    else if (J <= 2) DM(2);
+    else if (J <= 4) DM(4);
+    else if (J <= 8) DM(8);
+    else if (J <= 16) DM(16);
+    else DM(32);
+#undef DM
+    c->launches++;
+}
+
+}  // namespace frugal

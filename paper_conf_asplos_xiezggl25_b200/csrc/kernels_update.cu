@@ -1,0 +1,445 @@
+// kernels_update.cu -- backward (segment-reduce, mailbox, fused optimizer), final flush,
+// table/metadata initialisation, cross-rank flags and introspection kernels (sm_100a).
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <algorithm>
+
+#include "frugal_internal.cuh"
+#include "kutil.cuh"
+
+namespace frugal {
+
+__device__ __forceinline__ float4 add4(float4 a, float4 b) {
+    return make_float4(__fadd_rn(a.x, b.x), __fadd_rn(a.y, b.y), __fadd_rn(a.z, b.z), __fadd_rn(a.w, b.w));
+}
+
+// ============================================================================ a6 segment-reduce
+// P[q] = sum over the occurrences of unique row u in the canonical fixed order
+// (reading R23): positions ascending, cut into chunks of kChunk; each chunk summed
+// sequentially, chunk sums added sequentially.  world == 1: q = u.  world > 1: q walks
+// the owner-grouped order (gl); rows owned by this rank stay in HBM (Pp[q]), the others
+// go to this rank's host mailbox (zero-copy stores; §3.2 "update
+// staging queue").  Segments longer than one chunk (the Zipf head) are deferred to
+// k_segreduce_long, which computes their chunks in parallel.
+constexpr int kChunk = 64;
+
+template <int GS>
+__device__ __forceinline__ float4 chunk_sum(const float4* __restrict__ grad, const int32_t* __restrict__ pos, int b,
+                                            int e, int d4, int v) {
+    float4 acc = grad[(int64_t)pos[b] * d4 + v];
+    int j = b + 1;
+    for (; j + 8 <= e; j += 8) {  // 8 loads in flight, adds in position order
+        float4 x[8];
+#pragma unroll
+        for (int q = 0; q < 8; q++) x[q] = grad[(int64_t)pos[j + q] * d4 + v];
+#pragma unroll
+        for (int q = 0; q < 8; q++) acc = add4(acc, x[q]);
+    }
+    for (; j < e; j++) acc = add4(acc, grad[(int64_t)pos[j] * d4 + v]);
+    return acc;
+}
+
+template <int GS>
+__global__ void k_segreduce(const int32_t* __restrict__ off, const int32_t* __restrict__ pos,
+                            const int32_t* d_nu, const int32_t* __restrict__ gl, const int32_t* __restrict__ goff,
+                            int g, int d4, const float4* __restrict__ grad, float4* __restrict__ Pp, float4* mail,
+                            int32_t* long_q, int32_t* long_cnt) {
+    int64_t gid, gs;
+    int l;
+    RowGroup<GS>::ids(gid, gs, l);
+    const int n = *d_nu;
+    int own_lo = 0, own_hi = n;
+    if (gl) {
+        own_lo = goff[g];
+        own_hi = goff[g + 1];
+    }
+    for (int64_t q = gid; q < n; q += gs) {
+        const int u = gl ? gl[q] : (int)q;
+        const int b = off[u], e = off[u + 1];
+        if (e - b > kChunk) {
+            if (l == 0) long_q[atomicAdd(long_cnt, 1)] = (int32_t)q;
+            continue;
+        }
+        float4* dst = (q >= own_lo && q < own_hi) ? (Pp + q * d4) : (mail + q * d4);
+        for (int v = l; v < d4; v += GS) dst[v] = chunk_sum<GS>(grad, pos, b, e, d4, v);
+    }
+    if (gl) __threadfence_system();
+}
+
+// one block per long segment: row groups compute chunk sums into scratch (indexed by
+// the chunk's first position), then one group adds them in order
+template <int GS>
+__global__ void k_segreduce_long(const int32_t* __restrict__ off, const int32_t* __restrict__ pos,
+                                 const int32_t* __restrict__ gl, const int32_t* __restrict__ goff, int g, int d4,
+                                 const float4* __restrict__ grad, float4* __restrict__ Pp, float4* mail,
+                                 const int32_t* __restrict__ long_q, const int32_t* long_cnt,
+                                 float4* __restrict__ scratch) {
+    const int grp = threadIdx.x / GS, ngrp = blockDim.x / GS, l = threadIdx.x & (GS - 1);
+    const int nl = *long_cnt;
+    int own_lo = 0, own_hi = 0x7fffffff;
+    if (gl) {
+        own_lo = goff[g];
+        own_hi = goff[g + 1];
+    }
+    for (int t = blockIdx.x; t < nl; t += gridDim.x) {
+        const int q = long_q[t];
+        const int u = gl ? gl[q] : q;
+        const int b = off[u], e = off[u + 1];
+        const int nch = (e - b + kChunk - 1) / kChunk;
+        for (int c = grp; c < nch; c += ngrp) {
+            const int c0 = b + c * kChunk, c1 = min(e, c0 + kChunk);
+            for (int v = l; v < d4; v += GS) scratch[(int64_t)c0 * d4 + v] = chunk_sum<GS>(grad, pos, c0, c1, d4, v);
+        }
+        __syncthreads();
+        if (grp == 0) {
+            float4* dst = (q >= own_lo && q < own_hi) ? (Pp + (int64_t)q * d4) : (mail + (int64_t)q * d4);
+            for (int v = l; v < d4; v += GS) {
+                float4 acc = scratch[(int64_t)b * d4 + v];
+                for (int c = 1; c < nch; c++) acc = add4(acc, scratch[(int64_t)(b + c * kChunk) * d4 + v]);
+                dst[v] = acc;
+            }
+        }
+        __syncthreads();
+    }
+    if (gl) __threadfence_system();
+}
+
+void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, cudaStream_t st) {
+    const int d4 = c->d / 4, gs = group_size(d4);
+    int grid = grid_for((int64_t)c->M * gs, 256, 8);
+    const bool multi = c->n > 1;
+    float4* mail = multi ? (float4*)(c->dh_mail + ((size_t)par * c->n + c->g) * c->mail_stride + 256) : nullptr;
+    cudaMemsetAsync(c->long_cnt, 0, 4, st);
+    DISPATCH_GS(gs, (k_segreduce<GS><<<grid, 256, 0, st>>>(q.off, q.pos, q.n_uniq, multi ? q.gl : nullptr, q.goff,
+                                                           c->g, d4, (const float4*)grad, (float4*)c->Pp, mail,
+                                                           c->long_q, c->long_cnt)));
+    int lgrid = (int)std::min<int64_t>(c->M / (kChunk + 1) + 1, kSMs * 4);
+    DISPATCH_GS(gs, (k_segreduce_long<GS><<<lgrid, 256, 0, st>>>(q.off, q.pos, multi ? q.gl : nullptr, q.goff, c->g,
+                                                                 d4, (const float4*)grad, (float4*)c->Pp, mail,
+                                                                 c->long_q, c->long_cnt,
+                                                                 (float4*)c->chunk_scratch)));
+    c->launches += 2;
+}
+
+// mailbox header of (parity, this sender): goff[0..world]
+__global__ void k_mail_header(const int32_t* __restrict__ goff, int world, int32_t* hdr) {
+    if (threadIdx.x <= world) hdr[threadIdx.x] = goff[threadIdx.x];
+    __threadfence_system();
+}
+void launch_mail_header(frugal_ctx* c, QueueSlot& q, int par, cudaStream_t st) {
+    int32_t* hdr = (int32_t*)(c->dh_mail + ((size_t)par * c->n + c->g) * c->mail_stride);
+    k_mail_header<<<1, 64, 0, st>>>(q.goff, c->n, hdr);
+    c->launches++;
+}
+
+// ============================================================================ a8 merge + fused optimizer
+// For each owned row touched at s (T, ascending): g = sum of partials over ranks in
+// ascending order (own from HBM, others from their host mailboxes), then SGD/Adagrad
+// (elementwise, each op rounded separately).  Hot rows update the HBM cache in place;
+// cold rows read (w, G) fresh from the host table and go to pool segment s % P.
+// Marks dirty (last update s) and consumes read bit s.
+template <int GS>
+__global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, const uint32_t* __restrict__ Tmask,
+                            const int32_t* __restrict__ Tidx, int64_t capT, int world, int g, int d4, int32_t s,
+                            int adagrad, float lr, float eps, const float4* __restrict__ Pp,
+                            const int32_t* __restrict__ goff_own, const char* mail_par, size_t mail_stride,
+                            const float4* __restrict__ rows_w, const int32_t* __restrict__ slot,
+                            int32_t* __restrict__ state, int32_t* __restrict__ last_upd, int32_t* __restrict__ pool_idx,
+                            uint64_t* __restrict__ rbits, float4* __restrict__ cw, float4* __restrict__ cG,
+                            float4* __restrict__ pw, float4* __restrict__ pG, int32_t* __restrict__ pkey,
+                            int32_t* pcount, const float4* hw, const float4* hG) {
+    int64_t gid, gs;
+    int l;
+    RowGroup<GS>::ids(gid, gs, l);
+    const int n = *d_nT;
+    const uint64_t clear = ~((1ull << (s & 31)) | (1ull << (32 + (s & 31))));
+    for (int64_t j = gid; j < n; j += gs) {
+        const int32_t lk = T[j];
+        const int64_t k = (int64_t)lk * world + g;
+        const int sl = slot[lk];
+        uint32_t mask = 1u;
+        if (world > 1) mask = Tmask[j];
+        for (int v = l; v < d4; v += GS) {
+            float4 acc;
+            if (world == 1) {
+                acc = Pp[j * d4 + v];
+            } else {
+                bool first = true;
+                for (int r = 0; r < world; r++) {
+                    if (!((mask >> r) & 1u)) continue;
+                    const int idx = Tidx[(int64_t)r * capT + j];
+                    float4 x;
+                    if (r == g) {
+                        x = Pp[(int64_t)(goff_own[g] + idx) * d4 + v];
+                    } else {
+                        const char* mb = mail_par + (size_t)r * mail_stride;
+                        const int base = ((const int32_t*)mb)[g];
+                        x = ((const float4*)(mb + 256))[(int64_t)(base + idx) * d4 + v];
+                    }
+                    acc = first ? x : add4(acc, x);
+                    first = false;
+                }
+            }
+            float4 w, G = make_float4(0.f, 0.f, 0.f, 0.f);
+            if (sl >= 0) {
+                w = cw[(int64_t)sl * d4 + v];
+                if (adagrad) G = cG[(int64_t)sl * d4 + v];
+            } else {
+                w = rows_w ? rows_w[j * d4 + v] : hw[k * d4 + v];
+                if (adagrad) G = hG[k * d4 + v];
+            }
+            float* wp = &w.x;
+            float* Gp = &G.x;
+            const float* gp = &acc.x;
+#pragma unroll
+            for (int c = 0; c < 4; c++) {
+                if (adagrad) {
+                    Gp[c] = __fadd_rn(Gp[c], __fmul_rn(gp[c], gp[c]));
+                    float num = __fmul_rn(lr, gp[c]);
+                    float den = __fadd_rn(__fsqrt_rn(Gp[c]), eps);
+                    wp[c] = __fsub_rn(wp[c], __fdiv_rn(num, den));
+                } else {
+                    wp[c] = __fsub_rn(wp[c], __fmul_rn(lr, gp[c]));
+                }
+            }
+            if (sl >= 0) {
+                cw[(int64_t)sl * d4 + v] = w;
+                if (adagrad) cG[(int64_t)sl * d4 + v] = G;
+            } else {
+                pw[j * d4 + v] = w;
+                if (adagrad) pG[j * d4 + v] = G;
+            }
+        }
+        if (l == 0) {
+            state[lk] = ST_UPDATED;
+            last_upd[lk] = s;
+            rbits[lk] &= clear;
+            if (sl < 0) pool_idx[lk] = (int32_t)j;
+            pkey[j] = sl < 0 ? lk : -1;
+        }
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) *pcount = n;
+}
+
+void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, cudaStream_t st) {
+    const int d4 = c->d / 4, gs = group_size(d4);
+    int grid = grid_for(c->capT * gs, 256, 8);
+    const int seg = (int)(s % c->P);
+    const size_t pofs = (size_t)seg * c->capT * d4;
+    const bool adag = c->cfg.opt == FRUGAL_ADAGRAD;
+    const char* mail_par = c->n > 1 ? c->dh_mail + (size_t)par * c->n * c->mail_stride : nullptr;
+    // world == 1: the owner gathered every touched row itself this step (T == uniq),
+    // so the cold rows' w is taken from the staging rows instead of a second host read.
+    const float4* rows_w = c->n == 1 ? (const float4*)c->rows : nullptr;
+    DISPATCH_GS(gs, (k_optimizer<GS><<<grid, 256, 0, st>>>(
+                        q.T, q.nT, q.Tmask, q.Tidx, c->capT, c->n, c->g, d4, (int32_t)s, adag, c->cfg.lr, c->cfg.eps,
+                        (const float4*)c->Pp, q.goff, mail_par, c->mail_stride, rows_w, c->slot, c->state,
+                        c->last_upd, c->pool_idx, c->rbits, (float4*)c->cw, (float4*)c->cG,
+                        (float4*)c->pw + pofs, adag ? (float4*)c->pG + pofs : nullptr,
+                        c->pkey + (size_t)seg * c->capT, c->pcount + seg, (const float4*)c->dh_w,
+                        (const float4*)c->dh_G)));
+    c->launches++;
+}
+
+// ============================================================================ a12 final flush
+__global__ void k_final_collect(int64_t No, int32_t* __restrict__ state, int32_t* rows, int32_t* cnt) {
+    for (int64_t lk = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; lk < ((No + 31) / 32) * 32;
+         lk += (int64_t)gridDim.x * blockDim.x) {
+        bool dirty = lk < No && state[lk] != ST_CLEAN;
+        if (dirty) state[lk] = ST_CLEAN;
+        unsigned m = __ballot_sync(FULL, dirty);
+        if (dirty) {
+            int leader = __ffs(m) - 1, lane = threadIdx.x & 31, base = 0;
+            if (lane == leader) base = atomicAdd(cnt, __popc(m));
+            base = __shfl_sync(m, base, leader);
+            rows[base + __popc(m & lanemask_lt())] = (int32_t)lk;
+        }
+    }
+}
+template <int GS>
+__global__ void k_hot_g_push(const int32_t* __restrict__ hot_lk, int64_t cap_hot, int world, int g, int d4,
+                             const float4* __restrict__ cG, float4* hG) {
+    int64_t gid, gs;
+    int l;
+    RowGroup<GS>::ids(gid, gs, l);
+    for (int64_t sl = gid; sl < cap_hot; sl += gs) {
+        int64_t k = (int64_t)hot_lk[sl] * world + g;
+        for (int v = l; v < d4; v += GS) hG[k * d4 + v] = cG[sl * d4 + v];
+    }
+    __threadfence_system();
+}
+
+void launch_final_flush(frugal_ctx* c, cudaStream_t st) {
+    cudaMemsetAsync(c->ff_cnt, 0, sizeof(int32_t), st);
+    k_final_collect<<<grid_for(c->No, 256, 8), 256, 0, st>>>(c->No, c->state, c->ff_rows, c->ff_cnt);
+    c->launches++;
+    launch_flush_rows(c, c->ff_rows, nullptr, c->ff_cnt, 1, st);
+    if (c->cfg.opt == FRUGAL_ADAGRAD && c->cap_hot > 0) {
+        const int d4 = c->d / 4, gs = group_size(d4);
+        int grid = grid_for(c->cap_hot * gs, 256, 8);
+        DISPATCH_GS(gs, (k_hot_g_push<GS><<<grid, 256, 0, st>>>(c->hot_lk, c->cap_hot, c->n, c->g, d4,
+                                                                (const float4*)c->cG, (float4*)c->dh_G)));
+        c->launches++;
+    }
+}
+
+// ============================================================================ initialisation
+// w0[k][j] = init_scale * (2u - 1), u = top 24 bits of splitmix64(seed ^ (k*d + j)) / 2^24
+__device__ __forceinline__ uint64_t splitmix64(uint64_t z) {
+    z += 0x9e3779b97f4a7c15ULL;
+    z = (z ^ (z >> 30)) * 0xbf58476d1ce4e5b9ULL;
+    z = (z ^ (z >> 27)) * 0x94d049bb133111ebULL;
+    return z ^ (z >> 31);
+}
+__device__ __forceinline__ float w0(uint64_t seed, int64_t k, int d, int j, float scale) {
+    uint64_t h = splitmix64(seed ^ (uint64_t)(k * (int64_t)d + j));
+    float u = (float)(h >> 40) * (1.0f / 16777216.0f);
+    return __fmul_rn(scale, __fsub_rn(__fmul_rn(2.0f, u), 1.0f));
+}
+
+__global__ void k_init_table(float4* hw, float4* hG, int64_t N, int d, uint64_t seed, float scale, float accum) {
+    const int d4 = d / 4;
+    const int64_t total = N * d4;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+        int64_t k = e / d4;
+        int j = (int)(e - k * d4) * 4;
+        hw[e] = make_float4(w0(seed, k, d, j, scale), w0(seed, k, d, j + 1, scale), w0(seed, k, d, j + 2, scale),
+                            w0(seed, k, d, j + 3, scale));
+        if (hG) hG[e] = make_float4(accum, accum, accum, accum);
+    }
+}
+void launch_init_table(frugal_ctx* c, cudaStream_t st) {
+    k_init_table<<<kSMs * 8, 256, 0, st>>>((float4*)c->dh_w,
+                                           c->cfg.opt == FRUGAL_ADAGRAD ? (float4*)c->dh_G : nullptr, c->N, c->d,
+                                           c->cfg.init_seed, c->cfg.init_scale, c->cfg.init_accum);
+    c->launches++;
+}
+
+__global__ void k_init_meta(int64_t No, int32_t* slot, int32_t* state, int32_t* last_upd, int32_t* pool_idx,
+                            uint64_t* rbits) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < No; i += (int64_t)gridDim.x * blockDim.x) {
+        slot[i] = -1;
+        state[i] = ST_CLEAN;
+        last_upd[i] = -1;
+        pool_idx[i] = -1;
+        rbits[i] = 0ull;
+    }
+}
+// hot slots: d_hot_lk sorted owned local ids; cache rows start at w0 (same pure function)
+__global__ void k_init_hot(const int32_t* __restrict__ hot_lk, int64_t cap_hot, int world, int g, int d,
+                           uint64_t seed, float scale, float accum, int32_t* slot, float* cw, float* cG) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < cap_hot * d;
+         e += (int64_t)gridDim.x * blockDim.x) {
+        int64_t sl = e / d;
+        int j = (int)(e - sl * d);
+        int64_t k = (int64_t)hot_lk[sl] * world + g;
+        cw[e] = w0(seed, k, d, j, scale);
+        if (cG) cG[e] = accum;
+        if (j == 0) slot[hot_lk[sl]] = (int32_t)sl;
+    }
+}
+void launch_init_meta(frugal_ctx* c, const int64_t* unused, int64_t n_hot, cudaStream_t st) {
+    (void)unused;
+    (void)n_hot;
+    k_init_meta<<<grid_for(c->No, 256, 8), 256, 0, st>>>(c->No, c->slot, c->state, c->last_upd, c->pool_idx,
+                                                          c->rbits);
+    c->launches++;
+    if (c->cap_hot > 0) {
+        k_init_hot<<<grid_for(c->cap_hot * c->d, 256, 8), 256, 0, st>>>(
+            c->hot_lk, c->cap_hot, c->n, c->g, c->d, c->cfg.init_seed, c->cfg.init_scale, c->cfg.init_accum,
+            c->slot, c->cw, c->cfg.opt == FRUGAL_ADAGRAD ? c->cG : nullptr);
+        c->launches++;
+    }
+}
+
+// ============================================================================ cross-rank flags (host memory)
+// flags layout: [which][rank] uint32, 16 words (64 B) apart
+__global__ void k_set_flag(uint32_t* f, uint32_t v) {
+    __threadfence_system();
+    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(f), "r"(v) : "memory");
+}
+__global__ void k_wait_flags(const uint32_t* f, int world, uint32_t v, int32_t* err) {
+    int r = threadIdx.x;
+    if (r < world) {
+        const uint32_t* p = f + r * 16;
+        uint64_t t0;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+        while (true) {
+            uint32_t x;
+            asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(x) : "l"(p) : "memory");
+            if ((int32_t)(x - v) >= 0) break;
+            uint64_t t1;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
+            if (t1 - t0 > 120ull * 1000000000ull) {  // 120 s: a peer is gone
+                atomicExch(err, 2);
+                break;
+            }
+            __nanosleep(256);
+        }
+    }
+    __syncwarp();
+    __threadfence_system();
+}
+void launch_set_flag(frugal_ctx* c, int which, uint32_t value, cudaStream_t st) {
+    k_set_flag<<<1, 1, 0, st>>>(c->dh_flags + (which * 32 + c->g) * 16, value);
+    c->launches++;
+}
+void launch_wait_flags(frugal_ctx* c, int which, uint32_t value, cudaStream_t st) {
+    k_wait_flags<<<1, 32, 0, st>>>(c->dh_flags + which * 32 * 16, c->n, value, c->err);
+    c->launches++;
+}
+
+// ============================================================================ introspection
+// authoritative value of owned rows: hot -> cache; cold & dirty -> pool; else host
+__global__ void k_read_rows(const int32_t* __restrict__ lks, int64_t n, int world, int g, int d, int P, int64_t capT,
+                            const int32_t* slot, const int32_t* state, const int32_t* last_upd,
+                            const int32_t* pool_idx, const float* cw, const float* cG, const float* pw,
+                            const float* pG, const float* hw, const float* hG, float* ow, float* oG) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < n * d; e += (int64_t)gridDim.x * blockDim.x) {
+        int64_t a = e / d;
+        int j = (int)(e - a * d);
+        int32_t lk = lks[a];
+        int64_t k = (int64_t)lk * world + g;
+        int sl = slot[lk];
+        float w, G = 0.f;
+        if (sl >= 0) {
+            w = cw[(int64_t)sl * d + j];
+            G = cG ? cG[(int64_t)sl * d + j] : 0.f;
+        } else if (state[lk] == ST_UPDATED || state[lk] == ST_INF) {
+            int64_t pr = (int64_t)(last_upd[lk] % P) * capT + pool_idx[lk];
+            w = pw[pr * d + j];
+            G = pG ? pG[pr * d + j] : 0.f;
+        } else {
+            w = hw[k * d + j];
+            G = hG ? hG[k * d + j] : 0.f;
+        }
+        ow[e] = w;
+        oG[e] = G;
+    }
+}
+void launch_read_rows(frugal_ctx* c, const int32_t* d_lk, int64_t n, float* d_w, float* d_G, cudaStream_t st) {
+    const bool ad = c->cfg.opt == FRUGAL_ADAGRAD;
+    k_read_rows<<<grid_for(n * c->d, 256, 8), 256, 0, st>>>(d_lk, n, c->n, c->g, c->d, c->P, c->capT, c->slot,
+                                                             c->state, c->last_upd, c->pool_idx, c->cw,
+                                                             ad ? c->cG : nullptr, c->pw, ad ? c->pG : nullptr,
+                                                             c->dh_w, ad ? c->dh_G : nullptr, d_w, d_G);
+    c->launches++;
+}
+__global__ void k_read_host(const int64_t* __restrict__ ks, int64_t n, int d, const float* hw, const float* hG,
+                            float* ow, float* oG) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < n * d; e += (int64_t)gridDim.x * blockDim.x) {
+        int64_t a = e / d;
+        int j = (int)(e - a * d);
+        ow[e] = hw[ks[a] * d + j];
+        oG[e] = hG ? hG[ks[a] * d + j] : 0.f;
+    }
+}
+void launch_read_host(frugal_ctx* c, const int64_t* d_k, int64_t n, float* d_w, float* d_G, cudaStream_t st) {
+    k_read_host<<<grid_for(n * c->d, 256, 8), 256, 0, st>>>(d_k, n, c->d, c->dh_w,
+                                                             c->cfg.opt == FRUGAL_ADAGRAD ? c->dh_G : nullptr, d_w,
+                                                             d_G);
+    c->launches++;
+}
+
+}  // namespace frugal

@@ -1,0 +1,62 @@
+// kutil.cuh -- small device helpers shared by the CUDA kernels (not by the oracle).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "frugal_internal.cuh"
+
+namespace frugal {
+
+#define FULL 0xffffffffu
+
+__device__ __forceinline__ unsigned lanemask_lt() {
+    unsigned m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+// grid sized as a multiple of the SM count, capped by the work
+static inline int grid_for(int64_t work, int per_block, int max_waves = 8) {
+    int64_t b = (work + per_block - 1) / per_block;
+    int64_t cap = (int64_t)kSMs * max_waves;
+    if (b > cap) b = cap;
+    if (b < 1) b = 1;
+    return (int)b;
+}
+
+__device__ __forceinline__ void chunk_range(int n, int nblk, int b, int& lo, int& hi) {
+    int per = (n + nblk - 1) / nblk;
+    per = (per + kTile - 1) / kTile * kTile;
+    lo = min(n, b * per);
+    hi = min(n, lo + per);
+}
+
+template <int GS>
+struct RowGroup {
+    // lanes [grp*GS, grp*GS+GS) of the warp handle one row; returns global group id/stride
+    static __device__ __forceinline__ void ids(int64_t& gid, int64_t& gstride, int& l) {
+        int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+        gid = t / GS;
+        gstride = ((int64_t)gridDim.x * blockDim.x) / GS;
+        l = threadIdx.x & (GS - 1);
+    }
+};
+
+static inline int group_size(int d4) {
+    int gs = 1;
+    while (gs < d4 && gs < 32) gs <<= 1;
+    return gs;
+}
+
+#define DISPATCH_GS(gs, ...)                  \
+    switch (gs) {                             \
+        case 1: { constexpr int GS = 1; __VA_ARGS__; } break;   \
+        case 2: { constexpr int GS = 2; __VA_ARGS__; } break;   \
+        case 4: { constexpr int GS = 4; __VA_ARGS__; } break;   \
+        case 8: { constexpr int GS = 8; __VA_ARGS__; } break;   \
+        case 16: { constexpr int GS = 16; __VA_ARGS__; } break; \
+        default: { constexpr int GS = 32; __VA_ARGS__; } break; \
+    }
+
+
+}  // namespace frugal

@@ -1,0 +1,758 @@
+// runtime.cu -- host runtime of libfrugal: the C ABI (include/frugal.h), context setup,
+// the shared host table, the sample queue and the per-step orchestration of the kernels.
+//
+// Process model (§3.2 Fig. 5, re-designed): one process per GPU; the
+// paper's controller process is replaced by device kernels on each rank plus host-memory
+// flags.  The host parameter table w[N][d] (+ G[N][d]) lives in a POSIX shm segment
+// registered mapped+portable in every rank (L772-774 "shared memory interface"), so every
+// GPU reads it with zero-copy loads and the owners flush into it with zero-copy stores.
+#include <cuda_runtime.h>
+#include <fcntl.h>
+#include <stdarg.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <string.h>
+#include <sys/mman.h>
+#include <sys/stat.h>
+#include <time.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <string>
+#include <vector>
+
+#include "frugal_internal.cuh"
+
+using namespace frugal;
+
+static thread_local std::string g_err;
+static void set_err(const char* fmt, ...) {
+    char buf[1024];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+}
+
+#define CK(call)                                                                  \
+    do {                                                                          \
+        cudaError_t e_ = (call);                                                  \
+        if (e_ != cudaSuccess) {                                                  \
+            set_err("%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, __LINE__); \
+            return FRUGAL_ECUDA;                                                  \
+        }                                                                         \
+    } while (0)
+
+#define CKL()                                                                     \
+    do {                                                                          \
+        cudaError_t e_ = cudaGetLastError();                                      \
+        if (e_ != cudaSuccess) {                                                  \
+            set_err("kernel launch failed: %s (%s:%d)", cudaGetErrorString(e_), __FILE__, __LINE__); \
+            return FRUGAL_ECUDA;                                                  \
+        }                                                                         \
+    } while (0)
+
+namespace {
+
+constexpr uint64_t kMagic = 0x46525547414c3235ULL;  // "FRUGAL25"
+constexpr size_t kHdr = 4096;
+constexpr size_t kFlags = 8192;  // 3 kinds x 32 ranks x 64 B
+enum { FLAG_URGENT = 0, FLAG_SIDE = 1, FLAG_MAIL = 2 };
+enum { PH_INGEST, PH_SCHED, PH_URGENT, PH_GATE, PH_GATHER, PH_EXPAND, PH_MODEL, PH_SEGRED, PH_EXCH, PH_OPT, PH_SIDE };
+
+struct ShmHeader {
+    uint64_t magic;
+    volatile uint64_t ready;
+    uint64_t total_bytes;
+    int64_t n_rows;
+    int32_t dim, world, opt, pad;
+};
+
+size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+double now_s() {
+    timespec ts;
+    clock_gettime(CLOCK_MONOTONIC, &ts);
+    return ts.tv_sec + 1e-9 * ts.tv_nsec;
+}
+
+int bits_for(int64_t maxval) {  // bits to represent values in [0, maxval]
+    int b = 1;
+    while (b < 62 && ((int64_t)1 << b) <= maxval) b++;
+    return b;
+}
+
+struct Timer {
+    frugal_ctx* c;
+    int ph;
+    cudaStream_t st;
+    cudaEvent_t a = nullptr;
+    Timer(frugal_ctx* c_, int ph_, cudaStream_t st_) : c(c_), ph(ph_), st(st_) {
+        if (!(c->cfg.flags & FRUGAL_F_TIMERS)) return;
+        if (c->ev_used + 2 > c->ev_pool.size()) {
+            for (int i = 0; i < 64; i++) {
+                cudaEvent_t e;
+                cudaEventCreate(&e);
+                c->ev_pool.push_back(e);
+            }
+        }
+        a = c->ev_pool[c->ev_used++];
+        cudaEventRecord(a, st);
+    }
+    ~Timer() {
+        if (!a) return;
+        cudaEvent_t b = c->ev_pool[c->ev_used++];
+        cudaEventRecord(b, st);
+        c->evs.push_back({ph, a, b});
+    }
+};
+
+}  // namespace
+
+// ================================================================================ helpers
+static frugal_status check_err_word(frugal_ctx* c) {
+    if (c->herr && *(volatile int32_t*)c->herr) {
+        int e = *(volatile int32_t*)c->herr;
+        if (e == 2) {
+            set_err("a peer rank did not publish its flag within 120 s");
+            return FRUGAL_ETIMEOUT;
+        }
+        set_err("a row id outside [0, n_rows) was passed in a sample batch");
+        return FRUGAL_EINVAL;
+    }
+    return FRUGAL_OK;
+}
+
+static void free_ctx(frugal_ctx* c) {
+    if (!c) return;
+    cudaSetDevice(c->cfg.device);
+    cudaDeviceSynchronize();
+    auto F = [](void* p) {
+        if (p) cudaFree(p);
+    };
+    F(c->slot); F(c->state); F(c->last_upd); F(c->pool_idx); F(c->rbits);
+    F(c->cw); F(c->cG); F(c->hot_lk); F(c->pw); F(c->pG); F(c->pkey); F(c->pcount);
+    for (auto& q : c->q) {
+        F(q.ids); F(q.counts); F(q.m); F(q.uniq); F(q.inv); F(q.off); F(q.pos); F(q.n_uniq);
+        if (c->n > 1) { F(q.T); F(q.Tmask); F(q.Tidx); F(q.nT); F(q.gl); F(q.goff); }
+    }
+    F(c->rows); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->owned_cnt); F(c->nb_rows); F(c->nb_p); F(c->nb_cnt);
+    for (int i = 0; i < 2; i++) { F(c->bk_rows[i]); F(c->bk_p[i]); F(c->bk_off[i]); F(c->age_rows[i]); F(c->age_cnt[i]); }
+    F(c->sched_info); F(c->ff_rows); F(c->ff_cnt); F(c->ids_stage);
+    if (c->herr) cudaFreeHost(c->herr);
+    if (c->counts_pin) cudaFreeHost(c->counts_pin);
+    for (auto e : c->ev_counts) cudaEventDestroy(e);
+    sort_free(c->sort);
+    scan_free(c->scan);
+    if (c->side) cudaStreamDestroy(c->side);
+    if (c->ev_sched) cudaEventDestroy(c->ev_sched);
+    for (int i = 0; i < 2; i++) if (c->ev_side[i]) cudaEventDestroy(c->ev_side[i]);
+    for (auto e : c->ev_pool) cudaEventDestroy(e);
+    if (c->shm_base) {
+        cudaHostUnregister(c->shm_base);
+        munmap(c->shm_base, c->shm_bytes);
+    }
+    if (c->shm_fd >= 0) close(c->shm_fd);
+    if (c->shm_owner && c->cfg.shm_name) shm_unlink(c->cfg.shm_name);
+    delete c;
+}
+
+#define DMALLOC(ptr, bytes)                                                                     \
+    do {                                                                                         \
+        size_t b_ = (bytes) < 16 ? 16 : (bytes);                                                 \
+        if (cudaMalloc((void**)&(ptr), b_) != cudaSuccess) {                                     \
+            cudaGetLastError();                                                                  \
+            set_err("cudaMalloc of %zu bytes failed (%s)", b_, #ptr);                            \
+            free_ctx(c);                                                                         \
+            return FRUGAL_ENOMEM;                                                                \
+        }                                                                                        \
+    } while (0)
+
+// ================================================================================ init
+extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out) {
+    if (!out) { set_err("out is NULL"); return FRUGAL_EINVAL; }
+    *out = nullptr;
+    if (!cfg) { set_err("cfg is NULL"); return FRUGAL_EINVAL; }
+    const frugal_config& k = *cfg;
+    if (k.world < 1 || k.world > 32 || k.rank < 0 || k.rank >= k.world) { set_err("bad world/rank"); return FRUGAL_EINVAL; }
+    if (k.dim < 4 || k.dim > 1024 || k.dim % 4) { set_err("dim must be a multiple of 4 in [4, 1024]"); return FRUGAL_EINVAL; }
+    if (k.n_rows < 1 || k.n_rows > 0x7fffffffLL) { set_err("n_rows must be in [1, 2^31-1]"); return FRUGAL_EINVAL; }
+    if (k.slots < 1 || k.batch < 1 || (int64_t)k.slots * k.batch * k.world > 0x7fffffffLL) { set_err("bad slots/batch"); return FRUGAL_EINVAL; }
+    if (k.lookahead < 2 || k.lookahead > 31) { set_err("lookahead must be in [2, 31]"); return FRUGAL_EINVAL; }
+    if (k.age_out < 1) { set_err("age_out must be >= 1"); return FRUGAL_EINVAL; }
+    if (k.opt != FRUGAL_SGD && k.opt != FRUGAL_ADAGRAD) { set_err("bad opt"); return FRUGAL_EINVAL; }
+    if (k.mode != FRUGAL_MODE_P2F && k.mode != FRUGAL_MODE_WRITE_THROUGH) { set_err("bad mode"); return FRUGAL_EINVAL; }
+    if (!k.shm_name && k.world != 1) { set_err("world > 1 needs shm_name"); return FRUGAL_EINVAL; }
+    if (k.n_hot < 0 || (k.n_hot > 0 && !k.hot_ids)) { set_err("bad hot set"); return FRUGAL_EINVAL; }
+    for (int64_t i = 0; i < k.n_hot; i++)
+        if (k.hot_ids[i] < 0 || k.hot_ids[i] >= k.n_rows) { set_err("hot id out of range"); return FRUGAL_EINVAL; }
+    if (cudaSetDevice(k.device) != cudaSuccess) { set_err("cudaSetDevice(%d) failed", k.device); return FRUGAL_ECUDA; }
+    int dev_major = 0;
+    cudaDeviceGetAttribute(&dev_major, cudaDevAttrComputeCapabilityMajor, k.device);
+
+    frugal_ctx* c = new frugal_ctx();
+    c->cfg = k;
+    c->cfg.hot_ids = nullptr;
+    c->n = k.world; c->g = k.rank; c->d = k.dim; c->F = k.slots; c->B = k.batch;
+    c->L = k.lookahead; c->D = k.age_out; c->M = k.batch * k.slots; c->N = k.n_rows;
+    c->No = c->g < c->N ? (c->N - c->g + c->n - 1) / c->n : 0;
+    c->P = c->D + 2;
+    c->capT = std::max<int64_t>(1, std::min<int64_t>((int64_t)c->n * c->M, c->No));
+    c->key_bits = bits_for(c->N - 1);
+    c->lk_bits = bits_for(std::max<int64_t>(c->No - 1, 0));
+    const bool adag = k.opt == FRUGAL_ADAGRAD;
+    const size_t rowb = (size_t)c->d * sizeof(float);
+
+    // ---------------------------------------------------------------- host table (shm)
+    c->mail_stride = c->n > 1 ? align_up(256 + (size_t)c->M * rowb, 4096) : 0;
+    const size_t mail_bytes = c->n > 1 ? 2 * (size_t)c->n * c->mail_stride : 0;
+    const size_t off_mail = kHdr + kFlags;
+    const size_t off_w = align_up(off_mail + mail_bytes, 2 << 20);
+    const size_t tab = (size_t)c->N * rowb;
+    const size_t off_G = align_up(off_w + tab, 2 << 20);
+    const size_t total = adag ? off_G + tab : off_w + tab;
+    c->shm_bytes = total;
+    if (k.shm_name) {
+        if (c->g == 0) {
+            shm_unlink(k.shm_name);
+            c->shm_fd = shm_open(k.shm_name, O_CREAT | O_EXCL | O_RDWR, 0600);
+            if (c->shm_fd < 0 || ftruncate(c->shm_fd, (off_t)total) != 0) {
+                set_err("shm_open/ftruncate(%s, %zu) failed", k.shm_name, total);
+                free_ctx(c);
+                return FRUGAL_ESHM;
+            }
+            c->shm_owner = true;
+        } else {
+            double t0 = now_s();
+            while (true) {
+                c->shm_fd = shm_open(k.shm_name, O_RDWR, 0600);
+                struct stat sb;
+                if (c->shm_fd >= 0 && fstat(c->shm_fd, &sb) == 0 && (size_t)sb.st_size == total) break;
+                if (c->shm_fd >= 0) { close(c->shm_fd); c->shm_fd = -1; }
+                if (now_s() - t0 > 600) { set_err("timed out attaching shm %s", k.shm_name); delete c; return FRUGAL_ESHM; }
+                usleep(20000);
+            }
+        }
+        c->shm_base = mmap(nullptr, total, PROT_READ | PROT_WRITE, MAP_SHARED, c->shm_fd, 0);
+    } else {
+        c->shm_base = mmap(nullptr, total, PROT_READ | PROT_WRITE, MAP_SHARED | MAP_ANONYMOUS, -1, 0);
+    }
+    if (c->shm_base == MAP_FAILED) {
+        c->shm_base = nullptr;
+        set_err("mmap of %zu bytes failed", total);
+        free_ctx(c);
+        return FRUGAL_ESHM;
+    }
+    madvise(c->shm_base, total, MADV_HUGEPAGE);
+    if (cudaHostRegister(c->shm_base, total, cudaHostRegisterMapped | cudaHostRegisterPortable) != cudaSuccess) {
+        cudaGetLastError();
+        munmap(c->shm_base, total);
+        c->shm_base = nullptr;
+        set_err("cudaHostRegister of %zu bytes failed", total);
+        free_ctx(c);
+        return FRUGAL_ENOMEM;
+    }
+    char* dbase = nullptr;
+    if (cudaHostGetDevicePointer((void**)&dbase, c->shm_base, 0) != cudaSuccess) {
+        set_err("cudaHostGetDevicePointer failed");
+        free_ctx(c);
+        return FRUGAL_ECUDA;
+    }
+    char* hbase = (char*)c->shm_base;
+    ShmHeader* hdr = (ShmHeader*)hbase;
+    c->h_flags = (volatile uint32_t*)(hbase + kHdr);
+    c->dh_flags = (uint32_t*)(dbase + kHdr);
+    c->h_mail = hbase + off_mail;
+    c->dh_mail = dbase + off_mail;
+    c->h_w = (float*)(hbase + off_w);
+    c->dh_w = (float*)(dbase + off_w);
+    if (adag) {
+        c->h_G = (float*)(hbase + off_G);
+        c->dh_G = (float*)(dbase + off_G);
+    }
+    if (cudaHostAlloc((void**)&c->herr, 64, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess ||
+        cudaHostAlloc((void**)&c->counts_pin, (size_t)(c->L + 1) * c->n * 4, cudaHostAllocPortable) != cudaSuccess) {
+        set_err("cudaHostAlloc(err/counts) failed");
+        free_ctx(c);
+        return FRUGAL_ENOMEM;
+    }
+    memset(c->herr, 0, 64);
+    cudaHostGetDevicePointer((void**)&c->err, c->herr, 0);
+
+    // ---------------------------------------------------------------- device state
+    DMALLOC(c->slot, c->No * 4);
+    DMALLOC(c->state, c->No * 4);
+    DMALLOC(c->last_upd, c->No * 4);
+    DMALLOC(c->pool_idx, c->No * 4);
+    DMALLOC(c->rbits, c->No * 8);
+    // owned share of the hot set, sorted, deduplicated
+    std::vector<int32_t> hot;
+    for (int64_t i = 0; i < k.n_hot; i++)
+        if (k.hot_ids[i] % c->n == c->g) hot.push_back((int32_t)(k.hot_ids[i] / c->n));
+    std::sort(hot.begin(), hot.end());
+    hot.erase(std::unique(hot.begin(), hot.end()), hot.end());
+    c->cap_hot = (int64_t)hot.size();
+    DMALLOC(c->hot_lk, c->cap_hot * 4);
+    DMALLOC(c->cw, c->cap_hot * rowb);
+    if (adag) DMALLOC(c->cG, c->cap_hot * rowb);
+    DMALLOC(c->pw, (size_t)c->P * c->capT * rowb);
+    if (adag) DMALLOC(c->pG, (size_t)c->P * c->capT * rowb);
+    DMALLOC(c->pkey, (size_t)c->P * c->capT * 4);
+    DMALLOC(c->pcount, (size_t)c->P * 4);
+    c->q.resize(c->L + 1);
+    for (auto& q : c->q) {
+        DMALLOC(q.ids, (size_t)c->n * c->M * 4);
+        DMALLOC(q.counts, (size_t)c->n * 4);
+        DMALLOC(q.m, 4);
+        DMALLOC(q.uniq, (size_t)c->M * 4);
+        DMALLOC(q.inv, (size_t)c->M * 4);
+        DMALLOC(q.off, ((size_t)c->M + 1) * 4);
+        DMALLOC(q.pos, (size_t)c->M * 4);
+        DMALLOC(q.n_uniq, 4);
+        if (c->n > 1) {
+            DMALLOC(q.T, c->capT * 4);
+            DMALLOC(q.Tmask, c->capT * 4);
+            DMALLOC(q.Tidx, (size_t)c->n * c->capT * 4);
+            DMALLOC(q.nT, 4);
+            DMALLOC(q.gl, (size_t)c->M * 4);
+            DMALLOC(q.goff, 64 * 4);
+        } else {
+            q.T = q.uniq;  // world 1: every row is owned, T(t) == uniq(t)
+            q.nT = q.n_uniq;
+        }
+        q.h_counts.assign(c->n, 0);
+    }
+    DMALLOC(c->rows, (size_t)c->M * rowb);
+    DMALLOC(c->Pp, (size_t)c->M * rowb);
+    DMALLOC(c->chunk_scratch, (size_t)c->M * rowb);
+    DMALLOC(c->long_q, (size_t)c->M * 4);
+    DMALLOC(c->long_cnt, 4);
+    DMALLOC(c->owned_cnt, 4);
+    DMALLOC(c->nb_rows, 2 * c->capT * 4);
+    DMALLOC(c->nb_p, 2 * c->capT * 4);
+    DMALLOC(c->nb_cnt, 4);
+    for (int i = 0; i < 2; i++) {
+        DMALLOC(c->bk_rows[i], 2 * c->capT * 4);
+        DMALLOC(c->bk_p[i], 2 * c->capT * 4);
+        DMALLOC(c->bk_off[i], 64 * 4);
+        DMALLOC(c->age_rows[i], c->capT * 4);
+        DMALLOC(c->age_cnt[i], 4);
+    }
+    DMALLOC(c->sched_info, 64 * 4);
+    DMALLOC(c->ff_rows, std::max<int64_t>(c->No, 1) * 4);
+    DMALLOC(c->ff_cnt, 4);
+    DMALLOC(c->ids_stage, (size_t)c->n * c->M * 8);
+    sort_alloc(c->sort, (int64_t)c->n * c->M);
+    scan_alloc(c->scan, (int64_t)c->n * c->M);
+    if (!c->sort.hist || !c->scan.part) {
+        set_err("scratch allocation failed");
+        free_ctx(c);
+        return FRUGAL_ENOMEM;
+    }
+    int lo_prio, hi_prio;
+    cudaDeviceGetStreamPriorityRange(&lo_prio, &hi_prio);
+    CK(cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, lo_prio));  // lowest priority
+    CK(cudaEventCreateWithFlags(&c->ev_sched, cudaEventDisableTiming));
+    for (int i = 0; i < 2; i++) CK(cudaEventCreateWithFlags(&c->ev_side[i], cudaEventDisableTiming));
+    c->ev_counts.resize(c->L + 1);
+    for (auto& e : c->ev_counts) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+
+    cudaStream_t st = 0;
+    if (cudaMemcpy(c->hot_lk, hot.data(), hot.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) {
+        set_err("hot upload failed");
+        free_ctx(c);
+        return FRUGAL_ECUDA;
+    }
+    launch_init_meta(c, nullptr, 0, st);
+    cudaMemset(c->pcount, 0, (size_t)c->P * 4);
+    cudaMemset(c->pkey, 0xff, (size_t)c->P * c->capT * 4);
+    if (c->g == 0 || !k.shm_name) {
+        memset(hbase + kHdr, 0, kFlags);
+        launch_init_table(c, st);
+        if (cudaDeviceSynchronize() != cudaSuccess) {
+                set_err("table init failed: %s", cudaGetErrorString(cudaGetLastError()));
+            free_ctx(c);
+            return FRUGAL_ECUDA;
+        }
+        hdr->magic = kMagic;
+        hdr->total_bytes = total;
+        hdr->n_rows = c->N;
+        hdr->dim = c->d;
+        hdr->world = c->n;
+        hdr->opt = k.opt;
+        __sync_synchronize();
+        hdr->ready = kMagic;
+    } else {
+        double t0 = now_s();
+        while (hdr->ready != kMagic) {
+            if (now_s() - t0 > 600) {
+                        set_err("timed out waiting for rank 0's table");
+                free_ctx(c);
+                return FRUGAL_ETIMEOUT;
+            }
+            usleep(20000);
+        }
+        if (hdr->n_rows != c->N || hdr->dim != c->d || hdr->world != c->n || hdr->opt != k.opt) {
+                set_err("shm table config mismatch with rank 0");
+            free_ctx(c);
+            return FRUGAL_ESHM;
+        }
+    }
+    if (cudaDeviceSynchronize() != cudaSuccess) {
+        set_err("init failed: %s", cudaGetErrorString(cudaGetLastError()));
+        free_ctx(c);
+        return FRUGAL_ECUDA;
+    }
+    *out = c;
+    (void)dev_major;
+    return FRUGAL_OK;
+}
+
+// ================================================================================ sample queue
+// ingest step t of all ranks into queue slot t % (L+1): convert + validate ids, own dedup,
+// owner-side T (world > 1), read-ring bits of step t and AdjustPriority inf -> t.
+static frugal_status ingest(frugal_ctx* c, int64_t t, const int64_t* ids_all, const int32_t* counts, int adjust,
+                            cudaStream_t st) {
+    for (int r = 0; r < c->n; r++)
+        if (counts[r] < 0 || counts[r] > c->B) {
+            set_err("counts[%d] = %d outside [0, batch=%d]", r, counts[r], c->B);
+            return FRUGAL_EINVAL;
+        }
+    const int qi = (int)(t % (c->L + 1));
+    QueueSlot& q = c->q[qi];
+    q.step = t;
+    q.h_counts.assign(counts, counts + c->n);
+    // the pinned counts staging of this slot is reused only after its last copy ran
+    CK(cudaEventSynchronize(c->ev_counts[qi]));
+    int32_t* pin = c->counts_pin + (size_t)qi * c->n;
+    memcpy(pin, counts, (size_t)c->n * 4);
+    CK(cudaMemcpyAsync(q.counts, pin, (size_t)c->n * 4, cudaMemcpyHostToDevice, st));
+    CK(cudaEventRecord(c->ev_counts[qi], st));
+    CK(cudaMemcpyAsync(c->ids_stage, ids_all, (size_t)c->n * c->M * 8, cudaMemcpyDefault, st));
+    launch_convert_ids(c, q, st);
+    launch_dedup(c, q, st);
+    if (c->n > 1) launch_owner_side(c, q, t, st);
+    launch_ingest_bits(c, q, t, adjust, st);
+    CKL();
+    return FRUGAL_OK;
+}
+
+extern "C" frugal_status frugal_prefetch(frugal_ctx* c, int64_t t, const int64_t* ids_all, const int32_t* counts,
+                                         frugal_stream stream) {
+    if (!c || !ids_all || !counts) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    if (c->cur_step != -1 || t != c->next_prefetch || t > c->L - 2) {
+        set_err("prefetch(%lld): expected t = %lld (only steps 0..L-2 before step 0)", (long long)t,
+                (long long)c->next_prefetch);
+        return FRUGAL_ESTATE;
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    Timer tm(c, PH_INGEST, st);
+    frugal_status r = ingest(c, t, ids_all, counts, 0, st);
+    if (r) return r;
+    c->next_prefetch++;
+    return check_err_word(c);
+}
+
+static void record_schedule(frugal_ctx* c, int par, cudaStream_t st) {
+    cudaStreamSynchronize(st);
+    int32_t off[64];
+    int32_t nage = 0;
+    cudaMemcpy(off, c->bk_off[par], (c->L + 1) * 4, cudaMemcpyDeviceToHost);
+    cudaMemcpy(&nage, c->age_cnt[par], 4, cudaMemcpyDeviceToHost);
+    std::vector<int32_t> rows(off[c->L]), ps(off[c->L]), age(nage);
+    if (off[c->L]) {
+        cudaMemcpy(rows.data(), c->bk_rows[par], off[c->L] * 4, cudaMemcpyDeviceToHost);
+        cudaMemcpy(ps.data(), c->bk_p[par], off[c->L] * 4, cudaMemcpyDeviceToHost);
+    }
+    if (nage) cudaMemcpy(age.data(), c->age_rows[par], nage * 4, cudaMemcpyDeviceToHost);
+    c->rec_urgent.assign(rows.begin(), rows.begin() + off[1]);
+    c->rec_deferred.assign(rows.begin() + off[1], rows.end());
+    c->rec_deferred_p.assign(ps.begin() + off[1], ps.end());
+    c->rec_ageout = age;
+    c->rec_gate_wait = off[1] > 0;
+    c->rows_urgent += off[1];
+    c->rows_deferred += off[c->L] - off[1];
+    c->rows_ageout += nage;
+}
+
+extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* ids_next_all, const int32_t* counts_next,
+                                     frugal_stream stream) {
+    if (!c) { set_err("NULL ctx"); return FRUGAL_EINVAL; }
+    if (c->phase_in_step != 0 || s != c->cur_step + 1) {
+        set_err("step(%lld) out of order (current step %lld, phase %d)", (long long)s, (long long)c->cur_step,
+                c->phase_in_step);
+        return FRUGAL_ESTATE;
+    }
+    const int64_t t = s + c->L - 1;
+    if (ids_next_all) {
+        if (c->ids_exhausted || c->next_prefetch != t || !counts_next) {
+            set_err("step(%lld): steps 0..%lld must be prefetched first (and counts given)", (long long)s,
+                    (long long)(t - 1));
+            return FRUGAL_ESTATE;
+        }
+    } else {
+        c->ids_exhausted = true;
+        if (c->next_prefetch <= s) { set_err("step(%lld) was never enqueued", (long long)s); return FRUGAL_ESTATE; }
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    const int par = (int)(s & 1);
+    CK(cudaMemsetAsync(c->nb_cnt, 0, 4, st));
+    if (ids_next_all) {
+        Timer tm(c, PH_INGEST, st);
+        frugal_status r = ingest(c, t, ids_next_all, counts_next, 1, st);
+        if (r) return r;
+        c->next_prefetch++;
+    }
+    {
+        Timer tm(c, PH_SCHED, st);
+        QueueSlot* prev = nullptr;
+        if (s >= 1) {
+            prev = &c->q[(s - 1) % (c->L + 1)];
+            if (prev->step != s - 1) { set_err("internal: queue slot of step %lld lost", (long long)(s - 1)); return FRUGAL_ESTATE; }
+        }
+        launch_bucket(c, prev, s, par, st);
+        CKL();
+    }
+    if (c->cfg.flags & FRUGAL_F_RECORD) record_schedule(c, par, st);
+    {
+        // a10: urgent bucket (priority == s) to the host table on the critical path
+        Timer tm(c, PH_URGENT, st);
+        launch_flush_rows(c, c->bk_rows[par], c->bk_off[par], c->bk_off[par] + 1, 0, st);
+        if (c->n > 1) launch_set_flag(c, FLAG_URGENT, (uint32_t)(s + 1), st);
+        CKL();
+    }
+    // a11: deferred buckets (priorities s+1 .. s+L-1, ascending) and age-outs on the side stream
+    CK(cudaEventRecord(c->ev_sched, st));
+    CK(cudaStreamWaitEvent(c->side, c->ev_sched, 0));
+    {
+        Timer tm(c, PH_SIDE, c->side);
+        launch_flush_rows(c, c->bk_rows[par], c->bk_off[par] + 1, c->bk_off[par] + c->L, 0, c->side);
+        launch_flush_rows(c, c->age_rows[par], nullptr, c->age_cnt[par], 0, c->side);
+        if (c->n > 1) launch_set_flag(c, FLAG_SIDE, (uint32_t)(s + 1), c->side);
+        CKL();
+    }
+    CK(cudaEventRecord(c->ev_side[par], c->side));
+    c->side_pending[par] = true;
+    {
+        // a3: gate of step s -- PQ front > s: every owner's urgent bucket s and every
+        // deferred bucket drained by its side stream at steps <= s-1
+        Timer tm(c, PH_GATE, st);
+        if (c->n == 1) {
+            if (s >= 1 && c->side_pending[par ^ 1]) CK(cudaStreamWaitEvent(st, c->ev_side[par ^ 1], 0));
+        } else {
+            launch_wait_flags(c, FLAG_URGENT, (uint32_t)(s + 1), st);
+            if (s >= 1) launch_wait_flags(c, FLAG_SIDE, (uint32_t)s, st);
+            CKL();
+        }
+    }
+    c->cur_step = s;
+    c->phase_in_step = 1;
+    return check_err_word(c);
+}
+
+extern "C" frugal_status frugal_lookup(frugal_ctx* c, int64_t s, float* d_out, frugal_stream stream) {
+    if (!c || !d_out) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    if (c->phase_in_step != 1 || s != c->cur_step) {
+        set_err("lookup(%lld) out of order", (long long)s);
+        return FRUGAL_ESTATE;
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    QueueSlot& q = c->q[s % (c->L + 1)];
+    {
+        Timer tm(c, PH_GATHER, st);
+        launch_gather(c, q, d_out, st);
+    }
+    {
+        Timer tm(c, PH_EXPAND, st);
+        launch_expand(c, q, d_out, st);
+    }
+    CKL();
+    c->phase_in_step = 2;
+    return check_err_word(c);
+}
+
+extern "C" frugal_status frugal_dot_model(frugal_ctx* c, int64_t s, const float* d_emb, const float* d_x,
+                                          const float* d_y, float* d_grad, double* d_loss, frugal_stream stream) {
+    if (!c || !d_emb || !d_x || !d_y || !d_grad || !d_loss) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    if (c->phase_in_step != 2 || s != c->cur_step) {
+        set_err("dot_model(%lld) must follow lookup(%lld)", (long long)s, (long long)s);
+        return FRUGAL_ESTATE;
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    QueueSlot& q = c->q[s % (c->L + 1)];
+    int64_t nb = 0;
+    for (int r = 0; r < c->n; r++) nb += q.h_counts[r];
+    Timer tm(c, PH_MODEL, st);
+    launch_dot_model(c, q, d_emb, d_x, d_y, d_grad, d_loss, nb, st);
+    CKL();
+    return FRUGAL_OK;
+}
+
+extern "C" frugal_status frugal_backward_update(frugal_ctx* c, int64_t s, const float* d_grad, frugal_stream stream) {
+    if (!c || !d_grad) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    if (c->phase_in_step != 2 || s != c->cur_step) {
+        set_err("backward_update(%lld) out of order", (long long)s);
+        return FRUGAL_ESTATE;
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    QueueSlot& q = c->q[s % (c->L + 1)];
+    const int par = (int)(s & 1);
+    {
+        Timer tm(c, PH_SEGRED, st);
+        launch_segreduce(c, q, d_grad, par, st);
+    }
+    if (c->n > 1) {
+        // a7: partials of rows owned by other ranks are in this rank's host mailbox;
+        // publish and wait for every sender (the update staging queue, L785-789)
+        Timer tm(c, PH_EXCH, st);
+        launch_mail_header(c, q, par, st);
+        launch_set_flag(c, FLAG_MAIL, (uint32_t)(s + 1), st);
+        launch_wait_flags(c, FLAG_MAIL, (uint32_t)(s + 1), st);
+    }
+    {
+        Timer tm(c, PH_OPT, st);
+        launch_optimizer(c, q, s, par, st);
+    }
+    CKL();
+    c->phase_in_step = 0;
+    c->timed_steps++;
+    return check_err_word(c);
+}
+
+extern "C" frugal_status frugal_flush(frugal_ctx* c, int32_t what, frugal_stream stream) {
+    if (!c) { set_err("NULL ctx"); return FRUGAL_EINVAL; }
+    if (what != FRUGAL_FLUSH_ALL) { set_err("unknown flush kind %d", what); return FRUGAL_EINVAL; }
+    if (c->phase_in_step != 0) { set_err("flush in the middle of a step"); return FRUGAL_ESTATE; }
+    cudaStream_t st = (cudaStream_t)stream;
+    for (int i = 0; i < 2; i++)
+        if (c->side_pending[i]) CK(cudaStreamWaitEvent(st, c->ev_side[i], 0));
+    launch_final_flush(c, st);
+    CKL();
+    CK(cudaStreamSynchronize(st));
+    int32_t nff = 0;
+    CK(cudaMemcpy(&nff, c->ff_cnt, 4, cudaMemcpyDeviceToHost));
+    c->rec_final.resize(nff);
+    if (nff) CK(cudaMemcpy(c->rec_final.data(), c->ff_rows, (size_t)nff * 4, cudaMemcpyDeviceToHost));
+    return check_err_word(c);
+}
+
+extern "C" frugal_status frugal_destroy(frugal_ctx* c) {
+    if (!c) return FRUGAL_OK;
+    free_ctx(c);
+    return FRUGAL_OK;
+}
+
+extern "C" const char* frugal_last_error(void) { return g_err.c_str(); }
+
+// ================================================================================ introspection
+extern "C" frugal_status frugal_get_dedup(frugal_ctx* c, int64_t t, int64_t* uniq, int32_t* inv, int64_t* n_uniq) {
+    if (!c || !n_uniq) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    QueueSlot& q = c->q[t % (c->L + 1)];
+    if (t < 0 || q.step != t) { set_err("step %lld is not in the sample queue", (long long)t); return FRUGAL_EINVAL; }
+    CK(cudaDeviceSynchronize());
+    int32_t nu = 0;
+    CK(cudaMemcpy(&nu, q.n_uniq, 4, cudaMemcpyDeviceToHost));
+    *n_uniq = nu;
+    if (uniq && nu) {
+        std::vector<int32_t> u(nu);
+        CK(cudaMemcpy(u.data(), q.uniq, (size_t)nu * 4, cudaMemcpyDeviceToHost));
+        for (int i = 0; i < nu; i++) uniq[i] = u[i];
+    }
+    const int m = q.h_counts[c->g] * c->F;
+    if (inv && m) CK(cudaMemcpy(inv, q.inv, (size_t)m * 4, cudaMemcpyDeviceToHost));
+    return check_err_word(c);
+}
+
+extern "C" frugal_status frugal_get_schedule(frugal_ctx* c, frugal_schedule_info* info, int64_t* urgent,
+                                             int64_t* deferred, int32_t* deferred_p, int64_t* ageout) {
+    if (!c || !info) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    if (!(c->cfg.flags & FRUGAL_F_RECORD)) { set_err("context was created without FRUGAL_F_RECORD"); return FRUGAL_ESTATE; }
+    info->n_urgent = (int64_t)c->rec_urgent.size();
+    info->n_deferred = (int64_t)c->rec_deferred.size();
+    info->n_ageout = (int64_t)c->rec_ageout.size();
+    info->gate_wait = c->rec_gate_wait;
+    auto glob = [c](int32_t lk) { return (int64_t)lk * c->n + c->g; };
+    if (urgent) for (size_t i = 0; i < c->rec_urgent.size(); i++) urgent[i] = glob(c->rec_urgent[i]);
+    if (deferred) for (size_t i = 0; i < c->rec_deferred.size(); i++) deferred[i] = glob(c->rec_deferred[i]);
+    if (deferred_p) for (size_t i = 0; i < c->rec_deferred_p.size(); i++) deferred_p[i] = c->rec_deferred_p[i];
+    if (ageout) for (size_t i = 0; i < c->rec_ageout.size(); i++) ageout[i] = glob(c->rec_ageout[i]);
+    return FRUGAL_OK;
+}
+
+extern "C" frugal_status frugal_get_final_flush(frugal_ctx* c, int64_t* rows, int64_t* n) {
+    if (!c || !n) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    *n = (int64_t)c->rec_final.size();
+    if (rows) for (size_t i = 0; i < c->rec_final.size(); i++) rows[i] = (int64_t)c->rec_final[i] * c->n + c->g;
+    return FRUGAL_OK;
+}
+
+extern "C" frugal_status frugal_read_rows(frugal_ctx* c, const int64_t* ids, int64_t n, float* w, float* G) {
+    if (!c || (n && (!ids || !w))) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    if (n == 0) return FRUGAL_OK;
+    std::vector<int32_t> lk(n);
+    for (int64_t i = 0; i < n; i++) {
+        if (ids[i] < 0 || ids[i] >= c->N || ids[i] % c->n != c->g) {
+            set_err("read_rows: id %lld is not owned by rank %d", (long long)ids[i], c->g);
+            return FRUGAL_EINVAL;
+        }
+        lk[i] = (int32_t)(ids[i] / c->n);
+    }
+    CK(cudaDeviceSynchronize());
+    int32_t* d_lk;
+    float *d_w, *d_G;
+    CK(cudaMalloc(&d_lk, n * 4));
+    CK(cudaMalloc(&d_w, n * c->d * 4));
+    CK(cudaMalloc(&d_G, n * c->d * 4));
+    cudaMemcpy(d_lk, lk.data(), n * 4, cudaMemcpyHostToDevice);
+    launch_read_rows(c, d_lk, n, d_w, d_G, 0);
+    cudaError_t e = cudaDeviceSynchronize();
+    if (e == cudaSuccess) {
+        cudaMemcpy(w, d_w, n * c->d * 4, cudaMemcpyDeviceToHost);
+        if (G) cudaMemcpy(G, d_G, n * c->d * 4, cudaMemcpyDeviceToHost);
+    }
+    cudaFree(d_lk);
+    cudaFree(d_w);
+    cudaFree(d_G);
+    if (e != cudaSuccess) { set_err("read_rows: %s", cudaGetErrorString(e)); return FRUGAL_ECUDA; }
+    return FRUGAL_OK;
+}
+
+extern "C" frugal_status frugal_read_host(frugal_ctx* c, const int64_t* ids, int64_t n, float* w, float* G) {
+    if (!c || (n && (!ids || !w))) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    CK(cudaDeviceSynchronize());
+    for (int64_t i = 0; i < n; i++) {
+        if (ids[i] < 0 || ids[i] >= c->N) { set_err("read_host: id out of range"); return FRUGAL_EINVAL; }
+        memcpy(w + i * c->d, c->h_w + ids[i] * c->d, c->d * 4);
+        if (G) {
+            if (c->h_G) memcpy(G + i * c->d, c->h_G + ids[i] * c->d, c->d * 4);
+            else memset(G + i * c->d, 0, c->d * 4);
+        }
+    }
+    return FRUGAL_OK;
+}
+
+extern "C" frugal_status frugal_get_stats(frugal_ctx* c, frugal_stats* out) {
+    if (!c || !out) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    CK(cudaDeviceSynchronize());
+    for (auto& e : c->evs) {
+        float ms = 0.f;
+        if (cudaEventElapsedTime(&ms, e.a, e.b) == cudaSuccess) c->phase_ms[e.phase] += ms;
+    }
+    cudaGetLastError();
+    c->evs.clear();
+    c->ev_used = 0;
+    for (int i = 0; i < FRUGAL_N_PHASES; i++) out->ms[i] = c->phase_ms[i];
+    out->steps = c->timed_steps;
+    out->kernel_launches = c->launches;
+    out->rows_urgent = c->rows_urgent;
+    out->rows_deferred = c->rows_deferred;
+    out->rows_ageout = c->rows_ageout;
+    out->host_read_rows = c->host_read_rows;
+    for (int i = 0; i < FRUGAL_N_PHASES; i++) c->phase_ms[i] = 0;
+    c->timed_steps = 0;
+    return FRUGAL_OK;
+}
+
+extern "C" int64_t frugal_owned_rows(frugal_ctx* c) { return c ? c->No : -1; }
+extern "C" int64_t frugal_hot_slots(frugal_ctx* c) { return c ? c->cap_hot : -1; }

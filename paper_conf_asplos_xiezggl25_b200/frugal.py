@@ -1,0 +1,243 @@
+"""Thin ctypes binding of libfrugal.so (include/frugal.h).  Argument marshalling only:
+every step of the hot path runs in the library's CUDA kernels.  There is no CPU
+fallback: if the library is missing this module raises on import of the context.
+
+Device buffers are torch CUDA tensors (PyTorch is plumbing: memory, streams,
+process groups); host buffers are numpy arrays or pinned torch tensors.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(PKG, "libfrugal.so")
+
+SGD, ADAGRAD = 0, 1
+MODE_P2F, MODE_WRITE_THROUGH = 0, 1
+F_RECORD, F_TIMERS = 1, 2
+FLUSH_ALL = 0
+PHASES = ["ingest", "schedule", "urgent", "gate", "gather", "expand", "model", "segred", "exchange",
+          "optimizer", "side"]
+_STATUS = {0: "FRUGAL_OK", -1: "FRUGAL_EINVAL", -2: "FRUGAL_ENOMEM", -3: "FRUGAL_ECUDA",
+           -4: "FRUGAL_ESTATE", -5: "FRUGAL_ETIMEOUT", -6: "FRUGAL_ESHM"}
+
+
+class FrugalError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"{_STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class Config(C.Structure):
+    _fields_ = [("world", C.c_int32), ("rank", C.c_int32), ("device", C.c_int32), ("dim", C.c_int32),
+                ("n_rows", C.c_int64), ("slots", C.c_int32), ("batch", C.c_int32), ("lookahead", C.c_int32),
+                ("age_out", C.c_int32), ("opt", C.c_int32), ("lr", C.c_float), ("eps", C.c_float),
+                ("init_accum", C.c_float), ("init_scale", C.c_float), ("init_seed", C.c_uint64),
+                ("hot_ids", C.c_void_p), ("n_hot", C.c_int64), ("shm_name", C.c_char_p), ("mode", C.c_int32),
+                ("flags", C.c_int32)]
+
+
+class ScheduleInfo(C.Structure):
+    _fields_ = [("n_urgent", C.c_int64), ("n_deferred", C.c_int64), ("n_ageout", C.c_int64),
+                ("gate_wait", C.c_int32)]
+
+
+class Stats(C.Structure):
+    _fields_ = [("ms", C.c_double * 11), ("steps", C.c_int64), ("kernel_launches", C.c_int64),
+                ("rows_urgent", C.c_int64), ("rows_deferred", C.c_int64), ("rows_ageout", C.c_int64),
+                ("host_read_rows", C.c_int64)]
+
+
+_lib = None
+
+
+def lib():
+    """Load libfrugal.so; raises if it was not built (no fallback path exists)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_asplos_xiezggl25_b200.build` "
+                               "(or __graft_entry__.build()); there is no CPU fallback")
+        L = C.CDLL(LIB_PATH)
+        P, I64, I32 = C.c_void_p, C.c_int64, C.c_int32
+        sig = {
+            "frugal_init": [C.POINTER(Config), C.POINTER(P)],
+            "frugal_prefetch": [P, I64, P, P, P],
+            "frugal_step": [P, I64, P, P, P],
+            "frugal_lookup": [P, I64, P, P],
+            "frugal_backward_update": [P, I64, P, P],
+            "frugal_flush": [P, I32, P],
+            "frugal_destroy": [P],
+            "frugal_dot_model": [P, I64, P, P, P, P, P, P],
+            "frugal_get_dedup": [P, I64, P, P, C.POINTER(I64)],
+            "frugal_get_schedule": [P, C.POINTER(ScheduleInfo), P, P, P, P],
+            "frugal_get_final_flush": [P, P, C.POINTER(I64)],
+            "frugal_read_rows": [P, P, I64, P, P],
+            "frugal_read_host": [P, P, I64, P, P],
+            "frugal_get_stats": [P, C.POINTER(Stats)],
+        }
+        for name, args in sig.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = C.c_int
+        L.frugal_last_error.restype = C.c_char_p
+        L.frugal_last_error.argtypes = []
+        L.frugal_owned_rows.restype = I64
+        L.frugal_owned_rows.argtypes = [P]
+        L.frugal_hot_slots.restype = I64
+        L.frugal_hot_slots.argtypes = [P]
+        _lib = L
+    return _lib
+
+
+EXPORTED = ["frugal_init", "frugal_prefetch", "frugal_step", "frugal_lookup", "frugal_backward_update",
+            "frugal_flush", "frugal_destroy", "frugal_last_error", "frugal_dot_model", "frugal_get_dedup",
+            "frugal_get_schedule", "frugal_get_final_flush", "frugal_read_rows", "frugal_read_host",
+            "frugal_get_stats", "frugal_owned_rows", "frugal_hot_slots"]
+
+
+def _check(status):
+    if status != 0:
+        raise FrugalError(status, lib().frugal_last_error().decode())
+
+
+def _ptr(x):
+    """Pointer of a torch tensor / numpy array / int (None -> NULL)."""
+    if x is None:
+        return None
+    if isinstance(x, int):
+        return x
+    if hasattr(x, "data_ptr"):
+        return x.data_ptr()
+    return x.ctypes.data
+
+
+def _stream(stream):
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+class Frugal:
+    """One rank's context (frugal_ctx).  Names follow frugal.h."""
+
+    def __init__(self, *, world, rank, device, dim, n_rows, slots, batch, lookahead=10, age_out=10,
+                 opt="adagrad", lr=0.05, eps=1e-10, init_accum=0.0, init_scale=0.05, init_seed=3, hot_ids=None,
+                 shm_name=None, mode=MODE_P2F, flags=0):
+        self.world, self.rank, self.dim, self.slots, self.batch = world, rank, dim, slots, batch
+        self.lookahead = lookahead
+        hot = np.ascontiguousarray(np.zeros(0, np.int64) if hot_ids is None else hot_ids, dtype=np.int64)
+        self._hot = hot
+        self._shm = shm_name.encode() if shm_name else None
+        c = Config(world=world, rank=rank, device=device, dim=dim, n_rows=n_rows, slots=slots, batch=batch,
+                   lookahead=lookahead, age_out=age_out, opt=ADAGRAD if opt == "adagrad" else SGD, lr=lr, eps=eps,
+                   init_accum=init_accum, init_scale=init_scale, init_seed=init_seed,
+                   hot_ids=hot.ctypes.data if hot.size else None, n_hot=hot.size, shm_name=self._shm, mode=mode,
+                   flags=flags)
+        self._cfg = c
+        h = C.c_void_p()
+        _check(lib().frugal_init(C.byref(c), C.byref(h)))
+        self.h = h
+
+    @classmethod
+    def from_workload(cls, wcfg, *, world=None, rank=0, device=0, hot_ids=None, **kw):
+        return cls(world=wcfg.world if world is None else world, rank=rank, device=device, dim=wcfg.dim,
+                   n_rows=wcfg.n_rows, slots=wcfg.slots, batch=wcfg.batch, lookahead=wcfg.lookahead,
+                   age_out=wcfg.age_out, opt=wcfg.opt, lr=wcfg.lr, eps=wcfg.eps, init_accum=wcfg.init_accum,
+                   init_scale=wcfg.init_scale, init_seed=wcfg.seed_init, hot_ids=hot_ids, **kw)
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().frugal_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # ---- the hot path ---------------------------------------------------------------
+    def prefetch(self, t, ids_all, counts, stream=None):
+        counts = np.ascontiguousarray(counts, dtype=np.int32)
+        _check(lib().frugal_prefetch(self.h, t, _ptr(ids_all), counts.ctypes.data, _stream(stream)))
+
+    def step(self, s, ids_next_all=None, counts_next=None, stream=None):
+        cn = None if counts_next is None else np.ascontiguousarray(counts_next, dtype=np.int32)
+        _check(lib().frugal_step(self.h, s, _ptr(ids_next_all), None if cn is None else cn.ctypes.data,
+                                 _stream(stream)))
+
+    def lookup(self, s, out, stream=None):
+        _check(lib().frugal_lookup(self.h, s, _ptr(out), _stream(stream)))
+
+    def dot_model(self, s, emb, x, y, grad, loss, stream=None):
+        _check(lib().frugal_dot_model(self.h, s, _ptr(emb), _ptr(x), _ptr(y), _ptr(grad), _ptr(loss),
+                                      _stream(stream)))
+
+    def backward_update(self, s, grad, stream=None):
+        _check(lib().frugal_backward_update(self.h, s, _ptr(grad), _stream(stream)))
+
+    def flush(self, what=FLUSH_ALL, stream=None):
+        _check(lib().frugal_flush(self.h, what, _stream(stream)))
+
+    # ---- introspection ---------------------------------------------------------------
+    def get_dedup(self, t):
+        n = C.c_int64()
+        _check(lib().frugal_get_dedup(self.h, t, None, None, C.byref(n)))
+        uq = np.empty(n.value, np.int64)
+        inv = np.empty(self.batch * self.slots, np.int32)
+        _check(lib().frugal_get_dedup(self.h, t, uq.ctypes.data, inv.ctypes.data, C.byref(n)))
+        return uq, inv
+
+    def get_schedule(self):
+        info = ScheduleInfo()
+        _check(lib().frugal_get_schedule(self.h, C.byref(info), None, None, None, None))
+        u = np.empty(info.n_urgent, np.int64)
+        dfr = np.empty(info.n_deferred, np.int64)
+        dp = np.empty(info.n_deferred, np.int32)
+        a = np.empty(info.n_ageout, np.int64)
+        _check(lib().frugal_get_schedule(self.h, C.byref(info), u.ctypes.data, dfr.ctypes.data, dp.ctypes.data,
+                                         a.ctypes.data))
+        return dict(urgent=u, deferred=dfr, deferred_p=dp, ageout=a, gate_wait=bool(info.gate_wait))
+
+    def get_final_flush(self):
+        n = C.c_int64()
+        _check(lib().frugal_get_final_flush(self.h, None, C.byref(n)))
+        out = np.empty(n.value, np.int64)
+        _check(lib().frugal_get_final_flush(self.h, out.ctypes.data, C.byref(n)))
+        return out
+
+    def read_rows(self, ids):
+        ids = np.ascontiguousarray(ids, dtype=np.int64)
+        w = np.empty((len(ids), self.dim), np.float32)
+        G = np.empty((len(ids), self.dim), np.float32)
+        _check(lib().frugal_read_rows(self.h, ids.ctypes.data, len(ids), w.ctypes.data, G.ctypes.data))
+        return w, G
+
+    def read_host(self, ids):
+        ids = np.ascontiguousarray(ids, dtype=np.int64)
+        w = np.empty((len(ids), self.dim), np.float32)
+        G = np.empty((len(ids), self.dim), np.float32)
+        _check(lib().frugal_read_host(self.h, ids.ctypes.data, len(ids), w.ctypes.data, G.ctypes.data))
+        return w, G
+
+    def get_stats(self):
+        s = Stats()
+        _check(lib().frugal_get_stats(self.h, C.byref(s)))
+        return dict(ms={p: s.ms[i] for i, p in enumerate(PHASES)}, steps=s.steps,
+                    kernel_launches=s.kernel_launches, rows_urgent=s.rows_urgent, rows_deferred=s.rows_deferred,
+                    rows_ageout=s.rows_ageout)
+
+    @property
+    def owned_rows(self):
+        return lib().frugal_owned_rows(self.h)
+
+    @property
+    def hot_slots(self):
+        return lib().frugal_hot_slots(self.h)

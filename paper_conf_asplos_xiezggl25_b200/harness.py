@@ -1,0 +1,66 @@
+"""Training-loop harness around the C ABI (used by tests, bench.py and smoke()).
+
+It only sequences the public calls of include/frugal.h for one rank:
+prefetch(0..L-2), then per step: step(s) -> lookup(s) -> dot_model(s) ->
+backward_update(s), and flush() at the end.  No arithmetic of the method
+happens here.
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+
+from . import frugal as F
+
+
+def make_context(st, rank=0, device=0, shm_name=None, flags=0, hot=None, mode=F.MODE_P2F, **over):
+    cfg = st.cfg
+    world = st.ids.shape[1]
+    kw = dict(world=world, rank=rank, device=device, dim=cfg.dim, n_rows=cfg.n_rows, slots=cfg.slots,
+              batch=st.ids.shape[2] // cfg.slots, lookahead=cfg.lookahead, age_out=cfg.age_out, opt=cfg.opt,
+              lr=cfg.lr, eps=cfg.eps, init_accum=cfg.init_accum, init_scale=cfg.init_scale,
+              init_seed=cfg.seed_init, hot_ids=st.hot if hot is None else hot, shm_name=shm_name, mode=mode,
+              flags=flags)
+    kw.update(over)
+    return F.Frugal(**kw)
+
+
+class Trainer:
+    """Runs the stream on one rank.  Inputs are uploaded per step from host arrays."""
+
+    def __init__(self, fr: F.Frugal, st, rank=0, device=0):
+        self.fr, self.st, self.rank = fr, st, rank
+        self.dev = torch.device("cuda", device)
+        B, Fs, d = st.ids.shape[2] // st.cfg.slots, st.cfg.slots, st.cfg.dim
+        self.emb = torch.empty(B * Fs, d, device=self.dev)
+        self.grad = torch.empty_like(self.emb)
+        self.loss = torch.zeros(st.steps, dtype=torch.float64, device=self.dev)
+        self.s = 0
+        L = fr.lookahead
+        for t in range(min(L - 1, st.steps)):
+            fr.prefetch(t, st.ids[t], st.counts[t])
+
+    def step(self, on_schedule=None):
+        st, fr, s = self.st, self.fr, self.s
+        t = s + fr.lookahead - 1
+        if t < st.steps:
+            fr.step(s, st.ids[t], st.counts[t])
+        else:
+            fr.step(s)
+        if on_schedule:
+            on_schedule(s)
+        fr.lookup(s, self.emb)
+        x = torch.from_numpy(st.x[s, self.rank]).to(self.dev, non_blocking=False)
+        y = torch.from_numpy(st.y[s, self.rank]).to(self.dev, non_blocking=False)
+        fr.dot_model(s, self.emb, x, y, self.grad, self.loss[s:s + 1])
+        fr.backward_update(s, self.grad)
+        self.s += 1
+
+    def run(self, steps=None, on_schedule=None):
+        n = self.st.steps if steps is None else steps
+        while self.s < n:
+            self.step(on_schedule)
+
+    def losses(self):
+        torch.cuda.synchronize(self.dev)
+        return self.loss.cpu().numpy()

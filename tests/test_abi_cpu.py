@@ -1,0 +1,82 @@
+"""CPU-only checks of the C ABI library: it loads, exports every symbol frugal.h
+declares, and validates configs without touching a GPU."""
+import ctypes as C
+import os
+import re
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _lib():
+    from paper_conf_asplos_xiezggl25_b200 import build as B
+    B.build()
+    from paper_conf_asplos_xiezggl25_b200 import frugal as F
+    return F
+
+
+def declared_symbols():
+    src = open(os.path.join(ROOT, "include", "frugal.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(frugal_[a-z_]+)\s*\(", src)))
+
+
+def test_every_declared_symbol_is_exported():
+    F = _lib()
+    L = F.lib()
+    syms = declared_symbols()
+    assert len(syms) >= 15
+    missing = [s for s in syms if not hasattr(L, s)]
+    assert not missing, missing
+    assert set(syms) == set(F.EXPORTED)
+
+
+def test_sass_is_sm100a():
+    import subprocess
+    F = _lib()
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", F.LIB_PATH], capture_output=True,
+                         text=True).stdout
+    assert "sm_100a" in out
+
+
+@pytest.mark.parametrize("field,value", [("world", 0), ("dim", 6), ("lookahead", 1), ("lookahead", 40),
+                                         ("age_out", 0), ("n_rows", 0), ("batch", 0), ("opt", 7)])
+def test_config_validation(field, value):
+    F = _lib()
+    cfg = F.Config(world=1, rank=0, device=0, dim=16, n_rows=100, slots=1, batch=4, lookahead=4, age_out=2,
+                   opt=1, lr=0.1, eps=1e-10, init_accum=0.0, init_scale=0.05, init_seed=3, hot_ids=None,
+                   n_hot=0, shm_name=None, mode=0, flags=0)
+    setattr(cfg, field, value)
+    h = C.c_void_p()
+    st = F.lib().frugal_init(C.byref(cfg), C.byref(h))
+    assert st == -1, F.lib().frugal_last_error()
+    assert not h.value
+
+
+def test_world_gt1_needs_shm():
+    F = _lib()
+    cfg = F.Config(world=2, rank=0, device=0, dim=16, n_rows=100, slots=1, batch=4, lookahead=4, age_out=2,
+                   opt=1, lr=0.1, eps=1e-10, init_accum=0.0, init_scale=0.05, init_seed=3, hot_ids=None,
+                   n_hot=0, shm_name=None, mode=0, flags=0)
+    h = C.c_void_p()
+    assert F.lib().frugal_init(C.byref(cfg), C.byref(h)) == -1
+    assert b"shm" in F.lib().frugal_last_error()
+
+
+def test_null_ctx_calls_fail_cleanly():
+    F = _lib()
+    L = F.lib()
+    assert L.frugal_step(None, 0, None, None, None) == -1
+    assert L.frugal_lookup(None, 0, None, None) == -1
+    assert L.frugal_destroy(None) == 0
+
+
+def test_product_path_does_not_import_oracle():
+    """The product (package + CUDA sources) never imports, links or loads oracle/."""
+    pkg = os.path.join(ROOT, "paper_conf_asplos_xiezggl25_b200")
+    pat = re.compile(r"^\s*(from\s+oracle|import\s+oracle)|liboracle|frugal_oracle", re.M)
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h")):
+                assert not pat.search(open(os.path.join(dirpath, f)).read()), f

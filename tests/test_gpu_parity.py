@@ -1,0 +1,214 @@
+"""Parity of the CUDA path (through the C ABI) against the CPU oracle, on a B200.
+
+Bars (BASELINE.json north_star): dedup indices, priority-bucket membership, flush
+sets bit-exact; fp32 tables (w, G) and per-step losses within 1e-5 max-abs after
+100 steps.
+"""
+import dataclasses
+import os
+
+import numpy as np
+import pytest
+
+from oracle.oracle import Oracle
+from paper_conf_asplos_xiezggl25_b200 import workload as W
+
+pytestmark = pytest.mark.gpu
+TOL = 1e-5
+
+
+def _F():
+    from paper_conf_asplos_xiezggl25_b200 import frugal as F
+    return F
+
+
+def run_parity(st, *, flags=None, mode=None, hot=None, check_dedup=True, check_sched=True, steps=None,
+               sample_rows=None, oracle_kw=None):
+    """Run the stream on cuda:0 (world 1) and on the oracle; assert the bars."""
+    F = _F()
+    from paper_conf_asplos_xiezggl25_b200.harness import Trainer, make_context
+    flags = F.F_RECORD if flags is None else flags
+    mode = F.MODE_P2F if mode is None else mode
+    hot = st.hot if hot is None else hot
+    fr = make_context(st, flags=flags, mode=mode, hot=hot)
+    o = Oracle(st, hot=hot, write_through=(mode == F.MODE_WRITE_THROUGH), **(oracle_kw or {}))
+    tr = Trainer(fr, st)
+    S = st.steps if steps is None else steps
+    L = st.cfg.lookahead
+    if check_dedup:
+        for t in range(min(L - 1, st.steps)):
+            uq, inv = fr.get_dedup(t)
+            ouq, oinv = o.dedup(t, 0)
+            assert np.array_equal(uq, ouq) and np.array_equal(inv[:len(oinv)], oinv), f"dedup differs at {t}"
+    gate_waits = 0
+    for s in range(S):
+        got = {}
+
+        def cb(s_):
+            if check_sched:
+                got.update(fr.get_schedule())
+            if check_dedup and s_ + L - 1 < st.steps:
+                t = s_ + L - 1
+                uq, inv = fr.get_dedup(t)
+                ouq, oinv = o.dedup(t, 0)
+                assert np.array_equal(uq, ouq), f"uniq differs at step {t}"
+                assert np.array_equal(inv[:len(oinv)], oinv), f"inv differs at step {t}"
+
+        tr.step(on_schedule=cb)
+        o.step()
+        if check_sched:
+            ref = o.schedule()
+            assert sorted(got["urgent"].tolist()) == ref["urgent"].tolist(), f"urgent set differs at {s}"
+            assert sorted(zip(got["deferred"].tolist(), got["deferred_p"].tolist())) == \
+                list(zip(ref["deferred"].tolist(), ref["deferred_p"].tolist())), f"deferred set differs at {s}"
+            assert sorted(got["ageout"].tolist()) == ref["ageout"].tolist(), f"age-out set differs at {s}"
+            assert got["gate_wait"] == ref["gate_wait"]
+            gate_waits += ref["gate_wait"]
+    assert o.violations == 0
+    lo = np.array([o.loss(s) for s in range(S)])
+    lg = tr.losses()[:S]
+    assert np.abs(lg - lo).max() <= TOL, f"loss differs by {np.abs(lg - lo).max()}"
+    out = dict(fr=fr, o=o, gate_waits=gate_waits)
+    if S == st.steps:
+        fr.flush()
+        ff = o.final_flush()
+        assert sorted(fr.get_final_flush().tolist()) == ff.tolist(), "final flush set differs"
+        ks = np.arange(st.cfg.n_rows) if sample_rows is None else sample_rows
+        w, G = fr.read_host(ks)
+        wo, Go = o.read_rows(ks)
+        out.update(dw=float(np.abs(w - wo).max()), dG=float(np.abs(G - Go).max()),
+                   exact=bool(np.array_equal(w, wo) and np.array_equal(G, Go)), w=w, wo=wo)
+        assert out["dw"] <= TOL and out["dG"] <= TOL, (out["dw"], out["dG"])
+    else:
+        ks = sample_rows
+        w, G = fr.read_rows(ks)
+        wo, Go = o.read_rows(ks)
+        out.update(dw=float(np.abs(w - wo).max()), dG=float(np.abs(G - Go).max()))
+        assert out["dw"] <= TOL and out["dG"] <= TOL, (out["dw"], out["dG"])
+    return out
+
+
+def tiny1(**over):
+    kw = dict(world=1)
+    kw.update(over)
+    return W.config("tiny", **kw)
+
+
+def test_tiny_100_steps_parity():
+    """configs[0] (tiny DLRM-style, 10^4 x 16, batch 256) at world 1, 100 parity steps."""
+    st = W.gen_stream(tiny1(), 100)
+    r = run_parity(st)
+    w0 = np.array([[r["o"].init_value(k, j) for j in range(16)] for k in range(st.cfg.n_rows)], np.float32)
+    assert np.abs(r["wo"] - w0).max() >= 1e-3  # non-vacuous: parameters moved
+    assert r["gate_waits"] > 0                 # the gate actually blocked on urgent flushes
+    assert r["exact"], "tables are expected bit-exact (canonical fixed-order arithmetic)"
+    r["fr"].close()
+
+
+def test_ragged_and_empty_batches():
+    cfg = tiny1(batch=64, lookahead=5, age_out=2)
+    rng = np.random.default_rng(7)
+    counts = rng.integers(0, 65, size=(40, 1)).astype(np.int32)
+    counts[3] = 0
+    counts[10:12] = 0
+    counts[-1] = 0
+    counts[20] = 64
+    st = W.gen_stream(cfg, 40, counts=counts)
+    run_parity(st)["fr"].close()
+
+
+@pytest.mark.parametrize("L,D", [(2, 1), (3, 5), (31, 1), (10, 40)])
+def test_lookahead_and_ageout(L, D):
+    st = W.gen_stream(tiny1(lookahead=L, age_out=D, batch=128), 50)
+    run_parity(st)["fr"].close()
+
+
+@pytest.mark.parametrize("dim", [4, 8, 64, 128, 400])
+def test_dims(dim):
+    cfg = W.WorkloadConfig("d", [3000, 500, 7], dim=dim, batch=96, world=1, lookahead=4, age_out=3)
+    st = W.gen_stream(cfg, 25)
+    run_parity(st)["fr"].close()
+
+
+def test_sgd():
+    st = W.gen_stream(tiny1(opt="sgd", lr=1.0, batch=128), 40)
+    run_parity(st)["fr"].close()
+
+
+def test_long_segments_chunked_order():
+    """A 1-row and a 3-row table: segments of 1000+ occurrences exercise the chunked
+    fixed-order reduction (R23) against the oracle bit for bit."""
+    cfg = W.WorkloadConfig("long", [1, 3, 5000], dim=32, batch=1500, world=1, lookahead=3, age_out=2)
+    st = W.gen_stream(cfg, 12)
+    r = run_parity(st)
+    assert r["exact"]
+    r["fr"].close()
+
+
+def test_metamorphic_tables_identical():
+    """P2F == write-through (Frugal-Sync) == no cache == large cache == L=2, bit for bit."""
+    F = _F()
+    base = W.gen_stream(tiny1(batch=128, lookahead=6, age_out=3), 30)
+    tabs = []
+    variants = [dict(), dict(mode=F.MODE_WRITE_THROUGH), dict(hot=np.zeros(0, np.int64)),
+                dict(hot=np.arange(0, 10_000, 2, dtype=np.int64))]
+    for v in variants:
+        r = run_parity(base, **v)
+        tabs.append(r["w"])
+        r["fr"].close()
+    st2 = dataclasses.replace(base, cfg=dataclasses.replace(base.cfg, lookahead=2))
+    r = run_parity(st2)
+    tabs.append(r["w"])
+    r["fr"].close()
+    for t in tabs[1:]:
+        assert np.array_equal(tabs[0], t)
+
+
+def test_write_through_flushes_every_update():
+    F = _F()
+    st = W.gen_stream(tiny1(batch=64, lookahead=4), 10)
+    r = run_parity(st, mode=F.MODE_WRITE_THROUGH)
+    r["fr"].close()
+
+
+def test_criteo_kaggle_full_size_sampled():
+    """configs[1] shape (26 tables, 33.8M rows, d=32, batch 8192) at world 1, the launch
+    configuration bench.py times: dedup and schedule sets bit-exact every step, sampled
+    touched rows within 1e-5 (oracle materialises rows lazily)."""
+    cfg = W.config("criteo_kaggle", world=1)
+    st = W.gen_stream(cfg, 14)
+    rng = np.random.default_rng(0)
+    touched = np.unique(st.ids[:6, 0].ravel())
+    sample = np.sort(rng.choice(touched, size=20000, replace=False))
+    r = run_parity(st, steps=6, sample_rows=sample)
+    r["fr"].close()
+
+
+def test_invalid_id_fails_loudly():
+    F = _F()
+    from paper_conf_asplos_xiezggl25_b200.harness import Trainer, make_context
+    st = W.gen_stream(tiny1(batch=32, lookahead=3), 6)
+    st.ids[4, 0, 5] = st.cfg.n_rows + 7
+    fr = make_context(st)
+    tr = Trainer(fr, st)
+    with pytest.raises(F.FrugalError) as e:
+        for _ in range(6):
+            tr.step()
+        fr.flush()
+    assert e.value.status == -1
+    fr.close()
+
+
+def test_call_order_enforced():
+    F = _F()
+    import torch
+    from paper_conf_asplos_xiezggl25_b200.harness import make_context
+    st = W.gen_stream(tiny1(batch=32, lookahead=3), 6)
+    fr = make_context(st)
+    out = torch.empty(32, 16, device="cuda")
+    with pytest.raises(F.FrugalError) as e:
+        fr.lookup(0, out)
+    assert e.value.status == -4
+    with pytest.raises(F.FrugalError):
+        fr.step(0, st.ids[2], st.counts[2])  # steps 0..L-2 not prefetched yet
+    fr.close()
