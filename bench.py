@@ -1,0 +1,385 @@
+#!/usr/bin/env python
+"""Benchmark of the Frugal training step on B200 (contract: one JSON line on rank 0).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+    torchrun --nproc-per-node N bench.py --gpus N ...            (N > 1)
+
+Workload: BASELINE.json configs[1], the Criteo-Kaggle-shaped DLRM embedding step
+(26 tables, 33,762,577 rows, d = 32, fp32, Adagrad, Zipf alpha = 0.9, batch 8192 per
+GPU, cache 5 %, L = 10), synthetic seeded ids.  A step is
+one pass of the whole hot path: frugal_step (lookahead ingest + dedup + P2F bucketing
++ urgent flush + deferred drain on the side stream + gate) -> frugal_lookup (cache /
+zero-copy host gather + expand) -> frugal_dot_model (glue) -> frugal_backward_update
+(segment-reduce, mailbox exchange for N > 1, fused Adagrad).  Weak scaling: every rank
+trains its own 8192-sample batch; all ranks share one host table in POSIX shm.
+
+value  = samples/s with the step's inputs (ids of all ranks, x, y) already in HBM;
+e2e    = samples/s through the same public calls with host (pinned) inputs copied
+         in each step and the step's loss read back to the host;
+roofline / per-phase rooflines use CUDA events recorded around every phase inside
+the timed region (FRUGAL_F_TIMERS) and device row counters; cpu_baseline is the
+oracle (oracle/, single thread) on a bounded sample of the same stream.
+"""
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "training samples/s at 1/2/4/8 B200; flush+gather GB/s vs HBM/host-link peak"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="criteo_kaggle")
+    ap.add_argument("--alpha", type=float, default=0.9)
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------------------ clocks
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, dev):
+        self.dev, self.rows, self.p = dev, [], None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.dev), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except FileNotFoundError:
+            self.p = None
+
+    def _read(self):
+        for line in self.p.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) == 6:
+                self.rows.append(parts)
+
+    def stop(self):
+        if not self.p:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.p.terminate()
+        self.p.wait()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[2 + i].lower() == "active"})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+# ------------------------------------------------------------------------------ peaks
+def host_link_peaks(torch, dev):
+    """Pinned-copy peaks (1 GPU): H2D, D2H (256 MiB, best of 5, CUDA events)."""
+    n = 256 << 20
+    h = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(n, dtype=torch.uint8, device=dev)
+    out = {}
+    for name, fn in [("h2d", lambda: d.copy_(h, non_blocking=True)), ("d2h", lambda: h.copy_(d, non_blocking=True))]:
+        fn()
+        torch.cuda.synchronize()
+        best = 1e9
+        for _ in range(5):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            fn()
+            b.record()
+            b.synchronize()
+            best = min(best, a.elapsed_time(b))
+        out[name] = n / best / 1e6
+    del h, d
+    return out
+
+
+def measured_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+# ------------------------------------------------------------------------------ cpu baseline
+def cpu_baseline(cfg, st, seconds):
+    """The oracle as it stands (single thread) on the first steps of the same stream."""
+    from oracle.oracle import Oracle
+    o = Oracle(st)
+    t0 = time.perf_counter()
+    n = 0
+    while n < st.steps and time.perf_counter() - t0 < seconds:
+        o.step()
+        n += 1
+    dt = time.perf_counter() - t0
+    B = st.ids.shape[2] // cfg.slots
+    return {"value": n * B * st.ids.shape[1] / dt, "unit": "samples/s", "cores": 1, "kind": "oracle",
+            "sample": f"first {n} steps of the {cfg.name} stream (world {st.ids.shape[1]}, batch {B}), "
+                      f"{dt:.1f} s of single-thread C oracle incl. brute-force P2F schedule"}
+
+
+# ------------------------------------------------------------------------------ reference arm
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    from paper_conf_asplos_xiezggl25_b200 import workload as W
+    cfg = W.config(args.config, world=1, alpha=args.alpha)
+    steps = args.warmup + args.steps
+    # bounded sample: each "step" is one oracle step; cap the run to a few minutes
+    per_step_budget = 60
+    st = W.gen_stream(cfg, min(steps, per_step_budget) + cfg.lookahead)
+    from oracle.oracle import Oracle
+    o = Oracle(st)
+    for _ in range(min(args.warmup, 3)):
+        o.step()
+    K = min(args.steps, per_step_budget - min(args.warmup, 3))
+    t0 = time.perf_counter()
+    for _ in range(K):
+        o.step()
+    dt = time.perf_counter() - t0
+    v = K * cfg.batch / dt
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "samples/s", "n_gpus": 1, "steps": K,
+            "warmup": min(args.warmup, 3), "ms_per_step": dt / K * 1e3, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": cfg.name, "global_batch": cfg.batch, "tables": cfg.slots,
+                       "rows": cfg.n_rows, "dim": cfg.dim, "alpha": cfg.alpha, "lookahead": cfg.lookahead,
+                       "cache_ratio": cfg.cache_ratio, "opt": cfg.opt, "parallelism": "oracle, 1 CPU thread"},
+            "e2e": {"value": v, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+            "cpu_baseline": {"value": v, "unit": "samples/s", "cores": 1, "kind": "oracle",
+                             "sample": f"{K} oracle steps of the {cfg.name} stream after {min(args.warmup, 3)} "
+                                       "warm-up steps (bounded sample)"}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------------------ our arm
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    if world != args.gpus and world == 1 and args.gpus > 1:
+        sys.exit("--gpus N > 1 must be launched under torchrun with N processes")
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    import torch
+    import torch.distributed as dist
+    from paper_conf_asplos_xiezggl25_b200 import frugal as F
+    from paper_conf_asplos_xiezggl25_b200 import workload as W
+    from paper_conf_asplos_xiezggl25_b200.harness import make_context
+
+    assert args.warmup >= 3, "timing rules: at least 3 warm-up steps"
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def max_over_ranks(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    cfg = W.config(args.config, world=world, alpha=args.alpha)
+    K, Wm, L = args.steps, args.warmup, cfg.lookahead
+    S = Wm + 2 * K + L + 1
+    t_gen = time.time()
+    st = W.gen_stream(cfg, S)  # every rank generates the same seeded stream of all ranks
+    t_gen = time.time() - t_gen
+    B, Fs, d = cfg.batch, cfg.slots, cfg.dim
+    shm = f"/frugal_bench_{os.environ.get('MASTER_PORT', '0')}" if world > 1 else None
+    fr = make_context(st, rank=rank, device=local, shm_name=shm, flags=F.F_TIMERS)
+    barrier()
+    stream = torch.cuda.current_stream(dev)
+
+    # inputs of the value leg resident in HBM
+    ids_d = torch.from_numpy(st.ids).to(dev)                       # [S][world][M] int64
+    x_d = torch.from_numpy(np.ascontiguousarray(st.x[:, rank])).to(dev)
+    y_d = torch.from_numpy(np.ascontiguousarray(st.y[:, rank])).to(dev)
+    emb = torch.empty(B * Fs, d, device=dev)
+    grad = torch.empty_like(emb)
+    loss = torch.zeros(S, dtype=torch.float64, device=dev)
+    # pinned host copies for the e2e leg
+    ids_h = torch.from_numpy(st.ids).pin_memory()
+    x_h = torch.from_numpy(np.ascontiguousarray(st.x[:, rank])).pin_memory()
+    y_h = torch.from_numpy(np.ascontiguousarray(st.y[:, rank])).pin_memory()
+    loss_h = torch.zeros(S, dtype=torch.float64).pin_memory()
+    x_e = torch.empty(B, d, device=dev)
+    y_e = torch.empty(B, device=dev)
+    counts = st.counts
+
+    for t in range(L - 1):
+        fr.prefetch(t, ids_d[t], counts[t])
+
+    def step_dev(s):
+        t = s + L - 1
+        fr.step(s, ids_d[t], counts[t])
+        fr.lookup(s, emb)
+        fr.dot_model(s, emb, x_d[s], y_d[s], grad, loss[s:s + 1])
+        fr.backward_update(s, grad)
+
+    def step_e2e(s):
+        t = s + L - 1
+        fr.step(s, ids_h[t], counts[t])       # ids copied from pinned host inside the call
+        fr.lookup(s, emb)
+        x_e.copy_(x_h[s], non_blocking=True)
+        y_e.copy_(y_h[s], non_blocking=True)
+        fr.dot_model(s, emb, x_e, y_e, grad, loss[s:s + 1])
+        fr.backward_update(s, grad)
+        loss_h[s:s + 1].copy_(loss[s:s + 1], non_blocking=True)
+
+    # ---- warm-up
+    for s in range(Wm):
+        step_dev(s)
+    torch.cuda.synchronize()
+    fr.get_stats()  # reset phase timers / read counters
+    st0 = fr.get_stats()
+    # ---- value leg (inputs in HBM)
+    clocks = Clocks(local)
+    clocks.start()
+    barrier()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for s in range(Wm, Wm + K):
+        step_dev(s)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    barrier()
+    ms = e0.elapsed_time(e1)
+    clk = clocks.stop()
+    st1 = fr.get_stats()
+    ms_max = max_over_ranks(ms)
+    value = world * B * K / (ms_max / 1e3)
+
+    # ---- e2e leg (host inputs, loss read back)
+    barrier()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    f0.record(stream)
+    for s in range(Wm + K, Wm + 2 * K):
+        step_e2e(s)
+    f1.record(stream)
+    torch.cuda.synchronize()
+    wall = time.perf_counter() - t0
+    barrier()
+    e2e_ms = max_over_ranks(max(f0.elapsed_time(f1), wall * 1e3))
+    e2e = world * B * K / (e2e_ms / 1e3)
+    fr.get_stats()
+    finite = bool(torch.isfinite(loss[Wm:Wm + 2 * K]).all().item())
+
+    # ---- per-phase rooflines for this rank
+    cnt = {k: st1["count"][k] - st0["count"][k] for k in st1["count"]}
+    ph = {k: v / K for k, v in st1["ms"].items()}  # ms per step (per launch of the phase)
+    r = 4 * d
+    adag = cfg.opt == "adagrad"
+    peaks = measured_peaks()
+    link = host_link_peaks(torch, dev)
+    hbm_peak = peaks.get("hbm_gbs", 6650.0)
+
+    def gbs(nbytes, ms_):
+        return nbytes / (ms_ * 1e-3) / 1e9 if ms_ > 0 else None
+
+    per = {}
+    # a4 gather: unique rows from host (zero-copy, PCIe H2D) -- the miss path
+    per["gather"] = dict(bound="host-link h2d", bytes=cnt["gather_host"] * r / K,
+                         hbm_bytes=(cnt["gather_cache"] + cnt["unique"]) * r / K, ms=ph["gather"],
+                         peak=link["h2d"])
+    # a10 urgent flush (D2H, critical path), a11 side drain (D2H, side stream)
+    for nm, h, c_ in [("urgent", "urgent_hot", "urgent_cold"), ("side", "side_hot", "side_cold")]:
+        per[nm] = dict(bound="host-link d2h", bytes=(cnt[h] * r + cnt[c_] * r * (2 if adag else 1)) / K,
+                       ms=ph[nm], peak=link["d2h"])
+    # a4 expand: out[i] = rows[inv[i]] -- HBM write of M rows + read of rows/inv
+    per["expand"] = dict(bound="hbm", bytes=(cnt["positions"] * (2 * r + 4)) / K, ms=ph["expand"], peak=hbm_peak)
+    # a6 segment-reduce: read M grad rows + pos, write U partial rows + offsets
+    per["segred"] = dict(bound="hbm", bytes=(cnt["positions"] * (r + 4) + cnt["unique"] * (r + 4)) / K,
+                         ms=ph["segred"], peak=hbm_peak)
+    # a8 optimizer: hot rows r/w (w,G) in HBM; cold rows read G over the link (+w when N>1)
+    per["optimizer"] = dict(bound="host-link h2d",
+                            bytes=cnt["opt_cold"] * r * ((1 if world == 1 else 2) if adag else (0 if world == 1 else 1)) / K,
+                            hbm_bytes=(cnt["opt_hot"] * r * (4 if adag else 2) + cnt["opt_cold"] * r * (3 if adag else 2)
+                                       + (cnt["opt_hot"] + cnt["opt_cold"]) * r) / K,
+                            ms=ph["optimizer"], peak=link["h2d"])
+    for k, v in per.items():
+        v["achieved_gbs"] = gbs(v["bytes"], v["ms"])
+        v["frac"] = v["achieved_gbs"] / v["peak"] if v["achieved_gbs"] else None
+    main_ms = {k: v for k, v in ph.items() if k != "side"}
+    dom = max(("gather", "urgent", "expand", "segred", "optimizer"), key=lambda k: per[k]["ms"])
+    top = max(main_ms, key=main_ms.get)
+    D = per[dom]
+    traffic = None
+    try:
+        prof = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
+        traffic = prof.get(dom, {}).get("dram_bytes_per_launch")
+    except Exception:
+        pass
+    roofline = {"bound": "hbm" if D["bound"] == "hbm" else "host-link", "kernel": dom,
+                "achieved": D["achieved_gbs"], "peak": D["peak"], "unit": "GB/s", "frac": D["frac"],
+                "traffic": traffic,
+                "peak_source": ("measured pinned cudaMemcpy H2D/D2H 256 MiB in this run" if D["bound"] != "hbm"
+                                else "MEASURED_PEAKS.json hbm_gbs")}
+    launches = st1["kernel_launches"] - st0["kernel_launches"]
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(cfg, W.gen_stream(cfg, 80), args.cpu_seconds)
+    h2d = int(world * B * Fs * 8 + B * d * 4 + B * 4 + world * 4)
+    line = {
+        "metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": world, "steps": K, "warmup": Wm,
+        "ms_per_step": ms_max / K, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "f32", "data": "synthetic",
+        "config": {"workload": f"{cfg.name} (BASELINE.json configs[1])", "global_batch": world * B,
+                   "batch_per_gpu": B, "tables": Fs, "rows": cfg.n_rows, "dim": d, "alpha": cfg.alpha,
+                   "lookahead": L, "age_out": cfg.age_out, "cache_ratio": cfg.cache_ratio, "opt": cfg.opt,
+                   "parallelism": f"dp{world} (owner-sharded rows, shared pinned host table)",
+                   "l2": "inputs larger than L2: host table %.1f GB, HBM cache %.0f MB, %d distinct id batches"
+                         % (cfg.n_rows * r * (2 if adag else 1) / 1e9, len(st.hot) * r * 2 / 1e6, K)},
+        "e2e": {"value": e2e, "unit": "samples/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": 8},
+        "gpu_launches": int(launches),
+        "roofline": roofline,
+        "phases_ms_per_step": {k: round(v, 5) for k, v in ph.items()},
+        "rooflines": {k: {kk: (round(vv, 4) if isinstance(vv, float) else vv) for kk, vv in v.items()}
+                      for k, v in per.items()},
+        "flush_gather_gbs": {"gather_host_h2d": per["gather"]["achieved_gbs"],
+                             "flush_urgent_d2h": per["urgent"]["achieved_gbs"],
+                             "flush_side_d2h": per["side"]["achieved_gbs"],
+                             "host_link_peak": link, "hbm_peak": hbm_peak},
+        "rows_per_step": {k: v / K for k, v in cnt.items() if k != "reserved"},
+        "top_main_stream_phase": top,
+        "clocks": clk,
+        "loss_finite": finite,
+        "gen_s": round(t_gen, 1),
+    }
+    if cpu:
+        line["cpu_baseline"] = cpu
+    fr.close()
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

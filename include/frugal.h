@@ -170,17 +170,35 @@ frugal_status frugal_read_rows(frugal_ctx* ctx, const int64_t* ids, int64_t n, f
 /* raw host-table contents (any row). */
 frugal_status frugal_read_host(frugal_ctx* ctx, const int64_t* ids, int64_t n, float* w, float* G);
 
-/* per-phase device time (ms) summed over the steps since the last call, plus launch
-   counts (needs FRUGAL_F_TIMERS).  Phases, in order: ingest (a1+a2), schedule (a9),
-   urgent (a10), gate (a3), gather (a4, unique rows), expand (a4, per position),
-   model (a5), segred (a6), exchange (a7), optimizer (a8), side (a11, side stream). */
+/* per-phase device time (ms) summed over the steps since the last call (needs
+   FRUGAL_F_TIMERS; CUDA events on the phase's stream).  Phases, in order: ingest (a1+a2),
+   schedule (a9), urgent (a10), gate (a3), gather (a4, unique rows), expand (a4, per
+   position), model (a5), segred (a6), exchange (a7), optimizer (a8), side (a11, side
+   stream).  Device counters are cumulative since init (always on; one atomic per block). */
 #define FRUGAL_N_PHASES 11
+enum {
+    FRUGAL_C_POSITIONS = 0,     /* lookups (positions) of this rank                         */
+    FRUGAL_C_UNIQUE = 1,        /* distinct rows of this rank (sum over steps)               */
+    FRUGAL_C_GATHER_HOST = 2,   /* unique rows gathered from the host table (zero-copy)      */
+    FRUGAL_C_GATHER_CACHE = 3,  /* unique rows gathered from the HBM cache                   */
+    FRUGAL_C_OPT_HOT = 4,       /* owned rows updated in the cache                           */
+    FRUGAL_C_OPT_COLD = 5,      /* owned rows updated via host (w,G) -> dirty pool           */
+    FRUGAL_C_URGENT_HOT = 6,    /* rows flushed on the critical path (hot: w)                */
+    FRUGAL_C_URGENT_COLD = 7,   /* (cold: w and G)                                           */
+    FRUGAL_C_SIDE_HOT = 8,      /* rows flushed by the side stream (deferred + age-out)      */
+    FRUGAL_C_SIDE_COLD = 9,
+    FRUGAL_C_FINAL_HOT = 10,    /* rows flushed by frugal_flush                              */
+    FRUGAL_C_FINAL_COLD = 11,
+    FRUGAL_C_LONG_SEGMENTS = 12,/* unique rows with > 64 occurrences (chunked reduction)     */
+    FRUGAL_C_MAIL_OUT = 13,     /* partial rows written to this rank's host mailbox          */
+    FRUGAL_C_MAIL_IN = 14,      /* partial rows read from other ranks' mailboxes             */
+    FRUGAL_N_COUNTERS = 16
+};
 typedef struct {
     double ms[FRUGAL_N_PHASES];
-    int64_t steps;
-    int64_t kernel_launches;       /* library kernels launched since init               */
-    int64_t rows_urgent, rows_deferred, rows_ageout; /* cumulative (FRUGAL_F_RECORD)    */
-    int64_t host_read_rows;        /* cumulative rows gathered from host (RECORD)        */
+    int64_t steps;                 /* backward_update calls since the last get_stats       */
+    int64_t kernel_launches;       /* library kernels launched since init                  */
+    int64_t count[FRUGAL_N_COUNTERS];
 } frugal_stats;
 frugal_status frugal_get_stats(frugal_ctx* ctx, frugal_stats* out);
 

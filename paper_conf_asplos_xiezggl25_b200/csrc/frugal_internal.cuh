@@ -83,6 +83,7 @@ struct frugal_ctx {
     int n, g, d, F, B, L, D, M;  // world, rank, dim, slots, batch, lookahead, age_out, B*F
     int64_t N, No;               // rows, owned rows
     int P;                       // pool segments = D + 2
+    int side_blocks = 32;        // grid cap of the side-stream drain
     int64_t capT;                // max owned rows touched per step
     int key_bits, lk_bits;       // bits of global ids / local ids
 
@@ -111,13 +112,12 @@ struct frugal_ctx {
 
     // HBM cache of owned hot rows
     int64_t cap_hot = 0;
-    float* cw = nullptr;
-    float* cG = nullptr;
+    float* cw = nullptr;        // [cap_hot][d] w of the owned hot rows
+    float* Gd = nullptr;        // [No][d] Adagrad state of every owned row (HBM-resident, R8)
     int32_t* hot_lk = nullptr;  // [cap_hot] local index of each slot
 
     // dirty-row pool for cold owned rows: P segments x capT rows
-    float* pw = nullptr;
-    float* pG = nullptr;
+    float* pw = nullptr;        // [P][capT][d] w of updated cold rows until flushed
     int32_t* pkey = nullptr;   // [P][capT] local index
     int32_t* pcount = nullptr; // [P]
 
@@ -170,7 +170,7 @@ struct frugal_ctx {
     size_t ev_used = 0;
     double phase_ms[FRUGAL_N_PHASES] = {0};
     int64_t timed_steps = 0;
-    int64_t rows_urgent = 0, rows_deferred = 0, rows_ageout = 0, host_read_rows = 0;
+    unsigned long long* dstats = nullptr;  // device counters [FRUGAL_N_COUNTERS]
     // recorded schedule artefacts (FRUGAL_F_RECORD)
     std::vector<int32_t> rec_urgent, rec_deferred, rec_deferred_p, rec_ageout, rec_final;
     int rec_gate_wait = 0;
@@ -184,7 +184,7 @@ void launch_owner_side(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st);
 void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, cudaStream_t st);
 void launch_bucket(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStream_t st);
 void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begin, const int32_t* d_end,
-                       int with_hot_g, cudaStream_t st);
+                       int max_blocks, int counter, cudaStream_t st);
 void launch_gather(frugal_ctx* c, QueueSlot& q, float* out, cudaStream_t st);
 void launch_expand(frugal_ctx* c, QueueSlot& q, float* out, cudaStream_t st);
 void launch_mail_header(frugal_ctx* c, QueueSlot& q, int par, cudaStream_t st);

@@ -10,6 +10,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <algorithm>
+
 #include "frugal_internal.cuh"
 #include "kutil.cuh"
 
@@ -149,11 +151,61 @@ void sort_free(SortScratch& s) {
     s = SortScratch();
 }
 
+// exclusive scan of the [256 digits][nblk] histogram in digit-major order: one warp per
+// digit row (coalesced), digit totals scanned by warp 0, then rows offset by their base
+__global__ void k_scan_digits(int32_t* __restrict__ hist, int nblk) {
+    __shared__ int tot[256];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    for (int dg = w; dg < 256; dg += nw) {
+        int32_t* row = hist + (size_t)dg * nblk;
+        int run = 0;
+        for (int b0 = 0; b0 < nblk; b0 += 32) {
+            int i = b0 + lane;
+            int v = i < nblk ? row[i] : 0, x = v;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                int y = __shfl_up_sync(FULL, x, o);
+                if (lane >= o) x += y;
+            }
+            if (i < nblk) row[i] = run + x - v;
+            run += __shfl_sync(FULL, x, 31);
+        }
+        if (lane == 0) tot[dg] = run;
+    }
+    __syncthreads();
+    if (w == 0) {
+        int v[8], s = 0;
+#pragma unroll
+        for (int q = 0; q < 8; q++) {
+            v[q] = tot[lane * 8 + q];
+            s += v[q];
+        }
+        int x = s;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            int y = __shfl_up_sync(FULL, x, o);
+            if (lane >= o) x += y;
+        }
+        int base = x - s;
+#pragma unroll
+        for (int q = 0; q < 8; q++) {
+            tot[lane * 8 + q] = base;
+            base += v[q];
+        }
+    }
+    __syncthreads();
+    for (int dg = w; dg < 256; dg += nw) {
+        int32_t* row = hist + (size_t)dg * nblk;
+        const int base = tot[dg];
+        for (int i = lane; i < nblk; i += 32) row[i] += base;
+    }
+}
+
 int sort_pairs(SortScratch& s, const int32_t* d_n, int bits, cudaStream_t st, int64_t* launches) {
     int cur = 0;
     for (int shift = 0; shift < bits; shift += 8) {
         k_radix_hist<<<s.nblk, 256, 0, st>>>(s.k[cur], d_n, shift, s.hist, s.nblk);
-        k_scan_small<<<1, 1024, 0, st>>>(s.hist, 256 * s.nblk, nullptr);
+        k_scan_digits<<<1, 1024, 0, st>>>(s.hist, s.nblk);
         k_radix_scatter<<<s.nblk, 256, 0, st>>>(s.k[cur], s.v[cur], s.k[cur ^ 1], s.v[cur ^ 1], d_n, shift,
                                                 s.hist, s.nblk);
         *launches += 3;
@@ -218,7 +270,7 @@ __global__ void k_head_count(const uint32_t* __restrict__ ks, const int32_t* d_n
 __global__ void k_dedup_emit(const uint32_t* __restrict__ ks, const int32_t* __restrict__ vs, const int32_t* d_n,
                              const int32_t* __restrict__ part, int nblk, int32_t* __restrict__ uniq,
                              int32_t* __restrict__ off, int32_t* __restrict__ inv, int32_t* __restrict__ pos,
-                             int32_t* d_nuniq) {
+                             int32_t* d_nuniq, unsigned long long* stats) {
     __shared__ int smw[8];
     const int n = *d_n;
     int lo, hi;
@@ -243,6 +295,8 @@ __global__ void k_dedup_emit(const uint32_t* __restrict__ ks, const int32_t* __r
             if (i == n - 1) {
                 off[seg + 1] = n;
                 *d_nuniq = seg + 1;
+                atomicAdd(&stats[FRUGAL_C_POSITIONS], (unsigned long long)n);
+                atomicAdd(&stats[FRUGAL_C_UNIQUE], (unsigned long long)(seg + 1));
             }
         }
         run += tot;
@@ -267,7 +321,7 @@ void launch_dedup(frugal_ctx* c, QueueSlot& q, cudaStream_t st) {
     k_head_count<<<nb, 256, 0, st>>>(c->sort.k[r], q.m, c->scan.part, nb);
     k_scan_small<<<1, 1024, 0, st>>>(c->scan.part, nb, nullptr);
     k_dedup_emit<<<nb, 256, 0, st>>>(c->sort.k[r], c->sort.v[r], q.m, c->scan.part, nb, q.uniq, q.off,
-                                     q.inv, q.pos, q.n_uniq);
+                                     q.inv, q.pos, q.n_uniq, c->dstats);
     c->launches += 3;
 }
 
@@ -618,51 +672,50 @@ void launch_bucket(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStrea
 }
 
 // ============================================================================ row movers
-// a10/a11/a12: flush rows (local ids) to the host table.  hot: w (and G if with_hot_g)
-// from the HBM cache; cold: w and G from the dirty pool.  Zero-copy stores to host.
+// a10/a11/a12: flush rows (local ids) to the host table: w of hot rows from the HBM
+// cache, w of cold rows from the dirty pool.  Zero-copy stores to host memory.  (The
+// owner's Adagrad state G never leaves HBM during training -- no other rank reads it;
+// frugal_flush writes it back once, reading R8.)
 template <int GS>
 __global__ void k_flush_rows(const int32_t* __restrict__ rows, const int32_t* d_begin, const int32_t* d_end,
-                             int world, int g, int d4, int with_hot_g, int adagrad,
-                             const int32_t* __restrict__ slot, const int32_t* __restrict__ last_upd,
-                             const int32_t* __restrict__ pool_idx, int P, int64_t capT,
-                             const float4* __restrict__ cw, const float4* __restrict__ cG,
-                             const float4* __restrict__ pw, const float4* __restrict__ pG, float4* hw, float4* hG) {
+                             int world, int g, int d4, const int32_t* __restrict__ slot,
+                             const int32_t* __restrict__ last_upd, const int32_t* __restrict__ pool_idx, int P,
+                             int64_t capT, const float4* __restrict__ cw, const float4* __restrict__ pw, float4* hw,
+                             unsigned long long* stats) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
     const int b = d_begin ? *d_begin : 0, e = *d_end;
+    unsigned nh = 0, nc = 0;
     for (int64_t a = b + gid; a < e; a += gs) {
         int32_t lk = rows[a];
         int64_t k = (int64_t)lk * world + g;
         int sl = slot[lk];
+        const float4* src;
         if (sl >= 0) {
-            const float4* sw = cw + (int64_t)sl * d4;
-            for (int v = l; v < d4; v += GS) hw[k * d4 + v] = sw[v];
-            if (with_hot_g && adagrad) {
-                const float4* sg = cG + (int64_t)sl * d4;
-                for (int v = l; v < d4; v += GS) hG[k * d4 + v] = sg[v];
-            }
+            src = cw + (int64_t)sl * d4;
+            nh += (l == 0);
         } else {
-            int64_t pr = (int64_t)(last_upd[lk] % P) * capT + pool_idx[lk];
-            const float4* sw = pw + pr * d4;
-            for (int v = l; v < d4; v += GS) hw[k * d4 + v] = sw[v];
-            if (adagrad) {
-                const float4* sg = pG + pr * d4;
-                for (int v = l; v < d4; v += GS) hG[k * d4 + v] = sg[v];
-            }
+            src = pw + ((int64_t)(last_upd[lk] % P) * capT + pool_idx[lk]) * d4;
+            nc += (l == 0);
         }
+        for (int v = l; v < d4; v += GS) hw[k * d4 + v] = src[v];
     }
     __threadfence_system();
+    if (stats) {
+        block_count(stats, nh);
+        block_count(stats + 1, nc);
+    }
 }
 
 void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begin, const int32_t* d_end,
-                       int with_hot_g, cudaStream_t st) {
+                       int max_blocks, int counter, cudaStream_t st) {
     const int d4 = c->d / 4, gs = group_size(d4);
-    int grid = grid_for(c->capT * (int64_t)gs, 256, 4);
+    int grid = std::min(grid_for(c->capT * (int64_t)gs, 256, 4), max_blocks);
     DISPATCH_GS(gs, (k_flush_rows<GS><<<grid, 256, 0, st>>>(
-                        rows, d_begin, d_end, c->n, c->g, d4, with_hot_g, c->cfg.opt == FRUGAL_ADAGRAD, c->slot,
-                        c->last_upd, c->pool_idx, c->P, c->capT, (const float4*)c->cw, (const float4*)c->cG,
-                        (const float4*)c->pw, (const float4*)c->pG, (float4*)c->dh_w, (float4*)c->dh_G)));
+                        rows, d_begin, d_end, c->n, c->g, d4, c->slot, c->last_upd, c->pool_idx, c->P, c->capT,
+                        (const float4*)c->cw, (const float4*)c->pw, (float4*)c->dh_w,
+                        counter >= 0 ? c->dstats + counter : nullptr)));
     c->launches++;
 }
 
@@ -670,20 +723,31 @@ void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begi
 template <int GS>
 __global__ void k_gather_uniq(const int32_t* __restrict__ uniq, const int32_t* d_nu, int world, int g, int d4,
                               const int32_t* __restrict__ slot, const float4* __restrict__ cw,
-                              const float4* hw, float4* __restrict__ rows) {
+                              const float4* hw, float4* __restrict__ rows, unsigned long long* stats) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
     const int n = *d_nu;
+    unsigned nh = 0, nc = 0;
     for (int64_t u = gid; u < n; u += gs) {
         int32_t k = uniq[u];
         const float4* src = hw + (int64_t)k * d4;
+        bool cached = false;
         if (k % world == g) {
             int sl = slot[k / world];
-            if (sl >= 0) src = cw + (int64_t)sl * d4;
+            if (sl >= 0) {
+                src = cw + (int64_t)sl * d4;
+                cached = true;
+            }
+        }
+        if (l == 0) {
+            if (cached) nc++;
+            else nh++;
         }
         for (int v = l; v < d4; v += GS) rows[u * d4 + v] = src[v];
     }
+    block_count(stats + FRUGAL_C_GATHER_HOST, nh);
+    block_count(stats + FRUGAL_C_GATHER_CACHE, nc);
 }
 // a4 expand: out[i] = rows[inv[i]]
 template <int GS>
@@ -704,7 +768,7 @@ void launch_gather(frugal_ctx* c, QueueSlot& q, float* out, cudaStream_t st) {
     int grid = grid_for((int64_t)c->M * gs, 256, 8);
     DISPATCH_GS(gs, (k_gather_uniq<GS><<<grid, 256, 0, st>>>(q.uniq, q.n_uniq, c->n, c->g, d4, c->slot,
                                                              (const float4*)c->cw, (const float4*)c->dh_w,
-                                                             (float4*)c->rows)));
+                                                             (float4*)c->rows, c->dstats)));
     c->launches++;
 }
 void launch_expand(frugal_ctx* c, QueueSlot& q, float* out, cudaStream_t st) {

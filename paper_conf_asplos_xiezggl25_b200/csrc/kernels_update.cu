@@ -29,12 +29,19 @@ __device__ __forceinline__ float4 chunk_sum(const float4* __restrict__ grad, con
                                             int e, int d4, int v) {
     float4 acc = grad[(int64_t)pos[b] * d4 + v];
     int j = b + 1;
-    for (; j + 8 <= e; j += 8) {  // 8 loads in flight, adds in position order
-        float4 x[8];
+    for (; j + 16 <= e; j += 16) {  // 16 loads in flight, adds in position order
+        float4 x[16];
 #pragma unroll
-        for (int q = 0; q < 8; q++) x[q] = grad[(int64_t)pos[j + q] * d4 + v];
+        for (int q = 0; q < 16; q++) x[q] = grad[(int64_t)pos[j + q] * d4 + v];
 #pragma unroll
-        for (int q = 0; q < 8; q++) acc = add4(acc, x[q]);
+        for (int q = 0; q < 16; q++) acc = add4(acc, x[q]);
+    }
+    for (; j + 4 <= e; j += 4) {
+        float4 x[4];
+#pragma unroll
+        for (int q = 0; q < 4; q++) x[q] = grad[(int64_t)pos[j + q] * d4 + v];
+#pragma unroll
+        for (int q = 0; q < 4; q++) acc = add4(acc, x[q]);
     }
     for (; j < e; j++) acc = add4(acc, grad[(int64_t)pos[j] * d4 + v]);
     return acc;
@@ -44,7 +51,7 @@ template <int GS>
 __global__ void k_segreduce(const int32_t* __restrict__ off, const int32_t* __restrict__ pos,
                             const int32_t* d_nu, const int32_t* __restrict__ gl, const int32_t* __restrict__ goff,
                             int g, int d4, const float4* __restrict__ grad, float4* __restrict__ Pp, float4* mail,
-                            int32_t* long_q, int32_t* long_cnt) {
+                            int32_t* long_q, int32_t* long_cnt, unsigned long long* stats) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
@@ -54,17 +61,24 @@ __global__ void k_segreduce(const int32_t* __restrict__ off, const int32_t* __re
         own_lo = goff[g];
         own_hi = goff[g + 1];
     }
+    unsigned nlong = 0, nout = 0;
     for (int64_t q = gid; q < n; q += gs) {
         const int u = gl ? gl[q] : (int)q;
         const int b = off[u], e = off[u + 1];
+        if (l == 0 && (q < own_lo || q >= own_hi)) nout++;
         if (e - b > kChunk) {
-            if (l == 0) long_q[atomicAdd(long_cnt, 1)] = (int32_t)q;
+            if (l == 0) {
+                long_q[atomicAdd(long_cnt, 1)] = (int32_t)q;
+                nlong++;
+            }
             continue;
         }
         float4* dst = (q >= own_lo && q < own_hi) ? (Pp + q * d4) : (mail + q * d4);
         for (int v = l; v < d4; v += GS) dst[v] = chunk_sum<GS>(grad, pos, b, e, d4, v);
     }
     if (gl) __threadfence_system();
+    block_count(stats + FRUGAL_C_LONG_SEGMENTS, nlong);
+    block_count(stats + FRUGAL_C_MAIL_OUT, nout);
 }
 
 // one block per long segment: row groups compute chunk sums into scratch (indexed by
@@ -96,7 +110,15 @@ __global__ void k_segreduce_long(const int32_t* __restrict__ off, const int32_t*
             float4* dst = (q >= own_lo && q < own_hi) ? (Pp + (int64_t)q * d4) : (mail + (int64_t)q * d4);
             for (int v = l; v < d4; v += GS) {
                 float4 acc = scratch[(int64_t)b * d4 + v];
-                for (int c = 1; c < nch; c++) acc = add4(acc, scratch[(int64_t)(b + c * kChunk) * d4 + v]);
+                int c = 1;
+                for (; c + 8 <= nch; c += 8) {  // chunk sums in order, 8 loads in flight
+                    float4 x[8];
+#pragma unroll
+                    for (int q2 = 0; q2 < 8; q2++) x[q2] = scratch[(int64_t)(b + (c + q2) * kChunk) * d4 + v];
+#pragma unroll
+                    for (int q2 = 0; q2 < 8; q2++) acc = add4(acc, x[q2]);
+                }
+                for (; c < nch; c++) acc = add4(acc, scratch[(int64_t)(b + c * kChunk) * d4 + v]);
                 dst[v] = acc;
             }
         }
@@ -113,9 +135,9 @@ void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, c
     cudaMemsetAsync(c->long_cnt, 0, 4, st);
     DISPATCH_GS(gs, (k_segreduce<GS><<<grid, 256, 0, st>>>(q.off, q.pos, q.n_uniq, multi ? q.gl : nullptr, q.goff,
                                                            c->g, d4, (const float4*)grad, (float4*)c->Pp, mail,
-                                                           c->long_q, c->long_cnt)));
-    int lgrid = (int)std::min<int64_t>(c->M / (kChunk + 1) + 1, kSMs * 4);
-    DISPATCH_GS(gs, (k_segreduce_long<GS><<<lgrid, 256, 0, st>>>(q.off, q.pos, multi ? q.gl : nullptr, q.goff, c->g,
+                                                           c->long_q, c->long_cnt, c->dstats)));
+    int lgrid = (int)std::min<int64_t>(c->M / (kChunk + 1) + 1, kSMs * 2);
+    DISPATCH_GS(gs, (k_segreduce_long<GS><<<lgrid, 1024, 0, st>>>(q.off, q.pos, multi ? q.gl : nullptr, q.goff, c->g,
                                                                  d4, (const float4*)grad, (float4*)c->Pp, mail,
                                                                  c->long_q, c->long_cnt,
                                                                  (float4*)c->chunk_scratch)));
@@ -146,13 +168,14 @@ __global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, 
                             const int32_t* __restrict__ goff_own, const char* mail_par, size_t mail_stride,
                             const float4* __restrict__ rows_w, const int32_t* __restrict__ slot,
                             int32_t* __restrict__ state, int32_t* __restrict__ last_upd, int32_t* __restrict__ pool_idx,
-                            uint64_t* __restrict__ rbits, float4* __restrict__ cw, float4* __restrict__ cG,
-                            float4* __restrict__ pw, float4* __restrict__ pG, int32_t* __restrict__ pkey,
-                            int32_t* pcount, const float4* hw, const float4* hG) {
+                            uint64_t* __restrict__ rbits, float4* __restrict__ cw, float4* __restrict__ Gd,
+                            float4* __restrict__ pw, int32_t* __restrict__ pkey, int32_t* pcount, const float4* hw,
+                            unsigned long long* stats) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
     const int n = *d_nT;
+    unsigned nhot = 0, ncold = 0, nin = 0;
     const uint64_t clear = ~((1ull << (s & 31)) | (1ull << (32 + (s & 31))));
     for (int64_t j = gid; j < n; j += gs) {
         const int32_t lk = T[j];
@@ -182,13 +205,9 @@ __global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, 
                 }
             }
             float4 w, G = make_float4(0.f, 0.f, 0.f, 0.f);
-            if (sl >= 0) {
-                w = cw[(int64_t)sl * d4 + v];
-                if (adagrad) G = cG[(int64_t)sl * d4 + v];
-            } else {
-                w = rows_w ? rows_w[j * d4 + v] : hw[k * d4 + v];
-                if (adagrad) G = hG[k * d4 + v];
-            }
+            if (sl >= 0) w = cw[(int64_t)sl * d4 + v];
+            else w = rows_w ? rows_w[j * d4 + v] : hw[k * d4 + v];
+            if (adagrad) G = Gd[(int64_t)lk * d4 + v];
             float* wp = &w.x;
             float* Gp = &G.x;
             const float* gp = &acc.x;
@@ -203,15 +222,14 @@ __global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, 
                     wp[c] = __fsub_rn(wp[c], __fmul_rn(lr, gp[c]));
                 }
             }
-            if (sl >= 0) {
-                cw[(int64_t)sl * d4 + v] = w;
-                if (adagrad) cG[(int64_t)sl * d4 + v] = G;
-            } else {
-                pw[j * d4 + v] = w;
-                if (adagrad) pG[j * d4 + v] = G;
-            }
+            if (sl >= 0) cw[(int64_t)sl * d4 + v] = w;
+            else pw[j * d4 + v] = w;
+            if (adagrad) Gd[(int64_t)lk * d4 + v] = G;
         }
         if (l == 0) {
+            if (sl >= 0) nhot++;
+            else ncold++;
+            nin += __popc(mask & ~(1u << g));
             state[lk] = ST_UPDATED;
             last_upd[lk] = s;
             rbits[lk] &= clear;
@@ -220,6 +238,9 @@ __global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, 
         }
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) *pcount = n;
+    block_count(stats + FRUGAL_C_OPT_HOT, nhot);
+    block_count(stats + FRUGAL_C_OPT_COLD, ncold);
+    block_count(stats + FRUGAL_C_MAIL_IN, world > 1 ? nin : 0u);
 }
 
 void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, cudaStream_t st) {
@@ -228,6 +249,7 @@ void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, cudaStrea
     const int seg = (int)(s % c->P);
     const size_t pofs = (size_t)seg * c->capT * d4;
     const bool adag = c->cfg.opt == FRUGAL_ADAGRAD;
+    (void)adag;
     const char* mail_par = c->n > 1 ? c->dh_mail + (size_t)par * c->n * c->mail_stride : nullptr;
     // world == 1: the owner gathered every touched row itself this step (T == uniq),
     // so the cold rows' w is taken from the staging rows instead of a second host read.
@@ -235,10 +257,8 @@ void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, cudaStrea
     DISPATCH_GS(gs, (k_optimizer<GS><<<grid, 256, 0, st>>>(
                         q.T, q.nT, q.Tmask, q.Tidx, c->capT, c->n, c->g, d4, (int32_t)s, adag, c->cfg.lr, c->cfg.eps,
                         (const float4*)c->Pp, q.goff, mail_par, c->mail_stride, rows_w, c->slot, c->state,
-                        c->last_upd, c->pool_idx, c->rbits, (float4*)c->cw, (float4*)c->cG,
-                        (float4*)c->pw + pofs, adag ? (float4*)c->pG + pofs : nullptr,
-                        c->pkey + (size_t)seg * c->capT, c->pcount + seg, (const float4*)c->dh_w,
-                        (const float4*)c->dh_G)));
+                        c->last_upd, c->pool_idx, c->rbits, (float4*)c->cw, (float4*)c->Gd, (float4*)c->pw + pofs,
+                        c->pkey + (size_t)seg * c->capT, c->pcount + seg, (const float4*)c->dh_w, c->dstats)));
     c->launches++;
 }
 
@@ -257,15 +277,15 @@ __global__ void k_final_collect(int64_t No, int32_t* __restrict__ state, int32_t
         }
     }
 }
+// G of every owned row (HBM) to the host table, once, at the end of training
 template <int GS>
-__global__ void k_hot_g_push(const int32_t* __restrict__ hot_lk, int64_t cap_hot, int world, int g, int d4,
-                             const float4* __restrict__ cG, float4* hG) {
+__global__ void k_g_push(int64_t No, int world, int g, int d4, const float4* __restrict__ Gd, float4* hG) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
-    for (int64_t sl = gid; sl < cap_hot; sl += gs) {
-        int64_t k = (int64_t)hot_lk[sl] * world + g;
-        for (int v = l; v < d4; v += GS) hG[k * d4 + v] = cG[sl * d4 + v];
+    for (int64_t lk = gid; lk < No; lk += gs) {
+        int64_t k = lk * world + g;
+        for (int v = l; v < d4; v += GS) hG[k * d4 + v] = Gd[lk * d4 + v];
     }
     __threadfence_system();
 }
@@ -274,12 +294,12 @@ void launch_final_flush(frugal_ctx* c, cudaStream_t st) {
     cudaMemsetAsync(c->ff_cnt, 0, sizeof(int32_t), st);
     k_final_collect<<<grid_for(c->No, 256, 8), 256, 0, st>>>(c->No, c->state, c->ff_rows, c->ff_cnt);
     c->launches++;
-    launch_flush_rows(c, c->ff_rows, nullptr, c->ff_cnt, 1, st);
-    if (c->cfg.opt == FRUGAL_ADAGRAD && c->cap_hot > 0) {
+    launch_flush_rows(c, c->ff_rows, nullptr, c->ff_cnt, 1 << 30, FRUGAL_C_FINAL_HOT, st);
+    if (c->cfg.opt == FRUGAL_ADAGRAD && c->No > 0) {
         const int d4 = c->d / 4, gs = group_size(d4);
-        int grid = grid_for(c->cap_hot * gs, 256, 8);
-        DISPATCH_GS(gs, (k_hot_g_push<GS><<<grid, 256, 0, st>>>(c->hot_lk, c->cap_hot, c->n, c->g, d4,
-                                                                (const float4*)c->cG, (float4*)c->dh_G)));
+        int grid = grid_for(c->No * gs, 256, 8);
+        DISPATCH_GS(gs, (k_g_push<GS><<<grid, 256, 0, st>>>(c->No, c->n, c->g, d4, (const float4*)c->Gd,
+                                                            (float4*)c->dh_G)));
         c->launches++;
     }
 }
@@ -316,6 +336,9 @@ void launch_init_table(frugal_ctx* c, cudaStream_t st) {
     c->launches++;
 }
 
+__global__ void k_fill(float* a, int64_t n, float v) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) a[i] = v;
+}
 __global__ void k_init_meta(int64_t No, int32_t* slot, int32_t* state, int32_t* last_upd, int32_t* pool_idx,
                             uint64_t* rbits) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < No; i += (int64_t)gridDim.x * blockDim.x) {
@@ -328,14 +351,13 @@ __global__ void k_init_meta(int64_t No, int32_t* slot, int32_t* state, int32_t* 
 }
 // hot slots: d_hot_lk sorted owned local ids; cache rows start at w0 (same pure function)
 __global__ void k_init_hot(const int32_t* __restrict__ hot_lk, int64_t cap_hot, int world, int g, int d,
-                           uint64_t seed, float scale, float accum, int32_t* slot, float* cw, float* cG) {
+                           uint64_t seed, float scale, int32_t* slot, float* cw) {
     for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < cap_hot * d;
          e += (int64_t)gridDim.x * blockDim.x) {
         int64_t sl = e / d;
         int j = (int)(e - sl * d);
         int64_t k = (int64_t)hot_lk[sl] * world + g;
         cw[e] = w0(seed, k, d, j, scale);
-        if (cG) cG[e] = accum;
         if (j == 0) slot[hot_lk[sl]] = (int32_t)sl;
     }
 }
@@ -347,8 +369,11 @@ void launch_init_meta(frugal_ctx* c, const int64_t* unused, int64_t n_hot, cudaS
     c->launches++;
     if (c->cap_hot > 0) {
         k_init_hot<<<grid_for(c->cap_hot * c->d, 256, 8), 256, 0, st>>>(
-            c->hot_lk, c->cap_hot, c->n, c->g, c->d, c->cfg.init_seed, c->cfg.init_scale, c->cfg.init_accum,
-            c->slot, c->cw, c->cfg.opt == FRUGAL_ADAGRAD ? c->cG : nullptr);
+            c->hot_lk, c->cap_hot, c->n, c->g, c->d, c->cfg.init_seed, c->cfg.init_scale, c->slot, c->cw);
+        c->launches++;
+    }
+    if (c->cfg.opt == FRUGAL_ADAGRAD) {
+        k_fill<<<grid_for(c->No * c->d, 256, 8), 256, 0, st>>>(c->Gd, c->No * c->d, c->cfg.init_accum);
         c->launches++;
     }
 }
@@ -394,26 +419,24 @@ void launch_wait_flags(frugal_ctx* c, int which, uint32_t value, cudaStream_t st
 // authoritative value of owned rows: hot -> cache; cold & dirty -> pool; else host
 __global__ void k_read_rows(const int32_t* __restrict__ lks, int64_t n, int world, int g, int d, int P, int64_t capT,
                             const int32_t* slot, const int32_t* state, const int32_t* last_upd,
-                            const int32_t* pool_idx, const float* cw, const float* cG, const float* pw,
-                            const float* pG, const float* hw, const float* hG, float* ow, float* oG) {
+                            const int32_t* pool_idx, const float* cw, const float* Gd, const float* pw,
+                            const float* hw, float* ow, float* oG) {
     for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < n * d; e += (int64_t)gridDim.x * blockDim.x) {
         int64_t a = e / d;
         int j = (int)(e - a * d);
         int32_t lk = lks[a];
         int64_t k = (int64_t)lk * world + g;
         int sl = slot[lk];
-        float w, G = 0.f;
+        float w;
         if (sl >= 0) {
             w = cw[(int64_t)sl * d + j];
-            G = cG ? cG[(int64_t)sl * d + j] : 0.f;
         } else if (state[lk] == ST_UPDATED || state[lk] == ST_INF) {
             int64_t pr = (int64_t)(last_upd[lk] % P) * capT + pool_idx[lk];
             w = pw[pr * d + j];
-            G = pG ? pG[pr * d + j] : 0.f;
         } else {
             w = hw[k * d + j];
-            G = hG ? hG[k * d + j] : 0.f;
         }
+        float G = Gd ? Gd[(int64_t)lk * d + j] : 0.f;
         ow[e] = w;
         oG[e] = G;
     }
@@ -422,8 +445,7 @@ void launch_read_rows(frugal_ctx* c, const int32_t* d_lk, int64_t n, float* d_w,
     const bool ad = c->cfg.opt == FRUGAL_ADAGRAD;
     k_read_rows<<<grid_for(n * c->d, 256, 8), 256, 0, st>>>(d_lk, n, c->n, c->g, c->d, c->P, c->capT, c->slot,
                                                              c->state, c->last_upd, c->pool_idx, c->cw,
-                                                             ad ? c->cG : nullptr, c->pw, ad ? c->pG : nullptr,
-                                                             c->dh_w, ad ? c->dh_G : nullptr, d_w, d_G);
+                                                             ad ? c->Gd : nullptr, c->pw, c->dh_w, d_w, d_G);
     c->launches++;
 }
 __global__ void k_read_host(const int64_t* __restrict__ ks, int64_t n, int d, const float* hw, const float* hG,

@@ -42,6 +42,17 @@ struct RowGroup {
     }
 };
 
+// block-aggregated counter: every thread passes its count, one atomic per block
+__device__ __forceinline__ void block_count(unsigned long long* dst, unsigned v) {
+    __shared__ unsigned s_cnt;
+    if (threadIdx.x == 0) s_cnt = 0;
+    __syncthreads();
+    for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if ((threadIdx.x & 31) == 0 && v) atomicAdd(&s_cnt, v);
+    __syncthreads();
+    if (threadIdx.x == 0 && s_cnt) atomicAdd(dst, (unsigned long long)s_cnt);
+}
+
 static inline int group_size(int d4) {
     int gs = 1;
     while (gs < d4 && gs < 32) gs <<= 1;

@@ -16,6 +16,7 @@
 #include <sys/stat.h>
 #include <time.h>
 #include <unistd.h>
+#include <stdlib.h>
 
 #include <algorithm>
 #include <string>
@@ -132,14 +133,14 @@ static void free_ctx(frugal_ctx* c) {
         if (p) cudaFree(p);
     };
     F(c->slot); F(c->state); F(c->last_upd); F(c->pool_idx); F(c->rbits);
-    F(c->cw); F(c->cG); F(c->hot_lk); F(c->pw); F(c->pG); F(c->pkey); F(c->pcount);
+    F(c->cw); F(c->Gd); F(c->hot_lk); F(c->pw); F(c->pkey); F(c->pcount);
     for (auto& q : c->q) {
         F(q.ids); F(q.counts); F(q.m); F(q.uniq); F(q.inv); F(q.off); F(q.pos); F(q.n_uniq);
         if (c->n > 1) { F(q.T); F(q.Tmask); F(q.Tidx); F(q.nT); F(q.gl); F(q.goff); }
     }
     F(c->rows); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->owned_cnt); F(c->nb_rows); F(c->nb_p); F(c->nb_cnt);
     for (int i = 0; i < 2; i++) { F(c->bk_rows[i]); F(c->bk_p[i]); F(c->bk_off[i]); F(c->age_rows[i]); F(c->age_cnt[i]); }
-    F(c->sched_info); F(c->ff_rows); F(c->ff_cnt); F(c->ids_stage);
+    F(c->dstats); F(c->sched_info); F(c->ff_rows); F(c->ff_cnt); F(c->ids_stage);
     if (c->herr) cudaFreeHost(c->herr);
     if (c->counts_pin) cudaFreeHost(c->counts_pin);
     for (auto e : c->ev_counts) cudaEventDestroy(e);
@@ -198,6 +199,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->L = k.lookahead; c->D = k.age_out; c->M = k.batch * k.slots; c->N = k.n_rows;
     c->No = c->g < c->N ? (c->N - c->g + c->n - 1) / c->n : 0;
     c->P = c->D + 2;
+    c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 32;
     c->capT = std::max<int64_t>(1, std::min<int64_t>((int64_t)c->n * c->M, c->No));
     c->key_bits = bits_for(c->N - 1);
     c->lk_bits = bits_for(std::max<int64_t>(c->No - 1, 0));
@@ -295,9 +297,8 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->cap_hot = (int64_t)hot.size();
     DMALLOC(c->hot_lk, c->cap_hot * 4);
     DMALLOC(c->cw, c->cap_hot * rowb);
-    if (adag) DMALLOC(c->cG, c->cap_hot * rowb);
+    if (adag) DMALLOC(c->Gd, (size_t)c->No * rowb);
     DMALLOC(c->pw, (size_t)c->P * c->capT * rowb);
-    if (adag) DMALLOC(c->pG, (size_t)c->P * c->capT * rowb);
     DMALLOC(c->pkey, (size_t)c->P * c->capT * 4);
     DMALLOC(c->pcount, (size_t)c->P * 4);
     c->q.resize(c->L + 1);
@@ -343,6 +344,8 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     DMALLOC(c->ff_rows, std::max<int64_t>(c->No, 1) * 4);
     DMALLOC(c->ff_cnt, 4);
     DMALLOC(c->ids_stage, (size_t)c->n * c->M * 8);
+    DMALLOC(c->dstats, FRUGAL_N_COUNTERS * 8);
+    cudaMemset(c->dstats, 0, FRUGAL_N_COUNTERS * 8);
     sort_alloc(c->sort, (int64_t)c->n * c->M);
     scan_alloc(c->scan, (int64_t)c->n * c->M);
     if (!c->sort.hist || !c->scan.part) {
@@ -471,9 +474,6 @@ static void record_schedule(frugal_ctx* c, int par, cudaStream_t st) {
     c->rec_deferred_p.assign(ps.begin() + off[1], ps.end());
     c->rec_ageout = age;
     c->rec_gate_wait = off[1] > 0;
-    c->rows_urgent += off[1];
-    c->rows_deferred += off[c->L] - off[1];
-    c->rows_ageout += nage;
 }
 
 extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* ids_next_all, const int32_t* counts_next,
@@ -518,7 +518,7 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
     {
         // a10: urgent bucket (priority == s) to the host table on the critical path
         Timer tm(c, PH_URGENT, st);
-        launch_flush_rows(c, c->bk_rows[par], c->bk_off[par], c->bk_off[par] + 1, 0, st);
+        launch_flush_rows(c, c->bk_rows[par], c->bk_off[par], c->bk_off[par] + 1, 1 << 30, FRUGAL_C_URGENT_HOT, st);
         if (c->n > 1) launch_set_flag(c, FLAG_URGENT, (uint32_t)(s + 1), st);
         CKL();
     }
@@ -527,8 +527,10 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
     CK(cudaStreamWaitEvent(c->side, c->ev_sched, 0));
     {
         Timer tm(c, PH_SIDE, c->side);
-        launch_flush_rows(c, c->bk_rows[par], c->bk_off[par] + 1, c->bk_off[par] + c->L, 0, c->side);
-        launch_flush_rows(c, c->age_rows[par], nullptr, c->age_cnt[par], 0, c->side);
+        // bounded grid: the drain trickles over the step instead of crowding out the main stream
+        launch_flush_rows(c, c->bk_rows[par], c->bk_off[par] + 1, c->bk_off[par] + c->L, c->side_blocks,
+                          FRUGAL_C_SIDE_HOT, c->side);
+        launch_flush_rows(c, c->age_rows[par], nullptr, c->age_cnt[par], c->side_blocks, FRUGAL_C_SIDE_HOT, c->side);
         if (c->n > 1) launch_set_flag(c, FLAG_SIDE, (uint32_t)(s + 1), c->side);
         CKL();
     }
@@ -745,10 +747,9 @@ extern "C" frugal_status frugal_get_stats(frugal_ctx* c, frugal_stats* out) {
     for (int i = 0; i < FRUGAL_N_PHASES; i++) out->ms[i] = c->phase_ms[i];
     out->steps = c->timed_steps;
     out->kernel_launches = c->launches;
-    out->rows_urgent = c->rows_urgent;
-    out->rows_deferred = c->rows_deferred;
-    out->rows_ageout = c->rows_ageout;
-    out->host_read_rows = c->host_read_rows;
+    unsigned long long cnt[FRUGAL_N_COUNTERS];
+    CK(cudaMemcpy(cnt, c->dstats, sizeof cnt, cudaMemcpyDeviceToHost));
+    for (int i = 0; i < FRUGAL_N_COUNTERS; i++) out->count[i] = (int64_t)cnt[i];
     for (int i = 0; i < FRUGAL_N_PHASES; i++) c->phase_ms[i] = 0;
     c->timed_steps = 0;
     return FRUGAL_OK;

@@ -45,10 +45,14 @@ class ScheduleInfo(C.Structure):
                 ("gate_wait", C.c_int32)]
 
 
+COUNTERS = ["positions", "unique", "gather_host", "gather_cache", "opt_hot", "opt_cold", "urgent_hot",
+            "urgent_cold", "side_hot", "side_cold", "final_hot", "final_cold", "long_segments", "mail_out",
+            "mail_in", "reserved"]
+
+
 class Stats(C.Structure):
     _fields_ = [("ms", C.c_double * 11), ("steps", C.c_int64), ("kernel_launches", C.c_int64),
-                ("rows_urgent", C.c_int64), ("rows_deferred", C.c_int64), ("rows_ageout", C.c_int64),
-                ("host_read_rows", C.c_int64)]
+                ("count", C.c_int64 * 16)]
 
 
 _lib = None
@@ -231,8 +235,7 @@ class Frugal:
         s = Stats()
         _check(lib().frugal_get_stats(self.h, C.byref(s)))
         return dict(ms={p: s.ms[i] for i, p in enumerate(PHASES)}, steps=s.steps,
-                    kernel_launches=s.kernel_launches, rows_urgent=s.rows_urgent, rows_deferred=s.rows_deferred,
-                    rows_ageout=s.rows_ageout)
+                    kernel_launches=s.kernel_launches, count={n: s.count[i] for i, n in enumerate(COUNTERS)})
 
     @property
     def owned_rows(self):

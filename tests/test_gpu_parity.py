@@ -60,7 +60,7 @@ def run_parity(st, *, flags=None, mode=None, hot=None, check_dedup=True, check_s
             ref = o.schedule()
             assert sorted(got["urgent"].tolist()) == ref["urgent"].tolist(), f"urgent set differs at {s}"
             assert sorted(zip(got["deferred"].tolist(), got["deferred_p"].tolist())) == \
-                list(zip(ref["deferred"].tolist(), ref["deferred_p"].tolist())), f"deferred set differs at {s}"
+                sorted(zip(ref["deferred"].tolist(), ref["deferred_p"].tolist())), f"deferred set differs at {s}"
             assert sorted(got["ageout"].tolist()) == ref["ageout"].tolist(), f"age-out set differs at {s}"
             assert got["gate_wait"] == ref["gate_wait"]
             gate_waits += ref["gate_wait"]
