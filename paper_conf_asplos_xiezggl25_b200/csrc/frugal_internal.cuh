@@ -84,6 +84,7 @@ struct frugal_ctx {
     int64_t N, No;               // rows, owned rows
     int P;                       // pool segments = D + 2
     int side_blocks = 32;        // grid cap of the side-stream drain
+    bool side_inline = false;    // experiment: drain on the caller stream
     int64_t capT;                // max owned rows touched per step
     int key_bits, lk_bits;       // bits of global ids / local ids
 
@@ -129,7 +130,8 @@ struct frugal_ctx {
     float* Pp = nullptr;    // [M][d] partials (grouped order for world > 1)
     float* chunk_scratch = nullptr;  // [M][d] chunk sums of long segments
     int32_t* long_q = nullptr;       // [M] long segments of the current step
-    int32_t* long_cnt = nullptr;
+    int32_t* long_cnt = nullptr;     // [2]: long segments, chunk tasks
+    int2* long_tasks = nullptr;      // [M/32 + 2] chunk [begin, end) positions
     int32_t* owned_cnt = nullptr;  // scalar
     // schedule lists (double buffered by step parity)
     int32_t* nb_rows = nullptr;  // newly bucketed rows [capT + capT]

@@ -77,50 +77,86 @@ __global__ void k_scan_small(int32_t* a, int len, int32_t* total) {
 }
 
 // ============================================================================ radix sort
+// Stable LSD radix sort, 9-bit digits (3 passes for the 26-bit ids of Criteo-Kaggle).
+// Per pass: k_radix_hist (per-block digit counts, digit-major), k_radix_scan_rows (one
+// block per digit: exclusive scan over blocks + digit total), k_radix_scatter (each block
+// derives the digit bases from the totals, then ranks its tiles stably with
+// __match_any_sync and scatters).  All counts are device-resident.
+constexpr int kRadixBits = 9;
+constexpr int kDigits = 1 << kRadixBits;
+
 __global__ void k_radix_hist(const uint32_t* __restrict__ keys, const int32_t* d_n, int shift,
                              int32_t* hist, int nblk) {
-    __shared__ int h[256];
-    h[threadIdx.x] = 0;
+    __shared__ int h[kDigits];
+    for (int i = threadIdx.x; i < kDigits; i += blockDim.x) h[i] = 0;
     __syncthreads();
     int lo, hi;
     chunk_range(*d_n, nblk, blockIdx.x, lo, hi);
-    for (int i = lo + threadIdx.x; i < hi; i += blockDim.x) atomicAdd(&h[(keys[i] >> shift) & 255], 1);
+    for (int i = lo + threadIdx.x; i < hi; i += blockDim.x) atomicAdd(&h[(keys[i] >> shift) & (kDigits - 1)], 1);
     __syncthreads();
-    hist[threadIdx.x * nblk + blockIdx.x] = h[threadIdx.x];
+    for (int i = threadIdx.x; i < kDigits; i += blockDim.x) hist[(size_t)i * nblk + blockIdx.x] = h[i];
 }
 
-__global__ void k_radix_scatter(const uint32_t* __restrict__ kin, const int32_t* __restrict__ vin,
+// block dg: exclusive scan of hist[dg][0..nblk) in place, total -> tot[dg]
+__global__ void k_radix_scan_rows(int32_t* __restrict__ hist, int nblk, int32_t* __restrict__ tot) {
+    __shared__ int smw[8];
+    int32_t* row = hist + (size_t)blockIdx.x * nblk;
+    int run = 0;
+    for (int b0 = 0; b0 < nblk; b0 += blockDim.x) {
+        int i = b0 + threadIdx.x;
+        int v = i < nblk ? row[i] : 0;
+        int t;
+        int ex = block_excl_scan(v, smw, &t);
+        if (i < nblk) row[i] = run + ex;
+        run += t;
+    }
+    if (threadIdx.x == 0) tot[blockIdx.x] = run;
+}
+
+__global__ void __launch_bounds__(256) k_radix_scatter(const uint32_t* __restrict__ kin, const int32_t* __restrict__ vin,
                                 uint32_t* __restrict__ kout, int32_t* __restrict__ vout, const int32_t* d_n,
-                                int shift, const int32_t* __restrict__ hist, int nblk) {
-    __shared__ int run[256];
-    __shared__ int wcnt[8][256];
-    __shared__ int tot[256];
+                                int shift, const int32_t* __restrict__ hist, const int32_t* __restrict__ dtot,
+                                int nblk) {
+    __shared__ int run[kDigits];
+    __shared__ int wcnt[8][kDigits];
+    __shared__ int tot[kDigits];
+    __shared__ int smw[8];
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    run[tid] = hist[tid * nblk + blockIdx.x];
+    {   // digit bases: exclusive scan of the digit totals (2 digits per thread)
+        int a0 = dtot[2 * tid], a1 = dtot[2 * tid + 1], t;
+        int ex = block_excl_scan(a0 + a1, smw, &t);
+        run[2 * tid] = ex + hist[(size_t)(2 * tid) * nblk + blockIdx.x];
+        run[2 * tid + 1] = ex + a0 + hist[(size_t)(2 * tid + 1) * nblk + blockIdx.x];
+    }
     int lo, hi;
     chunk_range(*d_n, nblk, blockIdx.x, lo, hi);
     for (int base = lo; base < hi; base += kTile) {
 #pragma unroll
-        for (int i = 0; i < 8; i++) wcnt[i][tid] = 0;
+        for (int i = 0; i < 8; i++) {
+            wcnt[i][tid] = 0;
+            wcnt[i][tid + 256] = 0;
+        }
         __syncthreads();
         const int i = base + tid;
         const bool valid = i < hi;
         uint32_t key = valid ? kin[i] : 0u;
         int32_t val = valid ? vin[i] : 0;
-        int dg = valid ? (int)((key >> shift) & 255u) : -1;
+        int dg = valid ? (int)((key >> shift) & (kDigits - 1)) : -1;
         unsigned peers = __match_any_sync(FULL, dg);
         int rank = __popc(peers & lanemask_lt());
         if (valid && rank == 0) wcnt[w][dg] = __popc(peers);
         __syncthreads();
-        {
+#pragma unroll
+        for (int h = 0; h < 2; h++) {
+            const int d = tid + h * 256;
             int acc = 0;
 #pragma unroll
             for (int q = 0; q < 8; q++) {
-                int c = wcnt[q][tid];
-                wcnt[q][tid] = acc;
+                int c = wcnt[q][d];
+                wcnt[q][d] = acc;
                 acc += c;
             }
-            tot[tid] = acc;
+            tot[d] = acc;
         }
         __syncthreads();
         if (valid) {
@@ -130,6 +166,7 @@ __global__ void k_radix_scatter(const uint32_t* __restrict__ kin, const int32_t*
         }
         __syncthreads();
         run[tid] += tot[tid];
+        run[tid + 256] += tot[tid + 256];
     }
 }
 
@@ -140,7 +177,7 @@ void sort_alloc(SortScratch& s, int64_t cap) {
         cudaMalloc(&s.v[i], s.cap * sizeof(int32_t));
     }
     s.nblk = grid_for(s.cap, kTile * 4, 2);
-    cudaMalloc(&s.hist, 256 * (size_t)s.nblk * sizeof(int32_t));
+    cudaMalloc(&s.hist, ((size_t)kDigits * s.nblk + kDigits) * sizeof(int32_t));
 }
 void sort_free(SortScratch& s) {
     for (int i = 0; i < 2; i++) {
@@ -151,63 +188,14 @@ void sort_free(SortScratch& s) {
     s = SortScratch();
 }
 
-// exclusive scan of the [256 digits][nblk] histogram in digit-major order: one warp per
-// digit row (coalesced), digit totals scanned by warp 0, then rows offset by their base
-__global__ void k_scan_digits(int32_t* __restrict__ hist, int nblk) {
-    __shared__ int tot[256];
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    for (int dg = w; dg < 256; dg += nw) {
-        int32_t* row = hist + (size_t)dg * nblk;
-        int run = 0;
-        for (int b0 = 0; b0 < nblk; b0 += 32) {
-            int i = b0 + lane;
-            int v = i < nblk ? row[i] : 0, x = v;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                int y = __shfl_up_sync(FULL, x, o);
-                if (lane >= o) x += y;
-            }
-            if (i < nblk) row[i] = run + x - v;
-            run += __shfl_sync(FULL, x, 31);
-        }
-        if (lane == 0) tot[dg] = run;
-    }
-    __syncthreads();
-    if (w == 0) {
-        int v[8], s = 0;
-#pragma unroll
-        for (int q = 0; q < 8; q++) {
-            v[q] = tot[lane * 8 + q];
-            s += v[q];
-        }
-        int x = s;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            int y = __shfl_up_sync(FULL, x, o);
-            if (lane >= o) x += y;
-        }
-        int base = x - s;
-#pragma unroll
-        for (int q = 0; q < 8; q++) {
-            tot[lane * 8 + q] = base;
-            base += v[q];
-        }
-    }
-    __syncthreads();
-    for (int dg = w; dg < 256; dg += nw) {
-        int32_t* row = hist + (size_t)dg * nblk;
-        const int base = tot[dg];
-        for (int i = lane; i < nblk; i += 32) row[i] += base;
-    }
-}
-
 int sort_pairs(SortScratch& s, const int32_t* d_n, int bits, cudaStream_t st, int64_t* launches) {
     int cur = 0;
-    for (int shift = 0; shift < bits; shift += 8) {
+    int32_t* tot = s.hist + (size_t)kDigits * s.nblk;
+    for (int shift = 0; shift < bits; shift += kRadixBits) {
         k_radix_hist<<<s.nblk, 256, 0, st>>>(s.k[cur], d_n, shift, s.hist, s.nblk);
-        k_scan_digits<<<1, 1024, 0, st>>>(s.hist, s.nblk);
+        k_radix_scan_rows<<<kDigits, 256, 0, st>>>(s.hist, s.nblk, tot);
         k_radix_scatter<<<s.nblk, 256, 0, st>>>(s.k[cur], s.v[cur], s.k[cur ^ 1], s.v[cur ^ 1], d_n, shift,
-                                                s.hist, s.nblk);
+                                                s.hist, tot, s.nblk);
         *launches += 3;
         cur ^= 1;
     }
@@ -681,7 +669,7 @@ __global__ void k_flush_rows(const int32_t* __restrict__ rows, const int32_t* d_
                              int world, int g, int d4, const int32_t* __restrict__ slot,
                              const int32_t* __restrict__ last_upd, const int32_t* __restrict__ pool_idx, int P,
                              int64_t capT, const float4* __restrict__ cw, const float4* __restrict__ pw, float4* hw,
-                             unsigned long long* stats) {
+                             unsigned long long* stats, int sysfence) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
@@ -701,7 +689,7 @@ __global__ void k_flush_rows(const int32_t* __restrict__ rows, const int32_t* d_
         }
         for (int v = l; v < d4; v += GS) hw[k * d4 + v] = src[v];
     }
-    __threadfence_system();
+    if (sysfence) block_fence_system();
     if (stats) {
         block_count(stats, nh);
         block_count(stats + 1, nc);
@@ -715,7 +703,7 @@ void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begi
     DISPATCH_GS(gs, (k_flush_rows<GS><<<grid, 256, 0, st>>>(
                         rows, d_begin, d_end, c->n, c->g, d4, c->slot, c->last_upd, c->pool_idx, c->P, c->capT,
                         (const float4*)c->cw, (const float4*)c->pw, (float4*)c->dh_w,
-                        counter >= 0 ? c->dstats + counter : nullptr)));
+                        counter >= 0 ? c->dstats + counter : nullptr, c->n > 1)));
     c->launches++;
 }
 
@@ -780,9 +768,14 @@ void launch_expand(frugal_ctx* c, QueueSlot& q, float* out, cudaStream_t st) {
 }
 
 // ============================================================================ model glue
-template <int J>
-__global__ void k_dot_model(const float* __restrict__ emb, const float* __restrict__ x, const float* __restrict__ y,
-                            float* __restrict__ grad, double* loss, int count, int F, int d, double nb) {
+// warp per sample; lane j holds element j (+32q) of S and, when F <= FC, of every e_f
+// in registers (one HBM read of the embeddings); the loss is block-reduced, one atomic
+// per block.
+template <int J, int FC>
+__global__ void __launch_bounds__(256) k_dot_model(const float* __restrict__ emb, const float* __restrict__ x,
+                                                   const float* __restrict__ y, float* __restrict__ grad,
+                                                   double* loss, int count, int F, int d, double nb) {
+    __shared__ double sl[8];
     const int lane = threadIdx.x & 31;
     const int wid = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int nw = (gridDim.x * blockDim.x) >> 5;
@@ -790,30 +783,53 @@ __global__ void k_dot_model(const float* __restrict__ emb, const float* __restri
     for (int b = wid; b < count; b += nw) {
         const float* e0 = emb + (int64_t)b * F * d;
         float S[J];
+        float ec[FC > 0 ? FC : 1][J];
 #pragma unroll
         for (int q = 0; q < J; q++) S[q] = 0.0f;
         double ee = 0.0;
-        for (int f = 0; f < F; f++) {
+        if (FC > 0) {
 #pragma unroll
-            for (int q = 0; q < J; q++) {
-                int j = lane + 32 * q;
-                if (j < d) {
-                    float v = e0[f * d + j];
-                    S[q] = __fadd_rn(S[q], v);
-                    ee += (double)v * (double)v;
+            for (int f = 0; f < FC; f++) {
+#pragma unroll
+                for (int q = 0; q < J; q++) {
+                    int j = lane + 32 * q;
+                    ec[f][q] = (f < F && j < d) ? e0[f * d + j] : 0.0f;
+                }
+            }
+#pragma unroll
+            for (int f = 0; f < FC; f++) {
+                if (f < F) {
+#pragma unroll
+                    for (int q = 0; q < J; q++) {
+                        S[q] = __fadd_rn(S[q], ec[f][q]);
+                        ee += (double)ec[f][q] * (double)ec[f][q];
+                    }
+                }
+            }
+        } else {
+            for (int f = 0; f < F; f++) {
+#pragma unroll
+                for (int q = 0; q < J; q++) {
+                    int j = lane + 32 * q;
+                    if (j < d) {
+                        float v = e0[f * d + j];
+                        S[q] = __fadd_rn(S[q], v);
+                        ee += (double)v * (double)v;
+                    }
                 }
             }
         }
         double sq = 0.0, xs = 0.0;
         const float* xb = x + (int64_t)b * d;
+        float xv[J];
 #pragma unroll
         for (int q = 0; q < J; q++) {
             int j = lane + 32 * q;
-            if (j < d) {
-                sq += (double)S[q] * (double)S[q];
-                xs += (double)xb[j] * (double)S[q];
-            }
+            xv[q] = j < d ? xb[j] : 0.0f;
+            sq += (double)S[q] * (double)S[q];
+            xs += (double)xv[q] * (double)S[q];
         }
+#pragma unroll
         for (int o = 16; o; o >>= 1) {
             sq += __shfl_xor_sync(FULL, sq, o);
             ee += __shfl_xor_sync(FULL, ee, o);
@@ -823,20 +839,36 @@ __global__ void k_dot_model(const float* __restrict__ emb, const float* __restri
         double p = 1.0 / (1.0 + exp(-z));
         double yb = (double)y[b];
         if (lane == 0) lsum += (z > 0 ? z + log1p(exp(-z)) : log1p(exp(z))) - yb * z;
-        float cc = (float)((p - yb) / nb);  // same rounding as the definition
+        float cc = (float)((p - yb) / nb);  // same rounding as the definition (R16)
         float* g0 = grad + (int64_t)b * F * d;
-        for (int f = 0; f < F; f++) {
+        if (FC > 0) {
 #pragma unroll
-            for (int q = 0; q < J; q++) {
-                int j = lane + 32 * q;
-                if (j < d) {
-                    float t = __fadd_rn(__fsub_rn(S[q], e0[f * d + j]), xb[j]);
-                    g0[f * d + j] = __fmul_rn(cc, t);
+            for (int f = 0; f < FC; f++) {
+                if (f < F) {
+#pragma unroll
+                    for (int q = 0; q < J; q++) {
+                        int j = lane + 32 * q;
+                        if (j < d) g0[f * d + j] = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[q], ec[f][q]), xv[q]));
+                    }
+                }
+            }
+        } else {
+            for (int f = 0; f < F; f++) {
+#pragma unroll
+                for (int q = 0; q < J; q++) {
+                    int j = lane + 32 * q;
+                    if (j < d) g0[f * d + j] = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[q], e0[f * d + j]), xv[q]));
                 }
             }
         }
     }
-    if (lane == 0 && lsum != 0.0) atomicAdd(loss, lsum / nb);  // mean over the global batch (R17)
+    if (lane == 0) sl[threadIdx.x >> 5] = lsum;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int i = 0; i < 8; i++) t += sl[i];
+        if (t != 0.0) atomicAdd(loss, t / nb);  // mean over the global batch (R17)
+    }
 }
 
 void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const float* x, const float* y, float* grad,
@@ -844,15 +876,16 @@ void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const float
     int count = q.h_counts[c->g];
     if (count <= 0) return;
     int J = (c->d + 31) / 32;
-    int grid = grid_for((int64_t)count * 32, 256, 8);
+    int grid = grid_for((int64_t)count * 32, 256, 4);
     const double nbd = (double)nb;
-#define DM(JJ) k_dot_model<JJ><<<grid, 256, 0, st>>>(emb, x, y, grad, loss, count, c->F, c->d, nbd)
-    if (J <= 1) DM(1);
-    else if (J <= 2) DM(2);
-    else if (J <= 4) DM(4);
-    else if (J <= 8) DM(8);
-    else if (J <= 16) DM(16);
-    else DM(32);
+    const bool cache = c->F <= 32;
+#define DM(JJ, FC) k_dot_model<JJ, FC><<<grid, 256, 0, st>>>(emb, x, y, grad, loss, count, c->F, c->d, nbd)
+    if (J <= 1) { if (cache) DM(1, 32); else DM(1, 0); }
+    else if (J <= 2) { if (cache) DM(2, 32); else DM(2, 0); }
+    else if (J <= 4) DM(4, 0);
+    else if (J <= 8) DM(8, 0);
+    else if (J <= 16) DM(16, 0);
+    else DM(32, 0);
 #undef DM
     c->launches++;
 }

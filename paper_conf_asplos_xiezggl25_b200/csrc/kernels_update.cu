@@ -30,9 +30,13 @@ __device__ __forceinline__ float4 chunk_sum(const float4* __restrict__ grad, con
     float4 acc = grad[(int64_t)pos[b] * d4 + v];
     int j = b + 1;
     for (; j + 16 <= e; j += 16) {  // 16 loads in flight, adds in position order
+        int pq[16];
+#pragma unroll
+        for (int q = 0; q < 16; q++) pq[q] = pos[j + q];
         float4 x[16];
 #pragma unroll
-        for (int q = 0; q < 16; q++) x[q] = grad[(int64_t)pos[j + q] * d4 + v];
+        for (int q = 0; q < 16; q++) x[q] = grad[(int64_t)pq[q] * d4 + v];
+        asm volatile("" ::: "memory");  // keep all 16 loads issued before the first add
 #pragma unroll
         for (int q = 0; q < 16; q++) acc = add4(acc, x[q]);
     }
@@ -48,10 +52,11 @@ __device__ __forceinline__ float4 chunk_sum(const float4* __restrict__ grad, con
 }
 
 template <int GS>
-__global__ void k_segreduce(const int32_t* __restrict__ off, const int32_t* __restrict__ pos,
+__global__ void __launch_bounds__(256) k_segreduce(const int32_t* __restrict__ off, const int32_t* __restrict__ pos,
                             const int32_t* d_nu, const int32_t* __restrict__ gl, const int32_t* __restrict__ goff,
                             int g, int d4, const float4* __restrict__ grad, float4* __restrict__ Pp, float4* mail,
-                            int32_t* long_q, int32_t* long_cnt, unsigned long long* stats) {
+                            int32_t* long_q, int32_t* long_cnt, int2* tasks, int32_t* task_cnt,
+                            unsigned long long* stats) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
@@ -66,9 +71,12 @@ __global__ void k_segreduce(const int32_t* __restrict__ off, const int32_t* __re
         const int u = gl ? gl[q] : (int)q;
         const int b = off[u], e = off[u + 1];
         if (l == 0 && (q < own_lo || q >= own_hi)) nout++;
-        if (e - b > kChunk) {
+        if (e - b > kChunk) {  // Zipf head: chunk tasks for k_segred_chunks
             if (l == 0) {
                 long_q[atomicAdd(long_cnt, 1)] = (int32_t)q;
+                const int nch = (e - b + kChunk - 1) / kChunk;
+                const int t0 = atomicAdd(task_cnt, nch);
+                for (int cc = 0; cc < nch; cc++) tasks[t0 + cc] = make_int2(b + cc * kChunk, min(e, b + (cc + 1) * kChunk));
                 nlong++;
             }
             continue;
@@ -76,55 +84,107 @@ __global__ void k_segreduce(const int32_t* __restrict__ off, const int32_t* __re
         float4* dst = (q >= own_lo && q < own_hi) ? (Pp + q * d4) : (mail + q * d4);
         for (int v = l; v < d4; v += GS) dst[v] = chunk_sum<GS>(grad, pos, b, e, d4, v);
     }
-    if (gl) __threadfence_system();
+    if (gl) block_fence_system();
     block_count(stats + FRUGAL_C_LONG_SEGMENTS, nlong);
     block_count(stats + FRUGAL_C_MAIL_OUT, nout);
 }
 
-// one block per long segment: row groups compute chunk sums into scratch (indexed by
-// the chunk's first position), then one group adds them in order
+// Ordered sum of n rows (row(0) first, then row(1), ...) of src, column v, with the row
+// loads staged through shared memory by cp.async in double-buffered batches of 16, so
+// 16-32 row loads are in flight per lane while the adds stay strictly in order.
+// smem: [2][16][blockDim] float4, each thread touching only its own column.
+constexpr int kBatch = 16;
+
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+    unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+template <typename RowF>
+__device__ __forceinline__ float4 ordered_sum(RowF row, int n, const float4* __restrict__ src, int d4, int v,
+                                              float4* smem) {
+    const int nt = blockDim.x, t = threadIdx.x;
+    auto issue = [&](int k) {
+        const int q0 = k * kBatch, q1 = min(n, q0 + kBatch);
+        float4* bb = smem + (size_t)(k & 1) * kBatch * nt;
+        for (int q = q0; q < q1; q++) cp_async16(bb + (size_t)(q - q0) * nt + t, src + (int64_t)row(q) * d4 + v);
+        cp_async_commit();
+    };
+    const int nb = (n + kBatch - 1) / kBatch;
+    float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+    issue(0);
+    for (int k = 0; k < nb; k++) {
+        if (k + 1 < nb) {
+            issue(k + 1);
+            cp_async_wait<1>();
+        } else {
+            cp_async_wait<0>();
+        }
+        const float4* bb = smem + (size_t)(k & 1) * kBatch * nt;
+        const int q0 = k * kBatch, q1 = min(n, q0 + kBatch);
+        for (int q = q0; q < q1; q++) {
+            float4 x = bb[(size_t)(q - q0) * nt + t];
+            acc = (q == 0) ? x : add4(acc, x);
+        }
+    }
+    return acc;
+}
+constexpr size_t kOrderedSmem = 2 * kBatch * 256 * sizeof(float4);  // 128 KB for 256 threads
+
+// Long segments, phase 1: every chunk [j0, j1) of every long segment in parallel (task
+// list built by k_segreduce), summed in order into scratch[j0].
 template <int GS>
-__global__ void k_segreduce_long(const int32_t* __restrict__ off, const int32_t* __restrict__ pos,
-                                 const int32_t* __restrict__ gl, const int32_t* __restrict__ goff, int g, int d4,
-                                 const float4* __restrict__ grad, float4* __restrict__ Pp, float4* mail,
-                                 const int32_t* __restrict__ long_q, const int32_t* long_cnt,
-                                 float4* __restrict__ scratch) {
-    const int grp = threadIdx.x / GS, ngrp = blockDim.x / GS, l = threadIdx.x & (GS - 1);
+__global__ void __launch_bounds__(256) k_segred_chunks(const int32_t* __restrict__ pos, int d4,
+                                                       const float4* __restrict__ grad, float4* __restrict__ scratch,
+                                                       const int2* __restrict__ tasks, const int32_t* task_cnt) {
+    extern __shared__ float4 smem[];
+    int64_t gid, gs;
+    int l;
+    RowGroup<GS>::ids(gid, gs, l);
+    const int nt = *task_cnt;
+    const int64_t nloop = (nt + gs - 1) / gs * gs;  // uniform trip count: ordered_sum is per-thread
+    for (int64_t t = gid; t < nloop; t += gs) {
+        if (t >= nt) continue;
+        const int2 tk = tasks[t];
+        const int32_t* pj = pos + tk.x;
+        for (int v = l; v < d4; v += GS)
+            scratch[(int64_t)tk.x * d4 + v] = ordered_sum([&](int q) { return pj[q]; }, tk.y - tk.x, grad, d4, v, smem);
+    }
+}
+
+// Long segments, phase 2: per long segment, add its chunk sums in order
+template <int GS>
+__global__ void __launch_bounds__(256) k_segred_combine(const int32_t* __restrict__ off,
+                                                        const int32_t* __restrict__ gl,
+                                                        const int32_t* __restrict__ goff, int g, int d4,
+                                                        float4* __restrict__ Pp, float4* mail,
+                                                        const int32_t* __restrict__ long_q, const int32_t* long_cnt,
+                                                        const float4* __restrict__ scratch) {
+    extern __shared__ float4 smem[];
+    int64_t gid, gs;
+    int l;
+    RowGroup<GS>::ids(gid, gs, l);
     const int nl = *long_cnt;
     int own_lo = 0, own_hi = 0x7fffffff;
     if (gl) {
         own_lo = goff[g];
         own_hi = goff[g + 1];
     }
-    for (int t = blockIdx.x; t < nl; t += gridDim.x) {
+    const int64_t nloop = (nl + gs - 1) / gs * gs;
+    for (int64_t t = gid; t < nloop; t += gs) {
+        if (t >= nl) continue;
         const int q = long_q[t];
         const int u = gl ? gl[q] : q;
         const int b = off[u], e = off[u + 1];
         const int nch = (e - b + kChunk - 1) / kChunk;
-        for (int c = grp; c < nch; c += ngrp) {
-            const int c0 = b + c * kChunk, c1 = min(e, c0 + kChunk);
-            for (int v = l; v < d4; v += GS) scratch[(int64_t)c0 * d4 + v] = chunk_sum<GS>(grad, pos, c0, c1, d4, v);
-        }
-        __syncthreads();
-        if (grp == 0) {
-            float4* dst = (q >= own_lo && q < own_hi) ? (Pp + (int64_t)q * d4) : (mail + (int64_t)q * d4);
-            for (int v = l; v < d4; v += GS) {
-                float4 acc = scratch[(int64_t)b * d4 + v];
-                int c = 1;
-                for (; c + 8 <= nch; c += 8) {  // chunk sums in order, 8 loads in flight
-                    float4 x[8];
-#pragma unroll
-                    for (int q2 = 0; q2 < 8; q2++) x[q2] = scratch[(int64_t)(b + (c + q2) * kChunk) * d4 + v];
-#pragma unroll
-                    for (int q2 = 0; q2 < 8; q2++) acc = add4(acc, x[q2]);
-                }
-                for (; c < nch; c++) acc = add4(acc, scratch[(int64_t)(b + c * kChunk) * d4 + v]);
-                dst[v] = acc;
-            }
-        }
-        __syncthreads();
+        float4* dst = (q >= own_lo && q < own_hi) ? (Pp + (int64_t)q * d4) : (mail + (int64_t)q * d4);
+        for (int v = l; v < d4; v += GS)
+            dst[v] = ordered_sum([&](int c) { return b + c * kChunk; }, nch, scratch, d4, v, smem);
     }
-    if (gl) __threadfence_system();
+    if (gl) block_fence_system();
 }
 
 void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, cudaStream_t st) {
@@ -132,16 +192,27 @@ void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, c
     int grid = grid_for((int64_t)c->M * gs, 256, 8);
     const bool multi = c->n > 1;
     float4* mail = multi ? (float4*)(c->dh_mail + ((size_t)par * c->n + c->g) * c->mail_stride + 256) : nullptr;
-    cudaMemsetAsync(c->long_cnt, 0, 4, st);
+    cudaMemsetAsync(c->long_cnt, 0, 8, st);  // long_cnt[0] = long segments, long_cnt[1] = chunk tasks
     DISPATCH_GS(gs, (k_segreduce<GS><<<grid, 256, 0, st>>>(q.off, q.pos, q.n_uniq, multi ? q.gl : nullptr, q.goff,
                                                            c->g, d4, (const float4*)grad, (float4*)c->Pp, mail,
-                                                           c->long_q, c->long_cnt, c->dstats)));
-    int lgrid = (int)std::min<int64_t>(c->M / (kChunk + 1) + 1, kSMs * 2);
-    DISPATCH_GS(gs, (k_segreduce_long<GS><<<lgrid, 1024, 0, st>>>(q.off, q.pos, multi ? q.gl : nullptr, q.goff, c->g,
-                                                                 d4, (const float4*)grad, (float4*)c->Pp, mail,
-                                                                 c->long_q, c->long_cnt,
-                                                                 (float4*)c->chunk_scratch)));
-    c->launches += 2;
+                                                           c->long_q, c->long_cnt, c->long_tasks, c->long_cnt + 1,
+                                                           c->dstats)));
+    static unsigned attr_mask = 0;
+    if (!(attr_mask & gs)) {
+        DISPATCH_GS(gs, (cudaFuncSetAttribute(k_segred_chunks<GS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                              (int)kOrderedSmem),
+                         cudaFuncSetAttribute(k_segred_combine<GS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                              (int)kOrderedSmem)));
+        attr_mask |= gs;
+    }
+    DISPATCH_GS(gs, (k_segred_chunks<GS><<<kSMs, 256, kOrderedSmem, st>>>(q.pos, d4, (const float4*)grad,
+                                                                          (float4*)c->chunk_scratch, c->long_tasks,
+                                                                          c->long_cnt + 1)));
+    DISPATCH_GS(gs, (k_segred_combine<GS><<<kSMs, 256, kOrderedSmem, st>>>(q.off, multi ? q.gl : nullptr, q.goff, c->g,
+                                                                           d4, (float4*)c->Pp, mail, c->long_q,
+                                                                           c->long_cnt,
+                                                                           (const float4*)c->chunk_scratch)));
+    c->launches += 3;
 }
 
 // mailbox header of (parity, this sender): goff[0..world]
@@ -287,7 +358,7 @@ __global__ void k_g_push(int64_t No, int world, int g, int d4, const float4* __r
         int64_t k = lk * world + g;
         for (int v = l; v < d4; v += GS) hG[k * d4 + v] = Gd[lk * d4 + v];
     }
-    __threadfence_system();
+    block_fence_system();
 }
 
 void launch_final_flush(frugal_ctx* c, cudaStream_t st) {

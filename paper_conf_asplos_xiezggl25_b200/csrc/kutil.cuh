@@ -53,6 +53,15 @@ __device__ __forceinline__ void block_count(unsigned long long* dst, unsigned v)
     if (threadIdx.x == 0 && s_cnt) atomicAdd(dst, (unsigned long long)s_cnt);
 }
 
+// make this block's prior (host-memory) writes visible system-wide before anything the
+// block's thread 0 -- or a later kernel in stream order -- publishes: CTA barrier, then one
+// fence.sc.sys (cumulative over the writes ordered before it by the barrier).  Needed
+// only when other processes read the host table (world > 1); all threads must call it.
+__device__ __forceinline__ void block_fence_system() {
+    __syncthreads();
+    if (threadIdx.x == 0) __threadfence_system();
+}
+
 static inline int group_size(int d4) {
     int gs = 1;
     while (gs < d4 && gs < 32) gs <<= 1;

@@ -138,7 +138,7 @@ static void free_ctx(frugal_ctx* c) {
         F(q.ids); F(q.counts); F(q.m); F(q.uniq); F(q.inv); F(q.off); F(q.pos); F(q.n_uniq);
         if (c->n > 1) { F(q.T); F(q.Tmask); F(q.Tidx); F(q.nT); F(q.gl); F(q.goff); }
     }
-    F(c->rows); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->owned_cnt); F(c->nb_rows); F(c->nb_p); F(c->nb_cnt);
+    F(c->rows); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->long_tasks); F(c->owned_cnt); F(c->nb_rows); F(c->nb_p); F(c->nb_cnt);
     for (int i = 0; i < 2; i++) { F(c->bk_rows[i]); F(c->bk_p[i]); F(c->bk_off[i]); F(c->age_rows[i]); F(c->age_cnt[i]); }
     F(c->dstats); F(c->sched_info); F(c->ff_rows); F(c->ff_cnt); F(c->ids_stage);
     if (c->herr) cudaFreeHost(c->herr);
@@ -200,6 +200,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->No = c->g < c->N ? (c->N - c->g + c->n - 1) / c->n : 0;
     c->P = c->D + 2;
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 32;
+    c->side_inline = getenv("FRUGAL_SIDE_INLINE") && atoi(getenv("FRUGAL_SIDE_INLINE"));
     c->capT = std::max<int64_t>(1, std::min<int64_t>((int64_t)c->n * c->M, c->No));
     c->key_bits = bits_for(c->N - 1);
     c->lk_bits = bits_for(std::max<int64_t>(c->No - 1, 0));
@@ -328,7 +329,8 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     DMALLOC(c->Pp, (size_t)c->M * rowb);
     DMALLOC(c->chunk_scratch, (size_t)c->M * rowb);
     DMALLOC(c->long_q, (size_t)c->M * 4);
-    DMALLOC(c->long_cnt, 4);
+    DMALLOC(c->long_cnt, 8);
+    DMALLOC(c->long_tasks, ((size_t)c->M / 32 + 2) * sizeof(int2));
     DMALLOC(c->owned_cnt, 4);
     DMALLOC(c->nb_rows, 2 * c->capT * 4);
     DMALLOC(c->nb_p, 2 * c->capT * 4);
@@ -526,15 +528,17 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
     CK(cudaEventRecord(c->ev_sched, st));
     CK(cudaStreamWaitEvent(c->side, c->ev_sched, 0));
     {
-        Timer tm(c, PH_SIDE, c->side);
+        // FRUGAL_SIDE_INLINE=1 (experiments): drain on the caller's stream instead
+        cudaStream_t sd = c->side_inline ? st : c->side;
+        Timer tm(c, PH_SIDE, sd);
         // bounded grid: the drain trickles over the step instead of crowding out the main stream
         launch_flush_rows(c, c->bk_rows[par], c->bk_off[par] + 1, c->bk_off[par] + c->L, c->side_blocks,
-                          FRUGAL_C_SIDE_HOT, c->side);
-        launch_flush_rows(c, c->age_rows[par], nullptr, c->age_cnt[par], c->side_blocks, FRUGAL_C_SIDE_HOT, c->side);
-        if (c->n > 1) launch_set_flag(c, FLAG_SIDE, (uint32_t)(s + 1), c->side);
+                          FRUGAL_C_SIDE_HOT, sd);
+        launch_flush_rows(c, c->age_rows[par], nullptr, c->age_cnt[par], c->side_blocks, FRUGAL_C_SIDE_HOT, sd);
+        if (c->n > 1) launch_set_flag(c, FLAG_SIDE, (uint32_t)(s + 1), sd);
         CKL();
     }
-    CK(cudaEventRecord(c->ev_side[par], c->side));
+    CK(cudaEventRecord(c->ev_side[par], c->side_inline ? st : c->side));
     c->side_pending[par] = true;
     {
         // a3: gate of step s -- PQ front > s: every owner's urgent bucket s and every

@@ -1,0 +1,99 @@
+"""world = 2 on ONE B200: two rank processes share device 0 and one POSIX-shm host
+table; mailboxes, flags and gates go through host memory exactly as across GPUs.
+Compared against the oracle run with world 2: per-rank schedule sets (each rank owns
+k mod 2 == rank), final flush, host table (w, G) and the global loss."""
+import multiprocessing as mp
+import os
+import traceback
+
+import numpy as np
+import pytest
+
+from paper_conf_asplos_xiezggl25_b200 import workload as W
+
+pytestmark = pytest.mark.gpu
+
+
+def _rank_main(rank, st, shm, barrier, q):
+    try:
+        import torch
+        from paper_conf_asplos_xiezggl25_b200 import frugal as F
+        from paper_conf_asplos_xiezggl25_b200.harness import Trainer, make_context
+        torch.cuda.set_device(0)
+        fr = make_context(st, rank=rank, device=0, shm_name=shm, flags=F.F_RECORD)
+        barrier.wait()
+        tr = Trainer(fr, st, rank=rank)
+        sched = []
+        for s in range(st.steps):
+            got = {}
+            tr.step(on_schedule=lambda s_: got.update(fr.get_schedule()))
+            sched.append(got)
+        fr.flush()
+        ff = fr.get_final_flush()
+        losses = tr.losses()
+        barrier.wait()  # both ranks flushed: the host table is authoritative
+        w = G = None
+        if rank == 0:
+            w, G = fr.read_host(np.arange(st.cfg.n_rows))
+        barrier.wait()
+        fr.close()
+        q.put((rank, dict(sched=sched, ff=ff, losses=losses, w=w, G=G)))
+    except Exception:
+        q.put((rank, traceback.format_exc()))
+
+
+def run_two_ranks(st, timeout=600):
+    ctx = mp.get_context("spawn")
+    barrier = ctx.Barrier(2)
+    q = ctx.Queue()
+    shm = f"/frugal_test_{os.getpid()}"
+    ps = [ctx.Process(target=_rank_main, args=(r, st, shm, barrier, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    out = {}
+    try:
+        for _ in range(2):
+            r, v = q.get(timeout=timeout)
+            out[r] = v
+    finally:
+        for p in ps:
+            p.join(timeout=30)
+            if p.is_alive():
+                p.kill()
+    for r, v in out.items():
+        assert not isinstance(v, str), f"rank {r} failed:\n{v}"
+    return out
+
+
+@pytest.mark.parametrize("opt", ["adagrad", "sgd"])
+def test_two_ranks_one_gpu_parity(opt):
+    from oracle.oracle import Oracle
+    cfg = W.config("tiny", world=2, batch=64, lookahead=4, age_out=3, opt=opt,
+                   lr=0.05 if opt == "adagrad" else 1.0)
+    rng = np.random.default_rng(3)
+    counts = rng.integers(0, 65, size=(24, 2)).astype(np.int32)
+    counts[5, 1] = 0
+    st = W.gen_stream(cfg, 24, counts=counts)
+    out = run_two_ranks(st)
+    o = Oracle(st)
+    for s in range(st.steps):
+        o.step()
+        ref = o.schedule()
+        urg = sorted(sum((out[r]["sched"][s]["urgent"].tolist() for r in range(2)), []))
+        assert urg == ref["urgent"].tolist(), f"urgent differs at {s}"
+        dfr = sorted(sum((list(zip(out[r]["sched"][s]["deferred"].tolist(),
+                                   out[r]["sched"][s]["deferred_p"].tolist())) for r in range(2)), []))
+        assert dfr == sorted(zip(ref["deferred"].tolist(), ref["deferred_p"].tolist())), f"deferred differs at {s}"
+        age = sorted(sum((out[r]["sched"][s]["ageout"].tolist() for r in range(2)), []))
+        assert age == ref["ageout"].tolist()
+        for r in range(2):  # each rank only schedules rows it owns
+            assert all(k % 2 == r for k in out[r]["sched"][s]["urgent"].tolist())
+    ff = sorted(out[0]["ff"].tolist() + out[1]["ff"].tolist())
+    assert ff == o.final_flush().tolist()
+    lo = np.array([o.loss(s) for s in range(st.steps)])
+    lg = out[0]["losses"] + out[1]["losses"]
+    assert np.abs(lg - lo).max() <= 1e-5
+    wo, Go = o.read_rows(np.arange(cfg.n_rows))
+    assert np.abs(out[0]["w"] - wo).max() <= 1e-5
+    assert np.abs(out[0]["G"] - Go).max() <= 1e-5
+    assert o.violations == 0
