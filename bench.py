@@ -204,7 +204,7 @@ def main():
 
     cfg = W.config(args.config, world=world, alpha=args.alpha)
     K, Wm, L = args.steps, args.warmup, cfg.lookahead
-    S = Wm + 2 * K + L + 1
+    S = Wm + 2 * K + L + 2
     t_gen = time.time()
     st = W.gen_stream(cfg, S)  # every rank generates the same seeded stream of all ranks
     t_gen = time.time() - t_gen
@@ -230,18 +230,18 @@ def main():
     y_e = torch.empty(B, device=dev)
     counts = st.counts
 
-    for t in range(L - 1):
+    for t in range(L):
         fr.prefetch(t, ids_d[t], counts[t])
 
     def step_dev(s):
-        t = s + L - 1
+        t = s + L
         fr.step(s, ids_d[t], counts[t])
         fr.lookup(s, emb)
         fr.dot_model(s, emb, x_d[s], y_d[s], grad, loss[s:s + 1])
         fr.backward_update(s, grad)
 
     def step_e2e(s):
-        t = s + L - 1
+        t = s + L
         fr.step(s, ids_h[t], counts[t])       # ids copied from pinned host inside the call
         fr.lookup(s, emb)
         x_e.copy_(x_h[s], non_blocking=True)

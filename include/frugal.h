@@ -19,8 +19,9 @@
  * Rank g owns row k iff k mod world == g (reading R12 in DESIGN.md): the owner
  * caches it if hot and applies its optimizer update (R6).
  *
- * Per-step call order (after frugal_prefetch(t) for t = 0 .. L-2):
- *     frugal_step(s) -> frugal_lookup(s) -> [model] -> frugal_backward_update(s)
+ * Per-step call order (after frugal_prefetch(t) for t = 0 .. L-1):
+ *     frugal_step(s) [enqueues step s+L] -> frugal_lookup(s) -> [model] ->
+ *     frugal_backward_update(s)
  * and frugal_flush(FRUGAL_FLUSH_ALL) at the end of training.  Any other order
  * returns FRUGAL_ESTATE.
  */
@@ -95,18 +96,21 @@ typedef struct {
 frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out);
 
 /* Sample queue (§3.2, §3.3): enqueue the ids of step t of ALL
-   ranks.  ids_all: int64 [world][batch*slots], host (pinned) or device pointer,
-   copied before return to the stream's order (caller may reuse it after the stream
-   reaches this point).  counts: host int32[world], samples of each rank (0..batch).
-   Only used for t = 0..L-2 before step 0. */
+   ranks.  ids_all: int64 [world][batch*slots], host (pageable or pinned) or device
+   pointer; it is read after the work already on `stream` and `stream`'s later work is
+   ordered after the read, so the caller may overwrite it once `stream` gets there.
+   counts: host int32[world], samples of each rank (0..batch).  Only for t = 0..L-1
+   before step 0.  The queue holds L+1 future steps: the ingest of step t (id
+   conversion, dedup, read bits) runs on a library stream one step ahead, overlapping
+   the previous step; priorities still only see the L steps [s, s+L-1] (R1). */
 frugal_status frugal_prefetch(frugal_ctx* ctx, int64_t t, const int64_t* ids_all,
                               const int32_t* counts, frugal_stream stream);
 
-/* Begin step s: enqueue step t = s+L-1 (ids_next_all/counts_next as in prefetch; NULL
-   past the end of the stream), run the P2F scheduler for the rows updated at s-1
-   (priority buckets, AdjustPriority inf->t, age-out), flush the urgent bucket on
-   `stream`, hand the deferred buckets to the side stream, and enqueue the gate
-   (PQ front > s, §3.3) on `stream`.  Returns once enqueued. */
+/* Begin step s: run the P2F scheduler for the rows updated at s-1 (priority buckets over
+   [s, s+L-1], AdjustPriority inf->s+L-1, age-out), flush the urgent bucket on `stream`,
+   hand the deferred buckets to the side stream, enqueue step s+L (ids_next_all /
+   counts_next as in prefetch; NULL past the end of the stream) and the gate (PQ front
+   > s, §3.3) on `stream`.  Returns once enqueued. */
 frugal_status frugal_step(frugal_ctx* ctx, int64_t s, const int64_t* ids_next_all,
                           const int32_t* counts_next, frugal_stream stream);
 

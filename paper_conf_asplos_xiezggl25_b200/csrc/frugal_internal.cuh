@@ -83,6 +83,7 @@ struct frugal_ctx {
     int n, g, d, F, B, L, D, M;  // world, rank, dim, slots, batch, lookahead, age_out, B*F
     int64_t N, No;               // rows, owned rows
     int P;                       // pool segments = D + 2
+    int QN;                      // sample-queue slots = L + 2 (steps s-1 .. s+L)
     int side_blocks = 32;        // grid cap of the side-stream drain
     bool side_inline = false;    // experiment: drain on the caller stream
     int64_t capT;                // max owned rows touched per step
@@ -137,6 +138,9 @@ struct frugal_ctx {
     int32_t* nb_rows = nullptr;  // newly bucketed rows [capT + capT]
     int32_t* nb_p = nullptr;
     int32_t* nb_cnt = nullptr;   // scalar
+    int32_t* adj_rows[2] = {nullptr, nullptr};  // AdjustPriority inf -> t rows, by consuming step parity
+    int32_t* adj_p[2] = {nullptr, nullptr};
+    int32_t* adj_cnt[2] = {nullptr, nullptr};
     int32_t* bk_rows[2] = {nullptr, nullptr};  // bucket-sorted rows
     int32_t* bk_p[2] = {nullptr, nullptr};
     int32_t* bk_off[2] = {nullptr, nullptr};   // [L+1]
@@ -155,6 +159,9 @@ struct frugal_ctx {
     frugal::ScanScratch scan;
 
     cudaStream_t side = nullptr;
+    cudaStream_t istream = nullptr;  // sample-queue ingest, one step ahead
+    cudaEvent_t ev_call = nullptr, ev_copied = nullptr;
+    std::vector<cudaEvent_t> ev_ingest;  // per queue slot: ingest complete
     cudaEvent_t ev_sched = nullptr;
     cudaEvent_t ev_side[2] = {nullptr, nullptr};
     bool side_pending[2] = {false, false};
@@ -183,7 +190,8 @@ namespace frugal {
 void launch_convert_ids(frugal_ctx* c, QueueSlot& q, cudaStream_t st);
 void launch_dedup(frugal_ctx* c, QueueSlot& q, cudaStream_t st);
 void launch_owner_side(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st);
-void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, cudaStream_t st);
+void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, int32_t* adj_rows, int32_t* adj_p,
+                        int32_t* adj_cnt, cudaStream_t st);
 void launch_bucket(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStream_t st);
 void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begin, const int32_t* d_end,
                        int max_blocks, int counter, cudaStream_t st);

@@ -517,7 +517,7 @@ __global__ void k_ingest_bits(const int32_t* __restrict__ T, const uint32_t* __r
             uint32_t mask = (world > 1) ? Tmask[j] : 1u;
             bool host = (mask & ~(1u << g)) != 0u || slot[lk] < 0;
             uint64_t b = (1ull << bit) | (host ? (1ull << (32 + bit)) : 0ull);
-            rbits[lk] |= b;
+            atomicOr((unsigned long long*)&rbits[lk], (unsigned long long)b);  // races with k_optimizer's clear
             if (adjust && state[lk] == ST_INF) {
                 if (host) {
                     state[lk] = ST_CLEAN;
@@ -569,14 +569,15 @@ __global__ void k_bucket_prev(const int32_t* __restrict__ T, const int32_t* d_nT
 }
 
 // two-level PQ level 1: counting sort of the newly bucketed rows by deadline p - s in [0, L)
-__global__ void k_bucket_hist(const int32_t* __restrict__ nb_p, const int32_t* nb_cnt, int32_t s, int L,
+__global__ void k_bucket_hist(const int32_t* __restrict__ nb_p, const int32_t* nb_cnt,
+                              const int32_t* __restrict__ adj_p, const int32_t* adj_cnt, int32_t s, int L,
                               int32_t* bk_off /*[L+1], zeroed*/) {
     __shared__ int h[32];
     if (threadIdx.x < 32) h[threadIdx.x] = 0;
     __syncthreads();
-    int n = *nb_cnt;
+    const int n1 = *nb_cnt, n = n1 + *adj_cnt;
     for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
-        atomicAdd(&h[nb_p[i] - s], 1);
+        atomicAdd(&h[(i < n1 ? nb_p[i] : adj_p[i - n1]) - s], 1);
     __syncthreads();
     if (threadIdx.x < L && h[threadIdx.x]) atomicAdd(&bk_off[threadIdx.x + 1], h[threadIdx.x]);
 }
@@ -588,13 +589,15 @@ __global__ void k_bucket_scan(int32_t* bk_off, int L, int32_t* cursor) {
     }
 }
 __global__ void k_bucket_scatter(const int32_t* __restrict__ nb_rows, const int32_t* __restrict__ nb_p,
-                                 const int32_t* nb_cnt, int32_t s, int32_t* cursor, int32_t* __restrict__ bk_rows,
-                                 int32_t* __restrict__ bk_p) {
-    int n = *nb_cnt;
+                                 const int32_t* nb_cnt, const int32_t* __restrict__ adj_rows,
+                                 const int32_t* __restrict__ adj_p, const int32_t* adj_cnt, int32_t s,
+                                 int32_t* cursor, int32_t* __restrict__ bk_rows, int32_t* __restrict__ bk_p) {
+    const int n1 = *nb_cnt, n = n1 + *adj_cnt;
     for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
-        int p = nb_p[i];
+        const bool a = i >= n1;
+        const int p = a ? adj_p[i - n1] : nb_p[i];
         int at = atomicAdd(&cursor[p - s], 1);
-        bk_rows[at] = nb_rows[i];
+        bk_rows[at] = a ? adj_rows[i - n1] : nb_rows[i];
         bk_p[at] = p;
     }
 }
@@ -625,10 +628,11 @@ __global__ void k_ageout(const int32_t* __restrict__ pkey, const int32_t* pcount
     }
 }
 
-void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, cudaStream_t st) {
+void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, int32_t* adj_rows, int32_t* adj_p,
+                        int32_t* adj_cnt, cudaStream_t st) {
     k_ingest_bits<<<grid_for(c->capT, 256), 256, 0, st>>>(q.T, q.Tmask, q.nT, c->n, c->g, (int)(t & 31), (int32_t)t,
-                                                           adjust, c->slot, c->rbits, c->state, c->nb_rows,
-                                                           c->nb_p, c->nb_cnt);
+                                                           adjust, c->slot, c->rbits, c->state, adj_rows, adj_p,
+                                                           adj_cnt);
     c->launches++;
 }
 
@@ -642,9 +646,11 @@ void launch_bucket(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStrea
     }
     cudaMemsetAsync(c->bk_off[par], 0, (L + 1) * sizeof(int32_t), st);
     int32_t* cursor = c->sched_info + 8;  // [L] scratch
-    k_bucket_hist<<<grid_for(2 * c->capT, 256, 2), 256, 0, st>>>(c->nb_p, c->nb_cnt, (int32_t)s, L, c->bk_off[par]);
+    k_bucket_hist<<<grid_for(2 * c->capT, 256, 2), 256, 0, st>>>(c->nb_p, c->nb_cnt, c->adj_p[par], c->adj_cnt[par],
+                                                                  (int32_t)s, L, c->bk_off[par]);
     k_bucket_scan<<<1, 32, 0, st>>>(c->bk_off[par], L, cursor);
-    k_bucket_scatter<<<grid_for(2 * c->capT, 256, 2), 256, 0, st>>>(c->nb_rows, c->nb_p, c->nb_cnt, (int32_t)s,
+    k_bucket_scatter<<<grid_for(2 * c->capT, 256, 2), 256, 0, st>>>(c->nb_rows, c->nb_p, c->nb_cnt, c->adj_rows[par],
+                                                                     c->adj_p[par], c->adj_cnt[par], (int32_t)s,
                                                                      cursor, c->bk_rows[par], c->bk_p[par]);
     c->launches += 3;
     // age-out of cold rows updated at u = s-1-D

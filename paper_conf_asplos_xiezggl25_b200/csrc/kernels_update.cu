@@ -303,7 +303,7 @@ __global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, 
             nin += __popc(mask & ~(1u << g));
             state[lk] = ST_UPDATED;
             last_upd[lk] = s;
-            rbits[lk] &= clear;
+            atomicAnd((unsigned long long*)&rbits[lk], (unsigned long long)clear);  // races with k_ingest_bits
             if (sl < 0) pool_idx[lk] = (int32_t)j;
             pkey[j] = sl < 0 ? lk : -1;
         }

@@ -139,6 +139,7 @@ static void free_ctx(frugal_ctx* c) {
         if (c->n > 1) { F(q.T); F(q.Tmask); F(q.Tidx); F(q.nT); F(q.gl); F(q.goff); }
     }
     F(c->rows); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->long_tasks); F(c->owned_cnt); F(c->nb_rows); F(c->nb_p); F(c->nb_cnt);
+    for (int i = 0; i < 2; i++) { F(c->adj_rows[i]); F(c->adj_p[i]); F(c->adj_cnt[i]); }
     for (int i = 0; i < 2; i++) { F(c->bk_rows[i]); F(c->bk_p[i]); F(c->bk_off[i]); F(c->age_rows[i]); F(c->age_cnt[i]); }
     F(c->dstats); F(c->sched_info); F(c->ff_rows); F(c->ff_cnt); F(c->ids_stage);
     if (c->herr) cudaFreeHost(c->herr);
@@ -147,6 +148,10 @@ static void free_ctx(frugal_ctx* c) {
     sort_free(c->sort);
     scan_free(c->scan);
     if (c->side) cudaStreamDestroy(c->side);
+    if (c->istream) cudaStreamDestroy(c->istream);
+    if (c->ev_call) cudaEventDestroy(c->ev_call);
+    if (c->ev_copied) cudaEventDestroy(c->ev_copied);
+    for (auto e : c->ev_ingest) cudaEventDestroy(e);
     if (c->ev_sched) cudaEventDestroy(c->ev_sched);
     for (int i = 0; i < 2; i++) if (c->ev_side[i]) cudaEventDestroy(c->ev_side[i]);
     for (auto e : c->ev_pool) cudaEventDestroy(e);
@@ -199,6 +204,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->L = k.lookahead; c->D = k.age_out; c->M = k.batch * k.slots; c->N = k.n_rows;
     c->No = c->g < c->N ? (c->N - c->g + c->n - 1) / c->n : 0;
     c->P = c->D + 2;
+    c->QN = c->L + 2;
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 32;
     c->side_inline = getenv("FRUGAL_SIDE_INLINE") && atoi(getenv("FRUGAL_SIDE_INLINE"));
     c->capT = std::max<int64_t>(1, std::min<int64_t>((int64_t)c->n * c->M, c->No));
@@ -275,7 +281,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         c->dh_G = (float*)(dbase + off_G);
     }
     if (cudaHostAlloc((void**)&c->herr, 64, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess ||
-        cudaHostAlloc((void**)&c->counts_pin, (size_t)(c->L + 1) * c->n * 4, cudaHostAllocPortable) != cudaSuccess) {
+        cudaHostAlloc((void**)&c->counts_pin, (size_t)(c->L + 2) * c->n * 4, cudaHostAllocPortable) != cudaSuccess) {
         set_err("cudaHostAlloc(err/counts) failed");
         free_ctx(c);
         return FRUGAL_ENOMEM;
@@ -302,7 +308,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     DMALLOC(c->pw, (size_t)c->P * c->capT * rowb);
     DMALLOC(c->pkey, (size_t)c->P * c->capT * 4);
     DMALLOC(c->pcount, (size_t)c->P * 4);
-    c->q.resize(c->L + 1);
+    c->q.resize(c->QN);
     for (auto& q : c->q) {
         DMALLOC(q.ids, (size_t)c->n * c->M * 4);
         DMALLOC(q.counts, (size_t)c->n * 4);
@@ -336,6 +342,12 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     DMALLOC(c->nb_p, 2 * c->capT * 4);
     DMALLOC(c->nb_cnt, 4);
     for (int i = 0; i < 2; i++) {
+        DMALLOC(c->adj_rows[i], c->capT * 4);
+        DMALLOC(c->adj_p[i], c->capT * 4);
+        DMALLOC(c->adj_cnt[i], 4);
+        cudaMemset(c->adj_cnt[i], 0, 4);
+    }
+    for (int i = 0; i < 2; i++) {
         DMALLOC(c->bk_rows[i], 2 * c->capT * 4);
         DMALLOC(c->bk_p[i], 2 * c->capT * 4);
         DMALLOC(c->bk_off[i], 64 * 4);
@@ -359,9 +371,14 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     cudaDeviceGetStreamPriorityRange(&lo_prio, &hi_prio);
     CK(cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, lo_prio));  // lowest priority
     CK(cudaEventCreateWithFlags(&c->ev_sched, cudaEventDisableTiming));
+    CK(cudaStreamCreateWithFlags(&c->istream, cudaStreamNonBlocking));
+    CK(cudaEventCreateWithFlags(&c->ev_call, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&c->ev_copied, cudaEventDisableTiming));
     for (int i = 0; i < 2; i++) CK(cudaEventCreateWithFlags(&c->ev_side[i], cudaEventDisableTiming));
-    c->ev_counts.resize(c->L + 1);
+    c->ev_counts.resize(c->QN);
     for (auto& e : c->ev_counts) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    c->ev_ingest.resize(c->QN);
+    for (auto& e : c->ev_ingest) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
 
     cudaStream_t st = 0;
     if (cudaMemcpy(c->hot_lk, hot.data(), hot.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) {
@@ -415,30 +432,46 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
 }
 
 // ================================================================================ sample queue
-// ingest step t of all ranks into queue slot t % (L+1): convert + validate ids, own dedup,
-// owner-side T (world > 1), read-ring bits of step t and AdjustPriority inf -> t.
+// Ingest step t of all ranks into queue slot t % (L+2) on the ingest stream: copy + convert
+// + validate ids, own dedup, owner-side T (world > 1), read-ring bits of step t and
+// AdjustPriority inf -> t (into the adjust list consumed by frugal_step(t-L+1)).  The
+// ingest of step s+L runs one step ahead, overlapping step s's gather.
+// `after`: an event the ingest must follow (the scheduler of the current step).
 static frugal_status ingest(frugal_ctx* c, int64_t t, const int64_t* ids_all, const int32_t* counts, int adjust,
-                            cudaStream_t st) {
+                            cudaStream_t caller, cudaEvent_t after) {
     for (int r = 0; r < c->n; r++)
         if (counts[r] < 0 || counts[r] > c->B) {
             set_err("counts[%d] = %d outside [0, batch=%d]", r, counts[r], c->B);
             return FRUGAL_EINVAL;
         }
-    const int qi = (int)(t % (c->L + 1));
+    const int qi = (int)(t % c->QN);
     QueueSlot& q = c->q[qi];
     q.step = t;
     q.h_counts.assign(counts, counts + c->n);
-    // the pinned counts staging of this slot is reused only after its last copy ran
-    CK(cudaEventSynchronize(c->ev_counts[qi]));
+    cudaStream_t is = c->istream;
+    // the caller's buffer: copied after the caller's prior work, and the caller's later
+    // work is ordered after the copy (so it may reuse the buffer)
+    CK(cudaEventRecord(c->ev_call, caller));
+    CK(cudaStreamWaitEvent(is, c->ev_call, 0));
+    CK(cudaEventSynchronize(c->ev_counts[qi]));  // pinned counts staging of this slot is free
     int32_t* pin = c->counts_pin + (size_t)qi * c->n;
     memcpy(pin, counts, (size_t)c->n * 4);
-    CK(cudaMemcpyAsync(q.counts, pin, (size_t)c->n * 4, cudaMemcpyHostToDevice, st));
-    CK(cudaEventRecord(c->ev_counts[qi], st));
-    CK(cudaMemcpyAsync(c->ids_stage, ids_all, (size_t)c->n * c->M * 8, cudaMemcpyDefault, st));
-    launch_convert_ids(c, q, st);
-    launch_dedup(c, q, st);
-    if (c->n > 1) launch_owner_side(c, q, t, st);
-    launch_ingest_bits(c, q, t, adjust, st);
+    CK(cudaMemcpyAsync(q.counts, pin, (size_t)c->n * 4, cudaMemcpyHostToDevice, is));
+    CK(cudaEventRecord(c->ev_counts[qi], is));
+    CK(cudaMemcpyAsync(c->ids_stage, ids_all, (size_t)c->n * c->M * 8, cudaMemcpyDefault, is));
+    CK(cudaEventRecord(c->ev_copied, is));
+    CK(cudaStreamWaitEvent(caller, c->ev_copied, 0));
+    if (after) CK(cudaStreamWaitEvent(is, after, 0));
+    {
+        Timer tm(c, PH_INGEST, is);
+        launch_convert_ids(c, q, is);
+        launch_dedup(c, q, is);
+        if (c->n > 1) launch_owner_side(c, q, t, is);
+        const int apar = (int)((t - c->L + 1) & 1);  // consumed by frugal_step(t - L + 1)
+        CK(cudaMemsetAsync(c->adj_cnt[apar], 0, 4, is));
+        launch_ingest_bits(c, q, t, adjust, c->adj_rows[apar], c->adj_p[apar], c->adj_cnt[apar], is);
+    }
+    CK(cudaEventRecord(c->ev_ingest[qi], is));
     CKL();
     return FRUGAL_OK;
 }
@@ -446,14 +479,12 @@ static frugal_status ingest(frugal_ctx* c, int64_t t, const int64_t* ids_all, co
 extern "C" frugal_status frugal_prefetch(frugal_ctx* c, int64_t t, const int64_t* ids_all, const int32_t* counts,
                                          frugal_stream stream) {
     if (!c || !ids_all || !counts) { set_err("NULL argument"); return FRUGAL_EINVAL; }
-    if (c->cur_step != -1 || t != c->next_prefetch || t > c->L - 2) {
-        set_err("prefetch(%lld): expected t = %lld (only steps 0..L-2 before step 0)", (long long)t,
+    if (c->cur_step != -1 || t != c->next_prefetch || t > c->L - 1) {
+        set_err("prefetch(%lld): expected t = %lld (only steps 0..L-1 before step 0)", (long long)t,
                 (long long)c->next_prefetch);
         return FRUGAL_ESTATE;
     }
-    cudaStream_t st = (cudaStream_t)stream;
-    Timer tm(c, PH_INGEST, st);
-    frugal_status r = ingest(c, t, ids_all, counts, 0, st);
+    frugal_status r = ingest(c, t, ids_all, counts, 0, (cudaStream_t)stream, nullptr);
     if (r) return r;
     c->next_prefetch++;
     return check_err_word(c);
@@ -486,31 +517,30 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
                 c->phase_in_step);
         return FRUGAL_ESTATE;
     }
-    const int64_t t = s + c->L - 1;
+    const int64_t t = s + c->L;  // the step enqueued by this call (ingested during step s)
     if (ids_next_all) {
         if (c->ids_exhausted || c->next_prefetch != t || !counts_next) {
-            set_err("step(%lld): steps 0..%lld must be prefetched first (and counts given)", (long long)s,
+            set_err("step(%lld): steps 0..%lld must be enqueued first (and counts given)", (long long)s,
                     (long long)(t - 1));
             return FRUGAL_ESTATE;
         }
     } else {
-        c->ids_exhausted = true;
         if (c->next_prefetch <= s) { set_err("step(%lld) was never enqueued", (long long)s); return FRUGAL_ESTATE; }
     }
     cudaStream_t st = (cudaStream_t)stream;
     const int par = (int)(s & 1);
-    CK(cudaMemsetAsync(c->nb_cnt, 0, 4, st));
-    if (ids_next_all) {
-        Timer tm(c, PH_INGEST, st);
-        frugal_status r = ingest(c, t, ids_next_all, counts_next, 1, st);
-        if (r) return r;
-        c->next_prefetch++;
+    // the read bits of steps <= s+L-1 and the adjust list of this step are complete
+    {
+        const int64_t last = std::min<int64_t>(s + c->L - 1, c->next_prefetch - 1);
+        CK(cudaStreamWaitEvent(st, c->ev_ingest[last % c->QN], 0));
     }
+    CK(cudaMemsetAsync(c->nb_cnt, 0, 4, st));
+    if (s + c->L - 1 >= c->next_prefetch) CK(cudaMemsetAsync(c->adj_cnt[par], 0, 4, st));  // stream end: no adjust
     {
         Timer tm(c, PH_SCHED, st);
         QueueSlot* prev = nullptr;
         if (s >= 1) {
-            prev = &c->q[(s - 1) % (c->L + 1)];
+            prev = &c->q[(s - 1) % c->QN];
             if (prev->step != s - 1) { set_err("internal: queue slot of step %lld lost", (long long)(s - 1)); return FRUGAL_ESTATE; }
         }
         launch_bucket(c, prev, s, par, st);
@@ -540,6 +570,15 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
     }
     CK(cudaEventRecord(c->ev_side[par], c->side_inline ? st : c->side));
     c->side_pending[par] = true;
+    // a1/a2: ingest step s+L on the ingest stream, after this step's scheduler, so it
+    // overlaps the gate, the gather and the backward of step s
+    if (ids_next_all) {
+        frugal_status r = ingest(c, t, ids_next_all, counts_next, 1, st, c->ev_sched);
+        if (r) return r;
+        c->next_prefetch++;
+    } else {
+        c->ids_exhausted = true;
+    }
     {
         // a3: gate of step s -- PQ front > s: every owner's urgent bucket s and every
         // deferred bucket drained by its side stream at steps <= s-1
@@ -564,7 +603,7 @@ extern "C" frugal_status frugal_lookup(frugal_ctx* c, int64_t s, float* d_out, f
         return FRUGAL_ESTATE;
     }
     cudaStream_t st = (cudaStream_t)stream;
-    QueueSlot& q = c->q[s % (c->L + 1)];
+    QueueSlot& q = c->q[s % c->QN];
     {
         Timer tm(c, PH_GATHER, st);
         launch_gather(c, q, d_out, st);
@@ -586,7 +625,7 @@ extern "C" frugal_status frugal_dot_model(frugal_ctx* c, int64_t s, const float*
         return FRUGAL_ESTATE;
     }
     cudaStream_t st = (cudaStream_t)stream;
-    QueueSlot& q = c->q[s % (c->L + 1)];
+    QueueSlot& q = c->q[s % c->QN];
     int64_t nb = 0;
     for (int r = 0; r < c->n; r++) nb += q.h_counts[r];
     Timer tm(c, PH_MODEL, st);
@@ -602,7 +641,7 @@ extern "C" frugal_status frugal_backward_update(frugal_ctx* c, int64_t s, const 
         return FRUGAL_ESTATE;
     }
     cudaStream_t st = (cudaStream_t)stream;
-    QueueSlot& q = c->q[s % (c->L + 1)];
+    QueueSlot& q = c->q[s % c->QN];
     const int par = (int)(s & 1);
     {
         Timer tm(c, PH_SEGRED, st);
@@ -654,7 +693,7 @@ extern "C" const char* frugal_last_error(void) { return g_err.c_str(); }
 // ================================================================================ introspection
 extern "C" frugal_status frugal_get_dedup(frugal_ctx* c, int64_t t, int64_t* uniq, int32_t* inv, int64_t* n_uniq) {
     if (!c || !n_uniq) { set_err("NULL argument"); return FRUGAL_EINVAL; }
-    QueueSlot& q = c->q[t % (c->L + 1)];
+    QueueSlot& q = c->q[t % c->QN];
     if (t < 0 || q.step != t) { set_err("step %lld is not in the sample queue", (long long)t); return FRUGAL_EINVAL; }
     CK(cudaDeviceSynchronize());
     int32_t nu = 0;

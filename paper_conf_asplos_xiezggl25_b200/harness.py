@@ -1,8 +1,8 @@
 """Training-loop harness around the C ABI (used by tests, bench.py and smoke()).
 
 It only sequences the public calls of include/frugal.h for one rank:
-prefetch(0..L-2), then per step: step(s) -> lookup(s) -> dot_model(s) ->
-backward_update(s), and flush() at the end.  No arithmetic of the method
+prefetch(0..L-1), then per step: step(s) [enqueues step s+L] -> lookup(s) ->
+dot_model(s) -> backward_update(s), and flush() at the end.  No arithmetic of the method
 happens here.
 """
 from __future__ import annotations
@@ -37,12 +37,12 @@ class Trainer:
         self.loss = torch.zeros(st.steps, dtype=torch.float64, device=self.dev)
         self.s = 0
         L = fr.lookahead
-        for t in range(min(L - 1, st.steps)):
+        for t in range(min(L, st.steps)):
             fr.prefetch(t, st.ids[t], st.counts[t])
 
     def step(self, on_schedule=None):
         st, fr, s = self.st, self.fr, self.s
-        t = s + fr.lookahead - 1
+        t = s + fr.lookahead
         if t < st.steps:
             fr.step(s, st.ids[t], st.counts[t])
         else:

@@ -36,7 +36,7 @@ def run_parity(st, *, flags=None, mode=None, hot=None, check_dedup=True, check_s
     S = st.steps if steps is None else steps
     L = st.cfg.lookahead
     if check_dedup:
-        for t in range(min(L - 1, st.steps)):
+        for t in range(min(L, st.steps)):
             uq, inv = fr.get_dedup(t)
             ouq, oinv = o.dedup(t, 0)
             assert np.array_equal(uq, ouq) and np.array_equal(inv[:len(oinv)], oinv), f"dedup differs at {t}"
@@ -47,8 +47,8 @@ def run_parity(st, *, flags=None, mode=None, hot=None, check_dedup=True, check_s
         def cb(s_):
             if check_sched:
                 got.update(fr.get_schedule())
-            if check_dedup and s_ + L - 1 < st.steps:
-                t = s_ + L - 1
+            if check_dedup and s_ + L < st.steps:
+                t = s_ + L
                 uq, inv = fr.get_dedup(t)
                 ouq, oinv = o.dedup(t, 0)
                 assert np.array_equal(uq, ouq), f"uniq differs at step {t}"
@@ -210,5 +210,5 @@ def test_call_order_enforced():
         fr.lookup(0, out)
     assert e.value.status == -4
     with pytest.raises(F.FrugalError):
-        fr.step(0, st.ids[2], st.counts[2])  # steps 0..L-2 not prefetched yet
+        fr.step(0, st.ids[3], st.counts[3])  # steps 0..L-1 not prefetched yet
     fr.close()
