@@ -304,43 +304,50 @@ def main():
         return nbytes / (ms_ * 1e-3) / 1e9 if ms_ > 0 else None
 
     per = {}
-    # a4 gather: unique rows from host (zero-copy, PCIe H2D) -- the miss path
+    # Algorithmic bytes per unit, times the units the device counters saw.
+    # a4 gather: r per unique row served from the host table (zero-copy, PCIe H2D) -- the miss path
     per["gather"] = dict(bound="host-link h2d", bytes=cnt["gather_host"] * r / K,
                          hbm_bytes=(cnt["gather_cache"] + cnt["unique"]) * r / K, ms=ph["gather"],
                          peak=link["h2d"])
-    # a10 urgent flush (D2H, critical path), a11 side drain (D2H, side stream)
+    # a10 urgent flush (critical path) / a11 side drain: r per flushed row (w only, R8), D2H
     for nm, h, c_ in [("urgent", "urgent_hot", "urgent_cold"), ("side", "side_hot", "side_cold")]:
-        per[nm] = dict(bound="host-link d2h", bytes=(cnt[h] * r + cnt[c_] * r * (2 if adag else 1)) / K,
-                       ms=ph[nm], peak=link["d2h"])
-    # a4 expand: out[i] = rows[inv[i]] -- HBM write of M rows + read of rows/inv
+        per[nm] = dict(bound="host-link d2h", bytes=(cnt[h] + cnt[c_]) * r / K, ms=ph[nm], peak=link["d2h"])
+    # a4 expand: out[i] = rows[inv[i]]: write r + read r + 4 B index per position
     per["expand"] = dict(bound="hbm", bytes=(cnt["positions"] * (2 * r + 4)) / K, ms=ph["expand"], peak=hbm_peak)
-    # a6 segment-reduce: read M grad rows + pos, write U partial rows + offsets
+    # a6 segment-reduce: read r + 4 B per position, write r + 4 B per unique row
     per["segred"] = dict(bound="hbm", bytes=(cnt["positions"] * (r + 4) + cnt["unique"] * (r + 4)) / K,
                          ms=ph["segred"], peak=hbm_peak)
-    # a8 optimizer: hot rows r/w (w,G) in HBM; cold rows read G over the link (+w when N>1)
-    per["optimizer"] = dict(bound="host-link h2d",
-                            bytes=cnt["opt_cold"] * r * ((1 if world == 1 else 2) if adag else (0 if world == 1 else 1)) / K,
-                            hbm_bytes=(cnt["opt_hot"] * r * (4 if adag else 2) + cnt["opt_cold"] * r * (3 if adag else 2)
-                                       + (cnt["opt_hot"] + cnt["opt_cold"]) * r) / K,
-                            ms=ph["optimizer"], peak=link["h2d"])
+    # a8 optimizer: per touched owned row: partial r, w r (cache / staged rows), G r+r, w out r,
+    # + 28 B metadata; cold rows of other ranks' reads come over the link when N > 1
+    touched = cnt["opt_hot"] + cnt["opt_cold"]
+    per["optimizer"] = dict(bound="hbm", bytes=touched * (5 * r + 28) / K,
+                            link_bytes=(cnt["opt_cold"] * r + cnt["mail_in"] * r) / K if world > 1 else 0.0,
+                            ms=ph["optimizer"], peak=hbm_peak)
+    # a5 glue: read r per position (embeddings, register-cached), write r (grads), x per sample
+    per["model"] = dict(bound="hbm", bytes=(cnt["positions"] * 2 * r + B * (r + 4)) / K, ms=ph["model"],
+                        peak=hbm_peak)
     for k, v in per.items():
         v["achieved_gbs"] = gbs(v["bytes"], v["ms"])
         v["frac"] = v["achieved_gbs"] / v["peak"] if v["achieved_gbs"] else None
     main_ms = {k: v for k, v in ph.items() if k != "side"}
-    dom = max(("gather", "urgent", "expand", "segred", "optimizer"), key=lambda k: per[k]["ms"])
+    dom = max(("gather", "urgent", "expand", "segred", "optimizer", "model"), key=lambda k: per[k]["ms"])
     top = max(main_ms, key=main_ms.get)
     D = per[dom]
-    traffic = None
-    try:
-        prof = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
-        traffic = prof.get(dom, {}).get("dram_bytes_per_launch")
+    traffic, tnote = None, None
+    try:  # committed ncu --set full capture (profiles/, tools/ncu_summary.py)
+        prof = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json"))).get(dom, {})
+        traffic = prof.get("traffic_bytes_per_launch")
+        if traffic is not None:
+            tnote = (f"{prof['traffic_kind']} per launch of {prof['kernel']} in profiles/r1_ncu_full_summary.txt "
+                     f"(a warm-up-phase launch; its own algorithmic sysmem bytes: {prof['sysmem_bytes_per_launch']:.0f})")
     except Exception:
         pass
     roofline = {"bound": "hbm" if D["bound"] == "hbm" else "host-link", "kernel": dom,
                 "achieved": D["achieved_gbs"], "peak": D["peak"], "unit": "GB/s", "frac": D["frac"],
-                "traffic": traffic,
-                "peak_source": ("measured pinned cudaMemcpy H2D/D2H 256 MiB in this run" if D["bound"] != "hbm"
-                                else "MEASURED_PEAKS.json hbm_gbs")}
+                "traffic": traffic, "traffic_note": tnote,
+                "peak_source": ("measured pinned cudaMemcpy (256 MiB, best of 5) in this run; random 128-B rows "
+                                "measure 12-33 GB/s on this box (profiles/r1_zc_probe_*.txt)" if D["bound"] != "hbm"
+                                else "MEASURED_PEAKS.json hbm_gbs (burst)")}
     launches = st1["kernel_launches"] - st0["kernel_launches"]
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

@@ -178,8 +178,9 @@ frugal_status frugal_read_host(frugal_ctx* ctx, const int64_t* ids, int64_t n, f
    FRUGAL_F_TIMERS; CUDA events on the phase's stream).  Phases, in order: ingest (a1+a2),
    schedule (a9), urgent (a10), gate (a3), gather (a4, unique rows), expand (a4, per
    position), model (a5), segred (a6), exchange (a7), optimizer (a8), side (a11, side
-   stream).  Device counters are cumulative since init (always on; one atomic per block). */
-#define FRUGAL_N_PHASES 11
+   stream), prefetch (a4, the early part of the next step's gather, prefetch stream).
+   Device counters are cumulative since init (always on; one atomic per block). */
+#define FRUGAL_N_PHASES 12
 enum {
     FRUGAL_C_POSITIONS = 0,     /* lookups (positions) of this rank                         */
     FRUGAL_C_UNIQUE = 1,        /* distinct rows of this rank (sum over steps)               */

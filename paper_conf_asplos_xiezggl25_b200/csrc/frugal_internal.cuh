@@ -64,6 +64,11 @@ struct QueueSlot {
     uint32_t* Tmask = nullptr; // [capT] rank mask
     int32_t* Tidx = nullptr;   // [world][capT] index of T[j] in rank r's owner segment
     int32_t* nT = nullptr;     // device scalar
+    // gather split (world 1): uniq indices whose row was not read at t-1 ("early": can be
+    // gathered during step t-1) and the rest ("late": after gate t)
+    int32_t* eidx = nullptr;   // [M]
+    int32_t* lidx = nullptr;   // [M]
+    int32_t* elcnt = nullptr;  // [2] early, late counts
     // sender side grouping (world > 1): uniq positions grouped by owner
     int32_t* gl = nullptr;     // [M] grouped position -> uniq index
     int32_t* goff = nullptr;   // [world+1]
@@ -85,7 +90,9 @@ struct frugal_ctx {
     int P;                       // pool segments = D + 2
     int QN;                      // sample-queue slots = L + 2 (steps s-1 .. s+L)
     int side_blocks = 32;        // grid cap of the side-stream drain
+    int gather_blocks = 296;     // grid cap of the zero-copy gathers
     bool side_inline = false;    // experiment: drain on the caller stream
+    bool drain_after_gather = false;  // side drain ordered after the step's gather (FRUGAL_DRAIN_AT=gather)
     int64_t capT;                // max owned rows touched per step
     int key_bits, lk_bits;       // bits of global ids / local ids
 
@@ -127,7 +134,7 @@ struct frugal_ctx {
     std::vector<frugal::QueueSlot> q;
 
     // per-step scratch
-    float* rows = nullptr;  // [M][d] gathered unique rows
+    float* rows_buf[2] = {nullptr, nullptr};  // [M][d] gathered unique rows, by step parity
     float* Pp = nullptr;    // [M][d] partials (grouped order for world > 1)
     float* chunk_scratch = nullptr;  // [M][d] chunk sums of long segments
     int32_t* long_q = nullptr;       // [M] long segments of the current step
@@ -160,10 +167,17 @@ struct frugal_ctx {
 
     cudaStream_t side = nullptr;
     cudaStream_t istream = nullptr;  // sample-queue ingest, one step ahead
-    cudaEvent_t ev_call = nullptr, ev_copied = nullptr;
+    cudaEvent_t ev_call = nullptr, ev_copied = nullptr, ev_gathered = nullptr;
     std::vector<cudaEvent_t> ev_ingest;  // per queue slot: ingest complete
     cudaEvent_t ev_sched = nullptr;
     cudaEvent_t ev_side[2] = {nullptr, nullptr};
+    cudaEvent_t ev_side_first[2] = {nullptr, nullptr};  // side drain of the next step's deadline done
+    cudaStream_t pstream = nullptr;                     // early gather of the next step
+    cudaEvent_t ev_early[2] = {nullptr, nullptr};
+    cudaEvent_t ev_opt[2] = {nullptr, nullptr};         // optimizer of a step done (rows_buf free)
+    bool opt_pending[2] = {false, false};
+    int64_t early_issued = -1;                          // last step whose early gather was launched
+    bool early = false;                                 // pipelined gather enabled (world 1)
     bool side_pending[2] = {false, false};
 
     // call-order state
@@ -195,8 +209,9 @@ void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, int3
 void launch_bucket(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStream_t st);
 void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begin, const int32_t* d_end,
                        int max_blocks, int counter, cudaStream_t st);
-void launch_gather(frugal_ctx* c, QueueSlot& q, float* out, cudaStream_t st);
-void launch_expand(frugal_ctx* c, QueueSlot& q, float* out, cudaStream_t st);
+void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32_t* cnt, float* rows, cudaStream_t st);
+void launch_expand(frugal_ctx* c, QueueSlot& q, const float* rows, float* out, cudaStream_t st);
+void launch_split_early(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st);
 void launch_mail_header(frugal_ctx* c, QueueSlot& q, int par, cudaStream_t st);
 void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const float* x, const float* y,
                       float* grad, double* loss, int64_t nb, cudaStream_t st);

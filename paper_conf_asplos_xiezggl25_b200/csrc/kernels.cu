@@ -713,17 +713,20 @@ void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begi
     c->launches++;
 }
 
-// a4 gather: unique rows -> staging (owned hot: HBM cache; else host, zero-copy)
+// a4 gather: unique rows -> staging (owned hot: HBM cache; else host, zero-copy).
+// list: the uniq indices to gather (early or late part), cnt: its device count.
 template <int GS>
-__global__ void k_gather_uniq(const int32_t* __restrict__ uniq, const int32_t* d_nu, int world, int g, int d4,
-                              const int32_t* __restrict__ slot, const float4* __restrict__ cw,
-                              const float4* hw, float4* __restrict__ rows, unsigned long long* stats) {
+__global__ void k_gather_uniq(const int32_t* __restrict__ uniq, const int32_t* __restrict__ list, const int32_t* cnt,
+                              int world, int g, int d4, const int32_t* __restrict__ slot,
+                              const float4* __restrict__ cw, const float4* hw, float4* __restrict__ rows,
+                              unsigned long long* stats) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
-    const int n = *d_nu;
+    const int n = *cnt;
     unsigned nh = 0, nc = 0;
-    for (int64_t u = gid; u < n; u += gs) {
+    for (int64_t a = gid; a < n; a += gs) {
+        const int u = list ? list[a] : (int)a;
         int32_t k = uniq[u];
         const float4* src = hw + (int64_t)k * d4;
         bool cached = false;
@@ -738,7 +741,7 @@ __global__ void k_gather_uniq(const int32_t* __restrict__ uniq, const int32_t* d
             if (cached) nc++;
             else nh++;
         }
-        for (int v = l; v < d4; v += GS) rows[u * d4 + v] = src[v];
+        for (int v = l; v < d4; v += GS) rows[(int64_t)u * d4 + v] = src[v];
     }
     block_count(stats + FRUGAL_C_GATHER_HOST, nh);
     block_count(stats + FRUGAL_C_GATHER_CACHE, nc);
@@ -757,19 +760,53 @@ __global__ void k_expand(const int32_t* __restrict__ inv, const int32_t* d_m, in
     }
 }
 
-void launch_gather(frugal_ctx* c, QueueSlot& q, float* out, cudaStream_t st) {
+void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32_t* cnt, float* rows,
+                   cudaStream_t st) {
     const int d4 = c->d / 4, gs = group_size(d4);
-    int grid = grid_for((int64_t)c->M * gs, 256, 8);
-    DISPATCH_GS(gs, (k_gather_uniq<GS><<<grid, 256, 0, st>>>(q.uniq, q.n_uniq, c->n, c->g, d4, c->slot,
+    // zero-copy host loads are latency-bound: ~148x256 threads already keep the link's
+    // read requests in flight (tools/zc_probe: 148 vs 1184 CTAs, same GB/s), and a
+    // bigger grid only parks stalled warps on SMs other streams need
+    int grid = std::min(grid_for((int64_t)c->M * gs, 256, 8), c->gather_blocks);
+    DISPATCH_GS(gs, (k_gather_uniq<GS><<<grid, 256, 0, st>>>(q.uniq, list, cnt, c->n, c->g, d4, c->slot,
                                                              (const float4*)c->cw, (const float4*)c->dh_w,
-                                                             (float4*)c->rows, c->dstats)));
+                                                             (float4*)rows, c->dstats)));
     c->launches++;
 }
-void launch_expand(frugal_ctx* c, QueueSlot& q, float* out, cudaStream_t st) {
+void launch_expand(frugal_ctx* c, QueueSlot& q, const float* rows, float* out, cudaStream_t st) {
     const int d4 = c->d / 4, gs = group_size(d4);
     int grid = grid_for((int64_t)c->M * gs, 256, 8);
-    DISPATCH_GS(gs, (k_expand<GS><<<grid, 256, 0, st>>>(q.inv, q.m, d4, (const float4*)c->rows,
-                                                        (float4*)out)));
+    DISPATCH_GS(gs, (k_expand<GS><<<grid, 256, 0, st>>>(q.inv, q.m, d4, (const float4*)rows, (float4*)out)));
+    c->launches++;
+}
+
+// world 1: split uniq(t) into rows not read at t-1 (early) and rows read at t-1 (late;
+// they are updated at t-1 and may be urgent at t).  Read-ring bit t-1 is still set: it is
+// cleared by the optimizer of step t-1, which runs after this ingest (one step ahead).
+__global__ void k_split_early(const int32_t* __restrict__ uniq, const int32_t* d_nu, int64_t t,
+                              const uint64_t* __restrict__ rbits, int32_t* eidx, int32_t* lidx, int32_t* elcnt) {
+    const int n = *d_nu;
+    const int nloop = (n + blockDim.x * gridDim.x - 1) / (blockDim.x * gridDim.x) * (blockDim.x * gridDim.x);
+    const uint64_t bit = t > 0 ? (1ull << ((t - 1) & 31)) : 0ull;
+    for (int u = blockIdx.x * blockDim.x + threadIdx.x; u < nloop; u += gridDim.x * blockDim.x) {
+        bool valid = u < n;
+        bool late = valid && (rbits[uniq[valid ? u : 0]] & bit);
+        bool early = valid && !late;
+        unsigned me = __ballot_sync(FULL, early), ml = __ballot_sync(FULL, late);
+        const int lane = threadIdx.x & 31;
+        int be = 0, bl = 0;
+        if (lane == 0) {
+            if (me) be = atomicAdd(&elcnt[0], __popc(me));
+            if (ml) bl = atomicAdd(&elcnt[1], __popc(ml));
+        }
+        be = __shfl_sync(FULL, be, 0);
+        bl = __shfl_sync(FULL, bl, 0);
+        if (early) eidx[be + __popc(me & lanemask_lt())] = u;
+        if (late) lidx[bl + __popc(ml & lanemask_lt())] = u;
+    }
+}
+void launch_split_early(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st) {
+    cudaMemsetAsync(q.elcnt, 0, 8, st);
+    k_split_early<<<grid_for(c->M, 256, 4), 256, 0, st>>>(q.uniq, q.n_uniq, t, c->rbits, q.eidx, q.lidx, q.elcnt);
     c->launches++;
 }
 

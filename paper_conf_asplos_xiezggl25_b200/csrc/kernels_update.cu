@@ -324,7 +324,7 @@ void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, cudaStrea
     const char* mail_par = c->n > 1 ? c->dh_mail + (size_t)par * c->n * c->mail_stride : nullptr;
     // world == 1: the owner gathered every touched row itself this step (T == uniq),
     // so the cold rows' w is taken from the staging rows instead of a second host read.
-    const float4* rows_w = c->n == 1 ? (const float4*)c->rows : nullptr;
+    const float4* rows_w = c->n == 1 ? (const float4*)c->rows_buf[s & 1] : nullptr;
     DISPATCH_GS(gs, (k_optimizer<GS><<<grid, 256, 0, st>>>(
                         q.T, q.nT, q.Tmask, q.Tidx, c->capT, c->n, c->g, d4, (int32_t)s, adag, c->cfg.lr, c->cfg.eps,
                         (const float4*)c->Pp, q.goff, mail_par, c->mail_stride, rows_w, c->slot, c->state,

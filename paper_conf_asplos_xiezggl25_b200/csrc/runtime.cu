@@ -60,7 +60,8 @@ constexpr uint64_t kMagic = 0x46525547414c3235ULL;  // "FRUGAL25"
 constexpr size_t kHdr = 4096;
 constexpr size_t kFlags = 8192;  // 3 kinds x 32 ranks x 64 B
 enum { FLAG_URGENT = 0, FLAG_SIDE = 1, FLAG_MAIL = 2 };
-enum { PH_INGEST, PH_SCHED, PH_URGENT, PH_GATE, PH_GATHER, PH_EXPAND, PH_MODEL, PH_SEGRED, PH_EXCH, PH_OPT, PH_SIDE };
+enum { PH_INGEST, PH_SCHED, PH_URGENT, PH_GATE, PH_GATHER, PH_EXPAND, PH_MODEL, PH_SEGRED, PH_EXCH, PH_OPT, PH_SIDE,
+       PH_PREFETCH };
 
 struct ShmHeader {
     uint64_t magic;
@@ -135,10 +136,11 @@ static void free_ctx(frugal_ctx* c) {
     F(c->slot); F(c->state); F(c->last_upd); F(c->pool_idx); F(c->rbits);
     F(c->cw); F(c->Gd); F(c->hot_lk); F(c->pw); F(c->pkey); F(c->pcount);
     for (auto& q : c->q) {
+        F(q.eidx); F(q.lidx); F(q.elcnt);
         F(q.ids); F(q.counts); F(q.m); F(q.uniq); F(q.inv); F(q.off); F(q.pos); F(q.n_uniq);
         if (c->n > 1) { F(q.T); F(q.Tmask); F(q.Tidx); F(q.nT); F(q.gl); F(q.goff); }
     }
-    F(c->rows); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->long_tasks); F(c->owned_cnt); F(c->nb_rows); F(c->nb_p); F(c->nb_cnt);
+    F(c->rows_buf[0]); F(c->rows_buf[1]); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->long_tasks); F(c->owned_cnt); F(c->nb_rows); F(c->nb_p); F(c->nb_cnt);
     for (int i = 0; i < 2; i++) { F(c->adj_rows[i]); F(c->adj_p[i]); F(c->adj_cnt[i]); }
     for (int i = 0; i < 2; i++) { F(c->bk_rows[i]); F(c->bk_p[i]); F(c->bk_off[i]); F(c->age_rows[i]); F(c->age_cnt[i]); }
     F(c->dstats); F(c->sched_info); F(c->ff_rows); F(c->ff_cnt); F(c->ids_stage);
@@ -151,9 +153,16 @@ static void free_ctx(frugal_ctx* c) {
     if (c->istream) cudaStreamDestroy(c->istream);
     if (c->ev_call) cudaEventDestroy(c->ev_call);
     if (c->ev_copied) cudaEventDestroy(c->ev_copied);
+    if (c->ev_gathered) cudaEventDestroy(c->ev_gathered);
     for (auto e : c->ev_ingest) cudaEventDestroy(e);
     if (c->ev_sched) cudaEventDestroy(c->ev_sched);
-    for (int i = 0; i < 2; i++) if (c->ev_side[i]) cudaEventDestroy(c->ev_side[i]);
+    for (int i = 0; i < 2; i++) {
+        if (c->ev_side[i]) cudaEventDestroy(c->ev_side[i]);
+        if (c->ev_side_first[i]) cudaEventDestroy(c->ev_side_first[i]);
+        if (c->ev_early[i]) cudaEventDestroy(c->ev_early[i]);
+        if (c->ev_opt[i]) cudaEventDestroy(c->ev_opt[i]);
+    }
+    if (c->pstream) cudaStreamDestroy(c->pstream);
     for (auto e : c->ev_pool) cudaEventDestroy(e);
     if (c->shm_base) {
         cudaHostUnregister(c->shm_base);
@@ -205,8 +214,13 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->No = c->g < c->N ? (c->N - c->g + c->n - 1) / c->n : 0;
     c->P = c->D + 2;
     c->QN = c->L + 2;
+    // pipelined early gather (world 1): off by default -- measured no gain on a PCIe-bound
+    // box (the zero-copy loads of the next step only delay this step's); FRUGAL_EARLY=1
+    c->early = c->n == 1 && getenv("FRUGAL_EARLY") && atoi(getenv("FRUGAL_EARLY"));
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 32;
+    c->gather_blocks = getenv("FRUGAL_GATHER_BLOCKS") ? atoi(getenv("FRUGAL_GATHER_BLOCKS")) : 296;
     c->side_inline = getenv("FRUGAL_SIDE_INLINE") && atoi(getenv("FRUGAL_SIDE_INLINE"));
+    c->drain_after_gather = getenv("FRUGAL_DRAIN_AT") && !strcmp(getenv("FRUGAL_DRAIN_AT"), "gather");
     c->capT = std::max<int64_t>(1, std::min<int64_t>((int64_t)c->n * c->M, c->No));
     c->key_bits = bits_for(c->N - 1);
     c->lk_bits = bits_for(std::max<int64_t>(c->No - 1, 0));
@@ -318,6 +332,9 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         DMALLOC(q.off, ((size_t)c->M + 1) * 4);
         DMALLOC(q.pos, (size_t)c->M * 4);
         DMALLOC(q.n_uniq, 4);
+        DMALLOC(q.eidx, (size_t)c->M * 4);
+        DMALLOC(q.lidx, (size_t)c->M * 4);
+        DMALLOC(q.elcnt, 8);
         if (c->n > 1) {
             DMALLOC(q.T, c->capT * 4);
             DMALLOC(q.Tmask, c->capT * 4);
@@ -331,7 +348,8 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         }
         q.h_counts.assign(c->n, 0);
     }
-    DMALLOC(c->rows, (size_t)c->M * rowb);
+    DMALLOC(c->rows_buf[0], (size_t)c->M * rowb);
+    DMALLOC(c->rows_buf[1], (size_t)c->M * rowb);
     DMALLOC(c->Pp, (size_t)c->M * rowb);
     DMALLOC(c->chunk_scratch, (size_t)c->M * rowb);
     DMALLOC(c->long_q, (size_t)c->M * 4);
@@ -369,12 +387,27 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     }
     int lo_prio, hi_prio;
     cudaDeviceGetStreamPriorityRange(&lo_prio, &hi_prio);
-    CK(cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, lo_prio));  // lowest priority
+    // side-stream priority (FRUGAL_SIDE_PRIO=low|normal|high): low by default; measured
+    // within noise of the others on a PCIe-bound step
+    {
+        const char* sp = getenv("FRUGAL_SIDE_PRIO");
+        int prio = lo_prio;
+        if (sp && !strcmp(sp, "high")) prio = hi_prio;
+        if (sp && !strcmp(sp, "normal")) prio = 0;
+        CK(cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, prio));
+    }
     CK(cudaEventCreateWithFlags(&c->ev_sched, cudaEventDisableTiming));
     CK(cudaStreamCreateWithFlags(&c->istream, cudaStreamNonBlocking));
     CK(cudaEventCreateWithFlags(&c->ev_call, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&c->ev_copied, cudaEventDisableTiming));
-    for (int i = 0; i < 2; i++) CK(cudaEventCreateWithFlags(&c->ev_side[i], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&c->ev_gathered, cudaEventDisableTiming));
+    for (int i = 0; i < 2; i++) {
+        CK(cudaEventCreateWithFlags(&c->ev_side[i], cudaEventDisableTiming));
+        CK(cudaEventCreateWithFlags(&c->ev_side_first[i], cudaEventDisableTiming));
+        CK(cudaEventCreateWithFlags(&c->ev_early[i], cudaEventDisableTiming));
+        CK(cudaEventCreateWithFlags(&c->ev_opt[i], cudaEventDisableTiming));
+    }
+    CK(cudaStreamCreateWithPriority(&c->pstream, cudaStreamNonBlocking, hi_prio));
     c->ev_counts.resize(c->QN);
     for (auto& e : c->ev_counts) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     c->ev_ingest.resize(c->QN);
@@ -470,6 +503,7 @@ static frugal_status ingest(frugal_ctx* c, int64_t t, const int64_t* ids_all, co
         const int apar = (int)((t - c->L + 1) & 1);  // consumed by frugal_step(t - L + 1)
         CK(cudaMemsetAsync(c->adj_cnt[apar], 0, 4, is));
         launch_ingest_bits(c, q, t, adjust, c->adj_rows[apar], c->adj_p[apar], c->adj_cnt[apar], is);
+        if (c->early) launch_split_early(c, q, t, is);
     }
     CK(cudaEventRecord(c->ev_ingest[qi], is));
     CKL();
@@ -507,6 +541,54 @@ static void record_schedule(frugal_ctx* c, int par, cudaStream_t st) {
     c->rec_deferred_p.assign(ps.begin() + off[1], ps.end());
     c->rec_ageout = age;
     c->rec_gate_wait = off[1] > 0;
+}
+
+// a4 (pipelined, world 1): gather the rows of step u that were not read at u-1 into
+// rows_buf[u&1] on the prefetch stream, once (i) the ingest of u is done, (ii) the side
+// stream has drained every flush with deadline u, (iii) the optimizer of u-2 released
+// rows_buf[u&1].  None of these rows is updated at u-1, so the host table / cache already
+// hold their step-u values (invariant (2)); the rest is gathered after gate u.
+static frugal_status launch_early_gather(frugal_ctx* c, int64_t u, cudaEvent_t side_first) {
+    QueueSlot& q = c->q[u % c->QN];
+    cudaStream_t ps = c->pstream;
+    CK(cudaStreamWaitEvent(ps, c->ev_ingest[u % c->QN], 0));
+    if (side_first) CK(cudaStreamWaitEvent(ps, side_first, 0));
+    if (c->opt_pending[u & 1]) CK(cudaStreamWaitEvent(ps, c->ev_opt[u & 1], 0));
+    {
+        Timer tm(c, PH_PREFETCH, ps);
+        launch_gather(c, q, q.eidx, q.elcnt, c->rows_buf[u & 1], ps);
+    }
+    CK(cudaEventRecord(c->ev_early[u & 1], ps));
+    c->early_issued = u;
+    CKL();
+    return FRUGAL_OK;
+}
+
+// a11: deferred buckets (priorities s+1 .. s+L-1, ascending) and age-outs of step s on the
+// side stream, after `after` (the scheduler, or -- default -- the step's gather, so the
+// zero-copy stores of the drain do not compete with the zero-copy loads of the gather:
+// measured, a concurrent random gather and scatter over PCIe take longer than the two in
+// sequence).  Deadline s+1 is drained first; the next step's early gather
+// waits only for that part.
+static frugal_status launch_drain(frugal_ctx* c, int64_t s, cudaStream_t st, cudaEvent_t after) {
+    const int par = (int)(s & 1);
+    cudaStream_t sd = c->side_inline ? st : c->side;
+    if (!c->side_inline) CK(cudaStreamWaitEvent(c->side, after, 0));
+    static const bool no_drain = getenv("FRUGAL_EXPERIMENT_NO_DRAIN") != nullptr;  // WRONG RESULTS: upper bound only
+    if (!no_drain) {
+        Timer tm(c, PH_SIDE, sd);
+        launch_flush_rows(c, c->bk_rows[par], c->bk_off[par] + 1, c->bk_off[par] + 2, c->side_blocks,
+                          FRUGAL_C_SIDE_HOT, sd);
+        CK(cudaEventRecord(c->ev_side_first[par], sd));
+        launch_flush_rows(c, c->bk_rows[par], c->bk_off[par] + 2, c->bk_off[par] + c->L, c->side_blocks,
+                          FRUGAL_C_SIDE_HOT, sd);
+        launch_flush_rows(c, c->age_rows[par], nullptr, c->age_cnt[par], c->side_blocks, FRUGAL_C_SIDE_HOT, sd);
+        if (c->n > 1) launch_set_flag(c, FLAG_SIDE, (uint32_t)(s + 1), sd);
+        CKL();
+    }
+    CK(cudaEventRecord(c->ev_side[par], sd));
+    c->side_pending[par] = true;
+    return FRUGAL_OK;
 }
 
 extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* ids_next_all, const int32_t* counts_next,
@@ -554,22 +636,11 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
         if (c->n > 1) launch_set_flag(c, FLAG_URGENT, (uint32_t)(s + 1), st);
         CKL();
     }
-    // a11: deferred buckets (priorities s+1 .. s+L-1, ascending) and age-outs on the side stream
     CK(cudaEventRecord(c->ev_sched, st));
-    CK(cudaStreamWaitEvent(c->side, c->ev_sched, 0));
-    {
-        // FRUGAL_SIDE_INLINE=1 (experiments): drain on the caller's stream instead
-        cudaStream_t sd = c->side_inline ? st : c->side;
-        Timer tm(c, PH_SIDE, sd);
-        // bounded grid: the drain trickles over the step instead of crowding out the main stream
-        launch_flush_rows(c, c->bk_rows[par], c->bk_off[par] + 1, c->bk_off[par] + c->L, c->side_blocks,
-                          FRUGAL_C_SIDE_HOT, sd);
-        launch_flush_rows(c, c->age_rows[par], nullptr, c->age_cnt[par], c->side_blocks, FRUGAL_C_SIDE_HOT, sd);
-        if (c->n > 1) launch_set_flag(c, FLAG_SIDE, (uint32_t)(s + 1), sd);
-        CKL();
+    if (!c->drain_after_gather) {
+        frugal_status r = launch_drain(c, s, st, c->ev_sched);
+        if (r) return r;
     }
-    CK(cudaEventRecord(c->ev_side[par], c->side_inline ? st : c->side));
-    c->side_pending[par] = true;
     // a1/a2: ingest step s+L on the ingest stream, after this step's scheduler, so it
     // overlaps the gate, the gather and the backward of step s
     if (ids_next_all) {
@@ -578,6 +649,14 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
         c->next_prefetch++;
     } else {
         c->ids_exhausted = true;
+    }
+    if (c->early && c->early_issued < s) {  // step 0: nothing precedes it
+        frugal_status r = launch_early_gather(c, s, nullptr);
+        if (r) return r;
+    }
+    if (c->early && !c->drain_after_gather && s + 1 < c->next_prefetch) {
+        frugal_status r = launch_early_gather(c, s + 1, c->ev_side_first[par]);
+        if (r) return r;
     }
     {
         // a3: gate of step s -- PQ front > s: every owner's urgent bucket s and every
@@ -604,13 +683,28 @@ extern "C" frugal_status frugal_lookup(frugal_ctx* c, int64_t s, float* d_out, f
     }
     cudaStream_t st = (cudaStream_t)stream;
     QueueSlot& q = c->q[s % c->QN];
+    float* rows = c->rows_buf[s & 1];
     {
         Timer tm(c, PH_GATHER, st);
-        launch_gather(c, q, d_out, st);
+        if (c->early) {
+            CK(cudaStreamWaitEvent(st, c->ev_early[s & 1], 0));
+            launch_gather(c, q, q.lidx, q.elcnt + 1, rows, st);  // rows read at s-1 (updated then)
+        } else {
+            launch_gather(c, q, nullptr, q.n_uniq, rows, st);
+        }
+    }
+    if (c->drain_after_gather) {
+        CK(cudaEventRecord(c->ev_gathered, st));
+        frugal_status r = launch_drain(c, s, st, c->ev_gathered);
+        if (r) return r;
+        if (c->early && s + 1 < c->next_prefetch) {
+            r = launch_early_gather(c, s + 1, c->ev_side_first[s & 1]);
+            if (r) return r;
+        }
     }
     {
         Timer tm(c, PH_EXPAND, st);
-        launch_expand(c, q, d_out, st);
+        launch_expand(c, q, rows, d_out, st);
     }
     CKL();
     c->phase_in_step = 2;
@@ -659,6 +753,8 @@ extern "C" frugal_status frugal_backward_update(frugal_ctx* c, int64_t s, const 
         Timer tm(c, PH_OPT, st);
         launch_optimizer(c, q, s, par, st);
     }
+    CK(cudaEventRecord(c->ev_opt[s & 1], st));
+    c->opt_pending[s & 1] = true;
     CKL();
     c->phase_in_step = 0;
     c->timed_steps++;

@@ -20,7 +20,7 @@ MODE_P2F, MODE_WRITE_THROUGH = 0, 1
 F_RECORD, F_TIMERS = 1, 2
 FLUSH_ALL = 0
 PHASES = ["ingest", "schedule", "urgent", "gate", "gather", "expand", "model", "segred", "exchange",
-          "optimizer", "side"]
+          "optimizer", "side", "prefetch"]
 _STATUS = {0: "FRUGAL_OK", -1: "FRUGAL_EINVAL", -2: "FRUGAL_ENOMEM", -3: "FRUGAL_ECUDA",
            -4: "FRUGAL_ESTATE", -5: "FRUGAL_ETIMEOUT", -6: "FRUGAL_ESHM"}
 
@@ -51,7 +51,7 @@ COUNTERS = ["positions", "unique", "gather_host", "gather_cache", "opt_hot", "op
 
 
 class Stats(C.Structure):
-    _fields_ = [("ms", C.c_double * 11), ("steps", C.c_int64), ("kernel_launches", C.c_int64),
+    _fields_ = [("ms", C.c_double * 12), ("steps", C.c_int64), ("kernel_launches", C.c_int64),
                 ("count", C.c_int64 * 16)]
 
 

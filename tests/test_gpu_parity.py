@@ -212,3 +212,22 @@ def test_call_order_enforced():
     with pytest.raises(F.FrugalError):
         fr.step(0, st.ids[3], st.counts[3])  # steps 0..L-1 not prefetched yet
     fr.close()
+
+
+@pytest.mark.parametrize("env", [{"FRUGAL_EARLY": "1"}, {"FRUGAL_DRAIN_AT": "gather"},
+                                 {"FRUGAL_EARLY": "1", "FRUGAL_DRAIN_AT": "gather"}, {"FRUGAL_SIDE_INLINE": "1"}])
+def test_pipeline_modes_parity(env):
+    """The optional schedules (early gather of the next step, drain after the gather,
+    inline drain) keep every artefact bit-exact (run in a subprocess: the knobs are read
+    at context creation)."""
+    import subprocess
+    import sys
+    code = ("import sys; sys.path.insert(0, '.');"
+            "from tests.test_gpu_parity import run_parity, tiny1; from paper_conf_asplos_xiezggl25_b200 import workload as W;"
+            "st = W.gen_stream(tiny1(batch=128, lookahead=4, age_out=2), 40); r = run_parity(st); r['fr'].close();"
+            "print('OK', r['exact'])")
+    e = dict(os.environ)
+    e.update(env)
+    out = subprocess.run([sys.executable, "-c", code], env=e, capture_output=True, text=True,
+                         cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=600)
+    assert "OK True" in out.stdout, out.stdout + out.stderr
