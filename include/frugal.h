@@ -97,8 +97,9 @@ frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out);
 
 /* Sample queue (§3.2, §3.3): enqueue the ids of step t of ALL
    ranks.  ids_all: int64 [world][batch*slots], host (pageable or pinned) or device
-   pointer; it is read after the work already on `stream` and `stream`'s later work is
-   ordered after the read, so the caller may overwrite it once `stream` gets there.
+   pointer; it is read after the work already on `stream`, asynchronously on a library
+   stream: the caller may overwrite it once the next frugal_prefetch/frugal_step call
+   has returned (pageable host memory: as soon as this call returns).
    counts: host int32[world], samples of each rank (0..batch).  Only for t = 0..L-1
    before step 0.  The queue holds L+1 future steps: the ingest of step t (id
    conversion, dedup, read bits) runs on a library stream one step ahead, overlapping
@@ -197,6 +198,7 @@ enum {
     FRUGAL_C_LONG_SEGMENTS = 12,/* unique rows with > 64 occurrences (chunked reduction)     */
     FRUGAL_C_MAIL_OUT = 13,     /* partial rows written to this rank's host mailbox          */
     FRUGAL_C_MAIL_IN = 14,      /* partial rows read from other ranks' mailboxes             */
+    FRUGAL_C_GATHER_POOL = 15,  /* unique owned cold rows gathered from the dirty pool (HBM)  */
     FRUGAL_N_COUNTERS = 16
 };
 typedef struct {
@@ -206,6 +208,12 @@ typedef struct {
     int64_t count[FRUGAL_N_COUNTERS];
 } frugal_stats;
 frugal_status frugal_get_stats(frugal_ctx* ctx, frugal_stats* out);
+
+/* timeline of the last `cap` recorded phase instances (FRUGAL_F_TIMERS): phase index,
+   start and end (ms) relative to the first returned one, across all library streams.
+   Arrays may be NULL to query *n.  Call before frugal_get_stats (which consumes them). */
+frugal_status frugal_get_timeline(frugal_ctx* ctx, int32_t* phase, double* t0, double* t1, int64_t cap,
+                                  int64_t* n);
 
 /* number of owned rows / hot slots of this rank */
 int64_t frugal_owned_rows(frugal_ctx* ctx);

@@ -87,12 +87,12 @@ struct frugal_ctx {
     frugal_config cfg;
     int n, g, d, F, B, L, D, M;  // world, rank, dim, slots, batch, lookahead, age_out, B*F
     int64_t N, No;               // rows, owned rows
-    int P;                       // pool segments = D + 2
+    int P;                       // pool segments = D + 3
     int QN;                      // sample-queue slots = L + 2 (steps s-1 .. s+L)
     int side_blocks = 32;        // grid cap of the side-stream drain
     int gather_blocks = 296;     // grid cap of the zero-copy gathers
     bool side_inline = false;    // experiment: drain on the caller stream
-    bool drain_after_gather = false;  // side drain ordered after the step's gather (FRUGAL_DRAIN_AT=gather)
+    bool drain_after_gather = true;  // side drain after the step's gather (FRUGAL_DRAIN_AT=sched: after the scheduler)
     int64_t capT;                // max owned rows touched per step
     int key_bits, lk_bits;       // bits of global ids / local ids
 
@@ -141,18 +141,16 @@ struct frugal_ctx {
     int32_t* long_cnt = nullptr;     // [2]: long segments, chunk tasks
     int2* long_tasks = nullptr;      // [M/32 + 2] chunk [begin, end) positions
     int32_t* owned_cnt = nullptr;  // scalar
-    // schedule lists (double buffered by step parity)
-    int32_t* nb_rows = nullptr;  // newly bucketed rows [capT + capT]
-    int32_t* nb_p = nullptr;
-    int32_t* nb_cnt = nullptr;   // scalar
+    // schedule lists (double buffered by step parity): 4 lists of sl_cap rows each --
+    // 0 urgent (deadline s), 1 next (deadline s+1), 2 later (> s+1), 3 age-out; deadlines
+    // of lists 0..2 in sl_p; the 4 counts in sl_cnt
+    int64_t sl_cap = 0;
+    int32_t* sl_rows[2] = {nullptr, nullptr};
+    int32_t* sl_p[2] = {nullptr, nullptr};
+    int32_t* sl_cnt[2] = {nullptr, nullptr};
     int32_t* adj_rows[2] = {nullptr, nullptr};  // AdjustPriority inf -> t rows, by consuming step parity
     int32_t* adj_p[2] = {nullptr, nullptr};
     int32_t* adj_cnt[2] = {nullptr, nullptr};
-    int32_t* bk_rows[2] = {nullptr, nullptr};  // bucket-sorted rows
-    int32_t* bk_p[2] = {nullptr, nullptr};
-    int32_t* bk_off[2] = {nullptr, nullptr};   // [L+1]
-    int32_t* age_rows[2] = {nullptr, nullptr};
-    int32_t* age_cnt[2] = {nullptr, nullptr};
     int32_t* err = nullptr;   // device alias of the error word (mapped pinned host memory)
     int32_t* herr = nullptr;  // host pointer of the same word
     int32_t* sched_info = nullptr;  // device [4]
@@ -178,6 +176,7 @@ struct frugal_ctx {
     bool opt_pending[2] = {false, false};
     int64_t early_issued = -1;                          // last step whose early gather was launched
     bool early = false;                                 // pipelined gather enabled (world 1)
+    bool pool_hits = true;                              // owner reads its dirty-pool rows from HBM
     bool side_pending[2] = {false, false};
 
     // call-order state
@@ -206,10 +205,11 @@ void launch_dedup(frugal_ctx* c, QueueSlot& q, cudaStream_t st);
 void launch_owner_side(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st);
 void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, int32_t* adj_rows, int32_t* adj_p,
                         int32_t* adj_cnt, cudaStream_t st);
-void launch_bucket(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStream_t st);
+void launch_schedule(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStream_t st);
 void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begin, const int32_t* d_end,
                        int max_blocks, int counter, cudaStream_t st);
-void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32_t* cnt, float* rows, cudaStream_t st);
+void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32_t* cnt, float* rows, int64_t step,
+                   cudaStream_t st);
 void launch_expand(frugal_ctx* c, QueueSlot& q, const float* rows, float* out, cudaStream_t st);
 void launch_split_early(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st);
 void launch_mail_header(frugal_ctx* c, QueueSlot& q, int par, cudaStream_t st);

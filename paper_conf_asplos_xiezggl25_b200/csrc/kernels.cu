@@ -531,99 +531,72 @@ __global__ void k_ingest_bits(const int32_t* __restrict__ T, const uint32_t* __r
     }
 }
 
-// a9: priority of the rows updated at s-1 = next access step within [s, s+L-1] (Eq. 1)
-__global__ void k_bucket_prev(const int32_t* __restrict__ T, const int32_t* d_nT, int32_t s, int write_through,
-                              const uint64_t* __restrict__ rbits, int32_t* __restrict__ state, int32_t* nb_rows,
-                              int32_t* nb_p, int32_t* nb_cnt) {
-    int n = *d_nT;
-    int nloop = (n + blockDim.x * gridDim.x - 1) / (blockDim.x * gridDim.x) * (blockDim.x * gridDim.x);
+// a9 + a11 scheduler of step s, one kernel.  Three inputs, one virtual index range:
+//  [0, nA)        rows updated at s-1 (T(s-1)): priority = next access step within
+//                 [s, s+L-1] (Eq. (1)) read off the read ring; host-read there
+//                 -> flush class by deadline; owner-only hot read -> EXEMPT; none -> INF;
+//  [nA, nA+nB)    rows AdjustPriority'd inf -> s+L-1 by the ingest of that step;
+//  [nA+nB, ...)   age-out candidates: cold rows of pool segment s-1-D still INF.
+// Level 1 of the two-level PQ (§3.4) is the deadline relative to s; the drain policy (R9)
+// needs three of its classes: 0 urgent (p == s), 1 next (p == s+1), 2 later (p > s+1),
+// plus 3 = age-out.  Rows are appended to the four lists with warp-aggregated atomics.
+__global__ void k_schedule(const int32_t* __restrict__ T, const int32_t* d_nT, const int32_t* __restrict__ adj_rows,
+                           const int32_t* __restrict__ adj_p, const int32_t* adj_cnt,
+                           const int32_t* __restrict__ pkey, const int32_t* pcount_seg, int32_t u_age, int32_t s,
+                           int write_through, const uint64_t* __restrict__ rbits, int32_t* __restrict__ state,
+                           const int32_t* __restrict__ last_upd, int32_t* __restrict__ lists,
+                           int32_t* __restrict__ plist, int32_t* cnt, int64_t cap) {
+    const int nA = d_nT ? *d_nT : 0;
+    const int nB = *adj_cnt;
+    const int nC = pcount_seg ? *pcount_seg : 0;
+    const int n = nA + nB + nC;
+    const int nloop = (n + blockDim.x * gridDim.x - 1) / (blockDim.x * gridDim.x) * (blockDim.x * gridDim.x);
     const int rot = s & 31;
-    for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < nloop; j += gridDim.x * blockDim.x) {
-        bool app = false;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < nloop; i += gridDim.x * blockDim.x) {
+        int cls = -1;
         int32_t lk = 0, p = s;
-        if (j < n) {
-            lk = T[j];
-            uint64_t b = rbits[lk];
-            uint32_t any = (uint32_t)b, hst = (uint32_t)(b >> 32);
+        if (i < nA) {
+            lk = T[i];
             if (write_through) {
                 state[lk] = ST_CLEAN;
-                app = true;
+                cls = 0;
             } else {
-                uint32_t r = (any >> rot) | (rot ? (any << (32 - rot)) : 0u);
+                const uint64_t b = rbits[lk];
+                const uint32_t any = (uint32_t)b, hst = (uint32_t)(b >> 32);
+                const uint32_t r = (any >> rot) | (rot ? (any << (32 - rot)) : 0u);
                 if (r == 0u) {
                     state[lk] = ST_INF;
                 } else {
-                    int off = __ffs(r) - 1;
+                    const int off = __ffs(r) - 1;
                     p = s + off;
                     if ((hst >> ((rot + off) & 31)) & 1u) {
-                        state[lk] = ST_CLEAN;  // flush scheduled before gate p
-                        app = true;
+                        state[lk] = ST_CLEAN;  // flushed before gate p
+                        cls = off == 0 ? 0 : (off == 1 ? 1 : 2);
                     } else {
                         state[lk] = ST_EXEMPT;
                     }
                 }
             }
-        }
-        nb_append(nb_rows, nb_p, nb_cnt, app, lk, p);
-    }
-}
-
-// two-level PQ level 1: counting sort of the newly bucketed rows by deadline p - s in [0, L)
-__global__ void k_bucket_hist(const int32_t* __restrict__ nb_p, const int32_t* nb_cnt,
-                              const int32_t* __restrict__ adj_p, const int32_t* adj_cnt, int32_t s, int L,
-                              int32_t* bk_off /*[L+1], zeroed*/) {
-    __shared__ int h[32];
-    if (threadIdx.x < 32) h[threadIdx.x] = 0;
-    __syncthreads();
-    const int n1 = *nb_cnt, n = n1 + *adj_cnt;
-    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
-        atomicAdd(&h[(i < n1 ? nb_p[i] : adj_p[i - n1]) - s], 1);
-    __syncthreads();
-    if (threadIdx.x < L && h[threadIdx.x]) atomicAdd(&bk_off[threadIdx.x + 1], h[threadIdx.x]);
-}
-__global__ void k_bucket_scan(int32_t* bk_off, int L, int32_t* cursor) {
-    if (threadIdx.x == 0) {
-        bk_off[0] = 0;
-        for (int i = 1; i <= L; i++) bk_off[i] += bk_off[i - 1];
-        for (int i = 0; i < L; i++) cursor[i] = bk_off[i];
-    }
-}
-__global__ void k_bucket_scatter(const int32_t* __restrict__ nb_rows, const int32_t* __restrict__ nb_p,
-                                 const int32_t* nb_cnt, const int32_t* __restrict__ adj_rows,
-                                 const int32_t* __restrict__ adj_p, const int32_t* adj_cnt, int32_t s,
-                                 int32_t* cursor, int32_t* __restrict__ bk_rows, int32_t* __restrict__ bk_p) {
-    const int n1 = *nb_cnt, n = n1 + *adj_cnt;
-    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
-        const bool a = i >= n1;
-        const int p = a ? adj_p[i - n1] : nb_p[i];
-        int at = atomicAdd(&cursor[p - s], 1);
-        bk_rows[at] = a ? adj_rows[i - n1] : nb_rows[i];
-        bk_p[at] = p;
-    }
-}
-
-// a11 age-out: cold rows of pool segment u still dirty with priority inf
-__global__ void k_ageout(const int32_t* __restrict__ pkey, const int32_t* pcount_seg, int32_t u,
-                         const int32_t* __restrict__ last_upd, int32_t* __restrict__ state, int32_t* age_rows,
-                         int32_t* age_cnt) {
-    int n = *pcount_seg;
-    int nloop = (n + blockDim.x * gridDim.x - 1) / (blockDim.x * gridDim.x) * (blockDim.x * gridDim.x);
-    for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < nloop; j += gridDim.x * blockDim.x) {
-        bool app = false;
-        int32_t lk = 0;
-        if (j < n) {
-            lk = pkey[j];
-            if (lk >= 0 && state[lk] == ST_INF && last_upd[lk] == u) {
+        } else if (i < nA + nB) {
+            lk = adj_rows[i - nA];
+            p = adj_p[i - nA];
+            cls = p == s + 1 ? 1 : 2;
+        } else if (i < n) {
+            lk = pkey[i - nA - nB];
+            if (lk >= 0 && state[lk] == ST_INF && last_upd[lk] == u_age) {
                 state[lk] = ST_CLEAN;
-                app = true;
+                cls = 3;
             }
         }
-        unsigned m = __ballot_sync(FULL, app);
-        if (app) {
-            int leader = __ffs(m) - 1, lane = threadIdx.x & 31, base = 0;
-            if (lane == leader) base = atomicAdd(age_cnt, __popc(m));
-            base = __shfl_sync(m, base, leader);
-            age_rows[base + __popc(m & lanemask_lt())] = lk;
+        const unsigned peers = __match_any_sync(FULL, cls);
+        if (cls >= 0) {
+            const int leader = __ffs(peers) - 1, lane = threadIdx.x & 31;
+            int base = 0;
+            if (lane == leader) base = atomicAdd(&cnt[cls], __popc(peers));
+            base = __shfl_sync(peers, base, leader);
+            const int64_t at = (int64_t)cls * cap + base + __popc(peers & lanemask_lt());
+            lists[at] = lk;
+            if (cls < 3) plist[at] = p;
         }
     }
 }
@@ -636,33 +609,16 @@ void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, int3
     c->launches++;
 }
 
-void launch_bucket(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStream_t st) {
-    const int L = c->L;
-    if (prev) {
-        k_bucket_prev<<<grid_for(c->capT, 256), 256, 0, st>>>(prev->T, prev->nT, (int32_t)s,
-                                                               c->cfg.mode == FRUGAL_MODE_WRITE_THROUGH, c->rbits,
-                                                               c->state, c->nb_rows, c->nb_p, c->nb_cnt);
-        c->launches++;
-    }
-    cudaMemsetAsync(c->bk_off[par], 0, (L + 1) * sizeof(int32_t), st);
-    int32_t* cursor = c->sched_info + 8;  // [L] scratch
-    k_bucket_hist<<<grid_for(2 * c->capT, 256, 2), 256, 0, st>>>(c->nb_p, c->nb_cnt, c->adj_p[par], c->adj_cnt[par],
-                                                                  (int32_t)s, L, c->bk_off[par]);
-    k_bucket_scan<<<1, 32, 0, st>>>(c->bk_off[par], L, cursor);
-    k_bucket_scatter<<<grid_for(2 * c->capT, 256, 2), 256, 0, st>>>(c->nb_rows, c->nb_p, c->nb_cnt, c->adj_rows[par],
-                                                                     c->adj_p[par], c->adj_cnt[par], (int32_t)s,
-                                                                     cursor, c->bk_rows[par], c->bk_p[par]);
-    c->launches += 3;
-    // age-out of cold rows updated at u = s-1-D
-    cudaMemsetAsync(c->age_cnt[par], 0, sizeof(int32_t), st);
-    int64_t u = s - 1 - c->D;
-    if (u >= 0) {
-        int seg = (int)(u % c->P);
-        k_ageout<<<grid_for(c->capT, 256), 256, 0, st>>>(c->pkey + (size_t)seg * c->capT, c->pcount + seg,
-                                                          (int32_t)u, c->last_upd, c->state, c->age_rows[par],
-                                                          c->age_cnt[par]);
-        c->launches++;
-    }
+void launch_schedule(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStream_t st) {
+    cudaMemsetAsync(c->sl_cnt[par], 0, 4 * sizeof(int32_t), st);
+    const int64_t u = s - 1 - c->D;
+    const int seg = u >= 0 ? (int)(u % c->P) : 0;
+    k_schedule<<<grid_for(3 * c->capT, 256, 4), 256, 0, st>>>(
+        prev ? prev->T : nullptr, prev ? prev->nT : nullptr, c->adj_rows[par], c->adj_p[par], c->adj_cnt[par],
+        c->pkey + (size_t)seg * c->capT, u >= 0 ? c->pcount + seg : nullptr, (int32_t)u, (int32_t)s,
+        c->cfg.mode == FRUGAL_MODE_WRITE_THROUGH, c->rbits, c->state, c->last_upd, c->sl_rows[par], c->sl_p[par],
+        c->sl_cnt[par], c->sl_cap);
+    c->launches++;
 }
 
 // ============================================================================ row movers
@@ -715,36 +671,53 @@ void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begi
 
 // a4 gather: unique rows -> staging (owned hot: HBM cache; else host, zero-copy).
 // list: the uniq indices to gather (early or late part), cnt: its device count.
+// An owned cold row whose latest update is still in the dirty pool is read from the pool
+// (HBM) instead of the host: the pool holds exactly the value the flush wrote (or will
+// write), so the result is bit-identical and the flush schedule unchanged; only where the
+// owner reads from moves (R7').  Segment last_upd % P is intact while
+// last_upd >= pool_min (the optimizer of step u overwrites segment u % P; pool_min = u-P+2
+// also covers a gather running concurrently with the optimizer of u-1).
 template <int GS>
 __global__ void k_gather_uniq(const int32_t* __restrict__ uniq, const int32_t* __restrict__ list, const int32_t* cnt,
                               int world, int g, int d4, const int32_t* __restrict__ slot,
                               const float4* __restrict__ cw, const float4* hw, float4* __restrict__ rows,
+                              const int32_t* __restrict__ last_upd, const int32_t* __restrict__ pool_idx,
+                              const float4* __restrict__ pw, int P, int64_t capT, int32_t pool_min,
                               unsigned long long* stats) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
     const int n = *cnt;
-    unsigned nh = 0, nc = 0;
+    unsigned nh = 0, nc = 0, np = 0;
     for (int64_t a = gid; a < n; a += gs) {
         const int u = list ? list[a] : (int)a;
         int32_t k = uniq[u];
         const float4* src = hw + (int64_t)k * d4;
-        bool cached = false;
+        int kind = 0;  // 0 host, 1 cache, 2 pool
         if (k % world == g) {
-            int sl = slot[k / world];
+            const int32_t lk = k / world;
+            int sl = slot[lk];
             if (sl >= 0) {
                 src = cw + (int64_t)sl * d4;
-                cached = true;
+                kind = 1;
+            } else if (pw) {
+                const int32_t lu = last_upd[lk];
+                if (lu >= 0 && lu >= pool_min) {
+                    src = pw + ((int64_t)(lu % P) * capT + pool_idx[lk]) * d4;
+                    kind = 2;
+                }
             }
         }
         if (l == 0) {
-            if (cached) nc++;
-            else nh++;
+            nh += kind == 0;
+            nc += kind == 1;
+            np += kind == 2;
         }
         for (int v = l; v < d4; v += GS) rows[(int64_t)u * d4 + v] = src[v];
     }
     block_count(stats + FRUGAL_C_GATHER_HOST, nh);
     block_count(stats + FRUGAL_C_GATHER_CACHE, nc);
+    block_count(stats + FRUGAL_C_GATHER_POOL, np);
 }
 // a4 expand: out[i] = rows[inv[i]]
 template <int GS>
@@ -760,16 +733,19 @@ __global__ void k_expand(const int32_t* __restrict__ inv, const int32_t* d_m, in
     }
 }
 
-void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32_t* cnt, float* rows,
+void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32_t* cnt, float* rows, int64_t step,
                    cudaStream_t st) {
     const int d4 = c->d / 4, gs = group_size(d4);
     // zero-copy host loads are latency-bound: ~148x256 threads already keep the link's
     // read requests in flight (tools/zc_probe: 148 vs 1184 CTAs, same GB/s), and a
     // bigger grid only parks stalled warps on SMs other streams need
     int grid = std::min(grid_for((int64_t)c->M * gs, 256, 8), c->gather_blocks);
+    const int32_t pool_min = (int32_t)std::max<int64_t>(0, step - c->P + 2);
     DISPATCH_GS(gs, (k_gather_uniq<GS><<<grid, 256, 0, st>>>(q.uniq, list, cnt, c->n, c->g, d4, c->slot,
                                                              (const float4*)c->cw, (const float4*)c->dh_w,
-                                                             (float4*)rows, c->dstats)));
+                                                             (float4*)rows, c->last_upd, c->pool_idx,
+                                                             c->pool_hits ? (const float4*)c->pw : nullptr, c->P,
+                                                             c->capT, pool_min, c->dstats)));
     c->launches++;
 }
 void launch_expand(frugal_ctx* c, QueueSlot& q, const float* rows, float* out, cudaStream_t st) {

@@ -58,8 +58,8 @@ namespace {
 
 constexpr uint64_t kMagic = 0x46525547414c3235ULL;  // "FRUGAL25"
 constexpr size_t kHdr = 4096;
-constexpr size_t kFlags = 8192;  // 3 kinds x 32 ranks x 64 B
-enum { FLAG_URGENT = 0, FLAG_SIDE = 1, FLAG_MAIL = 2 };
+constexpr size_t kFlags = 8192;  // 4 kinds x 32 ranks x 64 B
+enum { FLAG_URGENT = 0, FLAG_SIDE = 1, FLAG_MAIL = 2, FLAG_SIDE_FIRST = 3 };
 enum { PH_INGEST, PH_SCHED, PH_URGENT, PH_GATE, PH_GATHER, PH_EXPAND, PH_MODEL, PH_SEGRED, PH_EXCH, PH_OPT, PH_SIDE,
        PH_PREFETCH };
 
@@ -140,10 +140,10 @@ static void free_ctx(frugal_ctx* c) {
         F(q.ids); F(q.counts); F(q.m); F(q.uniq); F(q.inv); F(q.off); F(q.pos); F(q.n_uniq);
         if (c->n > 1) { F(q.T); F(q.Tmask); F(q.Tidx); F(q.nT); F(q.gl); F(q.goff); }
     }
-    F(c->rows_buf[0]); F(c->rows_buf[1]); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->long_tasks); F(c->owned_cnt); F(c->nb_rows); F(c->nb_p); F(c->nb_cnt);
+    F(c->rows_buf[0]); F(c->rows_buf[1]); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->long_tasks); F(c->owned_cnt);
     for (int i = 0; i < 2; i++) { F(c->adj_rows[i]); F(c->adj_p[i]); F(c->adj_cnt[i]); }
-    for (int i = 0; i < 2; i++) { F(c->bk_rows[i]); F(c->bk_p[i]); F(c->bk_off[i]); F(c->age_rows[i]); F(c->age_cnt[i]); }
-    F(c->dstats); F(c->sched_info); F(c->ff_rows); F(c->ff_cnt); F(c->ids_stage);
+    for (int i = 0; i < 2; i++) { F(c->sl_rows[i]); F(c->sl_p[i]); F(c->sl_cnt[i]); }
+    F(c->dstats); F(c->ff_rows); F(c->ff_cnt); F(c->ids_stage);
     if (c->herr) cudaFreeHost(c->herr);
     if (c->counts_pin) cudaFreeHost(c->counts_pin);
     for (auto e : c->ev_counts) cudaEventDestroy(e);
@@ -212,16 +212,20 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->n = k.world; c->g = k.rank; c->d = k.dim; c->F = k.slots; c->B = k.batch;
     c->L = k.lookahead; c->D = k.age_out; c->M = k.batch * k.slots; c->N = k.n_rows;
     c->No = c->g < c->N ? (c->N - c->g + c->n - 1) / c->n : 0;
-    c->P = c->D + 2;
+    // pool segments: a row updated at u sits in segment u % P until the optimizer of u+P;
+    // its last reader is the drain of step u+1+D (age-out), which step u+D+3 waits for
+    c->P = c->D + 3;
     c->QN = c->L + 2;
     // pipelined early gather (world 1): off by default -- measured no gain on a PCIe-bound
     // box (the zero-copy loads of the next step only delay this step's); FRUGAL_EARLY=1
     c->early = c->n == 1 && getenv("FRUGAL_EARLY") && atoi(getenv("FRUGAL_EARLY"));
+    c->pool_hits = !(getenv("FRUGAL_NO_POOL_HITS") && atoi(getenv("FRUGAL_NO_POOL_HITS")));
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 32;
     c->gather_blocks = getenv("FRUGAL_GATHER_BLOCKS") ? atoi(getenv("FRUGAL_GATHER_BLOCKS")) : 296;
     c->side_inline = getenv("FRUGAL_SIDE_INLINE") && atoi(getenv("FRUGAL_SIDE_INLINE"));
-    c->drain_after_gather = getenv("FRUGAL_DRAIN_AT") && !strcmp(getenv("FRUGAL_DRAIN_AT"), "gather");
+    c->drain_after_gather = !(getenv("FRUGAL_DRAIN_AT") && !strcmp(getenv("FRUGAL_DRAIN_AT"), "sched"));
     c->capT = std::max<int64_t>(1, std::min<int64_t>((int64_t)c->n * c->M, c->No));
+    c->sl_cap = 2 * c->capT;
     c->key_bits = bits_for(c->N - 1);
     c->lk_bits = bits_for(std::max<int64_t>(c->No - 1, 0));
     const bool adag = k.opt == FRUGAL_ADAGRAD;
@@ -356,9 +360,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     DMALLOC(c->long_cnt, 8);
     DMALLOC(c->long_tasks, ((size_t)c->M / 32 + 2) * sizeof(int2));
     DMALLOC(c->owned_cnt, 4);
-    DMALLOC(c->nb_rows, 2 * c->capT * 4);
-    DMALLOC(c->nb_p, 2 * c->capT * 4);
-    DMALLOC(c->nb_cnt, 4);
+
     for (int i = 0; i < 2; i++) {
         DMALLOC(c->adj_rows[i], c->capT * 4);
         DMALLOC(c->adj_p[i], c->capT * 4);
@@ -366,13 +368,12 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         cudaMemset(c->adj_cnt[i], 0, 4);
     }
     for (int i = 0; i < 2; i++) {
-        DMALLOC(c->bk_rows[i], 2 * c->capT * 4);
-        DMALLOC(c->bk_p[i], 2 * c->capT * 4);
-        DMALLOC(c->bk_off[i], 64 * 4);
-        DMALLOC(c->age_rows[i], c->capT * 4);
-        DMALLOC(c->age_cnt[i], 4);
+        DMALLOC(c->sl_rows[i], 4 * c->sl_cap * 4);
+        DMALLOC(c->sl_p[i], 3 * c->sl_cap * 4);
+        DMALLOC(c->sl_cnt[i], 4 * 4);
+        cudaMemset(c->sl_cnt[i], 0, 16);
     }
-    DMALLOC(c->sched_info, 64 * 4);
+
     DMALLOC(c->ff_rows, std::max<int64_t>(c->No, 1) * 4);
     DMALLOC(c->ff_cnt, 4);
     DMALLOC(c->ids_stage, (size_t)c->n * c->M * 8);
@@ -482,8 +483,10 @@ static frugal_status ingest(frugal_ctx* c, int64_t t, const int64_t* ids_all, co
     q.step = t;
     q.h_counts.assign(counts, counts + c->n);
     cudaStream_t is = c->istream;
-    // the caller's buffer: copied after the caller's prior work, and the caller's later
-    // work is ordered after the copy (so it may reuse the buffer)
+    // the caller's buffer is read after the caller's prior work on `caller`; the copy of the
+    // previous call has finished once this call returns (host wait, normally long done), so
+    // the caller may reuse a buffer after the next frugal_step/frugal_prefetch returns
+    CK(cudaEventSynchronize(c->ev_copied));
     CK(cudaEventRecord(c->ev_call, caller));
     CK(cudaStreamWaitEvent(is, c->ev_call, 0));
     CK(cudaEventSynchronize(c->ev_counts[qi]));  // pinned counts staging of this slot is free
@@ -493,7 +496,6 @@ static frugal_status ingest(frugal_ctx* c, int64_t t, const int64_t* ids_all, co
     CK(cudaEventRecord(c->ev_counts[qi], is));
     CK(cudaMemcpyAsync(c->ids_stage, ids_all, (size_t)c->n * c->M * 8, cudaMemcpyDefault, is));
     CK(cudaEventRecord(c->ev_copied, is));
-    CK(cudaStreamWaitEvent(caller, c->ev_copied, 0));
     if (after) CK(cudaStreamWaitEvent(is, after, 0));
     {
         Timer tm(c, PH_INGEST, is);
@@ -526,21 +528,30 @@ extern "C" frugal_status frugal_prefetch(frugal_ctx* c, int64_t t, const int64_t
 
 static void record_schedule(frugal_ctx* c, int par, cudaStream_t st) {
     cudaStreamSynchronize(st);
-    int32_t off[64];
-    int32_t nage = 0;
-    cudaMemcpy(off, c->bk_off[par], (c->L + 1) * 4, cudaMemcpyDeviceToHost);
-    cudaMemcpy(&nage, c->age_cnt[par], 4, cudaMemcpyDeviceToHost);
-    std::vector<int32_t> rows(off[c->L]), ps(off[c->L]), age(nage);
-    if (off[c->L]) {
-        cudaMemcpy(rows.data(), c->bk_rows[par], off[c->L] * 4, cudaMemcpyDeviceToHost);
-        cudaMemcpy(ps.data(), c->bk_p[par], off[c->L] * 4, cudaMemcpyDeviceToHost);
-    }
-    if (nage) cudaMemcpy(age.data(), c->age_rows[par], nage * 4, cudaMemcpyDeviceToHost);
-    c->rec_urgent.assign(rows.begin(), rows.begin() + off[1]);
-    c->rec_deferred.assign(rows.begin() + off[1], rows.end());
-    c->rec_deferred_p.assign(ps.begin() + off[1], ps.end());
-    c->rec_ageout = age;
-    c->rec_gate_wait = off[1] > 0;
+    int32_t cnt[4];
+    cudaMemcpy(cnt, c->sl_cnt[par], sizeof cnt, cudaMemcpyDeviceToHost);
+    auto get = [&](int which, std::vector<int32_t>& rows, std::vector<int32_t>* ps) {
+        rows.resize(cnt[which]);
+        if (cnt[which]) {
+            cudaMemcpy(rows.data(), c->sl_rows[par] + (size_t)which * c->sl_cap, cnt[which] * 4, cudaMemcpyDeviceToHost);
+            if (ps) {
+                ps->resize(cnt[which]);
+                cudaMemcpy(ps->data(), c->sl_p[par] + (size_t)which * c->sl_cap, cnt[which] * 4, cudaMemcpyDeviceToHost);
+            }
+        } else if (ps) {
+            ps->clear();
+        }
+    };
+    std::vector<int32_t> r1, p1, r2, p2;
+    get(0, c->rec_urgent, nullptr);
+    get(1, r1, &p1);
+    get(2, r2, &p2);
+    get(3, c->rec_ageout, nullptr);
+    c->rec_deferred = r1;
+    c->rec_deferred.insert(c->rec_deferred.end(), r2.begin(), r2.end());
+    c->rec_deferred_p = p1;
+    c->rec_deferred_p.insert(c->rec_deferred_p.end(), p2.begin(), p2.end());
+    c->rec_gate_wait = cnt[0] > 0;
 }
 
 // a4 (pipelined, world 1): gather the rows of step u that were not read at u-1 into
@@ -556,7 +567,7 @@ static frugal_status launch_early_gather(frugal_ctx* c, int64_t u, cudaEvent_t s
     if (c->opt_pending[u & 1]) CK(cudaStreamWaitEvent(ps, c->ev_opt[u & 1], 0));
     {
         Timer tm(c, PH_PREFETCH, ps);
-        launch_gather(c, q, q.eidx, q.elcnt, c->rows_buf[u & 1], ps);
+        launch_gather(c, q, q.eidx, q.elcnt, c->rows_buf[u & 1], u, ps);
     }
     CK(cudaEventRecord(c->ev_early[u & 1], ps));
     c->early_issued = u;
@@ -577,12 +588,14 @@ static frugal_status launch_drain(frugal_ctx* c, int64_t s, cudaStream_t st, cud
     static const bool no_drain = getenv("FRUGAL_EXPERIMENT_NO_DRAIN") != nullptr;  // WRONG RESULTS: upper bound only
     if (!no_drain) {
         Timer tm(c, PH_SIDE, sd);
-        launch_flush_rows(c, c->bk_rows[par], c->bk_off[par] + 1, c->bk_off[par] + 2, c->side_blocks,
+        launch_flush_rows(c, c->sl_rows[par] + c->sl_cap, nullptr, c->sl_cnt[par] + 1, c->side_blocks,
                           FRUGAL_C_SIDE_HOT, sd);
         CK(cudaEventRecord(c->ev_side_first[par], sd));
-        launch_flush_rows(c, c->bk_rows[par], c->bk_off[par] + 2, c->bk_off[par] + c->L, c->side_blocks,
+        if (c->n > 1) launch_set_flag(c, FLAG_SIDE_FIRST, (uint32_t)(s + 1), sd);
+        launch_flush_rows(c, c->sl_rows[par] + 2 * c->sl_cap, nullptr, c->sl_cnt[par] + 2, c->side_blocks,
                           FRUGAL_C_SIDE_HOT, sd);
-        launch_flush_rows(c, c->age_rows[par], nullptr, c->age_cnt[par], c->side_blocks, FRUGAL_C_SIDE_HOT, sd);
+        launch_flush_rows(c, c->sl_rows[par] + 3 * c->sl_cap, nullptr, c->sl_cnt[par] + 3, c->side_blocks,
+                          FRUGAL_C_SIDE_HOT, sd);
         if (c->n > 1) launch_set_flag(c, FLAG_SIDE, (uint32_t)(s + 1), sd);
         CKL();
     }
@@ -616,7 +629,8 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
         const int64_t last = std::min<int64_t>(s + c->L - 1, c->next_prefetch - 1);
         CK(cudaStreamWaitEvent(st, c->ev_ingest[last % c->QN], 0));
     }
-    CK(cudaMemsetAsync(c->nb_cnt, 0, 4, st));
+    // the bucket / age-out lists of this parity were last read by the whole drain of s-2
+    if (c->side_pending[par]) CK(cudaStreamWaitEvent(st, c->ev_side[par], 0));
     if (s + c->L - 1 >= c->next_prefetch) CK(cudaMemsetAsync(c->adj_cnt[par], 0, 4, st));  // stream end: no adjust
     {
         Timer tm(c, PH_SCHED, st);
@@ -625,14 +639,14 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
             prev = &c->q[(s - 1) % c->QN];
             if (prev->step != s - 1) { set_err("internal: queue slot of step %lld lost", (long long)(s - 1)); return FRUGAL_ESTATE; }
         }
-        launch_bucket(c, prev, s, par, st);
+        launch_schedule(c, prev, s, par, st);
         CKL();
     }
     if (c->cfg.flags & FRUGAL_F_RECORD) record_schedule(c, par, st);
     {
         // a10: urgent bucket (priority == s) to the host table on the critical path
         Timer tm(c, PH_URGENT, st);
-        launch_flush_rows(c, c->bk_rows[par], c->bk_off[par], c->bk_off[par] + 1, 1 << 30, FRUGAL_C_URGENT_HOT, st);
+        launch_flush_rows(c, c->sl_rows[par], nullptr, c->sl_cnt[par], 1 << 30, FRUGAL_C_URGENT_HOT, st);
         if (c->n > 1) launch_set_flag(c, FLAG_URGENT, (uint32_t)(s + 1), st);
         CKL();
     }
@@ -662,11 +676,13 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
         // a3: gate of step s -- PQ front > s: every owner's urgent bucket s and every
         // deferred bucket drained by its side stream at steps <= s-1
         Timer tm(c, PH_GATE, st);
+        // (deadline-s rows are the first part of drain s-1; the side stream is FIFO, so that
+        // event also covers every earlier drain)
         if (c->n == 1) {
-            if (s >= 1 && c->side_pending[par ^ 1]) CK(cudaStreamWaitEvent(st, c->ev_side[par ^ 1], 0));
+            if (s >= 1 && c->side_pending[par ^ 1]) CK(cudaStreamWaitEvent(st, c->ev_side_first[par ^ 1], 0));
         } else {
             launch_wait_flags(c, FLAG_URGENT, (uint32_t)(s + 1), st);
-            if (s >= 1) launch_wait_flags(c, FLAG_SIDE, (uint32_t)s, st);
+            if (s >= 1) launch_wait_flags(c, FLAG_SIDE_FIRST, (uint32_t)s, st);
             CKL();
         }
     }
@@ -688,9 +704,9 @@ extern "C" frugal_status frugal_lookup(frugal_ctx* c, int64_t s, float* d_out, f
         Timer tm(c, PH_GATHER, st);
         if (c->early) {
             CK(cudaStreamWaitEvent(st, c->ev_early[s & 1], 0));
-            launch_gather(c, q, q.lidx, q.elcnt + 1, rows, st);  // rows read at s-1 (updated then)
+            launch_gather(c, q, q.lidx, q.elcnt + 1, rows, s, st);  // rows read at s-1 (updated then)
         } else {
-            launch_gather(c, q, nullptr, q.n_uniq, rows, st);
+            launch_gather(c, q, nullptr, q.n_uniq, rows, s, st);
         }
     }
     if (c->drain_after_gather) {
@@ -870,6 +886,30 @@ extern "C" frugal_status frugal_read_host(frugal_ctx* c, const int64_t* ids, int
             else memset(G + i * c->d, 0, c->d * 4);
         }
     }
+    return FRUGAL_OK;
+}
+
+// timeline of the recorded phases (FRUGAL_F_TIMERS): for each of the last `cap` recorded
+// phase instances, (phase, start_ms, end_ms) relative to the first recorded event.  Call
+// before frugal_get_stats (which consumes the events).
+extern "C" frugal_status frugal_get_timeline(frugal_ctx* c, int32_t* phase, double* t0, double* t1, int64_t cap,
+                                             int64_t* n) {
+    if (!c || !n) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    CK(cudaDeviceSynchronize());
+    *n = (int64_t)c->evs.size();
+    if (!phase || c->evs.empty()) return FRUGAL_OK;
+    const size_t first = c->evs.size() > (size_t)cap ? c->evs.size() - (size_t)cap : 0;
+    cudaEvent_t ref = c->evs[first].a;
+    for (size_t i = first; i < c->evs.size(); i++) {
+        float a = 0.f, b = 0.f;
+        cudaEventElapsedTime(&a, ref, c->evs[i].a);
+        cudaEventElapsedTime(&b, ref, c->evs[i].b);
+        phase[i - first] = c->evs[i].phase;
+        t0[i - first] = a;
+        t1[i - first] = b;
+    }
+    cudaGetLastError();
+    *n = (int64_t)(c->evs.size() - first);
     return FRUGAL_OK;
 }
 

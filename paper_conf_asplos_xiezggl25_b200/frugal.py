@@ -47,7 +47,7 @@ class ScheduleInfo(C.Structure):
 
 COUNTERS = ["positions", "unique", "gather_host", "gather_cache", "opt_hot", "opt_cold", "urgent_hot",
             "urgent_cold", "side_hot", "side_cold", "final_hot", "final_cold", "long_segments", "mail_out",
-            "mail_in", "reserved"]
+            "mail_in", "gather_pool"]
 
 
 class Stats(C.Structure):
@@ -82,6 +82,7 @@ def lib():
             "frugal_read_rows": [P, P, I64, P, P],
             "frugal_read_host": [P, P, I64, P, P],
             "frugal_get_stats": [P, C.POINTER(Stats)],
+            "frugal_get_timeline": [P, P, P, P, I64, C.POINTER(I64)],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -100,7 +101,7 @@ def lib():
 EXPORTED = ["frugal_init", "frugal_prefetch", "frugal_step", "frugal_lookup", "frugal_backward_update",
             "frugal_flush", "frugal_destroy", "frugal_last_error", "frugal_dot_model", "frugal_get_dedup",
             "frugal_get_schedule", "frugal_get_final_flush", "frugal_read_rows", "frugal_read_host",
-            "frugal_get_stats", "frugal_owned_rows", "frugal_hot_slots"]
+            "frugal_get_stats", "frugal_get_timeline", "frugal_owned_rows", "frugal_hot_slots"]
 
 
 def _check(status):
@@ -236,6 +237,15 @@ class Frugal:
         _check(lib().frugal_get_stats(self.h, C.byref(s)))
         return dict(ms={p: s.ms[i] for i, p in enumerate(PHASES)}, steps=s.steps,
                     kernel_launches=s.kernel_launches, count={n: s.count[i] for i, n in enumerate(COUNTERS)})
+
+    def get_timeline(self, cap=4096):
+        """[(phase name, start ms, end ms)] of the last `cap` recorded phases (all streams)."""
+        ph = np.empty(cap, np.int32)
+        t0 = np.empty(cap, np.float64)
+        t1 = np.empty(cap, np.float64)
+        n = C.c_int64()
+        _check(lib().frugal_get_timeline(self.h, ph.ctypes.data, t0.ctypes.data, t1.ctypes.data, cap, C.byref(n)))
+        return [(PHASES[ph[i]], float(t0[i]), float(t1[i])) for i in range(n.value)]
 
     @property
     def owned_rows(self):
