@@ -90,7 +90,7 @@ struct frugal_ctx {
     int P;                       // pool segments = D + 3
     int QN;                      // sample-queue slots = L + 2 (steps s-1 .. s+L)
     int side_blocks = 32;        // grid cap of the side-stream drain
-    int gather_blocks = 296;     // grid cap of the zero-copy gathers
+    int gather_blocks = 74;      // grid cap of the zero-copy gathers (74 CTAs fill the link: profiles/r1_zc_probe_async.txt)
     bool side_inline = false;    // experiment: drain on the caller stream
     bool drain_after_gather = true;  // side drain after the step's gather (FRUGAL_DRAIN_AT=sched: after the scheduler)
     int64_t capT;                // max owned rows touched per step

@@ -221,7 +221,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->early = c->n == 1 && getenv("FRUGAL_EARLY") && atoi(getenv("FRUGAL_EARLY"));
     c->pool_hits = !(getenv("FRUGAL_NO_POOL_HITS") && atoi(getenv("FRUGAL_NO_POOL_HITS")));
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 32;
-    c->gather_blocks = getenv("FRUGAL_GATHER_BLOCKS") ? atoi(getenv("FRUGAL_GATHER_BLOCKS")) : 296;
+    c->gather_blocks = getenv("FRUGAL_GATHER_BLOCKS") ? atoi(getenv("FRUGAL_GATHER_BLOCKS")) : 74;
     c->side_inline = getenv("FRUGAL_SIDE_INLINE") && atoi(getenv("FRUGAL_SIDE_INLINE"));
     c->drain_after_gather = !(getenv("FRUGAL_DRAIN_AT") && !strcmp(getenv("FRUGAL_DRAIN_AT"), "sched"));
     c->capT = std::max<int64_t>(1, std::min<int64_t>((int64_t)c->n * c->M, c->No));
@@ -561,7 +561,10 @@ static void record_schedule(frugal_ctx* c, int par, cudaStream_t st) {
 // hold their step-u values (invariant (2)); the rest is gathered after gate u.
 static frugal_status launch_early_gather(frugal_ctx* c, int64_t u, cudaEvent_t side_first) {
     QueueSlot& q = c->q[u % c->QN];
-    cudaStream_t ps = c->pstream;
+    // with the drain placed after the gather, the early gather follows the drain on the
+    // side stream: one FIFO of host-link work (late gather, drain, early gather of the
+    // next step) that fills the link while the main stream runs the backward
+    cudaStream_t ps = c->drain_after_gather ? c->side : c->pstream;
     CK(cudaStreamWaitEvent(ps, c->ev_ingest[u % c->QN], 0));
     if (side_first) CK(cudaStreamWaitEvent(ps, side_first, 0));
     if (c->opt_pending[u & 1]) CK(cudaStreamWaitEvent(ps, c->ev_opt[u & 1], 0));
