@@ -34,6 +34,8 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "training samples/s at 1/2/4/8 B200; flush+gather GB/s vs HBM/host-link peak"
+CONFIG_NAMES = {"tiny": "BASELINE.json configs[0]", "criteo_kaggle": "BASELINE.json configs[1]",
+                "avazu": "BASELINE.json configs[2]", "criteo_tb": "BASELINE.json configs[4]"}
 
 
 def parse():
@@ -46,7 +48,27 @@ def parse():
     ap.add_argument("--alpha", type=float, default=0.9)
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--mode", default="p2f", choices=["p2f", "write_through"],
+                    help="write_through = Frugal-Sync (every update flushed on the next step's critical path)")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process-group backend for barriers / the max-over-ranks timing only")
     return ap.parse_args()
+
+
+def dist_max(x, world, dist=None, device="cpu"):
+    """Max of a per-rank float over all ranks (the contract's max-over-ranks timing)."""
+    if world == 1:
+        return x
+    import torch
+    t = torch.tensor([x], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def rank_device(local_rank):
+    """One GPU per rank; FRUGAL_BENCH_SAME_DEVICE=1 puts every rank on cuda:0 (testing the
+    multi-rank protocol on a one-GPU box)."""
+    return 0 if os.environ.get("FRUGAL_BENCH_SAME_DEVICE") == "1" else local_rank
 
 
 # ------------------------------------------------------------------------------ clocks
@@ -186,21 +208,22 @@ def main():
     from paper_conf_asplos_xiezggl25_b200.harness import make_context
 
     assert args.warmup >= 3, "timing rules: at least 3 warm-up steps"
+    local = rank_device(local)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    coll_dev = dev if args.dist_backend == "nccl" else torch.device("cpu")
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
 
     def barrier():
         if world > 1:
             dist.barrier()
 
     def max_over_ranks(x):
-        if world == 1:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
+        return dist_max(x, world, dist, coll_dev)
 
     cfg = W.config(args.config, world=world, alpha=args.alpha)
     K, Wm, L = args.steps, args.warmup, cfg.lookahead
@@ -210,7 +233,8 @@ def main():
     t_gen = time.time() - t_gen
     B, Fs, d = cfg.batch, cfg.slots, cfg.dim
     shm = f"/frugal_bench_{os.environ.get('MASTER_PORT', '0')}" if world > 1 else None
-    fr = make_context(st, rank=rank, device=local, shm_name=shm, flags=F.F_TIMERS)
+    fr = make_context(st, rank=rank, device=local, shm_name=shm, flags=F.F_TIMERS,
+                      mode=F.MODE_WRITE_THROUGH if args.mode == "write_through" else F.MODE_P2F)
     barrier()
     stream = torch.cuda.current_stream(dev)
 
@@ -372,9 +396,10 @@ def main():
         "metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": world, "steps": K, "warmup": Wm,
         "ms_per_step": ms_max / K, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "f32", "data": "synthetic",
-        "config": {"workload": f"{cfg.name} (BASELINE.json configs[1])", "global_batch": world * B,
+        "config": {"workload": f"{cfg.name} ({CONFIG_NAMES.get(cfg.name, '')})", "global_batch": world * B,
                    "batch_per_gpu": B, "tables": Fs, "rows": cfg.n_rows, "dim": d, "alpha": cfg.alpha,
                    "lookahead": L, "age_out": cfg.age_out, "cache_ratio": cfg.cache_ratio, "opt": cfg.opt,
+                   "flush_mode": args.mode,
                    "parallelism": f"dp{world} (owner-sharded rows, shared pinned host table)",
                    "l2": "inputs larger than L2: host table %.1f GB, HBM cache %.0f MB, %d distinct id batches"
                          % (cfg.n_rows * r * (2 if adag else 1) / 1e9, len(st.hot) * r * 2 / 1e6, K)},
