@@ -35,7 +35,8 @@ sys.path.insert(0, ROOT)
 
 METRIC = "training samples/s at 1/2/4/8 B200; flush+gather GB/s vs HBM/host-link peak"
 CONFIG_NAMES = {"tiny": "BASELINE.json configs[0]", "criteo_kaggle": "BASELINE.json configs[1]",
-                "avazu": "BASELINE.json configs[2]", "criteo_tb": "BASELINE.json configs[4]"}
+                "avazu": "BASELINE.json configs[2]", "freebase": "BASELINE.json configs[3]",
+                "fb15k": "FB15k-shaped KG, Table 2", "criteo_tb": "BASELINE.json configs[4]"}
 
 
 def parse():
@@ -255,11 +256,16 @@ def main():
     for t in range(L):
         fr.prefetch(t, ids_d[t], counts[t])
 
+    kg = cfg.model == "transe"
+
     def step_dev(s):
         t = s + L
         fr.step(s, ids_d[t], counts[t])
         fr.lookup(s, emb)
-        fr.dot_model(s, emb, x_d[s], y_d[s], grad, loss[s:s + 1])
+        if kg:
+            fr.transe_model(s, emb, cfg.neg_chunk, cfg.gamma, grad, loss[s:s + 1])
+        else:
+            fr.dot_model(s, emb, x_d[s], y_d[s], grad, loss[s:s + 1])
         fr.backward_update(s, grad)
 
     copy_stream = torch.cuda.Stream(dev)
@@ -283,7 +289,10 @@ def main():
         load_xy(s + 1)
         fr.lookup(s, emb)
         stream.wait_event(xy_ready[b])
-        fr.dot_model(s, emb, x_e[b], y_e[b], grad, loss[s:s + 1])
+        if kg:
+            fr.transe_model(s, emb, cfg.neg_chunk, cfg.gamma, grad, loss[s:s + 1])
+        else:
+            fr.dot_model(s, emb, x_e[b], y_e[b], grad, loss[s:s + 1])
         xy_free[b].record(stream)
         fr.backward_update(s, grad)
         loss_h[s:s + 1].copy_(loss[s:s + 1], non_blocking=True)  # the step's result back to the host

@@ -147,6 +147,14 @@ frugal_status frugal_dot_model(frugal_ctx* ctx, int64_t s, const float* d_emb, c
                                const float* d_y, float* d_grad, double* d_loss,
                                frugal_stream stream);
 
+/* KG glue (R26): TransE-L2, samples = triples with slots (h, r, t, neg), the
+   negatives of each chunk of `chunk` consecutive samples of this rank shared by the chunk:
+   score = gamma - |h + r - x|_2, loss_b = softplus(-score(h,r,t)) + mean_j softplus(
+   score(h,r,n_j)); *d_loss += sum_b loss_b / nb.  fp64 internally, d_grad fp32 [count*4][dim].
+   Requires slots == 4. */
+frugal_status frugal_transe_model(frugal_ctx* ctx, int64_t s, const float* d_emb, int32_t chunk, float gamma,
+                                  float* d_grad, double* d_loss, frugal_stream stream);
+
 /* ---- introspection (tests / bench only; synchronise and copy to caller-owned host
    buffers) ---------------------------------------------------------------------- */
 /* dedup of this rank's ids at step t (t within the sample queue): uniq ascending

@@ -49,7 +49,7 @@
 #define OR_INF INT32_MAX
 #define OR_CHUNK 64 /* R23: segment-reduce chunk length */
 enum { OR_SGD = 0, OR_ADAGRAD = 1 };
-enum { OR_MODEL_DOT = 0, OR_MODEL_CONST = 1, OR_MODEL_L2 = 2 };
+enum { OR_MODEL_DOT = 0, OR_MODEL_CONST = 1, OR_MODEL_L2 = 2, OR_MODEL_TRANSE = 3 };
 enum { OR_CLEAN = 0, OR_UPDATED = 1, OR_INFP = 2, OR_EXEMPT = 3 };
 enum { OR_L_URGENT = 0, OR_L_DEFERRED = 1, OR_L_DEFERRED_P = 2, OR_L_AGEOUT = 3,
        OR_L_FINAL = 4, OR_L_UPDATED = 5, OR_L_INF = 6, OR_L_EXEMPT = 7 };
@@ -61,6 +61,8 @@ typedef struct {
     uint64_t init_seed;
     int32_t write_through;    /* 1: every update flushed at the next step (Frugal-Sync, L1399-1402) */
     int32_t skip_urgent_step; /* negative test: urgent flush of this step is lost (-1: never) */
+    float gamma;              /* TransE margin */
+    int32_t neg_chunk;        /* TransE: triples per negative-sharing chunk */
 } oracle_config;
 
 typedef struct { int64_t key; int32_t state, last_update; } rowmeta;
@@ -351,6 +353,76 @@ static void schedule(oracle* o, int64_t s) {
     }
 }
 
+/* ---- TransE glue (reading R26; §4.1, DGL-KE TransE_l2): slots of a
+   sample are (h, r, t, neg); the negatives of a chunk of neg_chunk consecutive triples of
+   a rank are shared by the chunk (tail corruption).  score = gamma - |h + r - x|_2;
+   loss_b = softplus(-score(h,r,t)) + (1/nC) sum_j softplus(score(h,r,n_j)).
+   Everything in fp64, sums in the written order; gradients rounded to fp32 once. */
+static double sigm(double x) { return 1.0 / (1.0 + exp(-x)); }
+static double softplus(double x) { return x > 0 ? x + log1p(exp(-x)) : log1p(exp(x)); }
+static double transe(oracle* o, int64_t s, int64_t nb) {
+    const int n = o->c.world, F = o->c.slots, B = o->c.batch, C = o->c.neg_chunk;
+    const int64_t d = o->c.dim;
+    const double gamma = o->c.gamma;
+    double loss = 0.0;
+    double* P = malloc(d * sizeof(double));
+    double* v = malloc(d * sizeof(double));
+    double* u = malloc(d * sizeof(double));
+    double* gh = malloc(d * sizeof(double));
+    double* gn = malloc((size_t)C * d * sizeof(double));
+    for (int g = 0; g < n; g++) {
+        const int64_t* id = step_ids(o, s, g);
+        const int32_t cnt = o->counts[s * n + g];
+        float* grad = o->grad + (int64_t)g * B * F * d;
+        for (int b0 = 0; b0 < cnt; b0 += C) {
+            const int b1 = b0 + C < cnt ? b0 + C : cnt, nC = b1 - b0;
+            for (int64_t q = 0; q < (int64_t)nC * d; q++) gn[q] = 0.0;
+            for (int b = b0; b < b1; b++) {
+                int64_t ih = row(o, id[b * F + 0]), ir = row(o, id[b * F + 1]), it = row(o, id[b * F + 2]);
+                const float *h = o->W + ih * d, *r = o->W + ir * d, *t = o->W + it * d;
+                double dp = 0.0;
+                for (int64_t k = 0; k < d; k++) {
+                    P[k] = (double)h[k] + (double)r[k];
+                    v[k] = P[k] - (double)t[k];
+                    dp = dp + v[k] * v[k];
+                }
+                dp = sqrt(dp);
+                const double sp = gamma - dp;
+                loss += softplus(-sp);
+                const double a = dp > 0.0 ? (1.0 - sigm(sp)) / dp : 0.0;
+                for (int64_t k = 0; k < d; k++) gh[k] = a * v[k];
+                for (int j = b0; j < b1; j++) {
+                    const float* nj = o->W + row(o, id[j * F + 3]) * d;
+                    double dj = 0.0;
+                    for (int64_t k = 0; k < d; k++) {
+                        u[k] = P[k] - (double)nj[k];
+                        dj = dj + u[k] * u[k];
+                    }
+                    dj = sqrt(dj);
+                    const double sj = gamma - dj;
+                    loss += softplus(sj) / (double)nC;
+                    const double w = dj > 0.0 ? sigm(sj) / dj / (double)nC : 0.0;
+                    double* gj = gn + (int64_t)(j - b0) * d;
+                    for (int64_t k = 0; k < d; k++) {
+                        gh[k] = gh[k] - w * u[k];
+                        gj[k] = gj[k] + w * u[k];
+                    }
+                }
+                for (int64_t k = 0; k < d; k++) {
+                    grad[(b * F + 0) * d + k] = (float)(gh[k] / (double)nb);
+                    grad[(b * F + 1) * d + k] = (float)(gh[k] / (double)nb);
+                    grad[(b * F + 2) * d + k] = (float)(-(a * v[k]) / (double)nb);
+                }
+            }
+            for (int j = b0; j < b1; j++)
+                for (int64_t k = 0; k < d; k++)
+                    grad[(j * F + 3) * d + k] = (float)(gn[(int64_t)(j - b0) * d + k] / (double)nb);
+        }
+    }
+    free(P); free(v); free(u); free(gh); free(gn);
+    return loss;
+}
+
 /* ---- value part of step s: synchronous training (f)-(j) */
 static void train(oracle* o, int64_t s) {
     const int n = o->c.world, F = o->c.slots, B = o->c.batch;
@@ -387,6 +459,8 @@ static void train(oracle* o, int64_t s) {
                     int64_t ri = row(o, id[b * F + f]); const float* e = o->W + ri * d;
                     for (int64_t j = 0; j < d; j++) gr[f * d + j] = c * ((S[j] - e[j]) + xb[j]);
                 }
+            } else if (o->c.model == OR_MODEL_TRANSE) {
+                continue;  /* whole chunks below */
             } else if (o->c.model == OR_MODEL_CONST) {  /* linear loss <x_b, e_f>: grad = x_b */
                 for (int f = 0; f < F; f++)
                     for (int64_t j = 0; j < d; j++) gr[f * d + j] = xb[j];
@@ -404,6 +478,7 @@ static void train(oracle* o, int64_t s) {
         }
     }
     free(S);
+    if (o->c.model == OR_MODEL_TRANSE) loss += transe(o, s, nb);
     o->loss[s] = nb ? loss / (double)nb : 0.0;
     /* (g) per-rank partials, positions ascending, sequential fp32 */
     for (int g = 0; g < n; g++) {

@@ -20,7 +20,7 @@ LIB = os.path.join(HERE, "liboracle.so")
 INF = 2**31 - 1
 L_URGENT, L_DEFERRED, L_DEFERRED_P, L_AGEOUT, L_FINAL, L_UPDATED, L_INF, L_EXEMPT = range(8)
 CLEAN, UPDATED, INFP, EXEMPT = range(4)
-MODELS = {"dot": 0, "const": 1, "l2": 2}
+MODELS = {"dot": 0, "const": 1, "l2": 2, "transe": 3}
 OPTS = {"sgd": 0, "adagrad": 1}
 
 
@@ -29,7 +29,7 @@ class _Cfg(C.Structure):
                 ("lookahead", C.c_int32), ("age_out", C.c_int32), ("opt", C.c_int32), ("model", C.c_int32),
                 ("n_rows", C.c_int64), ("lr", C.c_float), ("eps", C.c_float), ("init_accum", C.c_float),
                 ("init_scale", C.c_float), ("init_seed", C.c_uint64), ("write_through", C.c_int32),
-                ("skip_urgent_step", C.c_int32)]
+                ("skip_urgent_step", C.c_int32), ("gamma", C.c_float), ("neg_chunk", C.c_int32)]
 
 
 def build(force: bool = False) -> str:
@@ -90,7 +90,7 @@ def _p(a):
 class Oracle:
     """Single-threaded synchronous trainer + brute-force P2F schedule."""
 
-    def __init__(self, stream, model="dot", opt=None, lookahead=None, age_out=None, lr=None,
+    def __init__(self, stream, model=None, opt=None, lookahead=None, age_out=None, lr=None,
                  write_through=False, skip_urgent_step=-1, hot=None):
         cfg = stream.cfg
         self.stream = stream
@@ -103,7 +103,8 @@ class Oracle:
         c.lookahead = cfg.lookahead if lookahead is None else lookahead
         c.age_out = cfg.age_out if age_out is None else age_out
         c.opt = OPTS[cfg.opt if opt is None else opt]
-        c.model = MODELS[model]
+        c.model = MODELS[cfg.model if model is None else model]
+        c.gamma, c.neg_chunk = cfg.gamma, cfg.neg_chunk
         c.n_rows = cfg.n_rows
         c.lr = cfg.lr if lr is None else lr
         c.eps, c.init_accum, c.init_scale = cfg.eps, cfg.init_accum, cfg.init_scale

@@ -7,7 +7,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libfrugal.so")
-SOURCES = ["kernels.cu", "kernels_update.cu", "runtime.cu"]
+SOURCES = ["kernels.cu", "kernels_update.cu", "kernels_kg.cu", "runtime.cu"]
 HEADERS = ["frugal_internal.cuh", "kutil.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",

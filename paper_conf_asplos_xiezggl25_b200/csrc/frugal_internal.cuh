@@ -185,6 +185,11 @@ struct frugal_ctx {
     int phase_in_step = 0;  // 0 = need step, 1 = need lookup, 2 = need backward
     bool ids_exhausted = false;
 
+    // KG glue scratch (allocated on first use): W [batch][C] and A [batch] (fp64)
+    double* kg_W = nullptr;
+    double* kg_A = nullptr;
+    int kg_C = 0;
+
     // instrumentation
     int64_t launches = 0;
     std::vector<frugal::PhaseEv> evs;
@@ -213,6 +218,8 @@ void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32
 void launch_expand(frugal_ctx* c, QueueSlot& q, const float* rows, float* out, cudaStream_t st);
 void launch_split_early(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st);
 void launch_mail_header(frugal_ctx* c, QueueSlot& q, int par, cudaStream_t st);
+void launch_transe_model(frugal_ctx* c, QueueSlot& q, const float* emb, int C, double gamma, float* grad,
+                         double* loss, int64_t nb, double* Wm, double* A, cudaStream_t st);
 void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const float* x, const float* y,
                       float* grad, double* loss, int64_t nb, cudaStream_t st);
 void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, cudaStream_t st);

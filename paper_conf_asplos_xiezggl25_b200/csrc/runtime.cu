@@ -143,7 +143,7 @@ static void free_ctx(frugal_ctx* c) {
     F(c->rows_buf[0]); F(c->rows_buf[1]); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->long_tasks); F(c->owned_cnt);
     for (int i = 0; i < 2; i++) { F(c->adj_rows[i]); F(c->adj_p[i]); F(c->adj_cnt[i]); }
     for (int i = 0; i < 2; i++) { F(c->sl_rows[i]); F(c->sl_p[i]); F(c->sl_cnt[i]); }
-    F(c->dstats); F(c->ff_rows); F(c->ff_cnt); F(c->ids_stage);
+    F(c->dstats); F(c->kg_W); F(c->kg_A); F(c->ff_rows); F(c->ff_cnt); F(c->ids_stage);
     if (c->herr) cudaFreeHost(c->herr);
     if (c->counts_pin) cudaFreeHost(c->counts_pin);
     for (auto e : c->ev_counts) cudaEventDestroy(e);
@@ -743,6 +743,33 @@ extern "C" frugal_status frugal_dot_model(frugal_ctx* c, int64_t s, const float*
     for (int r = 0; r < c->n; r++) nb += q.h_counts[r];
     Timer tm(c, PH_MODEL, st);
     launch_dot_model(c, q, d_emb, d_x, d_y, d_grad, d_loss, nb, st);
+    CKL();
+    return FRUGAL_OK;
+}
+
+extern "C" frugal_status frugal_transe_model(frugal_ctx* c, int64_t s, const float* d_emb, int32_t chunk, float gamma,
+                                             float* d_grad, double* d_loss, frugal_stream stream) {
+    if (!c || !d_emb || !d_grad || !d_loss) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    if (c->F != 4) { set_err("transe_model needs slots == 4 (h, r, t, neg)"); return FRUGAL_EINVAL; }
+    if (chunk < 1 || chunk > 4096) { set_err("chunk must be in [1, 4096]"); return FRUGAL_EINVAL; }
+    if (c->phase_in_step != 2 || s != c->cur_step) {
+        set_err("transe_model(%lld) must follow lookup(%lld)", (long long)s, (long long)s);
+        return FRUGAL_ESTATE;
+    }
+    if (c->kg_C != chunk) {
+        cudaFree(c->kg_W);
+        cudaFree(c->kg_A);
+        c->kg_W = c->kg_A = nullptr;
+        CK(cudaMalloc(&c->kg_W, ((size_t)c->B + chunk) * chunk * sizeof(double)));
+        CK(cudaMalloc(&c->kg_A, ((size_t)c->B + chunk) * sizeof(double)));
+        c->kg_C = chunk;
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    QueueSlot& q = c->q[s % c->QN];
+    int64_t nb = 0;
+    for (int r = 0; r < c->n; r++) nb += q.h_counts[r];
+    Timer tm(c, PH_MODEL, st);
+    launch_transe_model(c, q, d_emb, chunk, (double)gamma, d_grad, d_loss, nb, c->kg_W, c->kg_A, st);
     CKL();
     return FRUGAL_OK;
 }

@@ -76,6 +76,7 @@ def lib():
             "frugal_flush": [P, I32, P],
             "frugal_destroy": [P],
             "frugal_dot_model": [P, I64, P, P, P, P, P, P],
+            "frugal_transe_model": [P, I64, P, I32, C.c_float, P, P, P],
             "frugal_get_dedup": [P, I64, P, P, C.POINTER(I64)],
             "frugal_get_schedule": [P, C.POINTER(ScheduleInfo), P, P, P, P],
             "frugal_get_final_flush": [P, P, C.POINTER(I64)],
@@ -99,7 +100,8 @@ def lib():
 
 
 EXPORTED = ["frugal_init", "frugal_prefetch", "frugal_step", "frugal_lookup", "frugal_backward_update",
-            "frugal_flush", "frugal_destroy", "frugal_last_error", "frugal_dot_model", "frugal_get_dedup",
+            "frugal_flush", "frugal_destroy", "frugal_last_error", "frugal_dot_model", "frugal_transe_model",
+            "frugal_get_dedup",
             "frugal_get_schedule", "frugal_get_final_flush", "frugal_read_rows", "frugal_read_host",
             "frugal_get_stats", "frugal_get_timeline", "frugal_owned_rows", "frugal_hot_slots"]
 
@@ -184,6 +186,10 @@ class Frugal:
     def dot_model(self, s, emb, x, y, grad, loss, stream=None):
         _check(lib().frugal_dot_model(self.h, s, _ptr(emb), _ptr(x), _ptr(y), _ptr(grad), _ptr(loss),
                                       _stream(stream)))
+
+    def transe_model(self, s, emb, chunk, gamma, grad, loss, stream=None):
+        _check(lib().frugal_transe_model(self.h, s, _ptr(emb), chunk, gamma, _ptr(grad), _ptr(loss),
+                                         _stream(stream)))
 
     def backward_update(self, s, grad, stream=None):
         _check(lib().frugal_backward_update(self.h, s, _ptr(grad), _stream(stream)))

@@ -50,9 +50,12 @@ class Trainer:
         if on_schedule:
             on_schedule(s)
         fr.lookup(s, self.emb)
-        x = torch.from_numpy(st.x[s, self.rank]).to(self.dev, non_blocking=False)
-        y = torch.from_numpy(st.y[s, self.rank]).to(self.dev, non_blocking=False)
-        fr.dot_model(s, self.emb, x, y, self.grad, self.loss[s:s + 1])
+        if st.cfg.model == "transe":
+            fr.transe_model(s, self.emb, st.cfg.neg_chunk, st.cfg.gamma, self.grad, self.loss[s:s + 1])
+        else:
+            x = torch.from_numpy(st.x[s, self.rank]).to(self.dev, non_blocking=False)
+            y = torch.from_numpy(st.y[s, self.rank]).to(self.dev, non_blocking=False)
+            fr.dot_model(s, self.emb, x, y, self.grad, self.loss[s:s + 1])
         fr.backward_update(s, self.grad)
         self.s += 1
 

@@ -19,7 +19,10 @@ Workload recipe (DESIGN.md §"Input recipe"):
   (22 tables, ~9.4e6 rows, d=64), CriteoTB-shaped (Kaggle profile scaled to
   ~8.8e8 rows, d=128), plus the tiny 1-table config.
 * Labels: planted y = [sum_f h(id_f) > 0] with h = +-1 from a hash of the id
-  (SURVEY §8(c) Q15).  Dense features x_b ~ N(0, 0.1^2) in R^d, frozen (they
+  (SURVEY §8(c) Q15).  KG workloads (TransE, §4.1): samples are
+  triples (h, r, t) plus one corrupting entity "neg" per triple; the negatives of a
+  chunk of neg_chunk triples are shared by the chunk (DGL-KE chunked negative sampling,
+  "negative sampling batch size of 200").  Entities and relations are Zipf(alpha).  Dense features x_b ~ N(0, 0.1^2) in R^d, frozen (they
   stand in for DLRM's bottom-MLP output).
 * Hot (cached) set: the top floor(cache_ratio * N_f) rows of each table by
   frequency over the first min(S, 50) steps of the stream, ties broken by the
@@ -65,10 +68,19 @@ class WorkloadConfig:
     seed_labels: int = 2
     seed_init: int = 3
     seed_dense: int = 4
+    # slot f reads table slot_tables[f] (None: slot f reads table f).  KG workloads use
+    # slots (h, r, t, neg) -> tables (entities, relations, entities, entities).
+    slot_tables: Optional[List[int]] = None
+    model: str = "dot"       # "dot" (REC glue, R15) | "transe" (KG glue, R26)
+    neg_chunk: int = 200     # TransE: negatives shared by chunks of this many triples (L1287-1288)
+    gamma: float = 12.0      # TransE margin (DGL-KE default)
 
     @property
     def slots(self) -> int:
-        return len(self.table_rows)
+        return len(self.slot_tables) if self.slot_tables is not None else len(self.table_rows)
+
+    def slot_table(self, f: int) -> int:
+        return self.slot_tables[f] if self.slot_tables is not None else f
 
     @property
     def n_rows(self) -> int:
@@ -87,6 +99,15 @@ def config(name: str, **over) -> WorkloadConfig:
         c = WorkloadConfig("criteo_kaggle", list(CRITEO_KAGGLE_ROWS), dim=32, batch=8192, world=8)
     elif name == "avazu":       # configs[2]
         c = WorkloadConfig("avazu", list(AVAZU_ROWS), dim=64, batch=16384, world=8, cache_ratio=0.10)
+    elif name == "freebase":    # configs[3]: Freebase-shaped KG (Table 2: 86.1M entities, 14.8K relations)
+        c = WorkloadConfig("freebase", [86_100_000, 14_824], dim=400, batch=2000, world=8,
+                           slot_tables=[0, 1, 0, 0], model="transe", neg_chunk=200)
+    elif name == "fb15k":       # FB15k-shaped KG (Table 2, columns read as 15k entities, 1.3k relations)
+        c = WorkloadConfig("fb15k", [14_951, 1_345], dim=400, batch=1200, world=8,
+                           slot_tables=[0, 1, 0, 0], model="transe", neg_chunk=200)
+    elif name == "tiny_kg":     # small KG case for parity tests
+        c = WorkloadConfig("tiny_kg", [5_000, 40], dim=16, batch=96, world=1, slot_tables=[0, 1, 0, 0],
+                           model="transe", neg_chunk=32, lookahead=4, age_out=3)
     elif name == "criteo_tb":   # configs[4]
         scale = 8.8e8 / sum(CRITEO_KAGGLE_ROWS)
         rows = [max(1, int(round(r * scale))) for r in CRITEO_KAGGLE_ROWS]
@@ -207,10 +228,12 @@ def gen_ids(cfg: WorkloadConfig, steps: int, world: Optional[int] = None) -> np.
     offs = cfg.table_offsets
     ids = np.empty((steps, world, B, F), dtype=np.int64)
     for s in range(steps):
-        for f, nf in enumerate(cfg.table_rows):
+        for f in range(F):
+            tb = cfg.slot_table(f)
+            nf = cfg.table_rows[tb]
             r = zipf_ranks(rng, nf, cfg.alpha, world * B) - 1
-            local = feistel_permute(r, nf, cfg.seed_ids * 1000003 + f)
-            ids[s, :, :, f] = (offs[f] + local).reshape(world, B)
+            local = feistel_permute(r, nf, cfg.seed_ids * 1000003 + tb)
+            ids[s, :, :, f] = (offs[tb] + local).reshape(world, B)
     return ids.reshape(steps, world, B * F)
 
 
@@ -229,8 +252,8 @@ def hot_set(cfg: WorkloadConfig, ids: np.ndarray, counts: Optional[np.ndarray] =
         k = int(math.floor(cfg.cache_ratio * nf))
         if k <= 0:
             continue
-        col = sub[:, :, :, f][valid] - offs[f]
-        freq = np.bincount(col, minlength=nf)
+        cols = [sub[:, :, :, q][valid] - offs[f] for q in range(F) if cfg.slot_table(q) == f]
+        freq = np.bincount(np.concatenate(cols), minlength=nf)
         # sort by (-freq, id): stable argsort of -freq keeps smaller ids first
         order = np.argsort(-freq, kind="stable")[:k]
         hot.append(offs[f] + order)

@@ -232,3 +232,17 @@ def test_pipeline_modes_parity(env):
     out = subprocess.run([sys.executable, "-c", code], env=e, capture_output=True, text=True,
                          cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=600)
     assert "OK True" in out.stdout, out.stdout + out.stderr
+
+
+@pytest.mark.parametrize("opt", ["adagrad", "sgd"])
+def test_kg_transe_parity(opt):
+    """KG workload (configs[3] shape, small): TransE glue with chunked shared negatives;
+    entities and relations in one id space, slots (h, r, t, neg) -> tables (E, R, E, E)."""
+    cfg = W.config("tiny_kg", opt=opt, lr=0.05 if opt == "adagrad" else 0.5)
+    rng = np.random.default_rng(5)
+    counts = rng.integers(0, cfg.batch + 1, size=(30, 1)).astype(np.int32)
+    counts[4] = 0
+    st = W.gen_stream(cfg, 30, counts=counts)
+    r = run_parity(st)
+    assert r["exact"]
+    r["fr"].close()

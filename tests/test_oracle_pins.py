@@ -349,3 +349,40 @@ def test_cross_world_equivalence_sgd():
     np.testing.assert_allclose(w1, w2, rtol=0, atol=1e-6)
     for s in range(S):
         assert abs(o1.loss(s) - o2.loss(s)) < 1e-9
+
+
+# ----------------------------------------------------------------------------- TransE glue (R26)
+def test_transe_glue_vs_torch_fp64():
+    """KG glue: TransE-L2 with chunked shared negatives -- loss and
+    per-row gradients equal fp64 torch.autograd of the same objective."""
+    torch = pytest.importorskip("torch")
+    cfg = W.config("tiny_kg", batch=20, neg_chunk=8, dim=6, world=2, table_rows=[40, 5], alpha=0.5)
+    st = W.gen_stream(cfg, 3, counts=np.array([[20, 13], [7, 20], [0, 20]], dtype=np.int32))
+    o = Oracle(st)
+    F, d = 4, cfg.dim
+    for s in range(st.steps):
+        ks = np.arange(cfg.n_rows)
+        w0, _ = o.read_rows(ks)
+        o.step()
+        E = torch.tensor(w0, dtype=torch.float64, requires_grad=True)
+        nb = int(st.counts[s].sum())
+        loss = 0
+        for g in range(2):
+            cnt = int(st.counts[s, g])
+            ids = torch.tensor(st.ids[s, g, :cnt * F].reshape(cnt, F))
+            for b0 in range(0, cnt, cfg.neg_chunk):
+                c = ids[b0:b0 + cfg.neg_chunk]
+                h, r, t, neg = E[c[:, 0]], E[c[:, 1]], E[c[:, 2]], E[c[:, 3]]
+                pos = cfg.gamma - torch.linalg.norm(h + r - t, dim=1)
+                negs = cfg.gamma - torch.linalg.norm((h + r)[:, None, :] - neg[None, :, :], dim=2)
+                loss = loss + torch.nn.functional.softplus(-pos).sum() + torch.nn.functional.softplus(negs).mean(1).sum()
+        if nb == 0:
+            continue
+        (loss / nb).backward()
+        assert abs(o.loss(s) - float(loss.detach()) / nb) < 1e-9 * max(1.0, abs(float(loss.detach())))
+        acc = np.zeros_like(w0, dtype=np.float64)
+        for g in range(2):
+            cnt = int(st.counts[s, g])
+            np.add.at(acc, st.ids[s, g, :cnt * F], o.grad(g)[:cnt * F].astype(np.float64))
+        ref = E.grad.numpy()
+        assert np.abs(acc - ref).max() <= 1e-6 * max(1e-3, np.abs(ref).max())
