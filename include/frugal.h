@@ -56,8 +56,11 @@ typedef enum {
 } frugal_mode;
 
 enum {
-    FRUGAL_F_RECORD = 1, /* keep per-step schedule artefacts for frugal_get_schedule */
-    FRUGAL_F_TIMERS = 2  /* record CUDA events around every phase (frugal_get_timers) */
+    FRUGAL_F_RECORD = 1,        /* keep per-step schedule artefacts for frugal_get_schedule  */
+    FRUGAL_F_TIMERS = 2,        /* record CUDA events around every phase (frugal_get_stats)  */
+    FRUGAL_F_NO_HOST_STATE = 4  /* Adagrad: no host copy of G (it lives in HBM, R8); the final
+                                   flush then writes w only -- for tables whose w and G do not
+                                   both fit in host memory (e.g. configs[3], 2 x 138 GB)      */
 };
 
 enum { FRUGAL_FLUSH_ALL = 0 };

@@ -5,6 +5,7 @@
 // written (sums over k, j, b ascending), gradients rounded to fp32 once.
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "frugal_internal.cuh"
 #include "kutil.cuh"
@@ -97,16 +98,203 @@ __global__ void k_transe_grads(const float* __restrict__ emb, int count, int C, 
     }
 }
 
+// ---- tiled versions (default): 32x32 output tiles per CTA of 256 threads, each thread 2x2
+// outputs; operand tiles of 32 (k, j or b) staged in shared memory as fp64.  Every output
+// still accumulates in the written order (k / j / b ascending), so the results equal the
+// loops above bit for bit.
+constexpr int TT = 32;
+
+// distances of all (b, j) pairs of a chunk: W[b][j] = sigma(gamma - dist)/dist/nC, loss
+__global__ void __launch_bounds__(256) k_transe_pairs_tiled(const float* __restrict__ emb, int count, int C, int d,
+                                                            double gamma, double* __restrict__ Wm, double* loss,
+                                                            double nb) {
+    __shared__ double Ps[TT][TT + 1];
+    __shared__ double Ns[TT][TT + 1];
+    const int tiles = (C + TT - 1) / TT;
+    const int c = blockIdx.x / (tiles * tiles), tb = (blockIdx.x / tiles) % tiles, tj = blockIdx.x % tiles;
+    const int b0 = c * C, nC = min(C, count - b0);
+    if (tb * TT >= nC || tj * TT >= nC) return;
+    const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;  // thread owns b = ty*2+{0,1}, j = tx*2+{0,1}
+    double acc[2][2] = {{0.0, 0.0}, {0.0, 0.0}};
+    for (int k0 = 0; k0 < d; k0 += TT) {
+        for (int e = threadIdx.x; e < TT * TT; e += 256) {
+            const int r = e / TT, kk = e % TT, k = k0 + kk;
+            const int bl = tb * TT + r, jl = tj * TT + r;
+            double pv = 0.0, nv = 0.0;
+            if (k < d && bl < nC) {
+                const int64_t b = b0 + bl;
+                pv = __dadd_rn((double)emb[(b * 4 + 0) * d + k], (double)emb[(b * 4 + 1) * d + k]);
+            }
+            if (k < d && jl < nC) nv = (double)emb[((int64_t)(b0 + jl) * 4 + 3) * d + k];
+            Ps[r][kk] = pv;
+            Ns[r][kk] = nv;
+        }
+        __syncthreads();
+        const int kend = min(TT, d - k0);
+        for (int kk = 0; kk < kend; kk++) {
+#pragma unroll
+            for (int i = 0; i < 2; i++)
+#pragma unroll
+                for (int q = 0; q < 2; q++) {
+                    const double u = __dsub_rn(Ps[ty * 2 + i][kk], Ns[tx * 2 + q][kk]);
+                    acc[i][q] = __dadd_rn(acc[i][q], __dmul_rn(u, u));
+                }
+        }
+        __syncthreads();
+    }
+    double lsum = 0.0;
+#pragma unroll
+    for (int i = 0; i < 2; i++)
+#pragma unroll
+        for (int q = 0; q < 2; q++) {
+            const int bl = tb * TT + ty * 2 + i, jl = tj * TT + tx * 2 + q;
+            if (bl < nC && jl < nC) {
+                const double dist = __dsqrt_rn(acc[i][q]);
+                const double sc = __dsub_rn(gamma, dist);
+                lsum += __ddiv_rn(softplus(sc), (double)nC);
+                Wm[(int64_t)(b0 + bl) * C + jl] = dist > 0.0 ? __ddiv_rn(__ddiv_rn(sigm(sc), dist), (double)nC) : 0.0;
+            }
+        }
+    __shared__ double sl[8];
+    for (int o = 16; o; o >>= 1) lsum += __shfl_xor_sync(FULL, lsum, o);
+    if ((threadIdx.x & 31) == 0) sl[threadIdx.x >> 5] = lsum;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int i = 0; i < 8; i++) t += sl[i];
+        if (t != 0.0) atomicAdd(loss, t / nb);
+    }
+}
+
+// positive triples: a_b = (1 - sigma(gamma - |v|))/|v|, loss (thread per b, k sequential)
+__global__ void k_transe_pos(const float* __restrict__ emb, int count, int d, double gamma, double* __restrict__ A,
+                             double* loss, double nb) {
+    double lsum = 0.0;
+    for (int b = blockIdx.x * blockDim.x + threadIdx.x; b < count; b += gridDim.x * blockDim.x) {
+        double acc = 0.0;
+        for (int k = 0; k < d; k++) {
+            const double P = __dadd_rn((double)emb[((int64_t)b * 4 + 0) * d + k], (double)emb[((int64_t)b * 4 + 1) * d + k]);
+            const double v = __dsub_rn(P, (double)emb[((int64_t)b * 4 + 2) * d + k]);
+            acc = __dadd_rn(acc, __dmul_rn(v, v));
+        }
+        const double dist = __dsqrt_rn(acc);
+        const double sc = __dsub_rn(gamma, dist);
+        lsum += softplus(-sc);
+        A[b] = dist > 0.0 ? __ddiv_rn(__dsub_rn(1.0, sigm(sc)), dist) : 0.0;
+    }
+    for (int o = 16; o; o >>= 1) lsum += __shfl_xor_sync(FULL, lsum, o);
+    if ((threadIdx.x & 31) == 0 && lsum != 0.0) atomicAdd(loss, lsum / nb);
+}
+
+// gradients: MODE 0: (h, r, t) rows, output tile (b, k), reduction over j ascending;
+//            MODE 1: negative rows,  output tile (j, k), reduction over b ascending.
+template <int MODE>
+__global__ void __launch_bounds__(256) k_transe_grads_tiled(const float* __restrict__ emb, int count, int C, int d,
+                                                            const double* __restrict__ Wm,
+                                                            const double* __restrict__ A, float* __restrict__ grad,
+                                                            double nb) {
+    __shared__ double Ws[TT][TT + 1];  // [out row][red]
+    __shared__ double Xs[TT][TT + 1];  // [red][k]: N (mode 0) or P (mode 1)
+    const int rtiles = (C + TT - 1) / TT, ktiles = (d + TT - 1) / TT;
+    const int c = blockIdx.x / (rtiles * ktiles), tr = (blockIdx.x / ktiles) % rtiles, tk = blockIdx.x % ktiles;
+    const int b0 = c * C, nC = min(C, count - b0);
+    if (tr * TT >= nC) return;
+    const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;  // outputs rows ty*2+{0,1}, k tx*2+{0,1}
+    double own[2][2], accv[2][2];
+#pragma unroll
+    for (int i = 0; i < 2; i++)
+#pragma unroll
+        for (int q = 0; q < 2; q++) {
+            const int rl = tr * TT + ty * 2 + i, k = tk * TT + tx * 2 + q;
+            own[i][q] = 0.0;
+            accv[i][q] = 0.0;
+            if (rl < nC && k < d) {
+                const int64_t b = b0 + rl;
+                if (MODE == 0) {
+                    const double P = __dadd_rn((double)emb[(b * 4 + 0) * d + k], (double)emb[(b * 4 + 1) * d + k]);
+                    own[i][q] = P;
+                    accv[i][q] = __dmul_rn(A[b], __dsub_rn(P, (double)emb[(b * 4 + 2) * d + k]));  // a_b v
+                } else {
+                    own[i][q] = (double)emb[(b * 4 + 3) * d + k];  // n_j
+                }
+            }
+        }
+    const double keep[2][2] = {{accv[0][0], accv[0][1]}, {accv[1][0], accv[1][1]}};  // a_b v (mode 0)
+    for (int r0 = 0; r0 < nC; r0 += TT) {
+        for (int e = threadIdx.x; e < TT * TT; e += 256) {
+            const int x = e / TT, y = e % TT;
+            // Ws[x][y] = W[out row x][red y]   (mode 0: W[b][j]; mode 1: W[b=red][j=out])
+            const int ol = tr * TT + x, rl = r0 + y;
+            double wv = 0.0;
+            if (ol < nC && rl < nC) wv = MODE == 0 ? Wm[(int64_t)(b0 + ol) * C + rl] : Wm[(int64_t)(b0 + rl) * C + ol];
+            Ws[x][y] = wv;
+            // Xs[x][y] = operand of reduction row x at k = tk*TT + y
+            const int rl2 = r0 + x, k = tk * TT + y;
+            double xv = 0.0;
+            if (rl2 < nC && k < d) {
+                const int64_t rr = b0 + rl2;
+                xv = MODE == 0 ? (double)emb[(rr * 4 + 3) * d + k]
+                               : __dadd_rn((double)emb[(rr * 4 + 0) * d + k], (double)emb[(rr * 4 + 1) * d + k]);
+            }
+            Xs[x][y] = xv;
+        }
+        __syncthreads();
+        const int rend = min(TT, nC - r0);
+        for (int y = 0; y < rend; y++) {
+#pragma unroll
+            for (int i = 0; i < 2; i++)
+#pragma unroll
+                for (int q = 0; q < 2; q++) {
+                    const double w = Ws[ty * 2 + i][y];
+                    const double x = Xs[y][tx * 2 + q];
+                    if (MODE == 0) {  // gh -= W_bj (P_b - n_j)
+                        accv[i][q] = __dsub_rn(accv[i][q], __dmul_rn(w, __dsub_rn(own[i][q], x)));
+                    } else {          // gn += W_bj (P_b - n_j)
+                        accv[i][q] = __dadd_rn(accv[i][q], __dmul_rn(w, __dsub_rn(x, own[i][q])));
+                    }
+                }
+        }
+        __syncthreads();
+    }
+#pragma unroll
+    for (int i = 0; i < 2; i++)
+#pragma unroll
+        for (int q = 0; q < 2; q++) {
+            const int rl = tr * TT + ty * 2 + i, k = tk * TT + tx * 2 + q;
+            if (rl < nC && k < d) {
+                const int64_t b = b0 + rl;
+                if (MODE == 0) {
+                    const float g = (float)__ddiv_rn(accv[i][q], nb);
+                    grad[(b * 4 + 0) * d + k] = g;
+                    grad[(b * 4 + 1) * d + k] = g;
+                    grad[(b * 4 + 2) * d + k] = (float)__ddiv_rn(-keep[i][q], nb);
+                } else {
+                    grad[(b * 4 + 3) * d + k] = (float)__ddiv_rn(accv[i][q], nb);
+                }
+            }
+        }
+}
+
 void launch_transe_model(frugal_ctx* c, QueueSlot& q, const float* emb, int C, double gamma, float* grad,
                          double* loss, int64_t nb, double* Wm, double* A, cudaStream_t st) {
     const int count = q.h_counts[c->g];
     if (count <= 0) return;
     const int nchunks = (count + C - 1) / C;
-    k_transe_pairs<<<grid_for((int64_t)nchunks * C * (C + 1), 256, 8), 256, 0, st>>>(emb, count, C, c->d, gamma, Wm, A,
-                                                                                   loss, (double)nb);
-    k_transe_grads<<<grid_for(2 * (int64_t)count * c->d, 256, 8), 256, 0, st>>>(emb, count, C, c->d, Wm, A, grad,
-                                                                              (double)nb);
-    c->launches += 2;
+    static const bool naive = getenv("FRUGAL_TRANSE_NAIVE") != nullptr;  // reference loops (tests)
+    if (naive) {
+        k_transe_pairs<<<grid_for((int64_t)nchunks * C * (C + 1), 256, 8), 256, 0, st>>>(emb, count, C, c->d, gamma,
+                                                                                       Wm, A, loss, (double)nb);
+        k_transe_grads<<<grid_for(2 * (int64_t)count * c->d, 256, 8), 256, 0, st>>>(emb, count, C, c->d, Wm, A,
+                                                                                  grad, (double)nb);
+        c->launches += 2;
+        return;
+    }
+    const int tiles = (C + TT - 1) / TT, ktiles = (c->d + TT - 1) / TT;
+    k_transe_pos<<<grid_for(count, 256, 4), 256, 0, st>>>(emb, count, c->d, gamma, A, loss, (double)nb);
+    k_transe_pairs_tiled<<<nchunks * tiles * tiles, 256, 0, st>>>(emb, count, C, c->d, gamma, Wm, loss, (double)nb);
+    k_transe_grads_tiled<0><<<nchunks * tiles * ktiles, 256, 0, st>>>(emb, count, C, c->d, Wm, A, grad, (double)nb);
+    k_transe_grads_tiled<1><<<nchunks * tiles * ktiles, 256, 0, st>>>(emb, count, C, c->d, Wm, A, grad, (double)nb);
+    c->launches += 4;
 }
 
 }  // namespace frugal

@@ -366,7 +366,7 @@ void launch_final_flush(frugal_ctx* c, cudaStream_t st) {
     k_final_collect<<<grid_for(c->No, 256, 8), 256, 0, st>>>(c->No, c->state, c->ff_rows, c->ff_cnt);
     c->launches++;
     launch_flush_rows(c, c->ff_rows, nullptr, c->ff_cnt, 1 << 30, FRUGAL_C_FINAL_HOT, st);
-    if (c->cfg.opt == FRUGAL_ADAGRAD && c->No > 0) {
+    if (c->cfg.opt == FRUGAL_ADAGRAD && c->No > 0 && c->dh_G) {
         const int d4 = c->d / 4, gs = group_size(d4);
         int grid = grid_for(c->No * gs, 256, 8);
         DISPATCH_GS(gs, (k_g_push<GS><<<grid, 256, 0, st>>>(c->No, c->n, c->g, d4, (const float4*)c->Gd,
@@ -401,8 +401,7 @@ __global__ void k_init_table(float4* hw, float4* hG, int64_t N, int d, uint64_t 
     }
 }
 void launch_init_table(frugal_ctx* c, cudaStream_t st) {
-    k_init_table<<<kSMs * 8, 256, 0, st>>>((float4*)c->dh_w,
-                                           c->cfg.opt == FRUGAL_ADAGRAD ? (float4*)c->dh_G : nullptr, c->N, c->d,
+    k_init_table<<<kSMs * 8, 256, 0, st>>>((float4*)c->dh_w, (float4*)c->dh_G, c->N, c->d,
                                            c->cfg.init_seed, c->cfg.init_scale, c->cfg.init_accum);
     c->launches++;
 }
@@ -529,9 +528,7 @@ __global__ void k_read_host(const int64_t* __restrict__ ks, int64_t n, int d, co
     }
 }
 void launch_read_host(frugal_ctx* c, const int64_t* d_k, int64_t n, float* d_w, float* d_G, cudaStream_t st) {
-    k_read_host<<<grid_for(n * c->d, 256, 8), 256, 0, st>>>(d_k, n, c->d, c->dh_w,
-                                                             c->cfg.opt == FRUGAL_ADAGRAD ? c->dh_G : nullptr, d_w,
-                                                             d_G);
+    k_read_host<<<grid_for(n * c->d, 256, 8), 256, 0, st>>>(d_k, n, c->d, c->dh_w, c->dh_G, d_w, d_G);
     c->launches++;
 }
 

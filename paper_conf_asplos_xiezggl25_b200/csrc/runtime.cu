@@ -229,6 +229,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->key_bits = bits_for(c->N - 1);
     c->lk_bits = bits_for(std::max<int64_t>(c->No - 1, 0));
     const bool adag = k.opt == FRUGAL_ADAGRAD;
+    const bool host_G = adag && !(k.flags & FRUGAL_F_NO_HOST_STATE);
     const size_t rowb = (size_t)c->d * sizeof(float);
 
     // ---------------------------------------------------------------- host table (shm)
@@ -238,7 +239,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     const size_t off_w = align_up(off_mail + mail_bytes, 2 << 20);
     const size_t tab = (size_t)c->N * rowb;
     const size_t off_G = align_up(off_w + tab, 2 << 20);
-    const size_t total = adag ? off_G + tab : off_w + tab;
+    const size_t total = host_G ? off_G + tab : off_w + tab;
     c->shm_bytes = total;
     if (k.shm_name) {
         if (c->g == 0) {
@@ -294,7 +295,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->dh_mail = dbase + off_mail;
     c->h_w = (float*)(hbase + off_w);
     c->dh_w = (float*)(dbase + off_w);
-    if (adag) {
+    if (host_G) {
         c->h_G = (float*)(hbase + off_G);
         c->dh_G = (float*)(dbase + off_G);
     }

@@ -246,3 +246,13 @@ def test_kg_transe_parity(opt):
     r = run_parity(st)
     assert r["exact"]
     r["fr"].close()
+
+
+def test_kg_transe_tiles_ragged():
+    """Tiled TransE glue across tile boundaries: d = 72 (k tiles 32+32+8), chunks of 50 (b/j
+    tiles 32+18) and a ragged last chunk of 30, bit-exact against the oracle."""
+    cfg = W.config("tiny_kg", dim=72, neg_chunk=50, batch=130, table_rows=[3000, 30])
+    st = W.gen_stream(cfg, 10)
+    r = run_parity(st)
+    assert r["exact"]
+    r["fr"].close()
