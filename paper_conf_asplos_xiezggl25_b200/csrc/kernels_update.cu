@@ -241,7 +241,7 @@ __global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, 
                             int32_t* __restrict__ state, int32_t* __restrict__ last_upd, int32_t* __restrict__ pool_idx,
                             uint64_t* __restrict__ rbits, float4* __restrict__ cw, float4* __restrict__ Gd,
                             float4* __restrict__ pw, int32_t* __restrict__ pkey, int32_t* pcount, const float4* hw,
-                            unsigned long long* stats) {
+                            const float4* __restrict__ pw_all, int P, int32_t pool_min, unsigned long long* stats) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
@@ -252,6 +252,15 @@ __global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, 
         const int32_t lk = T[j];
         const int64_t k = (int64_t)lk * world + g;
         const int sl = slot[lk];
+        // world > 1: the latest w of a recently updated cold row is still in this owner's pool
+        // (segment last_upd % P, not this step's segment s % P); read before lane 0 rewrites it
+        const int32_t lu = last_upd[lk];
+        const int64_t prow = (sl < 0 && !rows_w && lu >= 0 && lu >= pool_min)
+                                 ? ((int64_t)(lu % P) * capT + pool_idx[lk]) : -1;
+        {  // the group's lanes all read `lu` before its lane 0 rewrites last_upd below
+            const unsigned gmask = GS == 32 ? 0xffffffffu : (((1u << GS) - 1u) << ((threadIdx.x & 31) & ~(GS - 1)));
+            __syncwarp(gmask);
+        }
         uint32_t mask = 1u;
         if (world > 1) mask = Tmask[j];
         for (int v = l; v < d4; v += GS) {
@@ -277,7 +286,8 @@ __global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, 
             }
             float4 w, G = make_float4(0.f, 0.f, 0.f, 0.f);
             if (sl >= 0) w = cw[(int64_t)sl * d4 + v];
-            else w = rows_w ? rows_w[j * d4 + v] : hw[k * d4 + v];
+            else if (rows_w) w = rows_w[j * d4 + v];  // world 1: staged by this step's gather
+            else w = prow >= 0 ? pw_all[prow * d4 + v] : hw[k * d4 + v];
             if (adagrad) G = Gd[(int64_t)lk * d4 + v];
             float* wp = &w.x;
             float* Gp = &G.x;
@@ -329,7 +339,8 @@ void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, cudaStrea
                         q.T, q.nT, q.Tmask, q.Tidx, c->capT, c->n, c->g, d4, (int32_t)s, adag, c->cfg.lr, c->cfg.eps,
                         (const float4*)c->Pp, q.goff, mail_par, c->mail_stride, rows_w, c->slot, c->state,
                         c->last_upd, c->pool_idx, c->rbits, (float4*)c->cw, (float4*)c->Gd, (float4*)c->pw + pofs,
-                        c->pkey + (size_t)seg * c->capT, c->pcount + seg, (const float4*)c->dh_w, c->dstats)));
+                        c->pkey + (size_t)seg * c->capT, c->pcount + seg, (const float4*)c->dh_w,
+                        (const float4*)c->pw, c->P, (int32_t)std::max<int64_t>(0, s - c->P + 2), c->dstats)));
     c->launches++;
 }
 

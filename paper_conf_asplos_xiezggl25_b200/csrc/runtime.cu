@@ -14,6 +14,7 @@
 #include <string.h>
 #include <sys/mman.h>
 #include <sys/stat.h>
+#include <sys/syscall.h>
 #include <time.h>
 #include <unistd.h>
 #include <stdlib.h>
@@ -113,6 +114,20 @@ struct Timer {
 }  // namespace
 
 // ================================================================================ helpers
+// Spread the host table over every NUMA node (best effort, before the pages are first
+// touched): on a two-socket host each GPU then finds half the rows behind its own root
+// complex instead of all of them behind rank 0's.
+static void interleave_numa(void* base, size_t bytes) {
+    FILE* f = fopen("/sys/devices/system/node/online", "r");
+    if (!f) return;
+    int lo = 0, hi = 0;
+    int got = fscanf(f, "%d-%d", &lo, &hi);
+    fclose(f);
+    if (got < 2 || hi <= lo || hi >= 64) return;
+    unsigned long mask = 0;
+    for (int n = lo; n <= hi; n++) mask |= 1ul << n;
+    syscall(SYS_mbind, base, bytes, 3 /* MPOL_INTERLEAVE */, &mask, 65ul, 0u);
+}
 static frugal_status check_err_word(frugal_ctx* c) {
     if (c->herr && *(volatile int32_t*)c->herr) {
         int e = *(volatile int32_t*)c->herr;
@@ -273,6 +288,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         return FRUGAL_ESHM;
     }
     madvise(c->shm_base, total, MADV_HUGEPAGE);
+    if (c->g == 0 || !k.shm_name) interleave_numa(c->shm_base, total);
     if (cudaHostRegister(c->shm_base, total, cudaHostRegisterMapped | cudaHostRegisterPortable) != cudaSuccess) {
         cudaGetLastError();
         munmap(c->shm_base, total);
