@@ -51,6 +51,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--mode", default="p2f", choices=["p2f", "write_through"],
                     help="write_through = Frugal-Sync (every update flushed on the next step's critical path)")
+    ap.add_argument("--exchange", default="host", choices=["host", "a2a"],
+                    help="a2a = the comparison path: rows/partials by all-to-all over the process group "
+                         "(NCCL/NVLink) instead of the host table and mailbox (N > 1)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for barriers / the max-over-ranks timing only")
     return ap.parse_args()
@@ -236,8 +239,11 @@ def main():
     shm = f"/frugal_bench_{os.environ.get('MASTER_PORT', '0')}" if world > 1 else None
     host_bytes = cfg.n_rows * 4 * d * (2 if cfg.opt == "adagrad" else 1)
     no_host_state = host_bytes > 150e9  # configs[3]: w + G do not both fit in host RAM
+    a2a = args.exchange == "a2a"
+    if a2a and world == 1:
+        sys.exit("--exchange a2a needs N > 1")
     fr = make_context(st, rank=rank, device=local, shm_name=shm,
-                      flags=F.F_TIMERS | (F.F_NO_HOST_STATE if no_host_state else 0),
+                      flags=F.F_TIMERS | (F.F_NO_HOST_STATE if no_host_state else 0) | (F.F_A2A if a2a else 0),
                       mode=F.MODE_WRITE_THROUGH if args.mode == "write_through" else F.MODE_P2F)
     barrier()
     stream = torch.cuda.current_stream(dev)
@@ -260,16 +266,54 @@ def main():
         fr.prefetch(t, ids_d[t], counts[t])
 
     kg = cfg.model == "transe"
+    host_staging = args.dist_backend == "gloo"
+    ids_send = torch.empty(B * Fs, dtype=torch.int32, device=dev)
+    part_send = torch.empty(B * Fs, d, device=dev)
+
+    def a2a(send, send_counts, recv_counts, inner):
+        rc = [int(c) * inner for c in recv_counts]
+        sc = [int(c) * inner for c in send_counts]
+        src = send.reshape(-1)[:sum(sc)]
+        if host_staging:
+            src = src.cpu()
+        out = torch.empty(sum(rc), dtype=send.dtype, device=src.device)
+        dist.all_to_all_single(out, src, rc, sc)
+        return out.to(dev, non_blocking=True)
+
+    def lookup(s):
+        if not a2a:
+            fr.lookup(s, emb)
+            return
+        sc = fr.a2a_requests(s, ids_send)
+        sct = torch.tensor(sc, dtype=torch.int64, device=coll_dev)
+        rct = torch.empty_like(sct)
+        dist.all_to_all_single(rct, sct)
+        rc = rct.cpu().numpy()
+        ids_in = a2a(ids_send, sc, rc, 1)
+        rows_out = torch.empty(int(rc.sum()), d, device=dev)
+        fr.a2a_serve(s, ids_in, int(rc.sum()), rows_out)
+        rows_in = a2a(rows_out, rc, sc, d)
+        fr.a2a_lookup(s, rows_in, emb)
+        lookup.counts = (sc, rc)
+
+    def backward(s):
+        if not a2a:
+            fr.backward_update(s, grad)
+            return
+        sc, rc = lookup.counts
+        fr.a2a_pack(s, grad, part_send)
+        part_in = a2a(part_send, sc, rc, d)
+        fr.a2a_update(s, part_in, rc)
 
     def step_dev(s):
         t = s + L
         fr.step(s, ids_d[t], counts[t])
-        fr.lookup(s, emb)
+        lookup(s)
         if kg:
             fr.transe_model(s, emb, cfg.neg_chunk, cfg.gamma, grad, loss[s:s + 1])
         else:
             fr.dot_model(s, emb, x_d[s], y_d[s], grad, loss[s:s + 1])
-        fr.backward_update(s, grad)
+        backward(s)
 
     copy_stream = torch.cuda.Stream(dev)
     x_e = [torch.empty(B, d, device=dev) for _ in range(2)]
@@ -290,14 +334,14 @@ def main():
         b = s & 1
         fr.step(s, ids_h[t], counts[t])       # ids copied from pinned host inside the call
         load_xy(s + 1)
-        fr.lookup(s, emb)
+        lookup(s)
         stream.wait_event(xy_ready[b])
         if kg:
             fr.transe_model(s, emb, cfg.neg_chunk, cfg.gamma, grad, loss[s:s + 1])
         else:
             fr.dot_model(s, emb, x_e[b], y_e[b], grad, loss[s:s + 1])
         xy_free[b].record(stream)
-        fr.backward_update(s, grad)
+        backward(s)
         loss_h[s:s + 1].copy_(loss[s:s + 1], non_blocking=True)  # the step's result back to the host
 
     # ---- warm-up
@@ -411,7 +455,8 @@ def main():
         "config": {"workload": f"{cfg.name} ({CONFIG_NAMES.get(cfg.name, '')})", "global_batch": world * B,
                    "batch_per_gpu": B, "tables": Fs, "rows": cfg.n_rows, "dim": d, "alpha": cfg.alpha,
                    "lookahead": L, "age_out": cfg.age_out, "cache_ratio": cfg.cache_ratio, "opt": cfg.opt,
-                   "flush_mode": args.mode,
+                   "flush_mode": args.mode, "exchange": "host table + mailbox (P2F)" if not a2a else
+                   "all-to-all over the process group (comparison path)",
                    "parallelism": f"dp{world} (owner-sharded rows, shared pinned host table)",
                    "l2": "inputs larger than L2: host table %.1f GB, HBM cache %.0f MB, %d distinct id batches"
                          % (cfg.n_rows * r * (1 if (no_host_state or not adag) else 2) / 1e9, len(st.hot) * r / 1e6, K),

@@ -58,9 +58,14 @@ typedef enum {
 enum {
     FRUGAL_F_RECORD = 1,        /* keep per-step schedule artefacts for frugal_get_schedule  */
     FRUGAL_F_TIMERS = 2,        /* record CUDA events around every phase (frugal_get_stats)  */
-    FRUGAL_F_NO_HOST_STATE = 4  /* Adagrad: no host copy of G (it lives in HBM, R8); the final
+    FRUGAL_F_NO_HOST_STATE = 4, /* Adagrad: no host copy of G (it lives in HBM, R8); the final
                                    flush then writes w only -- for tables whose w and G do not
                                    both fit in host memory (e.g. configs[3], 2 x 138 GB)      */
+    FRUGAL_F_A2A = 8            /* comparison path (the message pipeline of
+                                   PAPER.md Fig. 2b): rows and gradients move between
+                                   ranks by the caller's all-to-all (NCCL over NVLink) through
+                                   the frugal_a2a_* calls instead of the host table/mailbox;
+                                   world > 1 only                                           */
 };
 
 enum { FRUGAL_FLUSH_ALL = 0 };
@@ -157,6 +162,32 @@ frugal_status frugal_dot_model(frugal_ctx* ctx, int64_t s, const float* d_emb, c
    Requires slots == 4. */
 frugal_status frugal_transe_model(frugal_ctx* ctx, int64_t s, const float* d_emb, int32_t chunk, float gamma,
                                   float* d_grad, double* d_loss, frugal_stream stream);
+
+/* ---- comparison path (FRUGAL_F_A2A) -------------------------------------------------
+   Per step: frugal_step(s) -> frugal_a2a_requests(s) -> [caller: all-to-all of the ids] ->
+   frugal_a2a_serve(s) -> [all-to-all of the rows back] -> frugal_a2a_lookup(s) -> glue ->
+   frugal_a2a_pack(s) -> [all-to-all of the partials] -> frugal_a2a_update(s).  Segment r of
+   every buffer is the part to/from rank r, ids ascending within a segment.
+   requests: d_ids [n_uniq] (device, int32 global ids, grouped by owner), counts[world] (host)
+             = ids this rank asks each owner for.
+   serve:    d_ids_in [n_in]: ids other ranks asked this owner for (segments by requester);
+             d_rows [n_in][dim]: their current values (cache, pool or host).
+   lookup:   d_rows_in [n_uniq][dim] in the order of requests (NULL if none); d_out as
+             frugal_lookup.
+   pack:     d_partials [n_uniq][dim]: per distinct row, the segment-reduced gradient, in the
+             order of requests.
+   update:   d_partials_in: the partials other ranks sent this owner, segments by sender;
+             recv_counts[world] (host; d_partials_in may be NULL if they sum to 0).  Merge in
+             rank order + optimizer, as backward_update. */
+frugal_status frugal_a2a_requests(frugal_ctx* ctx, int64_t s, int32_t* d_ids, int64_t* counts, frugal_stream stream);
+frugal_status frugal_a2a_serve(frugal_ctx* ctx, int64_t s, const int32_t* d_ids_in, int64_t n_in, float* d_rows,
+                               frugal_stream stream);
+frugal_status frugal_a2a_lookup(frugal_ctx* ctx, int64_t s, const float* d_rows_in, float* d_out,
+                                frugal_stream stream);
+frugal_status frugal_a2a_pack(frugal_ctx* ctx, int64_t s, const float* d_grad, float* d_partials,
+                              frugal_stream stream);
+frugal_status frugal_a2a_update(frugal_ctx* ctx, int64_t s, const float* d_partials_in, const int64_t* recv_counts,
+                                frugal_stream stream);
 
 /* ---- introspection (tests / bench only; synchronise and copy to caller-owned host
    buffers) ---------------------------------------------------------------------- */

@@ -177,6 +177,9 @@ struct frugal_ctx {
     int64_t early_issued = -1;                          // last step whose early gather was launched
     bool early = false;                                 // pipelined gather enabled (world 1)
     bool pool_hits = true;                              // owner reads its dirty-pool rows from HBM
+    bool a2a = false;                                   // comparison path (FRUGAL_F_A2A)
+    bool xhost = false;                                 // world > 1 and host-bounced exchange
+    int32_t* a2a_roff = nullptr;                        // [world] receive offsets (device)
     bool side_pending[2] = {false, false};
 
     // call-order state
@@ -222,8 +225,12 @@ void launch_transe_model(frugal_ctx* c, QueueSlot& q, const float* emb, int C, d
                          double* loss, int64_t nb, double* Wm, double* A, cudaStream_t st);
 void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const float* x, const float* y,
                       float* grad, double* loss, int64_t nb, cudaStream_t st);
-void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, cudaStream_t st);
-void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, cudaStream_t st);
+void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, float* dest, cudaStream_t st);
+void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, const float* recv, const int32_t* roff,
+                      cudaStream_t st);
+void launch_a2a_ids(frugal_ctx* c, QueueSlot& q, int32_t* ids, cudaStream_t st);
+void launch_serve_rows(frugal_ctx* c, const int32_t* ids, int64_t n, int64_t s, float* out, cudaStream_t st);
+void launch_a2a_place(frugal_ctx* c, QueueSlot& q, const float* in, float* rows, cudaStream_t st);
 void launch_final_flush(frugal_ctx* c, cudaStream_t st);
 void launch_init_table(frugal_ctx* c, cudaStream_t st);
 void launch_init_meta(frugal_ctx* c, const int64_t* d_hot_global, int64_t n_hot, cudaStream_t st);

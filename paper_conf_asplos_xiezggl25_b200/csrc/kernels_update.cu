@@ -187,14 +187,17 @@ __global__ void __launch_bounds__(256) k_segred_combine(const int32_t* __restric
     if (gl) block_fence_system();
 }
 
-void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, cudaStream_t st) {
+void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, float* dest, cudaStream_t st) {
     const int d4 = c->d / 4, gs = group_size(d4);
     int grid = grid_for((int64_t)c->M * gs, 256, 8);
     const bool multi = c->n > 1;
-    float4* mail = multi ? (float4*)(c->dh_mail + ((size_t)par * c->n + c->g) * c->mail_stride + 256) : nullptr;
+    // dest (comparison path): every partial, own or not, to one device buffer in grouped order
+    float4* mail = dest ? (float4*)dest
+                        : multi ? (float4*)(c->dh_mail + ((size_t)par * c->n + c->g) * c->mail_stride + 256) : nullptr;
+    float* Pp = dest ? dest : c->Pp;
     cudaMemsetAsync(c->long_cnt, 0, 8, st);  // long_cnt[0] = long segments, long_cnt[1] = chunk tasks
     DISPATCH_GS(gs, (k_segreduce<GS><<<grid, 256, 0, st>>>(q.off, q.pos, q.n_uniq, multi ? q.gl : nullptr, q.goff,
-                                                           c->g, d4, (const float4*)grad, (float4*)c->Pp, mail,
+                                                           c->g, d4, (const float4*)grad, (float4*)Pp, mail,
                                                            c->long_q, c->long_cnt, c->long_tasks, c->long_cnt + 1,
                                                            c->dstats)));
     static unsigned attr_mask = 0;
@@ -209,7 +212,7 @@ void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, c
                                                                           (float4*)c->chunk_scratch, c->long_tasks,
                                                                           c->long_cnt + 1)));
     DISPATCH_GS(gs, (k_segred_combine<GS><<<kSMs, 256, kOrderedSmem, st>>>(q.off, multi ? q.gl : nullptr, q.goff, c->g,
-                                                                           d4, (float4*)c->Pp, mail, c->long_q,
+                                                                           d4, (float4*)Pp, mail, c->long_q,
                                                                            c->long_cnt,
                                                                            (const float4*)c->chunk_scratch)));
     c->launches += 3;
@@ -241,7 +244,9 @@ __global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, 
                             int32_t* __restrict__ state, int32_t* __restrict__ last_upd, int32_t* __restrict__ pool_idx,
                             uint64_t* __restrict__ rbits, float4* __restrict__ cw, float4* __restrict__ Gd,
                             float4* __restrict__ pw, int32_t* __restrict__ pkey, int32_t* pcount, const float4* hw,
-                            const float4* __restrict__ pw_all, int P, int32_t pool_min, unsigned long long* stats) {
+                            const float4* __restrict__ pw_all, int P, int32_t pool_min,
+                            const float4* __restrict__ recv, const int32_t* __restrict__ roff,
+                            unsigned long long* stats) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
@@ -273,7 +278,9 @@ __global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, 
                     if (!((mask >> r) & 1u)) continue;
                     const int idx = Tidx[(int64_t)r * capT + j];
                     float4 x;
-                    if (r == g) {
+                    if (recv) {  // comparison path: partials arrived by the caller's all-to-all
+                        x = recv[(int64_t)(roff[r] + idx) * d4 + v];
+                    } else if (r == g) {
                         x = Pp[(int64_t)(goff_own[g] + idx) * d4 + v];
                     } else {
                         const char* mb = mail_par + (size_t)r * mail_stride;
@@ -324,7 +331,8 @@ __global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, 
     block_count(stats + FRUGAL_C_MAIL_IN, world > 1 ? nin : 0u);
 }
 
-void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, cudaStream_t st) {
+void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, const float* recv, const int32_t* roff,
+                      cudaStream_t st) {
     const int d4 = c->d / 4, gs = group_size(d4);
     int grid = grid_for(c->capT * gs, 256, 8);
     const int seg = (int)(s % c->P);
@@ -340,7 +348,8 @@ void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, cudaStrea
                         (const float4*)c->Pp, q.goff, mail_par, c->mail_stride, rows_w, c->slot, c->state,
                         c->last_upd, c->pool_idx, c->rbits, (float4*)c->cw, (float4*)c->Gd, (float4*)c->pw + pofs,
                         c->pkey + (size_t)seg * c->capT, c->pcount + seg, (const float4*)c->dh_w,
-                        (const float4*)c->pw, c->P, (int32_t)std::max<int64_t>(0, s - c->P + 2), c->dstats)));
+                        (const float4*)c->pw, c->P, (int32_t)std::max<int64_t>(0, s - c->P + 2),
+                        (const float4*)recv, roff, c->dstats)));
     c->launches++;
 }
 
@@ -493,6 +502,82 @@ void launch_set_flag(frugal_ctx* c, int which, uint32_t value, cudaStream_t st) 
 }
 void launch_wait_flags(frugal_ctx* c, int which, uint32_t value, cudaStream_t st) {
     k_wait_flags<<<1, 32, 0, st>>>(c->dh_flags + which * 32 * 16, c->n, value, c->err);
+    c->launches++;
+}
+
+// ============================================================================ comparison path (a2a)
+__global__ void k_a2a_ids(const int32_t* __restrict__ uniq, const int32_t* __restrict__ gl, const int32_t* d_nu,
+                          int32_t* __restrict__ ids) {
+    const int n = *d_nu;
+    for (int q = blockIdx.x * blockDim.x + threadIdx.x; q < n; q += gridDim.x * blockDim.x) ids[q] = uniq[gl[q]];
+}
+// owner side: rows other ranks asked for (cache / pool / host, as k_gather_uniq)
+template <int GS>
+__global__ void k_serve_rows(const int32_t* __restrict__ ids, int64_t n, int world, int d4,
+                             const int32_t* __restrict__ slot, const float4* __restrict__ cw, const float4* hw,
+                             const int32_t* __restrict__ last_upd, const int32_t* __restrict__ pool_idx,
+                             const float4* __restrict__ pw, int P, int64_t capT, int32_t pool_min,
+                             float4* __restrict__ out, unsigned long long* stats) {
+    int64_t gid, gs;
+    int l;
+    RowGroup<GS>::ids(gid, gs, l);
+    unsigned nh = 0, nc = 0, np = 0;
+    for (int64_t a = gid; a < n; a += gs) {
+        const int32_t k = ids[a], lk = k / world;
+        const float4* src = hw + (int64_t)k * d4;
+        const int sl = slot[lk];
+        int kind = 0;
+        if (sl >= 0) {
+            src = cw + (int64_t)sl * d4;
+            kind = 1;
+        } else {
+            const int32_t lu = last_upd[lk];
+            if (lu >= 0 && lu >= pool_min) {
+                src = pw + ((int64_t)(lu % P) * capT + pool_idx[lk]) * d4;
+                kind = 2;
+            }
+        }
+        if (l == 0) {
+            nh += kind == 0;
+            nc += kind == 1;
+            np += kind == 2;
+        }
+        for (int v = l; v < d4; v += GS) out[a * d4 + v] = src[v];
+    }
+    block_count(stats + FRUGAL_C_GATHER_HOST, nh);
+    block_count(stats + FRUGAL_C_GATHER_CACHE, nc);
+    block_count(stats + FRUGAL_C_GATHER_POOL, np);
+}
+template <int GS>
+__global__ void k_a2a_place(const int32_t* __restrict__ gl, const int32_t* d_nu, int d4,
+                            const float4* __restrict__ in, float4* __restrict__ rows) {
+    int64_t gid, gs;
+    int l;
+    RowGroup<GS>::ids(gid, gs, l);
+    const int n = *d_nu;
+    for (int64_t q = gid; q < n; q += gs)
+        for (int v = l; v < d4; v += GS) rows[(int64_t)gl[q] * d4 + v] = in[q * d4 + v];
+}
+
+void launch_a2a_ids(frugal_ctx* c, QueueSlot& q, int32_t* ids, cudaStream_t st) {
+    k_a2a_ids<<<grid_for(c->M, 256, 4), 256, 0, st>>>(q.uniq, q.gl, q.n_uniq, ids);
+    c->launches++;
+}
+void launch_serve_rows(frugal_ctx* c, const int32_t* ids, int64_t n, int64_t s, float* out, cudaStream_t st) {
+    if (n <= 0) return;
+    const int d4 = c->d / 4, gs = group_size(d4);
+    int grid = std::min(grid_for(n * gs, 256, 8), c->gather_blocks);
+    const int32_t pool_min = (int32_t)std::max<int64_t>(0, s - c->P + 2);
+    DISPATCH_GS(gs, (k_serve_rows<GS><<<grid, 256, 0, st>>>(ids, n, c->n, d4, c->slot, (const float4*)c->cw,
+                                                            (const float4*)c->dh_w, c->last_upd, c->pool_idx,
+                                                            (const float4*)c->pw, c->P, c->capT, pool_min,
+                                                            (float4*)out, c->dstats)));
+    c->launches++;
+}
+void launch_a2a_place(frugal_ctx* c, QueueSlot& q, const float* in, float* rows, cudaStream_t st) {
+    const int d4 = c->d / 4, gs = group_size(d4);
+    DISPATCH_GS(gs, (k_a2a_place<GS><<<grid_for((int64_t)c->M * gs, 256, 8), 256, 0, st>>>(
+                        q.gl, q.n_uniq, d4, (const float4*)in, (float4*)rows)));
     c->launches++;
 }
 

@@ -158,7 +158,7 @@ static void free_ctx(frugal_ctx* c) {
     F(c->rows_buf[0]); F(c->rows_buf[1]); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->long_tasks); F(c->owned_cnt);
     for (int i = 0; i < 2; i++) { F(c->adj_rows[i]); F(c->adj_p[i]); F(c->adj_cnt[i]); }
     for (int i = 0; i < 2; i++) { F(c->sl_rows[i]); F(c->sl_p[i]); F(c->sl_cnt[i]); }
-    F(c->dstats); F(c->kg_W); F(c->kg_A); F(c->ff_rows); F(c->ff_cnt); F(c->ids_stage);
+    F(c->dstats); F(c->kg_W); F(c->kg_A); F(c->a2a_roff); F(c->ff_rows); F(c->ff_cnt); F(c->ids_stage);
     if (c->herr) cudaFreeHost(c->herr);
     if (c->counts_pin) cudaFreeHost(c->counts_pin);
     for (auto e : c->ev_counts) cudaEventDestroy(e);
@@ -214,6 +214,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     if (k.opt != FRUGAL_SGD && k.opt != FRUGAL_ADAGRAD) { set_err("bad opt"); return FRUGAL_EINVAL; }
     if (k.mode != FRUGAL_MODE_P2F && k.mode != FRUGAL_MODE_WRITE_THROUGH) { set_err("bad mode"); return FRUGAL_EINVAL; }
     if (!k.shm_name && k.world != 1) { set_err("world > 1 needs shm_name"); return FRUGAL_EINVAL; }
+    if ((k.flags & FRUGAL_F_A2A) && k.world < 2) { set_err("FRUGAL_F_A2A needs world > 1"); return FRUGAL_EINVAL; }
     if (k.n_hot < 0 || (k.n_hot > 0 && !k.hot_ids)) { set_err("bad hot set"); return FRUGAL_EINVAL; }
     for (int64_t i = 0; i < k.n_hot; i++)
         if (k.hot_ids[i] < 0 || k.hot_ids[i] >= k.n_rows) { set_err("hot id out of range"); return FRUGAL_EINVAL; }
@@ -235,6 +236,8 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     // box (the zero-copy loads of the next step only delay this step's); FRUGAL_EARLY=1
     c->early = c->n == 1 && getenv("FRUGAL_EARLY") && atoi(getenv("FRUGAL_EARLY"));
     c->pool_hits = !(getenv("FRUGAL_NO_POOL_HITS") && atoi(getenv("FRUGAL_NO_POOL_HITS")));
+    c->a2a = (k.flags & FRUGAL_F_A2A) != 0;
+    c->xhost = c->n > 1 && !c->a2a;
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 32;
     c->gather_blocks = getenv("FRUGAL_GATHER_BLOCKS") ? atoi(getenv("FRUGAL_GATHER_BLOCKS")) : 74;
     c->side_inline = getenv("FRUGAL_SIDE_INLINE") && atoi(getenv("FRUGAL_SIDE_INLINE"));
@@ -395,6 +398,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     DMALLOC(c->ff_cnt, 4);
     DMALLOC(c->ids_stage, (size_t)c->n * c->M * 8);
     DMALLOC(c->dstats, FRUGAL_N_COUNTERS * 8);
+    DMALLOC(c->a2a_roff, 64 * 4);
     cudaMemset(c->dstats, 0, FRUGAL_N_COUNTERS * 8);
     sort_alloc(c->sort, (int64_t)c->n * c->M);
     scan_alloc(c->scan, (int64_t)c->n * c->M);
@@ -611,12 +615,12 @@ static frugal_status launch_drain(frugal_ctx* c, int64_t s, cudaStream_t st, cud
         launch_flush_rows(c, c->sl_rows[par] + c->sl_cap, nullptr, c->sl_cnt[par] + 1, c->side_blocks,
                           FRUGAL_C_SIDE_HOT, sd);
         CK(cudaEventRecord(c->ev_side_first[par], sd));
-        if (c->n > 1) launch_set_flag(c, FLAG_SIDE_FIRST, (uint32_t)(s + 1), sd);
+        if (c->xhost) launch_set_flag(c, FLAG_SIDE_FIRST, (uint32_t)(s + 1), sd);
         launch_flush_rows(c, c->sl_rows[par] + 2 * c->sl_cap, nullptr, c->sl_cnt[par] + 2, c->side_blocks,
                           FRUGAL_C_SIDE_HOT, sd);
         launch_flush_rows(c, c->sl_rows[par] + 3 * c->sl_cap, nullptr, c->sl_cnt[par] + 3, c->side_blocks,
                           FRUGAL_C_SIDE_HOT, sd);
-        if (c->n > 1) launch_set_flag(c, FLAG_SIDE, (uint32_t)(s + 1), sd);
+        if (c->xhost) launch_set_flag(c, FLAG_SIDE, (uint32_t)(s + 1), sd);
         CKL();
     }
     CK(cudaEventRecord(c->ev_side[par], sd));
@@ -667,7 +671,7 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
         // a10: urgent bucket (priority == s) to the host table on the critical path
         Timer tm(c, PH_URGENT, st);
         launch_flush_rows(c, c->sl_rows[par], nullptr, c->sl_cnt[par], 1 << 30, FRUGAL_C_URGENT_HOT, st);
-        if (c->n > 1) launch_set_flag(c, FLAG_URGENT, (uint32_t)(s + 1), st);
+        if (c->xhost) launch_set_flag(c, FLAG_URGENT, (uint32_t)(s + 1), st);
         CKL();
     }
     CK(cudaEventRecord(c->ev_sched, st));
@@ -698,7 +702,7 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
         Timer tm(c, PH_GATE, st);
         // (deadline-s rows are the first part of drain s-1; the side stream is FIFO, so that
         // event also covers every earlier drain)
-        if (c->n == 1) {
+        if (!c->xhost) {  // world 1, or the comparison path: only this rank reads its host rows
             if (s >= 1 && c->side_pending[par ^ 1]) CK(cudaStreamWaitEvent(st, c->ev_side_first[par ^ 1], 0));
         } else {
             launch_wait_flags(c, FLAG_URGENT, (uint32_t)(s + 1), st);
@@ -713,6 +717,7 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
 
 extern "C" frugal_status frugal_lookup(frugal_ctx* c, int64_t s, float* d_out, frugal_stream stream) {
     if (!c || !d_out) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    if (c->a2a) { set_err("context uses FRUGAL_F_A2A: use frugal_a2a_requests/serve/lookup"); return FRUGAL_ESTATE; }
     if (c->phase_in_step != 1 || s != c->cur_step) {
         set_err("lookup(%lld) out of order", (long long)s);
         return FRUGAL_ESTATE;
@@ -793,6 +798,7 @@ extern "C" frugal_status frugal_transe_model(frugal_ctx* c, int64_t s, const flo
 
 extern "C" frugal_status frugal_backward_update(frugal_ctx* c, int64_t s, const float* d_grad, frugal_stream stream) {
     if (!c || !d_grad) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    if (c->a2a) { set_err("context uses FRUGAL_F_A2A: use frugal_a2a_pack/update"); return FRUGAL_ESTATE; }
     if (c->phase_in_step != 2 || s != c->cur_step) {
         set_err("backward_update(%lld) out of order", (long long)s);
         return FRUGAL_ESTATE;
@@ -802,7 +808,7 @@ extern "C" frugal_status frugal_backward_update(frugal_ctx* c, int64_t s, const 
     const int par = (int)(s & 1);
     {
         Timer tm(c, PH_SEGRED, st);
-        launch_segreduce(c, q, d_grad, par, st);
+        launch_segreduce(c, q, d_grad, par, nullptr, st);
     }
     if (c->n > 1) {
         // a7: partials of rows owned by other ranks are in this rank's host mailbox;
@@ -814,7 +820,102 @@ extern "C" frugal_status frugal_backward_update(frugal_ctx* c, int64_t s, const 
     }
     {
         Timer tm(c, PH_OPT, st);
-        launch_optimizer(c, q, s, par, st);
+        launch_optimizer(c, q, s, par, nullptr, nullptr, st);
+    }
+    CK(cudaEventRecord(c->ev_opt[s & 1], st));
+    c->opt_pending[s & 1] = true;
+    CKL();
+    c->phase_in_step = 0;
+    c->timed_steps++;
+    return check_err_word(c);
+}
+
+// ================================================================================ comparison path
+static frugal_status a2a_check(frugal_ctx* c, int64_t s, int phase, const char* what) {
+    if (!c) { set_err("NULL ctx"); return FRUGAL_EINVAL; }
+    if (!c->a2a) { set_err("%s needs a context created with FRUGAL_F_A2A", what); return FRUGAL_ESTATE; }
+    if (c->phase_in_step != phase || s != c->cur_step) { set_err("%s(%lld) out of order", what, (long long)s); return FRUGAL_ESTATE; }
+    return FRUGAL_OK;
+}
+
+extern "C" frugal_status frugal_a2a_requests(frugal_ctx* c, int64_t s, int32_t* d_ids, int64_t* counts,
+                                             frugal_stream stream) {
+    if (frugal_status r = a2a_check(c, s, 1, "a2a_requests")) return r;
+    if (!d_ids || !counts) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    cudaStream_t st = (cudaStream_t)stream;
+    QueueSlot& q = c->q[s % c->QN];
+    Timer tm(c, PH_EXCH, st);
+    launch_a2a_ids(c, q, d_ids, st);
+    int32_t goff[33];
+    CK(cudaMemcpyAsync(goff, q.goff, (size_t)(c->n + 1) * 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    for (int r = 0; r < c->n; r++) counts[r] = goff[r + 1] - goff[r];
+    CKL();
+    return FRUGAL_OK;
+}
+
+extern "C" frugal_status frugal_a2a_serve(frugal_ctx* c, int64_t s, const int32_t* d_ids_in, int64_t n_in, float* d_rows,
+                                          frugal_stream stream) {
+    if (frugal_status r = a2a_check(c, s, 1, "a2a_serve")) return r;
+    if (n_in < 0 || (n_in && (!d_ids_in || !d_rows))) { set_err("bad arguments"); return FRUGAL_EINVAL; }
+    cudaStream_t st = (cudaStream_t)stream;
+    Timer tm(c, PH_GATHER, st);
+    launch_serve_rows(c, d_ids_in, n_in, s, d_rows, st);
+    CKL();
+    return FRUGAL_OK;
+}
+
+extern "C" frugal_status frugal_a2a_lookup(frugal_ctx* c, int64_t s, const float* d_rows_in, float* d_out,
+                                           frugal_stream stream) {
+    if (frugal_status r = a2a_check(c, s, 1, "a2a_lookup")) return r;
+    QueueSlot& q0 = c->q[s % c->QN];
+    if ((!d_rows_in || !d_out) && q0.h_counts[c->g] > 0) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    cudaStream_t st = (cudaStream_t)stream;
+    QueueSlot& q = c->q[s % c->QN];
+    float* rows = c->rows_buf[s & 1];
+    {
+        Timer tm(c, PH_EXPAND, st);
+        launch_a2a_place(c, q, d_rows_in, rows, st);
+        launch_expand(c, q, rows, d_out, st);
+    }
+    if (c->drain_after_gather) {
+        CK(cudaEventRecord(c->ev_gathered, st));
+        frugal_status r = launch_drain(c, s, st, c->ev_gathered);
+        if (r) return r;
+    }
+    CKL();
+    c->phase_in_step = 2;
+    return check_err_word(c);
+}
+
+extern "C" frugal_status frugal_a2a_pack(frugal_ctx* c, int64_t s, const float* d_grad, float* d_partials,
+                                         frugal_stream stream) {
+    if (frugal_status r = a2a_check(c, s, 2, "a2a_pack")) return r;
+    if (!d_grad || !d_partials) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    cudaStream_t st = (cudaStream_t)stream;
+    QueueSlot& q = c->q[s % c->QN];
+    Timer tm(c, PH_SEGRED, st);
+    launch_segreduce(c, q, d_grad, (int)(s & 1), d_partials, st);
+    CKL();
+    return FRUGAL_OK;
+}
+
+extern "C" frugal_status frugal_a2a_update(frugal_ctx* c, int64_t s, const float* d_partials_in,
+                                           const int64_t* recv_counts, frugal_stream stream) {
+    if (frugal_status r = a2a_check(c, s, 2, "a2a_update")) return r;
+    if (!recv_counts) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    int64_t nrecv = 0;
+    for (int r = 0; r < c->n; r++) nrecv += recv_counts[r];
+    if (!d_partials_in && nrecv > 0) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    cudaStream_t st = (cudaStream_t)stream;
+    QueueSlot& q = c->q[s % c->QN];
+    int32_t roff[33];  // pageable source: the copy is staged before cudaMemcpyAsync returns
+    roff[0] = 0;
+    for (int r = 0; r < c->n; r++) roff[r + 1] = roff[r] + (int32_t)recv_counts[r];
+    CK(cudaMemcpyAsync(c->a2a_roff, roff, (size_t)c->n * 4, cudaMemcpyHostToDevice, st));
+    {
+        Timer tm(c, PH_OPT, st);
+        launch_optimizer(c, q, s, (int)(s & 1), d_partials_in, c->a2a_roff, st);
     }
     CK(cudaEventRecord(c->ev_opt[s & 1], st));
     c->opt_pending[s & 1] = true;

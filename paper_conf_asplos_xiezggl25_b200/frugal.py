@@ -17,7 +17,7 @@ LIB_PATH = os.path.join(PKG, "libfrugal.so")
 
 SGD, ADAGRAD = 0, 1
 MODE_P2F, MODE_WRITE_THROUGH = 0, 1
-F_RECORD, F_TIMERS, F_NO_HOST_STATE = 1, 2, 4
+F_RECORD, F_TIMERS, F_NO_HOST_STATE, F_A2A = 1, 2, 4, 8
 FLUSH_ALL = 0
 PHASES = ["ingest", "schedule", "urgent", "gate", "gather", "expand", "model", "segred", "exchange",
           "optimizer", "side", "prefetch"]
@@ -84,6 +84,11 @@ def lib():
             "frugal_read_host": [P, P, I64, P, P],
             "frugal_get_stats": [P, C.POINTER(Stats)],
             "frugal_get_timeline": [P, P, P, P, I64, C.POINTER(I64)],
+            "frugal_a2a_requests": [P, I64, P, P, P],
+            "frugal_a2a_serve": [P, I64, P, I64, P, P],
+            "frugal_a2a_lookup": [P, I64, P, P, P],
+            "frugal_a2a_pack": [P, I64, P, P, P],
+            "frugal_a2a_update": [P, I64, P, P, P],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -103,7 +108,8 @@ EXPORTED = ["frugal_init", "frugal_prefetch", "frugal_step", "frugal_lookup", "f
             "frugal_flush", "frugal_destroy", "frugal_last_error", "frugal_dot_model", "frugal_transe_model",
             "frugal_get_dedup",
             "frugal_get_schedule", "frugal_get_final_flush", "frugal_read_rows", "frugal_read_host",
-            "frugal_get_stats", "frugal_get_timeline", "frugal_owned_rows", "frugal_hot_slots"]
+            "frugal_get_stats", "frugal_get_timeline", "frugal_owned_rows", "frugal_hot_slots",
+            "frugal_a2a_requests", "frugal_a2a_serve", "frugal_a2a_lookup", "frugal_a2a_pack", "frugal_a2a_update"]
 
 
 def _check(status):
@@ -196,6 +202,26 @@ class Frugal:
 
     def flush(self, what=FLUSH_ALL, stream=None):
         _check(lib().frugal_flush(self.h, what, _stream(stream)))
+
+    # ---- comparison path (FRUGAL_F_A2A) -------------------------------------------------
+    def a2a_requests(self, s, ids_out, stream=None):
+        """Fills ids_out (int32 device, >= n_uniq) grouped by owner; returns counts per owner."""
+        counts = np.zeros(self.world, np.int64)
+        _check(lib().frugal_a2a_requests(self.h, s, _ptr(ids_out), counts.ctypes.data, _stream(stream)))
+        return counts
+
+    def a2a_serve(self, s, ids_in, n_in, rows_out, stream=None):
+        _check(lib().frugal_a2a_serve(self.h, s, _ptr(ids_in), n_in, _ptr(rows_out), _stream(stream)))
+
+    def a2a_lookup(self, s, rows_in, out, stream=None):
+        _check(lib().frugal_a2a_lookup(self.h, s, _ptr(rows_in), _ptr(out), _stream(stream)))
+
+    def a2a_pack(self, s, grad, partials_out, stream=None):
+        _check(lib().frugal_a2a_pack(self.h, s, _ptr(grad), _ptr(partials_out), _stream(stream)))
+
+    def a2a_update(self, s, partials_in, recv_counts, stream=None):
+        rc = np.ascontiguousarray(recv_counts, dtype=np.int64)
+        _check(lib().frugal_a2a_update(self.h, s, _ptr(partials_in), rc.ctypes.data, _stream(stream)))
 
     # ---- introspection ---------------------------------------------------------------
     def get_dedup(self, t):

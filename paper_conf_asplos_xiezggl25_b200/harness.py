@@ -67,3 +67,63 @@ class Trainer:
     def losses(self):
         torch.cuda.synchronize(self.dev)
         return self.loss.cpu().numpy()
+
+
+class A2ATrainer(Trainer):
+    """The comparison path (Fig. 2b ❶-❺, L278-336): ids to their
+    owners, rows back, partials to the owners, each by an all-to-all of the process group
+    `group` (NCCL over NVLink on GPUs; gloo with host staging when `host_staging`, e.g.
+    several ranks sharing one GPU in tests).  The context needs FRUGAL_F_A2A."""
+
+    def __init__(self, fr, st, rank=0, device=0, dist=None, host_staging=False):
+        super().__init__(fr, st, rank, device)
+        self.dist = dist
+        self.host = host_staging
+        M, d = self.emb.shape
+        self.ids_send = torch.empty(M, dtype=torch.int32, device=self.dev)
+        self.part_send = torch.empty(M, d, device=self.dev)
+        self.world = fr.world
+
+    def _a2a(self, send, send_counts, recv_counts, inner):
+        """all_to_all_single with per-rank row counts; inner = elements per row."""
+        rc = [int(c) * inner for c in recv_counts]
+        sc = [int(c) * inner for c in send_counts]
+        src = send.reshape(-1)[:sum(sc)]
+        if self.host:
+            src = src.cpu()
+        out = torch.empty(sum(rc), dtype=send.dtype, device=src.device)
+        self.dist.all_to_all_single(out, src, rc, sc)
+        return out.to(self.dev)
+
+    def step(self, on_schedule=None):
+        st, fr, s, D = self.st, self.fr, self.s, self.dist
+        t = s + fr.lookahead
+        if t < st.steps:
+            fr.step(s, st.ids[t], st.counts[t])
+        else:
+            fr.step(s)
+        if on_schedule:
+            on_schedule(s)
+        d = self.emb.shape[1]
+        send_counts = fr.a2a_requests(s, self.ids_send)                       # ❶ bucket by owner
+        sc = torch.tensor(send_counts, dtype=torch.int64)
+        rc = torch.empty_like(sc)
+        D.all_to_all_single(rc, sc)                                            # counts
+        recv_counts = rc.numpy()
+        ids_in = self._a2a(self.ids_send, send_counts, recv_counts, 1)        # ❷ ids to owners
+        rows_out = torch.empty(int(recv_counts.sum()), d, device=self.dev)
+        fr.a2a_serve(s, ids_in, int(recv_counts.sum()), rows_out)             # ❸ owner queries
+        torch.cuda.synchronize(self.dev)
+        rows_in = self._a2a(rows_out, recv_counts, send_counts, d)            # ❹ rows back
+        fr.a2a_lookup(s, rows_in, self.emb)                                    # ❺ reorder + expand
+        if st.cfg.model == "transe":
+            fr.transe_model(s, self.emb, st.cfg.neg_chunk, st.cfg.gamma, self.grad, self.loss[s:s + 1])
+        else:
+            x = torch.from_numpy(st.x[s, self.rank]).to(self.dev)
+            y = torch.from_numpy(st.y[s, self.rank]).to(self.dev)
+            fr.dot_model(s, self.emb, x, y, self.grad, self.loss[s:s + 1])
+        fr.a2a_pack(s, self.grad, self.part_send)
+        torch.cuda.synchronize(self.dev)
+        part_in = self._a2a(self.part_send, send_counts, recv_counts, d)      # partials to owners
+        fr.a2a_update(s, part_in, recv_counts)
+        self.s += 1

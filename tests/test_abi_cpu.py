@@ -19,7 +19,7 @@ def _lib():
 def declared_symbols():
     src = open(os.path.join(ROOT, "include", "frugal.h")).read()
     src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
-    return sorted(set(re.findall(r"\b(frugal_[a-z_]+)\s*\(", src)))
+    return sorted(set(re.findall(r"\b(frugal_[a-z0-9_]+)\s*\(", src)))
 
 
 def test_every_declared_symbol_is_exported():

@@ -14,15 +14,21 @@ from paper_conf_asplos_xiezggl25_b200 import workload as W
 pytestmark = pytest.mark.gpu
 
 
-def _rank_main(rank, st, shm, barrier, q):
+def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0):
     try:
         import torch
         from paper_conf_asplos_xiezggl25_b200 import frugal as F
-        from paper_conf_asplos_xiezggl25_b200.harness import Trainer, make_context
+        from paper_conf_asplos_xiezggl25_b200.harness import A2ATrainer, Trainer, make_context
         torch.cuda.set_device(0)
-        fr = make_context(st, rank=rank, device=0, shm_name=shm, flags=F.F_RECORD)
+        fr = make_context(st, rank=rank, device=0, shm_name=shm, flags=F.F_RECORD | (F.F_A2A if a2a else 0))
         barrier.wait()
-        tr = Trainer(fr, st, rank=rank)
+        if a2a:
+            import torch.distributed as dist
+            os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+            dist.init_process_group("gloo", rank=rank, world_size=2)
+            tr = A2ATrainer(fr, st, rank=rank, dist=dist, host_staging=True)
+        else:
+            tr = Trainer(fr, st, rank=rank)
         sched = []
         for s in range(st.steps):
             got = {}
@@ -42,12 +48,17 @@ def _rank_main(rank, st, shm, barrier, q):
         q.put((rank, traceback.format_exc()))
 
 
-def run_two_ranks(st, timeout=600):
+def run_two_ranks(st, timeout=600, a2a=False):
+    import socket
     ctx = mp.get_context("spawn")
     barrier = ctx.Barrier(2)
     q = ctx.Queue()
     shm = f"/frugal_test_{os.getpid()}"
-    ps = [ctx.Process(target=_rank_main, args=(r, st, shm, barrier, q)) for r in range(2)]
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    ps = [ctx.Process(target=_rank_main, args=(r, st, shm, barrier, q, a2a, port)) for r in range(2)]
     for p in ps:
         p.start()
     out = {}
@@ -65,8 +76,11 @@ def run_two_ranks(st, timeout=600):
     return out
 
 
-@pytest.mark.parametrize("opt", ["adagrad", "sgd"])
-def test_two_ranks_one_gpu_parity(opt):
+@pytest.mark.parametrize("opt,a2a", [("adagrad", False), ("sgd", False), ("adagrad", True)])
+def test_two_ranks_one_gpu_parity(opt, a2a):
+    """a2a=True: the comparison path (§8(e)) -- ids, rows and partials move by all-to-all
+    (gloo with host staging here; NCCL over NVLink on a multi-GPU box) instead of the host
+    table and mailbox; every artefact and table must be identical."""
     from oracle.oracle import Oracle
     cfg = W.config("tiny", world=2, batch=64, lookahead=4, age_out=3, opt=opt,
                    lr=0.05 if opt == "adagrad" else 1.0)
@@ -74,7 +88,7 @@ def test_two_ranks_one_gpu_parity(opt):
     counts = rng.integers(0, 65, size=(24, 2)).astype(np.int32)
     counts[5, 1] = 0
     st = W.gen_stream(cfg, 24, counts=counts)
-    out = run_two_ranks(st)
+    out = run_two_ranks(st, a2a=a2a)
     o = Oracle(st)
     for s in range(st.steps):
         o.step()
