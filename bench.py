@@ -270,7 +270,7 @@ def main():
     ids_send = torch.empty(B * Fs, dtype=torch.int32, device=dev)
     part_send = torch.empty(B * Fs, d, device=dev)
 
-    def a2a(send, send_counts, recv_counts, inner):
+    def a2a_xchg(send, send_counts, recv_counts, inner):
         rc = [int(c) * inner for c in recv_counts]
         sc = [int(c) * inner for c in send_counts]
         src = send.reshape(-1)[:sum(sc)]
@@ -289,10 +289,10 @@ def main():
         rct = torch.empty_like(sct)
         dist.all_to_all_single(rct, sct)
         rc = rct.cpu().numpy()
-        ids_in = a2a(ids_send, sc, rc, 1)
+        ids_in = a2a_xchg(ids_send, sc, rc, 1)
         rows_out = torch.empty(int(rc.sum()), d, device=dev)
         fr.a2a_serve(s, ids_in, int(rc.sum()), rows_out)
-        rows_in = a2a(rows_out, rc, sc, d)
+        rows_in = a2a_xchg(rows_out, rc, sc, d)
         fr.a2a_lookup(s, rows_in, emb)
         lookup.counts = (sc, rc)
 
@@ -302,7 +302,7 @@ def main():
             return
         sc, rc = lookup.counts
         fr.a2a_pack(s, grad, part_send)
-        part_in = a2a(part_send, sc, rc, d)
+        part_in = a2a_xchg(part_send, sc, rc, d)
         fr.a2a_update(s, part_in, rc)
 
     def step_dev(s):

@@ -177,6 +177,8 @@ struct frugal_ctx {
     int64_t early_issued = -1;                          // last step whose early gather was launched
     bool early = false;                                 // pipelined gather enabled (world 1)
     bool pool_hits = true;                              // owner reads its dirty-pool rows from HBM
+    int early_blocks = 16;                              // grid of the early gather
+    bool early_on_side = false;                         // early gather queued behind the drain
     bool a2a = false;                                   // comparison path (FRUGAL_F_A2A)
     bool xhost = false;                                 // world > 1 and host-bounced exchange
     int32_t* a2a_roff = nullptr;                        // [world] receive offsets (device)

@@ -236,6 +236,8 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     // box (the zero-copy loads of the next step only delay this step's); FRUGAL_EARLY=1
     c->early = c->n == 1 && getenv("FRUGAL_EARLY") && atoi(getenv("FRUGAL_EARLY"));
     c->pool_hits = !(getenv("FRUGAL_NO_POOL_HITS") && atoi(getenv("FRUGAL_NO_POOL_HITS")));
+    c->early_blocks = getenv("FRUGAL_EARLY_BLOCKS") ? atoi(getenv("FRUGAL_EARLY_BLOCKS")) : 16;
+    c->early_on_side = getenv("FRUGAL_EARLY_ON_SIDE") && atoi(getenv("FRUGAL_EARLY_ON_SIDE"));
     c->a2a = (k.flags & FRUGAL_F_A2A) != 0;
     c->xhost = c->n > 1 && !c->a2a;
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 32;
@@ -585,13 +587,16 @@ static frugal_status launch_early_gather(frugal_ctx* c, int64_t u, cudaEvent_t s
     // with the drain placed after the gather, the early gather follows the drain on the
     // side stream: one FIFO of host-link work (late gather, drain, early gather of the
     // next step) that fills the link while the main stream runs the backward
-    cudaStream_t ps = c->drain_after_gather ? c->side : c->pstream;
+    cudaStream_t ps = c->early_on_side ? c->side : c->pstream;
     CK(cudaStreamWaitEvent(ps, c->ev_ingest[u % c->QN], 0));
     if (side_first) CK(cudaStreamWaitEvent(ps, side_first, 0));
     if (c->opt_pending[u & 1]) CK(cudaStreamWaitEvent(ps, c->ev_opt[u & 1], 0));
     {
         Timer tm(c, PH_PREFETCH, ps);
+        const int keep = c->gather_blocks;
+        c->gather_blocks = c->early_blocks;  // few SMs: its loads must not crowd the backward
         launch_gather(c, q, q.eidx, q.elcnt, c->rows_buf[u & 1], u, ps);
+        c->gather_blocks = keep;
     }
     CK(cudaEventRecord(c->ev_early[u & 1], ps));
     c->early_issued = u;

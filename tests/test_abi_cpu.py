@@ -80,3 +80,14 @@ def test_product_path_does_not_import_oracle():
         for f in files:
             if f.endswith((".py", ".cu", ".cuh", ".h")):
                 assert not pat.search(open(os.path.join(dirpath, f)).read()), f
+
+
+def test_bench_module_imports_and_parses():
+    """bench.py must at least import and parse its arguments without a GPU."""
+    import importlib
+    import sys
+    sys.argv = ["bench.py"]
+    b = importlib.import_module("bench")
+    a = b.parse()
+    assert a.gpus == 1 and a.warmup >= 3 and a.exchange == "host"
+    assert b.dist_max(3.0, 1) == 3.0
