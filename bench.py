@@ -54,6 +54,9 @@ def parse():
     ap.add_argument("--exchange", default="host", choices=["host", "a2a"],
                     help="a2a = the comparison path: rows/partials by all-to-all over the process group "
                          "(NCCL/NVLink) instead of the host table and mailbox (N > 1)")
+    ap.add_argument("--peer", action="store_true",
+                    help="N4 NVLink-native variant: non-owned rows held in the owner's HBM are loaded "
+                         "over peer memory instead of from the host table (N > 1)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for barriers / the max-over-ranks timing only")
     return ap.parse_args()
@@ -247,7 +250,8 @@ def main():
     if a2a and world == 1:
         sys.exit("--exchange a2a needs N > 1")
     fr = make_context(st, rank=rank, device=local, shm_name=shm,
-                      flags=F.F_TIMERS | (F.F_NO_HOST_STATE if no_host_state else 0) | (F.F_A2A if a2a else 0),
+                      flags=F.F_TIMERS | (F.F_NO_HOST_STATE if no_host_state else 0) | (F.F_A2A if a2a else 0)
+                      | (F.F_PEER if (args.peer and world > 1) else 0),
                       mode=F.MODE_WRITE_THROUGH if args.mode == "write_through" else F.MODE_P2F)
     barrier()
     stream = torch.cuda.current_stream(dev)
@@ -461,6 +465,7 @@ def main():
                    "lookahead": L, "age_out": cfg.age_out, "cache_ratio": cfg.cache_ratio, "opt": cfg.opt,
                    "flush_mode": args.mode, "exchange": "host table + mailbox (P2F)" if not a2a else
                    "all-to-all over the process group (comparison path)",
+                   "peer_reads": bool(args.peer and world > 1),
                    "parallelism": f"dp{world} (owner-sharded rows, shared pinned host table)",
                    "l2": "inputs larger than L2: host table %.1f GB, HBM cache %.0f MB, %d distinct id batches "
                          "(%.0f MB) cycled" % (cfg.n_rows * r * (1 if (no_host_state or not adag) else 2) / 1e9,

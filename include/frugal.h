@@ -61,6 +61,10 @@ enum {
     FRUGAL_F_NO_HOST_STATE = 4, /* Adagrad: no host copy of G (it lives in HBM, R8); the final
                                    flush then writes w only -- for tables whose w and G do not
                                    both fit in host memory (e.g. configs[3], 2 x 138 GB)      */
+    FRUGAL_F_PEER = 16,         /* NVLink-native variant: a non-owned row
+                                   the owner holds in HBM (cache, or dirty pool) is loaded from
+                                   the owner's GPU over peer memory (CUDA IPC) instead of the
+                                   host table; flush schedule and results unchanged; world > 1 */
     FRUGAL_F_A2A = 8            /* comparison path (the message pipeline of
                                    PAPER.md Fig. 2b): rows and gradients move between
                                    ranks by the caller's all-to-all (NCCL over NVLink) through
@@ -241,7 +245,8 @@ enum {
     FRUGAL_C_MAIL_OUT = 13,     /* partial rows written to this rank's host mailbox          */
     FRUGAL_C_MAIL_IN = 14,      /* partial rows read from other ranks' mailboxes             */
     FRUGAL_C_GATHER_POOL = 15,  /* unique owned cold rows gathered from the dirty pool (HBM)  */
-    FRUGAL_N_COUNTERS = 16
+    FRUGAL_C_GATHER_PEER = 16,  /* unique non-owned rows loaded from the owner's HBM (PEER)  */
+    FRUGAL_N_COUNTERS = 20
 };
 typedef struct {
     double ms[FRUGAL_N_PHASES];

@@ -81,6 +81,16 @@ struct PhaseEv {
 
 struct HostShared;  // shm segment layout (runtime.cu)
 
+// NVLink-native variant (FRUGAL_F_PEER): every rank's HBM cache / pool / metadata, opened
+// through CUDA IPC (device pointers valid in this process)
+struct PeerTab {
+    const float4* cw[32];
+    const float4* pw[32];
+    const int32_t* lu[32];
+    const int32_t* pi[32];
+    int64_t capT[32];
+};
+
 }  // namespace frugal
 
 struct frugal_ctx {
@@ -180,6 +190,10 @@ struct frugal_ctx {
     int early_blocks = 16;                              // grid of the early gather
     bool early_on_side = false;                         // early gather queued behind the drain
     bool a2a = false;                                   // comparison path (FRUGAL_F_A2A)
+    bool peer = false;                                  // NVLink-native variant (FRUGAL_F_PEER)
+    frugal::PeerTab* peer_tab = nullptr;                // device copy
+    void* peer_open[32][4] = {};                        // opened IPC mappings (to close)
+    int32_t* gslot = nullptr;                           // [N] owner's cache slot of every hot row
     bool xhost = false;                                 // world > 1 and host-bounced exchange
     int32_t* a2a_roff = nullptr;                        // [world] receive offsets (device)
     bool side_pending[2] = {false, false};

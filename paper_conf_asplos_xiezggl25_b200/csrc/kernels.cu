@@ -683,12 +683,13 @@ __global__ void k_gather_uniq(const int32_t* __restrict__ uniq, const int32_t* _
                               const float4* __restrict__ cw, const float4* hw, float4* __restrict__ rows,
                               const int32_t* __restrict__ last_upd, const int32_t* __restrict__ pool_idx,
                               const float4* __restrict__ pw, int P, int64_t capT, int32_t pool_min,
+                              const int32_t* __restrict__ gslot, const PeerTab* __restrict__ pt,
                               unsigned long long* stats) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
     const int n = *cnt;
-    unsigned nh = 0, nc = 0, np = 0;
+    unsigned nh = 0, nc = 0, np = 0, npeer = 0;
     for (int64_t a = gid; a < n; a += gs) {
         const int u = list ? list[a] : (int)a;
         int32_t k = uniq[u];
@@ -707,17 +708,37 @@ __global__ void k_gather_uniq(const int32_t* __restrict__ uniq, const int32_t* _
                     kind = 2;
                 }
             }
+        } else if (pt) {
+            // N4: the owner's HBM holds this row (cache, or pool within the window) -> peer
+            // load over NVLink; its values are the post-(s-1) ones for as long as this gather
+            // runs (the gate waited for the owner's urgent flush, which follows its optimizer
+            // of s-1; its optimizer of s waits for this rank's mailbox flag of s)
+            const int o = k % world;
+            const int32_t lk = k / world;
+            const int sl = gslot[k];
+            if (sl >= 0) {
+                src = pt->cw[o] + (int64_t)sl * d4;
+                kind = 3;
+            } else {
+                const int32_t lu = pt->lu[o][lk];
+                if (lu >= 0 && lu >= pool_min) {
+                    src = pt->pw[o] + ((int64_t)(lu % P) * pt->capT[o] + pt->pi[o][lk]) * d4;
+                    kind = 3;
+                }
+            }
         }
         if (l == 0) {
             nh += kind == 0;
             nc += kind == 1;
             np += kind == 2;
+            npeer += kind == 3;
         }
         for (int v = l; v < d4; v += GS) rows[(int64_t)u * d4 + v] = src[v];
     }
     block_count(stats + FRUGAL_C_GATHER_HOST, nh);
     block_count(stats + FRUGAL_C_GATHER_CACHE, nc);
     block_count(stats + FRUGAL_C_GATHER_POOL, np);
+    block_count(stats + FRUGAL_C_GATHER_PEER, npeer);
 }
 // a4 expand: out[i] = rows[inv[i]]
 template <int GS>
@@ -745,7 +766,7 @@ void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32
                                                              (const float4*)c->cw, (const float4*)c->dh_w,
                                                              (float4*)rows, c->last_upd, c->pool_idx,
                                                              c->pool_hits ? (const float4*)c->pw : nullptr, c->P,
-                                                             c->capT, pool_min, c->dstats)));
+                                                             c->capT, pool_min, c->gslot, c->peer_tab, c->dstats)));
     c->launches++;
 }
 void launch_expand(frugal_ctx* c, QueueSlot& q, const float* rows, float* out, cudaStream_t st) {

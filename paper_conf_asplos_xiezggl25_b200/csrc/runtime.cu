@@ -60,6 +60,14 @@ namespace {
 constexpr uint64_t kMagic = 0x46525547414c3235ULL;  // "FRUGAL25"
 constexpr size_t kHdr = 4096;
 constexpr size_t kFlags = 8192;  // 4 kinds x 32 ranks x 64 B
+constexpr size_t kIpc = 32 * 512;  // per rank: IPC handles of cache / pool / last_upd / pool_idx (PEER)
+
+struct IpcRecord {
+    volatile uint64_t ready;
+    int64_t capT;
+    cudaIpcMemHandle_t h[4];
+};
+static_assert(sizeof(IpcRecord) <= 512, "IPC record");
 enum { FLAG_URGENT = 0, FLAG_SIDE = 1, FLAG_MAIL = 2, FLAG_SIDE_FIRST = 3 };
 enum { PH_INGEST, PH_SCHED, PH_URGENT, PH_GATE, PH_GATHER, PH_EXPAND, PH_MODEL, PH_SEGRED, PH_EXCH, PH_OPT, PH_SIDE,
        PH_PREFETCH };
@@ -158,7 +166,10 @@ static void free_ctx(frugal_ctx* c) {
     F(c->rows_buf[0]); F(c->rows_buf[1]); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->long_tasks); F(c->owned_cnt);
     for (int i = 0; i < 2; i++) { F(c->adj_rows[i]); F(c->adj_p[i]); F(c->adj_cnt[i]); }
     for (int i = 0; i < 2; i++) { F(c->sl_rows[i]); F(c->sl_p[i]); F(c->sl_cnt[i]); }
-    F(c->dstats); F(c->kg_W); F(c->kg_A); F(c->a2a_roff); F(c->ff_rows); F(c->ff_cnt); F(c->ids_stage);
+    F(c->dstats); F(c->kg_W); F(c->kg_A); F(c->a2a_roff); F(c->peer_tab); F(c->gslot);
+    for (int r = 0; r < 32; r++)
+        for (int i = 0; i < 4; i++)
+            if (c->peer_open[r][i]) cudaIpcCloseMemHandle(c->peer_open[r][i]); F(c->ff_rows); F(c->ff_cnt); F(c->ids_stage);
     if (c->herr) cudaFreeHost(c->herr);
     if (c->counts_pin) cudaFreeHost(c->counts_pin);
     for (auto e : c->ev_counts) cudaEventDestroy(e);
@@ -199,6 +210,59 @@ static void free_ctx(frugal_ctx* c) {
         }                                                                                        \
     } while (0)
 
+// ================================================================================ peers (N4)
+// Publish this rank's cache / pool / metadata as CUDA IPC handles in the shared segment,
+// wait for every rank, open the others' (lazy peer access), and build the dense map
+// gslot[k] = slot of hot row k in its owner's cache (owners number their hot rows in
+// ascending local id, as frugal_init does).
+static frugal_status setup_peers(frugal_ctx* c, char* ipc_base, std::vector<int64_t>& hot_global) {
+    IpcRecord* mine = (IpcRecord*)(ipc_base + (size_t)c->g * 512);
+    CK(cudaIpcGetMemHandle(&mine->h[0], c->cw));
+    CK(cudaIpcGetMemHandle(&mine->h[1], c->pw));
+    CK(cudaIpcGetMemHandle(&mine->h[2], c->last_upd));
+    CK(cudaIpcGetMemHandle(&mine->h[3], c->pool_idx));
+    mine->capT = c->capT;
+    __sync_synchronize();
+    mine->ready = kMagic;
+    PeerTab tab;
+    memset(&tab, 0, sizeof tab);
+    const double t0 = now_s();
+    for (int r = 0; r < c->n; r++) {
+        IpcRecord* rec = (IpcRecord*)(ipc_base + (size_t)r * 512);
+        while (rec->ready != kMagic) {
+            if (now_s() - t0 > 600) { set_err("timed out waiting for rank %d's IPC handles", r); return FRUGAL_ETIMEOUT; }
+            usleep(5000);
+        }
+        __sync_synchronize();
+        tab.capT[r] = rec->capT;
+        if (r == c->g) {
+            tab.cw[r] = (const float4*)c->cw;
+            tab.pw[r] = (const float4*)c->pw;
+            tab.lu[r] = c->last_upd;
+            tab.pi[r] = c->pool_idx;
+            continue;
+        }
+        for (int i = 0; i < 4; i++) {
+            void* p = nullptr;
+            CK(cudaIpcOpenMemHandle(&p, rec->h[i], cudaIpcMemLazyEnablePeerAccess));
+            c->peer_open[r][i] = p;
+        }
+        tab.cw[r] = (const float4*)c->peer_open[r][0];
+        tab.pw[r] = (const float4*)c->peer_open[r][1];
+        tab.lu[r] = (const int32_t*)c->peer_open[r][2];
+        tab.pi[r] = (const int32_t*)c->peer_open[r][3];
+    }
+    CK(cudaMalloc(&c->peer_tab, sizeof(PeerTab)));
+    CK(cudaMemcpy(c->peer_tab, &tab, sizeof tab, cudaMemcpyHostToDevice));
+    std::sort(hot_global.begin(), hot_global.end());
+    hot_global.erase(std::unique(hot_global.begin(), hot_global.end()), hot_global.end());
+    std::vector<int32_t> gslot((size_t)c->N, -1), next(c->n, 0);
+    for (int64_t k : hot_global) gslot[k] = next[k % c->n]++;  // ascending k == ascending local id per owner
+    CK(cudaMalloc(&c->gslot, (size_t)c->N * 4));
+    CK(cudaMemcpy(c->gslot, gslot.data(), (size_t)c->N * 4, cudaMemcpyHostToDevice));
+    return FRUGAL_OK;
+}
+
 // ================================================================================ init
 extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out) {
     if (!out) { set_err("out is NULL"); return FRUGAL_EINVAL; }
@@ -215,6 +279,10 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     if (k.mode != FRUGAL_MODE_P2F && k.mode != FRUGAL_MODE_WRITE_THROUGH) { set_err("bad mode"); return FRUGAL_EINVAL; }
     if (!k.shm_name && k.world != 1) { set_err("world > 1 needs shm_name"); return FRUGAL_EINVAL; }
     if ((k.flags & FRUGAL_F_A2A) && k.world < 2) { set_err("FRUGAL_F_A2A needs world > 1"); return FRUGAL_EINVAL; }
+    if ((k.flags & FRUGAL_F_PEER) && (k.world < 2 || (k.flags & FRUGAL_F_A2A))) {
+        set_err("FRUGAL_F_PEER needs world > 1 and the host-bounced exchange");
+        return FRUGAL_EINVAL;
+    }
     if (k.n_hot < 0 || (k.n_hot > 0 && !k.hot_ids)) { set_err("bad hot set"); return FRUGAL_EINVAL; }
     for (int64_t i = 0; i < k.n_hot; i++)
         if (k.hot_ids[i] < 0 || k.hot_ids[i] >= k.n_rows) { set_err("hot id out of range"); return FRUGAL_EINVAL; }
@@ -239,6 +307,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->early_blocks = getenv("FRUGAL_EARLY_BLOCKS") ? atoi(getenv("FRUGAL_EARLY_BLOCKS")) : 16;
     c->early_on_side = getenv("FRUGAL_EARLY_ON_SIDE") && atoi(getenv("FRUGAL_EARLY_ON_SIDE"));
     c->a2a = (k.flags & FRUGAL_F_A2A) != 0;
+    c->peer = (k.flags & FRUGAL_F_PEER) != 0;
     c->xhost = c->n > 1 && !c->a2a;
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 32;
     c->gather_blocks = getenv("FRUGAL_GATHER_BLOCKS") ? atoi(getenv("FRUGAL_GATHER_BLOCKS")) : 74;
@@ -255,7 +324,8 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     // ---------------------------------------------------------------- host table (shm)
     c->mail_stride = c->n > 1 ? align_up(256 + (size_t)c->M * rowb, 4096) : 0;
     const size_t mail_bytes = c->n > 1 ? 2 * (size_t)c->n * c->mail_stride : 0;
-    const size_t off_mail = kHdr + kFlags;
+    const size_t off_ipc = kHdr + kFlags;
+    const size_t off_mail = off_ipc + kIpc;
     const size_t off_w = align_up(off_mail + mail_bytes, 2 << 20);
     const size_t tab = (size_t)c->N * rowb;
     const size_t off_G = align_up(off_w + tab, 2 << 20);
@@ -335,6 +405,8 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     DMALLOC(c->last_upd, c->No * 4);
     DMALLOC(c->pool_idx, c->No * 4);
     DMALLOC(c->rbits, c->No * 8);
+    // the whole hot set (PEER: every owner's slot of every hot row) and this rank's share
+    std::vector<int64_t> hot_global(k.hot_ids, k.hot_ids + k.n_hot);
     // owned share of the hot set, sorted, deduplicated
     std::vector<int32_t> hot;
     for (int64_t i = 0; i < k.n_hot; i++)
@@ -447,7 +519,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     cudaMemset(c->pcount, 0, (size_t)c->P * 4);
     cudaMemset(c->pkey, 0xff, (size_t)c->P * c->capT * 4);
     if (c->g == 0 || !k.shm_name) {
-        memset(hbase + kHdr, 0, kFlags);
+        memset(hbase + kHdr, 0, kFlags + kIpc);
         launch_init_table(c, st);
         if (cudaDeviceSynchronize() != cudaSuccess) {
                 set_err("table init failed: %s", cudaGetErrorString(cudaGetLastError()));
@@ -482,6 +554,13 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         set_err("init failed: %s", cudaGetErrorString(cudaGetLastError()));
         free_ctx(c);
         return FRUGAL_ECUDA;
+    }
+    if (c->peer) {
+        frugal_status r = setup_peers(c, hbase + off_ipc, hot_global);
+        if (r) {
+            free_ctx(c);
+            return r;
+        }
     }
     *out = c;
     (void)dev_major;

@@ -17,7 +17,7 @@ LIB_PATH = os.path.join(PKG, "libfrugal.so")
 
 SGD, ADAGRAD = 0, 1
 MODE_P2F, MODE_WRITE_THROUGH = 0, 1
-F_RECORD, F_TIMERS, F_NO_HOST_STATE, F_A2A = 1, 2, 4, 8
+F_RECORD, F_TIMERS, F_NO_HOST_STATE, F_A2A, F_PEER = 1, 2, 4, 8, 16
 FLUSH_ALL = 0
 PHASES = ["ingest", "schedule", "urgent", "gate", "gather", "expand", "model", "segred", "exchange",
           "optimizer", "side", "prefetch"]
@@ -47,12 +47,12 @@ class ScheduleInfo(C.Structure):
 
 COUNTERS = ["positions", "unique", "gather_host", "gather_cache", "opt_hot", "opt_cold", "urgent_hot",
             "urgent_cold", "side_hot", "side_cold", "final_hot", "final_cold", "long_segments", "mail_out",
-            "mail_in", "gather_pool"]
+            "mail_in", "gather_pool", "gather_peer", "reserved17", "reserved18", "reserved19"]
 
 
 class Stats(C.Structure):
     _fields_ = [("ms", C.c_double * 12), ("steps", C.c_int64), ("kernel_launches", C.c_int64),
-                ("count", C.c_int64 * 16)]
+                ("count", C.c_int64 * 20)]
 
 
 _lib = None

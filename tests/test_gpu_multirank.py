@@ -14,13 +14,14 @@ from paper_conf_asplos_xiezggl25_b200 import workload as W
 pytestmark = pytest.mark.gpu
 
 
-def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0):
+def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False):
     try:
         import torch
         from paper_conf_asplos_xiezggl25_b200 import frugal as F
         from paper_conf_asplos_xiezggl25_b200.harness import A2ATrainer, Trainer, make_context
         torch.cuda.set_device(0)
-        fr = make_context(st, rank=rank, device=0, shm_name=shm, flags=F.F_RECORD | (F.F_A2A if a2a else 0))
+        fr = make_context(st, rank=rank, device=0, shm_name=shm,
+                          flags=F.F_RECORD | (F.F_A2A if a2a else 0) | (F.F_PEER if peer else 0))
         barrier.wait()
         if a2a:
             import torch.distributed as dist
@@ -37,18 +38,19 @@ def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0):
         fr.flush()
         ff = fr.get_final_flush()
         losses = tr.losses()
+        stats = fr.get_stats()["count"]
         barrier.wait()  # both ranks flushed: the host table is authoritative
         w = G = None
         if rank == 0:
             w, G = fr.read_host(np.arange(st.cfg.n_rows))
         barrier.wait()
         fr.close()
-        q.put((rank, dict(sched=sched, ff=ff, losses=losses, w=w, G=G)))
+        q.put((rank, dict(sched=sched, ff=ff, losses=losses, w=w, G=G, stats=stats)))
     except Exception:
         q.put((rank, traceback.format_exc()))
 
 
-def run_two_ranks(st, timeout=600, a2a=False):
+def run_two_ranks(st, timeout=600, a2a=False, peer=False):
     import socket
     ctx = mp.get_context("spawn")
     barrier = ctx.Barrier(2)
@@ -58,7 +60,7 @@ def run_two_ranks(st, timeout=600, a2a=False):
     sk.bind(("127.0.0.1", 0))
     port = sk.getsockname()[1]
     sk.close()
-    ps = [ctx.Process(target=_rank_main, args=(r, st, shm, barrier, q, a2a, port)) for r in range(2)]
+    ps = [ctx.Process(target=_rank_main, args=(r, st, shm, barrier, q, a2a, port, peer)) for r in range(2)]
     for p in ps:
         p.start()
     out = {}
@@ -76,11 +78,14 @@ def run_two_ranks(st, timeout=600, a2a=False):
     return out
 
 
-@pytest.mark.parametrize("opt,a2a", [("adagrad", False), ("sgd", False), ("adagrad", True)])
-def test_two_ranks_one_gpu_parity(opt, a2a):
+@pytest.mark.parametrize("opt,a2a,peer", [("adagrad", False, False), ("sgd", False, False), ("adagrad", True, False),
+                                          ("adagrad", False, True)])
+def test_two_ranks_one_gpu_parity(opt, a2a, peer):
     """a2a=True: the comparison path (§8(e)) -- ids, rows and partials move by all-to-all
     (gloo with host staging here; NCCL over NVLink on a multi-GPU box) instead of the host
-    table and mailbox; every artefact and table must be identical."""
+    table and mailbox; every artefact and table must be identical.  peer=True: the N4
+    variant -- non-owned rows the owner holds in HBM are loaded from the owner's device
+    memory (CUDA IPC; NVLink on a multi-GPU box); every artefact and table identical."""
     from oracle.oracle import Oracle
     cfg = W.config("tiny", world=2, batch=64, lookahead=4, age_out=3, opt=opt,
                    lr=0.05 if opt == "adagrad" else 1.0)
@@ -88,7 +93,9 @@ def test_two_ranks_one_gpu_parity(opt, a2a):
     counts = rng.integers(0, 65, size=(24, 2)).astype(np.int32)
     counts[5, 1] = 0
     st = W.gen_stream(cfg, 24, counts=counts)
-    out = run_two_ranks(st, a2a=a2a)
+    out = run_two_ranks(st, a2a=a2a, peer=peer)
+    if peer:  # the variant actually served rows from the other rank's HBM
+        assert out[0]["stats"]["gather_peer"] > 0 and out[1]["stats"]["gather_peer"] > 0
     o = Oracle(st)
     for s in range(st.steps):
         o.step()
