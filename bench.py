@@ -401,6 +401,10 @@ def main():
     adag = cfg.opt == "adagrad"
     peaks = measured_peaks()
     link = host_link_peaks(torch, dev)
+    # random-row ceiling of this box: fresh pseudo-random rows of the host table, gather pattern
+    nprobe = max(1, int(cnt["gather_host"] / K))
+    probe = [fr.probe_host_reads(nprobe, seed=1000 + i) for i in range(3)]
+    link["random_rows_h2d"] = nprobe * r / (min(probe) * 1e-3) / 1e9
     hbm_peak = peaks.get("hbm_gbs", 6650.0)
 
     def gbs(nbytes, ms_):
@@ -447,6 +451,9 @@ def main():
         pass
     roofline = {"bound": "hbm" if D["bound"] == "hbm" else "host-link", "kernel": dom,
                 "achieved": D["achieved_gbs"], "peak": D["peak"], "unit": "GB/s", "frac": D["frac"],
+                "random_row_ceiling": link["random_rows_h2d"] if D["bound"] != "hbm" else None,
+                "frac_of_random_row_ceiling": (D["achieved_gbs"] / link["random_rows_h2d"])
+                if D["bound"] != "hbm" and D["achieved_gbs"] else None,
                 "traffic": traffic, "traffic_note": tnote,
                 "peak_source": ("measured pinned cudaMemcpy (256 MiB, best of 5) in this run; random 128-B rows "
                                 "measure 12-33 GB/s on this box (profiles/r1_zc_probe_*.txt)" if D["bound"] != "hbm"

@@ -262,6 +262,11 @@ frugal_status frugal_get_stats(frugal_ctx* ctx, frugal_stats* out);
 frugal_status frugal_get_timeline(frugal_ctx* ctx, int32_t* phase, double* t0, double* t1, int64_t cap,
                                   int64_t* n);
 
+/* host-link calibration (bench only): time (*ms) to read n pseudo-random rows of the host
+   table with the gather's access pattern and grid (read-only; between steps) -- the
+   random-row ceiling of this machine's host link, next to the sequential pinned-copy peak */
+frugal_status frugal_probe_host_reads(frugal_ctx* ctx, int64_t n, uint64_t seed, double* ms);
+
 /* number of owned rows / hot slots of this rank */
 int64_t frugal_owned_rows(frugal_ctx* ctx);
 int64_t frugal_hot_slots(frugal_ctx* ctx);

@@ -235,6 +235,7 @@ void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begi
 void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32_t* cnt, float* rows, int64_t step,
                    cudaStream_t st);
 void launch_expand(frugal_ctx* c, QueueSlot& q, const float* rows, float* out, cudaStream_t st);
+void launch_probe_rows(frugal_ctx* c, int64_t n, uint64_t seed, float* out, int64_t out_rows, cudaStream_t st);
 void launch_split_early(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st);
 void launch_mail_header(frugal_ctx* c, QueueSlot& q, int par, cudaStream_t st);
 void launch_transe_model(frugal_ctx* c, QueueSlot& q, const float* emb, int C, double gamma, float* grad,

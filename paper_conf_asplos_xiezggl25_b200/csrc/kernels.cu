@@ -769,6 +769,31 @@ void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32
                                                              c->capT, pool_min, c->gslot, c->peer_tab, c->dstats)));
     c->launches++;
 }
+// host-link calibration: n pseudo-random rows of the host table (hash of i and seed) read
+// with the gather's access pattern (row groups, zero-copy, same grid cap) into scratch
+template <int GS>
+__global__ void k_probe_rows(int64_t n, int64_t N, uint64_t seed, int d4, const float4* hw, float4* __restrict__ out,
+                             int64_t out_rows) {
+    int64_t gid, gs;
+    int l;
+    RowGroup<GS>::ids(gid, gs, l);
+    for (int64_t i = gid; i < n; i += gs) {
+        uint64_t z = seed + 0x9e3779b97f4a7c15ULL * (uint64_t)(i + 1);
+        z = (z ^ (z >> 30)) * 0xbf58476d1ce4e5b9ULL;
+        z = (z ^ (z >> 27)) * 0x94d049bb133111ebULL;
+        z ^= z >> 31;
+        const int64_t k = (int64_t)(z % (uint64_t)N);
+        for (int v = l; v < d4; v += GS) out[(i % out_rows) * d4 + v] = hw[k * d4 + v];
+    }
+}
+void launch_probe_rows(frugal_ctx* c, int64_t n, uint64_t seed, float* out, int64_t out_rows, cudaStream_t st) {
+    const int d4 = c->d / 4, gs = group_size(d4);
+    int grid = std::min(grid_for(n * gs, 256, 8), c->gather_blocks);
+    DISPATCH_GS(gs, (k_probe_rows<GS><<<grid, 256, 0, st>>>(n, c->N, seed, d4, (const float4*)c->dh_w, (float4*)out,
+                                                            out_rows)));
+    c->launches++;
+}
+
 void launch_expand(frugal_ctx* c, QueueSlot& q, const float* rows, float* out, cudaStream_t st) {
     const int d4 = c->d / 4, gs = group_size(d4);
     int grid = grid_for((int64_t)c->M * gs, 256, 8);

@@ -1166,5 +1166,26 @@ extern "C" frugal_status frugal_get_stats(frugal_ctx* c, frugal_stats* out) {
     return FRUGAL_OK;
 }
 
+extern "C" frugal_status frugal_probe_host_reads(frugal_ctx* c, int64_t n, uint64_t seed, double* ms) {
+    if (!c || !ms || n <= 0) { set_err("bad arguments"); return FRUGAL_EINVAL; }
+    if (c->phase_in_step != 0) { set_err("probe in the middle of a step"); return FRUGAL_ESTATE; }
+    CK(cudaDeviceSynchronize());
+    cudaEvent_t a, b;
+    CK(cudaEventCreate(&a));
+    CK(cudaEventCreate(&b));
+    const int64_t out_rows = std::min<int64_t>(n, c->M);
+    CK(cudaEventRecord(a, 0));
+    launch_probe_rows(c, n, seed, c->chunk_scratch, out_rows, 0);
+    CK(cudaEventRecord(b, 0));
+    CK(cudaEventSynchronize(b));
+    float f = 0.f;
+    cudaEventElapsedTime(&f, a, b);
+    cudaEventDestroy(a);
+    cudaEventDestroy(b);
+    *ms = f;
+    CKL();
+    return FRUGAL_OK;
+}
+
 extern "C" int64_t frugal_owned_rows(frugal_ctx* c) { return c ? c->No : -1; }
 extern "C" int64_t frugal_hot_slots(frugal_ctx* c) { return c ? c->cap_hot : -1; }

@@ -84,6 +84,7 @@ def lib():
             "frugal_read_host": [P, P, I64, P, P],
             "frugal_get_stats": [P, C.POINTER(Stats)],
             "frugal_get_timeline": [P, P, P, P, I64, C.POINTER(I64)],
+            "frugal_probe_host_reads": [P, I64, C.c_uint64, C.POINTER(C.c_double)],
             "frugal_a2a_requests": [P, I64, P, P, P],
             "frugal_a2a_serve": [P, I64, P, I64, P, P],
             "frugal_a2a_lookup": [P, I64, P, P, P],
@@ -109,7 +110,8 @@ EXPORTED = ["frugal_init", "frugal_prefetch", "frugal_step", "frugal_lookup", "f
             "frugal_get_dedup",
             "frugal_get_schedule", "frugal_get_final_flush", "frugal_read_rows", "frugal_read_host",
             "frugal_get_stats", "frugal_get_timeline", "frugal_owned_rows", "frugal_hot_slots",
-            "frugal_a2a_requests", "frugal_a2a_serve", "frugal_a2a_lookup", "frugal_a2a_pack", "frugal_a2a_update"]
+            "frugal_a2a_requests", "frugal_a2a_serve", "frugal_a2a_lookup", "frugal_a2a_pack", "frugal_a2a_update",
+            "frugal_probe_host_reads"]
 
 
 def _check(status):
@@ -278,6 +280,12 @@ class Frugal:
         n = C.c_int64()
         _check(lib().frugal_get_timeline(self.h, ph.ctypes.data, t0.ctypes.data, t1.ctypes.data, cap, C.byref(n)))
         return [(PHASES[ph[i]], float(t0[i]), float(t1[i])) for i in range(n.value)]
+
+    def probe_host_reads(self, n, seed=12345):
+        """ms to read n random host-table rows with the gather's pattern (calibration)."""
+        ms = C.c_double()
+        _check(lib().frugal_probe_host_reads(self.h, n, seed, C.byref(ms)))
+        return ms.value
 
     @property
     def owned_rows(self):
