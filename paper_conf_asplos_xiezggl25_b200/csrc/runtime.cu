@@ -299,6 +299,9 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     // pool segments: a row updated at u sits in segment u % P until the optimizer of u+P;
     // its last reader is the drain of step u+1+D (age-out), which step u+D+3 waits for
     c->P = c->D + 3;
+    // FRUGAL_POOL_STEPS=P' > D+3 keeps every segment for P' steps: owned cold rows updated
+    // within the last P'-2 steps are then read from HBM (R7') -- more HBM, fewer host reads
+    if (getenv("FRUGAL_POOL_STEPS")) c->P = std::max(c->P, atoi(getenv("FRUGAL_POOL_STEPS")));
     c->QN = c->L + 2;
     // pipelined early gather (world 1): off by default -- measured no gain on a PCIe-bound
     // box (the zero-copy loads of the next step only delay this step's); FRUGAL_EARLY=1
@@ -493,7 +496,13 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         CK(cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, prio));
     }
     CK(cudaEventCreateWithFlags(&c->ev_sched, cudaEventDisableTiming));
-    CK(cudaStreamCreateWithFlags(&c->istream, cudaStreamNonBlocking));
+    {   // ingest-stream priority (FRUGAL_INGEST_PRIO=low|normal|high, default normal)
+        const char* ip = getenv("FRUGAL_INGEST_PRIO");
+        int prio = 0;
+        if (ip && !strcmp(ip, "high")) prio = hi_prio;
+        if (ip && !strcmp(ip, "low")) prio = lo_prio;
+        CK(cudaStreamCreateWithPriority(&c->istream, cudaStreamNonBlocking, prio));
+    }
     CK(cudaEventCreateWithFlags(&c->ev_call, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&c->ev_copied, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&c->ev_gathered, cudaEventDisableTiming));
@@ -584,7 +593,9 @@ static frugal_status ingest(frugal_ctx* c, int64_t t, const int64_t* ids_all, co
     QueueSlot& q = c->q[qi];
     q.step = t;
     q.h_counts.assign(counts, counts + c->n);
-    cudaStream_t is = c->istream;
+    // FRUGAL_INGEST_SERIAL=1 (diagnostic): ingest on the caller's stream, no overlap
+    static const bool serial = getenv("FRUGAL_INGEST_SERIAL") && atoi(getenv("FRUGAL_INGEST_SERIAL"));
+    cudaStream_t is = serial ? caller : c->istream;
     // the caller's buffer is read after the caller's prior work on `caller`; the copy of the
     // previous call has finished once this call returns (host wait, normally long done), so
     // the caller may reuse a buffer after the next frugal_step/frugal_prefetch returns

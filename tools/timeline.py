@@ -2,6 +2,7 @@
 bench workload: which phase runs when, on which stream, in the steady state."""
 import os
 import sys
+import time
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np
@@ -11,8 +12,9 @@ from paper_conf_asplos_xiezggl25_b200 import frugal as F
 from paper_conf_asplos_xiezggl25_b200 import workload as W
 from paper_conf_asplos_xiezggl25_b200.harness import make_context
 
+SLEEP = float(os.environ.get("TL_SLEEP", "0"))
 cfg = W.config("criteo_kaggle", world=1)
-S, L = 60, cfg.lookahead
+S, L = int(os.environ.get("TL_STEPS", "60")), cfg.lookahead
 st = W.gen_stream(cfg, S + L + 2)
 fr = make_context(st, flags=F.F_TIMERS)
 dev = torch.device("cuda", 0)
@@ -26,6 +28,9 @@ for t in range(L):
     fr.prefetch(t, ids[t], st.counts[t])
 for s in range(S):
     fr.step(s, ids[s + L], st.counts[s + L])
+    if SLEEP:  # diagnostic: let the step's flushes settle before the gather
+        torch.cuda.synchronize()
+        time.sleep(SLEEP)
     fr.lookup(s, emb)
     fr.dot_model(s, emb, x[s], y[s], grad, loss[s:s + 1])
     fr.backward_update(s, grad)
