@@ -36,6 +36,11 @@
  *     L1074-1077) -> D(s) (or EXEMPT);
  *   * age-out A(s): cold INF rows whose last update <= s-1-D (reading R9);
  *   * final flush: every still-dirty row (L1082-1083); hot rows also push G.
+ *   * dynamic cache (reading R27): the hot set H_t is a
+ *     step function (epochs starting at t0); every "hot" above means "hot at the step in
+ *     question".  At an epoch boundary t0, before anything else of step t0, every row
+ *     whose hotness changes and that is dirty is flushed (w and G) -- the transition set
+ *     X(t0) -- and an evicted row's G is pushed to the host (G follows w out of the cache).
  *  A simulated host table Hw/HG is written only by flushes; invariant (2)
  *  (L1104-1108) is checked on every host read: no host-read of a dirty row and
  *  Hw == W bit-for-bit.
@@ -52,7 +57,9 @@ enum { OR_SGD = 0, OR_ADAGRAD = 1 };
 enum { OR_MODEL_DOT = 0, OR_MODEL_CONST = 1, OR_MODEL_L2 = 2, OR_MODEL_TRANSE = 3 };
 enum { OR_CLEAN = 0, OR_UPDATED = 1, OR_INFP = 2, OR_EXEMPT = 3 };
 enum { OR_L_URGENT = 0, OR_L_DEFERRED = 1, OR_L_DEFERRED_P = 2, OR_L_AGEOUT = 3,
-       OR_L_FINAL = 4, OR_L_UPDATED = 5, OR_L_INF = 6, OR_L_EXEMPT = 7 };
+       OR_L_FINAL = 4, OR_L_UPDATED = 5, OR_L_INF = 6, OR_L_EXEMPT = 7, OR_L_TRANSITION = 8 };
+#define OR_NLISTS 9
+#define OR_MAX_EPOCHS 4096
 
 typedef struct {
     int32_t world, dim, slots, batch, lookahead, age_out, opt, model;
@@ -60,7 +67,7 @@ typedef struct {
     float lr, eps, init_accum, init_scale;
     uint64_t init_seed;
     int32_t write_through;    /* 1: every update flushed at the next step (Frugal-Sync, L1399-1402) */
-    int32_t skip_urgent_step; /* negative test: urgent flush of this step is lost (-1: never) */
+    int32_t skip_urgent_step; /* negative test: urgent (and transition) flushes of this step are lost (-1: never) */
     float gamma;              /* TransE margin */
     int32_t neg_chunk;        /* TransE: triples per negative-sharing chunk */
 } oracle_config;
@@ -70,7 +77,8 @@ typedef struct { int64_t v; int64_t p; } pair64;
 
 typedef struct {
     oracle_config c;
-    int64_t* hot; int64_t n_hot;
+    /* hot sets by epoch: epoch e is in force for steps [ep_t0[e], ep_t0[e+1]) (N3) */
+    int64_t n_ep; int64_t ep_t0[OR_MAX_EPOCHS]; int64_t* ep_hot[OR_MAX_EPOCHS]; int64_t ep_n[OR_MAX_EPOCHS];
     /* lazily materialised rows: open-addressing map key -> index */
     int64_t* hkeys; int64_t* hidx; int64_t hcap;
     int64_t n, cap; rowmeta* meta; float *W, *G, *Hw, *HG;
@@ -80,7 +88,7 @@ typedef struct {
     int64_t cur;                  /* next step to run */
     int64_t* upd; int64_t n_upd;  /* rows updated at cur-1 (sorted) */
     /* artefacts of the last step() */
-    int64_t* lists[8]; int64_t nl[8], capl[8];
+    int64_t* lists[OR_NLISTS]; int64_t nl[OR_NLISTS], capl[OR_NLISTS];
     int gate_wait;
     double* loss;
     float* grad; /* last step grads [world][batch*slots][dim] */
@@ -118,8 +126,15 @@ static void push(oracle* o, int which, int64_t v) {
     }
     o->lists[which][o->nl[which]++] = v;
 }
-static int is_hot(const oracle* o, int64_t k) {
-    return o->n_hot && bsearch(&k, o->hot, o->n_hot, sizeof(int64_t), cmp_i64) != NULL;
+/* k is hot (cached by its owner) at step t: the hot set of t's epoch */
+static int is_hot(const oracle* o, int64_t k, int64_t t) {
+    int64_t e = o->n_ep - 1;
+    while (e > 0 && o->ep_t0[e] > t) e--;
+    return o->ep_n[e] && bsearch(&k, o->ep_hot[e], o->ep_n[e], sizeof(int64_t), cmp_i64) != NULL;
+}
+static int epoch_starts_at(const oracle* o, int64_t t) {
+    for (int64_t e = 1; e < o->n_ep; e++) if (o->ep_t0[e] == t) return 1;
+    return 0;
 }
 static int owner(const oracle* o, int64_t k) { return (int)(k % o->c.world); }
 
@@ -206,13 +221,13 @@ static int any_read(oracle* o, int64_t k, int64_t t) {
     for (int g = 0; g < o->c.world; g++) if (read_by(o, k, t, g)) return 1;
     return 0;
 }
-/* a host-reader: any reader except the owner reading its own hot row (R7) */
-static int host_reader(const oracle* o, int64_t k, int g) {
-    return !(g == owner(o, k) && is_hot(o, k));
+/* a host-reader at t: any reader except the owner reading its own hot row (R7) */
+static int host_reader(const oracle* o, int64_t k, int g, int64_t t) {
+    return !(g == owner(o, k) && is_hot(o, k, t));
 }
 static int needs_host(oracle* o, int64_t k, int64_t t) {
     for (int g = 0; g < o->c.world; g++)
-        if (read_by(o, k, t, g) && host_reader(o, k, g)) return 1;
+        if (read_by(o, k, t, g) && host_reader(o, k, g, t)) return 1;
     return 0;
 }
 static int32_t next_access(oracle* o, int64_t k, int64_t u) {
@@ -241,10 +256,12 @@ static int host_fresh_g(const oracle* o, int64_t i) {
 void* oracle_new(const oracle_config* c, const int64_t* hot, int64_t n_hot) {
     oracle* o = calloc(1, sizeof(oracle));
     o->c = *c;
-    o->n_hot = n_hot;
-    o->hot = malloc((n_hot ? n_hot : 1) * sizeof(int64_t));
-    memcpy(o->hot, hot, n_hot * sizeof(int64_t));
-    qsort(o->hot, n_hot, sizeof(int64_t), cmp_i64);
+    o->n_ep = 1;
+    o->ep_t0[0] = 0;
+    o->ep_n[0] = n_hot;
+    o->ep_hot[0] = malloc((n_hot ? n_hot : 1) * sizeof(int64_t));
+    memcpy(o->ep_hot[0], hot, n_hot * sizeof(int64_t));
+    qsort(o->ep_hot[0], n_hot, sizeof(int64_t), cmp_i64);
     rehash(o);
     return o;
 }
@@ -253,13 +270,27 @@ void oracle_free(void* p) {
     oracle* o = p;
     if (!o) return;
     for (int64_t i = 0; i < o->S * o->c.world; i++) free(o->uq[i]);
-    for (int i = 0; i < 8; i++) free(o->lists[i]);
+    for (int i = 0; i < OR_NLISTS; i++) free(o->lists[i]);
+    for (int64_t e = 0; e < o->n_ep; e++) free(o->ep_hot[e]);
     for (int g = 0; g < o->c.world && o->pk; g++) { free(o->pk[g]); free(o->pv[g]); }
     free(o->pk); free(o->pv); free(o->pn);
     free(o->uq); free(o->uq_n); free(o->upd); free(o->loss); free(o->grad);
-    free(o->hot); free(o->hkeys); free(o->hidx);
+    free(o->hkeys); free(o->hidx);
     free(o->meta); free(o->W); free(o->G); free(o->Hw); free(o->HG);
     free(o);
+}
+
+/* N3: from step t0 on the hot set is hot[0..n) (t0 after every earlier epoch start) */
+int oracle_set_hot(void* p, int64_t t0, const int64_t* hot, int64_t n) {
+    oracle* o = p;
+    if (o->n_ep >= OR_MAX_EPOCHS || t0 <= o->ep_t0[o->n_ep - 1]) return -1;
+    int64_t e = o->n_ep++;
+    o->ep_t0[e] = t0;
+    o->ep_n[e] = n;
+    o->ep_hot[e] = malloc((n ? n : 1) * sizeof(int64_t));
+    memcpy(o->ep_hot[e], hot, n * sizeof(int64_t));
+    qsort(o->ep_hot[e], n, sizeof(int64_t), cmp_i64);
+    return 0;
 }
 
 /* the whole stream is given up front: the lookahead reads future steps */
@@ -281,11 +312,27 @@ int oracle_set_stream(void* p, int64_t S, const int64_t* ids, const int32_t* cou
 /* ---- schedule part of step s: (b) bucketing of Upd(s-1), (c) AdjustPriority, (d) age-out, (e) gate */
 static void schedule(oracle* o, int64_t s) {
     const int L = o->c.lookahead;
-    for (int i = 0; i < 8; i++) o->nl[i] = 0;
+    for (int i = 0; i < OR_NLISTS; i++) o->nl[i] = 0;
+    /* (N3) epoch boundary: rows changing hotness are made clean first (reading R27) */
+    if (s >= 1 && epoch_starts_at(o, s)) {
+        for (int64_t i = 0; i < o->n; i++) {
+            int64_t k = o->meta[i].key;
+            int was = is_hot(o, k, s - 1), now = is_hot(o, k, s);
+            if (was == now) continue;
+            if (o->meta[i].state != OR_CLEAN) {
+                push(o, OR_L_TRANSITION, k);
+                if (s == o->c.skip_urgent_step) o->meta[i].state = OR_CLEAN; /* negative test: lost */
+                else flush_row(o, i, 1);
+            }
+            if (was) memcpy(o->HG + i * o->c.dim, o->G + i * o->c.dim, o->c.dim * sizeof(float));
+        }
+        qsort(o->lists[OR_L_TRANSITION], o->nl[OR_L_TRANSITION], sizeof(int64_t), cmp_i64);
+    }
     /* (b) rows updated at s-1: priority = next access (Eq. 1) */
     for (int64_t a = 0; a < o->n_upd; a++) {
         int64_t k = o->upd[a], i = find_row(o, k);
-        int cold = !is_hot(o, k);
+        if (o->meta[i].state == OR_CLEAN) continue; /* flushed by the transition above */
+        int cold = !is_hot(o, k, s);
         if (o->c.write_through) { push(o, OR_L_URGENT, k); flush_row(o, i, cold); continue; }
         int32_t pr = next_access(o, k, s - 1);
         if (pr == OR_INF) { o->meta[i].state = OR_INFP; continue; }
@@ -308,7 +355,7 @@ static void schedule(oracle* o, int64_t s) {
                 if (i < 0 || o->meta[i].state != OR_INFP) continue;
                 if (needs_host(o, k, t)) {
                     push(o, OR_L_DEFERRED, k); push(o, OR_L_DEFERRED_P, t);
-                    flush_row(o, i, !is_hot(o, k));
+                    flush_row(o, i, !is_hot(o, k, s));
                 } else {
                     o->meta[i].state = OR_EXEMPT;
                 }
@@ -318,7 +365,7 @@ static void schedule(oracle* o, int64_t s) {
     /* (d) age-out of cold rows still dirty with INF priority */
     for (int64_t i = 0; i < o->n; i++) {
         rowmeta* m = &o->meta[i];
-        if (m->state == OR_INFP && !is_hot(o, m->key) && m->last_update <= s - 1 - o->c.age_out) {
+        if (m->state == OR_INFP && !is_hot(o, m->key, s) && m->last_update <= s - 1 - o->c.age_out) {
             push(o, OR_L_AGEOUT, m->key);
             flush_row(o, i, 1);
         }
@@ -346,7 +393,7 @@ static void schedule(oracle* o, int64_t s) {
         int64_t n; const int64_t* u = uniq(o, s, g, &n);
         for (int64_t q = 0; q < n; q++) {
             int64_t k = u[q];
-            if (!host_reader(o, k, g)) continue;
+            if (!host_reader(o, k, g, s)) continue;
             int64_t i = row(o, k);
             if (o->meta[i].state != OR_CLEAN || !host_fresh_w(o, i)) o->violations++;
         }
@@ -541,7 +588,7 @@ static void train(oracle* o, int64_t s) {
             }
         }
         /* a cold row is read from the host at update time: it must be fresh */
-        if (!is_hot(o, k) && (o->meta[i].state != OR_CLEAN || !host_fresh_w(o, i) || !host_fresh_g(o, i)))
+        if (!is_hot(o, k, s) && (o->meta[i].state != OR_CLEAN || !host_fresh_w(o, i) || !host_fresh_g(o, i)))
             o->violations++;
         /* (i) optimizer, elementwise fp32 */
         float* w = o->W + i * d;
@@ -581,13 +628,14 @@ int64_t oracle_step(void* p) {
 /* end of training: every dirty row to the host (L1082-1083); hot rows also push G (R8) */
 int64_t oracle_final_flush(void* p) {
     oracle* o = p;
-    for (int i = 0; i < 8; i++) o->nl[i] = 0;
+    const int64_t last = o->cur > 0 ? o->cur - 1 : 0;
+    for (int i = 0; i < OR_NLISTS; i++) o->nl[i] = 0;
     for (int64_t i = 0; i < o->n; i++) {
         if (o->meta[i].state != OR_CLEAN) {
             push(o, OR_L_FINAL, o->meta[i].key);
             flush_row(o, i, 1);
         }
-        if (is_hot(o, o->meta[i].key)) {
+        if (is_hot(o, o->meta[i].key, last)) {
             int64_t d = o->c.dim;
             memcpy(o->HG + i * d, o->G + i * d, d * sizeof(float));
         }

@@ -18,7 +18,7 @@ SRC = os.path.join(HERE, "frugal_oracle.c")
 LIB = os.path.join(HERE, "liboracle.so")
 
 INF = 2**31 - 1
-L_URGENT, L_DEFERRED, L_DEFERRED_P, L_AGEOUT, L_FINAL, L_UPDATED, L_INF, L_EXEMPT = range(8)
+L_URGENT, L_DEFERRED, L_DEFERRED_P, L_AGEOUT, L_FINAL, L_UPDATED, L_INF, L_EXEMPT, L_TRANSITION = range(9)
 CLEAN, UPDATED, INFP, EXEMPT = range(4)
 MODELS = {"dot": 0, "const": 1, "l2": 2, "transe": 3}
 OPTS = {"sgd": 0, "adagrad": 1}
@@ -78,6 +78,8 @@ def lib():
         _lib.oracle_get_grad.argtypes = [P, I32, P]
         _lib.oracle_get_partial.restype = I64
         _lib.oracle_get_partial.argtypes = [P, I32, P, P]
+        _lib.oracle_set_hot.restype = C.c_int
+        _lib.oracle_set_hot.argtypes = [P, I64, P, I64]
         _lib.oracle_init_value.restype = C.c_float
         _lib.oracle_init_value.argtypes = [P, I64, I32]
     return _lib
@@ -121,6 +123,14 @@ class Oracle:
         L = lib()
         self.h = L.oracle_new(C.byref(c), _p(self._hot), len(self._hot))
         L.oracle_set_stream(self.h, stream.ids.shape[0], *[_p(a) for a in self._keep])
+        for t0, ids in getattr(stream, "hot_schedule", None) or []:
+            self.set_hot(t0, ids)
+
+    def set_hot(self, t0, ids):
+        """N3: the hot set from step t0 on (reading R27)."""
+        a = np.ascontiguousarray(ids, dtype=np.int64)
+        if lib().oracle_set_hot(self.h, int(t0), _p(a), len(a)) != 0:
+            raise ValueError(f"oracle_set_hot({t0}): epochs must start after the previous one")
 
     def __del__(self):
         if getattr(self, "h", None):
@@ -151,7 +161,8 @@ class Oracle:
         return dict(urgent=self.get_list(L_URGENT), deferred=self.get_list(L_DEFERRED),
                     deferred_p=self.get_list(L_DEFERRED_P), ageout=self.get_list(L_AGEOUT),
                     inf=self.get_list(L_INF), exempt=self.get_list(L_EXEMPT),
-                    updated=self.get_list(L_UPDATED), gate_wait=bool(lib().oracle_gate_wait(self.h)))
+                    updated=self.get_list(L_UPDATED), transition=self.get_list(L_TRANSITION),
+                    gate_wait=bool(lib().oracle_gate_wait(self.h)))
 
     def loss(self, s) -> float:
         return lib().oracle_loss(self.h, s)

@@ -215,6 +215,8 @@ class Stream:
     x: np.ndarray
     y: np.ndarray
     hot: np.ndarray
+    # N3 dynamic cache (reading R27): [(t0, hot ids)], the hot set in force from step t0 on
+    hot_schedule: list = dataclasses.field(default_factory=list)
 
     @property
     def steps(self) -> int:
@@ -237,9 +239,10 @@ def gen_ids(cfg: WorkloadConfig, steps: int, world: Optional[int] = None) -> np.
     return ids.reshape(steps, world, B * F)
 
 
-def hot_set(cfg: WorkloadConfig, ids: np.ndarray, counts: Optional[np.ndarray] = None) -> np.ndarray:
-    """Top floor(ratio*N_f) rows per table by frequency over the first min(S,50) steps."""
-    S = min(ids.shape[0], 50)
+def hot_set(cfg: WorkloadConfig, ids: np.ndarray, counts: Optional[np.ndarray] = None,
+            window: int = 50) -> np.ndarray:
+    """Top floor(ratio*N_f) rows per table by frequency over the first min(S, window) steps."""
+    S = min(ids.shape[0], window)
     F, B = cfg.slots, cfg.batch
     sub = ids[:S].reshape(S, -1, B, F)
     if counts is not None:
@@ -283,6 +286,19 @@ def gen_stream(cfg: WorkloadConfig, steps: int, world: Optional[int] = None,
     x[~valid] = 0
     hot = hot_set(cfg, ids, counts)
     return Stream(cfg, np.ascontiguousarray(ids), counts, x, y, hot)
+
+
+def with_dynamic_hot(st: Stream, epoch: int, window: Optional[int] = None) -> Stream:
+    """N3 cache policy (reading R27; the paper's cache "follows HugeCTR", L1412-1414): every
+    `epoch` steps the hot set is recomputed as the same per-table top-frequency rule (R10)
+    over the `window` (default: epoch) steps just before the boundary t0 -- an LFU over a
+    sliding window, decided from past traffic only.  Returns a copy carrying the schedule."""
+    window = epoch if window is None else window
+    sched = []
+    for t0 in range(epoch, st.steps, epoch):
+        lo = max(0, t0 - window)
+        sched.append((t0, hot_set(st.cfg, st.ids[lo:t0], st.counts[lo:t0], window=t0 - lo)))
+    return dataclasses.replace(st, hot_schedule=sched)
 
 
 def stream_from_lists(cfg: WorkloadConfig, per_step: List[List[List[int]]],
