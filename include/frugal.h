@@ -65,6 +65,9 @@ enum {
                                    the owner holds in HBM (cache, or dirty pool) is loaded from
                                    the owner's GPU over peer memory (CUDA IPC) instead of the
                                    host table; flush schedule and results unchanged; world > 1 */
+    FRUGAL_F_DYNAMIC_CACHE = 32,/* N3: the hot set may change at epoch
+                                   boundaries (frugal_set_hot); the cache gets 25% spare
+                                   slots; not with FRUGAL_F_PEER or the early gather      */
     FRUGAL_F_A2A = 8            /* comparison path (the message pipeline of
                                    PAPER.md Fig. 2b): rows and gradients move between
                                    ranks by the caller's all-to-all (NCCL over NVLink) through
@@ -141,6 +144,18 @@ frugal_status frugal_lookup(frugal_ctx* ctx, int64_t s, float* d_out, frugal_str
 frugal_status frugal_backward_update(frugal_ctx* ctx, int64_t s, const float* d_grad,
                                      frugal_stream stream);
 
+/* N3 dynamic cache (needs FRUGAL_F_DYNAMIC_CACHE; reading R27).  From step t0
+   on, the hot (cached) set is hot_ids (host array of global ids, any order; each owner
+   keeps its share) instead of the previous one.  The reads of steps >= t0 are classified
+   against it as soon as they are ingested, so this must be called before the ingest of t0
+   is enqueued (before frugal_step(t0 - L), or frugal_prefetch(t0) for t0 < L) and at most
+   one change may be pending.  At the start of frugal_step(t0) the owner flushes every row
+   whose hotness changes and whose host copy is not current (the transition set, on the
+   critical path, like the urgent bucket), then evicts and admits rows.  Results (tables,
+   losses) do not depend on the hot sets.  FRUGAL_EINVAL: the owned share exceeds the slot
+   capacity (1.25x the initial share + 64); FRUGAL_ESTATE: too late / one already pending. */
+frugal_status frugal_set_hot(frugal_ctx* ctx, int64_t t0, const int64_t* hot_ids, int64_t n_hot);
+
 /* End of training (L1082-1083): every dirty owned row (w and G) and the G of every
    hot row to the host table; waits for the side stream.  Afterwards the host table
    is authoritative. */
@@ -211,6 +226,10 @@ typedef struct {
 frugal_status frugal_get_schedule(frugal_ctx* ctx, frugal_schedule_info* info, int64_t* urgent,
                                   int64_t* deferred, int32_t* deferred_p, int64_t* ageout);
 
+/* rows flushed by the cache transition of the last frugal_step (global ids, any order;
+   empty unless that step was an epoch boundary; needs FRUGAL_F_RECORD) */
+frugal_status frugal_get_transition(frugal_ctx* ctx, int64_t* rows, int64_t* n);
+
 /* rows flushed by the last frugal_flush(FRUGAL_FLUSH_ALL) (global ids, any order) */
 frugal_status frugal_get_final_flush(frugal_ctx* ctx, int64_t* rows, int64_t* n);
 
@@ -246,6 +265,8 @@ enum {
     FRUGAL_C_MAIL_IN = 14,      /* partial rows read from other ranks' mailboxes             */
     FRUGAL_C_GATHER_POOL = 15,  /* unique owned cold rows gathered from the dirty pool (HBM)  */
     FRUGAL_C_GATHER_PEER = 16,  /* unique non-owned rows loaded from the owner's HBM (PEER)  */
+    FRUGAL_C_TRANSITION_HOT = 17,  /* rows flushed by cache transitions (N3), from the cache */
+    FRUGAL_C_TRANSITION_COLD = 18, /* ... from the dirty pool                               */
     FRUGAL_N_COUNTERS = 20
 };
 typedef struct {

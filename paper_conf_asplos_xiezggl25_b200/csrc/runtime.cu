@@ -143,6 +143,10 @@ static frugal_status check_err_word(frugal_ctx* c) {
             set_err("a peer rank did not publish its flag within 120 s");
             return FRUGAL_ETIMEOUT;
         }
+        if (e == 3) {
+            set_err("dynamic cache: more admitted rows than free slots");
+            return FRUGAL_EINVAL;
+        }
         set_err("a row id outside [0, n_rows) was passed in a sample batch");
         return FRUGAL_EINVAL;
     }
@@ -158,6 +162,7 @@ static void free_ctx(frugal_ctx* c) {
     };
     F(c->slot); F(c->state); F(c->last_upd); F(c->pool_idx); F(c->rbits);
     F(c->cw); F(c->Gd); F(c->hot_lk); F(c->pw); F(c->pkey); F(c->pcount);
+    F(c->hot_map[0]); F(c->hot_map[1]); F(c->new_lk); F(c->free_slots); F(c->tr_cnt); F(c->tr_rows);
     for (auto& q : c->q) {
         F(q.eidx); F(q.lidx); F(q.elcnt);
         F(q.ids); F(q.counts); F(q.m); F(q.uniq); F(q.inv); F(q.off); F(q.pos); F(q.n_uniq);
@@ -190,6 +195,7 @@ static void free_ctx(frugal_ctx* c) {
     }
     if (c->pstream) cudaStreamDestroy(c->pstream);
     for (auto e : c->ev_pool) cudaEventDestroy(e);
+    if (c->ev_hot) cudaEventDestroy(c->ev_hot);
     if (c->shm_base) {
         cudaHostUnregister(c->shm_base);
         munmap(c->shm_base, c->shm_bytes);
@@ -283,6 +289,10 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         set_err("FRUGAL_F_PEER needs world > 1 and the host-bounced exchange");
         return FRUGAL_EINVAL;
     }
+    if ((k.flags & FRUGAL_F_DYNAMIC_CACHE) && (k.flags & FRUGAL_F_PEER)) {
+        set_err("FRUGAL_F_DYNAMIC_CACHE does not combine with FRUGAL_F_PEER");
+        return FRUGAL_EINVAL;
+    }
     if (k.n_hot < 0 || (k.n_hot > 0 && !k.hot_ids)) { set_err("bad hot set"); return FRUGAL_EINVAL; }
     for (int64_t i = 0; i < k.n_hot; i++)
         if (k.hot_ids[i] < 0 || k.hot_ids[i] >= k.n_rows) { set_err("hot id out of range"); return FRUGAL_EINVAL; }
@@ -299,6 +309,10 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     // pool segments: a row updated at u sits in segment u % P until the optimizer of u+P;
     // its last reader is the drain of step u+1+D (age-out), which step u+D+3 waits for
     c->P = c->D + 3;
+    // N3: a cold dirty row may wait for a cache transition instead of its age-out (EXEMPT
+    // for a read under the next hot set): its pool copy must live until that boundary,
+    // at most D + L steps after its update
+    if (k.flags & FRUGAL_F_DYNAMIC_CACHE) c->P = std::max(c->P, c->D + c->L + 1);
     // FRUGAL_POOL_STEPS=P' > D+3 keeps every segment for P' steps: owned cold rows updated
     // within the last P'-2 steps are then read from HBM (R7') -- more HBM, fewer host reads
     if (getenv("FRUGAL_POOL_STEPS")) c->P = std::max(c->P, atoi(getenv("FRUGAL_POOL_STEPS")));
@@ -311,6 +325,8 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->early_on_side = getenv("FRUGAL_EARLY_ON_SIDE") && atoi(getenv("FRUGAL_EARLY_ON_SIDE"));
     c->a2a = (k.flags & FRUGAL_F_A2A) != 0;
     c->peer = (k.flags & FRUGAL_F_PEER) != 0;
+    c->dyn = (k.flags & FRUGAL_F_DYNAMIC_CACHE) != 0;
+    if (c->dyn) c->early = false;
     c->xhost = c->n > 1 && !c->a2a;
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 32;
     c->gather_blocks = getenv("FRUGAL_GATHER_BLOCKS") ? atoi(getenv("FRUGAL_GATHER_BLOCKS")) : 74;
@@ -417,8 +433,17 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     std::sort(hot.begin(), hot.end());
     hot.erase(std::unique(hot.begin(), hot.end()), hot.end());
     c->cap_hot = (int64_t)hot.size();
-    DMALLOC(c->hot_lk, c->cap_hot * 4);
-    DMALLOC(c->cw, c->cap_hot * rowb);
+    c->cap_slots = c->dyn ? c->cap_hot + std::max<int64_t>(64, c->cap_hot / 4) : c->cap_hot;
+    DMALLOC(c->hot_lk, c->cap_slots * 4);
+    DMALLOC(c->cw, c->cap_slots * rowb);
+    if (c->dyn) {
+        DMALLOC(c->hot_map[0], c->No);
+        DMALLOC(c->hot_map[1], c->No);
+        DMALLOC(c->new_lk, c->cap_slots * 4);
+        DMALLOC(c->free_slots, c->cap_slots * 4);
+        DMALLOC(c->tr_cnt, 8);
+        DMALLOC(c->tr_rows, ((size_t)c->capT + 2 * c->cap_slots) * 4);
+    }
     if (adag) DMALLOC(c->Gd, (size_t)c->No * rowb);
     DMALLOC(c->pw, (size_t)c->P * c->capT * rowb);
     DMALLOC(c->pkey, (size_t)c->P * c->capT * 4);
@@ -519,12 +544,22 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     for (auto& e : c->ev_ingest) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
 
     cudaStream_t st = 0;
+    cudaMemset(c->hot_lk, 0xff, c->cap_slots * 4);  // spare slots (N3) are free
+    if (c->dyn) {
+        std::vector<int32_t> fr;
+        for (int64_t j = c->cap_slots - 1; j >= c->cap_hot; j--) fr.push_back((int32_t)j);
+        const int32_t cnt2[2] = {(int32_t)fr.size(), 0};
+        cudaMemcpy(c->free_slots, fr.data(), fr.size() * 4, cudaMemcpyHostToDevice);
+        cudaMemcpy(c->tr_cnt, cnt2, 8, cudaMemcpyHostToDevice);
+        CK(cudaEventCreateWithFlags(&c->ev_hot, cudaEventDisableTiming));
+    }
     if (cudaMemcpy(c->hot_lk, hot.data(), hot.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) {
         set_err("hot upload failed");
         free_ctx(c);
         return FRUGAL_ECUDA;
     }
     launch_init_meta(c, nullptr, 0, st);
+    if (c->dyn) launch_hot_map(c, 0, c->hot_lk, c->cap_hot, st);
     cudaMemset(c->pcount, 0, (size_t)c->P * 4);
     cudaMemset(c->pkey, 0xff, (size_t)c->P * c->capT * 4);
     if (c->g == 0 || !k.shm_name) {
@@ -751,6 +786,26 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
     // the bucket / age-out lists of this parity were last read by the whole drain of s-2
     if (c->side_pending[par]) CK(cudaStreamWaitEvent(st, c->ev_side[par], 0));
     if (s + c->L - 1 >= c->next_prefetch) CK(cudaMemsetAsync(c->adj_cnt[par], 0, 4, st));  // stream end: no adjust
+    c->rec_transition.clear();
+    if (c->dyn && c->hot_pending && s == c->hot_t0) {
+        // N3 epoch boundary: the whole drain of s-1 (it reads cache slots) and the upload
+        // of the new set precede the transition; it runs on the critical path
+        Timer tm(c, PH_URGENT, st);
+        if (s >= 1 && c->side_pending[par ^ 1]) CK(cudaStreamWaitEvent(st, c->ev_side[par ^ 1], 0));
+        CK(cudaStreamWaitEvent(st, c->ev_hot, 0));
+        launch_cache_transition(c, s, par, st);
+        CK(cudaEventRecord(c->ev_hot, st));  // the next frugal_set_hot reuses new_lk after it
+        CKL();
+        c->hot_cur ^= 1;
+        c->hot_pending = false;
+        if (c->cfg.flags & FRUGAL_F_RECORD) {
+            CK(cudaStreamSynchronize(st));
+            int32_t nx = 0;
+            CK(cudaMemcpy(&nx, c->tr_cnt + 1, 4, cudaMemcpyDeviceToHost));
+            c->rec_transition.resize(nx);
+            if (nx) CK(cudaMemcpy(c->rec_transition.data(), c->tr_rows, (size_t)nx * 4, cudaMemcpyDeviceToHost));
+        }
+    }
     {
         Timer tm(c, PH_SCHED, st);
         QueueSlot* prev = nullptr;
@@ -1077,6 +1132,47 @@ extern "C" frugal_status frugal_get_schedule(frugal_ctx* c, frugal_schedule_info
     if (deferred) for (size_t i = 0; i < c->rec_deferred.size(); i++) deferred[i] = glob(c->rec_deferred[i]);
     if (deferred_p) for (size_t i = 0; i < c->rec_deferred_p.size(); i++) deferred_p[i] = c->rec_deferred_p[i];
     if (ageout) for (size_t i = 0; i < c->rec_ageout.size(); i++) ageout[i] = glob(c->rec_ageout[i]);
+    return FRUGAL_OK;
+}
+
+extern "C" frugal_status frugal_set_hot(frugal_ctx* c, int64_t t0, const int64_t* hot_ids, int64_t n_hot) {
+    if (!c || n_hot < 0 || (n_hot > 0 && !hot_ids)) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    if (!c->dyn) { set_err("frugal_set_hot needs FRUGAL_F_DYNAMIC_CACHE"); return FRUGAL_ESTATE; }
+    if (c->hot_pending) { set_err("set_hot(%lld): a change is already pending", (long long)t0); return FRUGAL_ESTATE; }
+    if (t0 < 1 || t0 < c->next_prefetch) {
+        set_err("set_hot(%lld): the ingest of that step was already enqueued (next: %lld)", (long long)t0,
+                (long long)c->next_prefetch);
+        return FRUGAL_ESTATE;
+    }
+    std::vector<int32_t> own;
+    for (int64_t i = 0; i < n_hot; i++) {
+        if (hot_ids[i] < 0 || hot_ids[i] >= c->N) { set_err("hot id out of range"); return FRUGAL_EINVAL; }
+        if (hot_ids[i] % c->n == c->g) own.push_back((int32_t)(hot_ids[i] / c->n));
+    }
+    std::sort(own.begin(), own.end());
+    own.erase(std::unique(own.begin(), own.end()), own.end());
+    if ((int64_t)own.size() > c->cap_slots) {
+        set_err("set_hot: owned share %zu exceeds the %lld cache slots", own.size(), (long long)c->cap_slots);
+        return FRUGAL_EINVAL;
+    }
+    // the map of the previous epoch is free: every ingest that read it precedes this on the
+    // in-order ingest stream; the pinned staging keeps the upload asynchronous
+    CK(cudaStreamSynchronize(c->istream));
+    CK(cudaEventSynchronize(c->ev_hot));  // the previous transition has read new_lk
+    if (!own.empty()) CK(cudaMemcpy(c->new_lk, own.data(), own.size() * 4, cudaMemcpyHostToDevice));
+    c->n_new = (int64_t)own.size();
+    launch_hot_map(c, c->hot_cur ^ 1, c->new_lk, c->n_new, c->istream);
+    CK(cudaEventRecord(c->ev_hot, c->istream));
+    CKL();
+    c->hot_t0 = t0;
+    c->hot_pending = true;
+    return FRUGAL_OK;
+}
+
+extern "C" frugal_status frugal_get_transition(frugal_ctx* c, int64_t* rows, int64_t* n) {
+    if (!c || !n) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    *n = (int64_t)c->rec_transition.size();
+    if (rows) for (size_t i = 0; i < c->rec_transition.size(); i++) rows[i] = (int64_t)c->rec_transition[i] * c->n + c->g;
     return FRUGAL_OK;
 }
 

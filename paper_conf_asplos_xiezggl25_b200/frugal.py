@@ -17,7 +17,7 @@ LIB_PATH = os.path.join(PKG, "libfrugal.so")
 
 SGD, ADAGRAD = 0, 1
 MODE_P2F, MODE_WRITE_THROUGH = 0, 1
-F_RECORD, F_TIMERS, F_NO_HOST_STATE, F_A2A, F_PEER = 1, 2, 4, 8, 16
+F_RECORD, F_TIMERS, F_NO_HOST_STATE, F_A2A, F_PEER, F_DYNAMIC_CACHE = 1, 2, 4, 8, 16, 32
 FLUSH_ALL = 0
 PHASES = ["ingest", "schedule", "urgent", "gate", "gather", "expand", "model", "segred", "exchange",
           "optimizer", "side", "prefetch"]
@@ -47,7 +47,7 @@ class ScheduleInfo(C.Structure):
 
 COUNTERS = ["positions", "unique", "gather_host", "gather_cache", "opt_hot", "opt_cold", "urgent_hot",
             "urgent_cold", "side_hot", "side_cold", "final_hot", "final_cold", "long_segments", "mail_out",
-            "mail_in", "gather_pool", "gather_peer", "reserved17", "reserved18", "reserved19"]
+            "mail_in", "gather_pool", "gather_peer", "transition_hot", "transition_cold", "reserved19"]
 
 
 class Stats(C.Structure):
@@ -80,6 +80,8 @@ def lib():
             "frugal_get_dedup": [P, I64, P, P, C.POINTER(I64)],
             "frugal_get_schedule": [P, C.POINTER(ScheduleInfo), P, P, P, P],
             "frugal_get_final_flush": [P, P, C.POINTER(I64)],
+            "frugal_get_transition": [P, P, C.POINTER(I64)],
+            "frugal_set_hot": [P, I64, P, I64],
             "frugal_read_rows": [P, P, I64, P, P],
             "frugal_read_host": [P, P, I64, P, P],
             "frugal_get_stats": [P, C.POINTER(Stats)],
@@ -111,7 +113,7 @@ EXPORTED = ["frugal_init", "frugal_prefetch", "frugal_step", "frugal_lookup", "f
             "frugal_get_schedule", "frugal_get_final_flush", "frugal_read_rows", "frugal_read_host",
             "frugal_get_stats", "frugal_get_timeline", "frugal_owned_rows", "frugal_hot_slots",
             "frugal_a2a_requests", "frugal_a2a_serve", "frugal_a2a_lookup", "frugal_a2a_pack", "frugal_a2a_update",
-            "frugal_probe_host_reads"]
+            "frugal_probe_host_reads", "frugal_set_hot", "frugal_get_transition"]
 
 
 def _check(status):
@@ -244,6 +246,18 @@ class Frugal:
         _check(lib().frugal_get_schedule(self.h, C.byref(info), u.ctypes.data, dfr.ctypes.data, dp.ctypes.data,
                                          a.ctypes.data))
         return dict(urgent=u, deferred=dfr, deferred_p=dp, ageout=a, gate_wait=bool(info.gate_wait))
+
+    def set_hot(self, t0, hot_ids):
+        """N3: the hot set from step t0 on (before step(t0 - L) / prefetch(t0))."""
+        h = np.ascontiguousarray(hot_ids, dtype=np.int64)
+        _check(lib().frugal_set_hot(self.h, int(t0), h.ctypes.data, len(h)))
+
+    def get_transition(self):
+        n = C.c_int64()
+        _check(lib().frugal_get_transition(self.h, None, C.byref(n)))
+        out = np.empty(n.value, np.int64)
+        _check(lib().frugal_get_transition(self.h, out.ctypes.data, C.byref(n)))
+        return out
 
     def get_final_flush(self):
         n = C.c_int64()

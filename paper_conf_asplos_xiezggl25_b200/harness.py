@@ -21,6 +21,8 @@ def make_context(st, rank=0, device=0, shm_name=None, flags=0, hot=None, mode=F.
               lr=cfg.lr, eps=cfg.eps, init_accum=cfg.init_accum, init_scale=cfg.init_scale,
               init_seed=cfg.seed_init, hot_ids=st.hot if hot is None else hot, shm_name=shm_name, mode=mode,
               flags=flags)
+    if getattr(st, "hot_schedule", None):
+        kw["flags"] |= F.F_DYNAMIC_CACHE  # N3: the stream carries hot-set changes
     kw.update(over)
     return F.Frugal(**kw)
 
@@ -36,14 +38,22 @@ class Trainer:
         self.grad = torch.empty_like(self.emb)
         self.loss = torch.zeros(st.steps, dtype=torch.float64, device=self.dev)
         self.s = 0
+        # N3: hot set changes, handed to the library before the ingest of their t0
+        self._hot = dict((int(t0), ids) for t0, ids in (getattr(st, "hot_schedule", None) or []))
         L = fr.lookahead
         for t in range(min(L, st.steps)):
+            self._set_hot_before_ingest(t)
             fr.prefetch(t, st.ids[t], st.counts[t])
+
+    def _set_hot_before_ingest(self, t):
+        if t in self._hot:
+            self.fr.set_hot(t, self._hot[t])
 
     def step(self, on_schedule=None):
         st, fr, s = self.st, self.fr, self.s
         t = s + fr.lookahead
         if t < st.steps:
+            self._set_hot_before_ingest(t)
             fr.step(s, st.ids[t], st.counts[t])
         else:
             fr.step(s)
@@ -99,6 +109,7 @@ class A2ATrainer(Trainer):
         st, fr, s, D = self.st, self.fr, self.s, self.dist
         t = s + fr.lookahead
         if t < st.steps:
+            self._set_hot_before_ingest(t)
             fr.step(s, st.ids[t], st.counts[t])
         else:
             fr.step(s)

@@ -33,7 +33,11 @@ def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False):
         sched = []
         for s in range(st.steps):
             got = {}
-            tr.step(on_schedule=lambda s_: got.update(fr.get_schedule()))
+
+            def cb(s_):
+                got.update(fr.get_schedule())
+                got["transition"] = fr.get_transition()
+            tr.step(on_schedule=cb)
             sched.append(got)
         fr.flush()
         ff = fr.get_final_flush()
@@ -78,9 +82,10 @@ def run_two_ranks(st, timeout=600, a2a=False, peer=False):
     return out
 
 
-@pytest.mark.parametrize("opt,a2a,peer", [("adagrad", False, False), ("sgd", False, False), ("adagrad", True, False),
-                                          ("adagrad", False, True)])
-def test_two_ranks_one_gpu_parity(opt, a2a, peer):
+@pytest.mark.parametrize("opt,a2a,peer,dyn", [("adagrad", False, False, False), ("sgd", False, False, False),
+                                              ("adagrad", True, False, False), ("adagrad", False, True, False),
+                                              ("adagrad", False, False, True)])
+def test_two_ranks_one_gpu_parity(opt, a2a, peer, dyn):
     """a2a=True: the comparison path (§8(e)) -- ids, rows and partials move by all-to-all
     (gloo with host staging here; NCCL over NVLink on a multi-GPU box) instead of the host
     table and mailbox; every artefact and table must be identical.  peer=True: the N4
@@ -93,6 +98,8 @@ def test_two_ranks_one_gpu_parity(opt, a2a, peer):
     counts = rng.integers(0, 65, size=(24, 2)).astype(np.int32)
     counts[5, 1] = 0
     st = W.gen_stream(cfg, 24, counts=counts)
+    if dyn:  # N3: hot set recomputed every 6 steps (each owner moves its own share)
+        st = W.with_dynamic_hot(st, epoch=6)
     out = run_two_ranks(st, a2a=a2a, peer=peer)
     if peer:  # the variant actually served rows from the other rank's HBM
         assert out[0]["stats"]["gather_peer"] > 0 and out[1]["stats"]["gather_peer"] > 0
@@ -107,6 +114,8 @@ def test_two_ranks_one_gpu_parity(opt, a2a, peer):
         assert dfr == sorted(zip(ref["deferred"].tolist(), ref["deferred_p"].tolist())), f"deferred differs at {s}"
         age = sorted(sum((out[r]["sched"][s]["ageout"].tolist() for r in range(2)), []))
         assert age == ref["ageout"].tolist()
+        xs = sorted(sum((out[r]["sched"][s]["transition"].tolist() for r in range(2)), []))
+        assert xs == ref["transition"].tolist(), f"transition differs at {s}"
         for r in range(2):  # each rank only schedules rows it owns
             assert all(k % 2 == r for k in out[r]["sched"][s]["urgent"].tolist())
     ff = sorted(out[0]["ff"].tolist() + out[1]["ff"].tolist())

@@ -47,6 +47,7 @@ def run_parity(st, *, flags=None, mode=None, hot=None, check_dedup=True, check_s
         def cb(s_):
             if check_sched:
                 got.update(fr.get_schedule())
+                got["transition"] = fr.get_transition()
             if check_dedup and s_ + L < st.steps:
                 t = s_ + L
                 uq, inv = fr.get_dedup(t)
@@ -62,6 +63,7 @@ def run_parity(st, *, flags=None, mode=None, hot=None, check_dedup=True, check_s
             assert sorted(zip(got["deferred"].tolist(), got["deferred_p"].tolist())) == \
                 sorted(zip(ref["deferred"].tolist(), ref["deferred_p"].tolist())), f"deferred set differs at {s}"
             assert sorted(got["ageout"].tolist()) == ref["ageout"].tolist(), f"age-out set differs at {s}"
+            assert sorted(got["transition"].tolist()) == ref["transition"].tolist(), f"transition differs at {s}"
             assert got["gate_wait"] == ref["gate_wait"]
             gate_waits += ref["gate_wait"]
     assert o.violations == 0
@@ -279,3 +281,58 @@ def test_fb15k_kg_full_size():
     r = run_parity(st)
     assert r["exact"]
     r["fr"].close()
+
+
+# ----------------------------------------------------------------------------- N3 dynamic cache
+def test_dynamic_cache_parity():
+    """SURVEY §8(f) N3 (reading R27): the hot set is recomputed every E steps from the
+    previous window (LFU over a sliding window); every schedule artefact, the transition
+    sets X(t0), the losses and the final tables match the oracle; the tables are also
+    bit-identical to a static-cache run (values cannot depend on the cache)."""
+    cfg = tiny1(lookahead=4, age_out=3, cache_ratio=0.05)
+    st = W.gen_stream(cfg, 60)
+    dyn = W.with_dynamic_hot(st, epoch=7)
+    r = run_parity(dyn)
+    assert r["exact"]
+    c = r["fr"].get_stats()["count"]
+    assert c["transition_hot"] + c["transition_cold"] > 0  # rows actually moved dirty
+    r["fr"].close()
+    s0 = run_parity(st, check_dedup=False)
+    assert np.array_equal(s0["w"], r["w"])
+    s0["fr"].close()
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_dynamic_cache_random_sets(seed):
+    """Random hot sets (any turnover, growing and shrinking) at random epoch lengths > L."""
+    rng = np.random.default_rng(900 + seed)
+    L = int(rng.choice([2, 3, 5]))
+    D = int(rng.choice([1, L, 2 * L]))
+    cfg = tiny1(batch=48, lookahead=L, age_out=D, cache_ratio=0.05, seed_ids=seed + 11)
+    st = W.gen_stream(cfg, 40)
+    E = int(rng.integers(L + 1, L + 5))
+    sched = []
+    for t0 in range(E, st.steps, E):
+        k = int(rng.integers(100, 600))  # <= the 625 slots (500 + 25%)
+        sched.append((t0, np.sort(rng.choice(cfg.n_rows, size=k, replace=False)).astype(np.int64)))
+    r = run_parity(dataclasses.replace(st, hot_schedule=sched))
+    assert r["exact"]
+    r["fr"].close()
+
+
+def test_dynamic_cache_capacity_and_order_errors():
+    F = _F()
+    from paper_conf_asplos_xiezggl25_b200.harness import make_context
+    cfg = tiny1(lookahead=3)
+    st = W.gen_stream(cfg, 10)
+    fr = make_context(st)  # static cache: set_hot is refused
+    with pytest.raises(F.FrugalError):
+        fr.set_hot(5, st.hot)
+    fr.close()
+    fr = make_context(st, flags=F.F_DYNAMIC_CACHE)
+    with pytest.raises(F.FrugalError):  # far more rows than slots
+        fr.set_hot(5, np.arange(cfg.n_rows))
+    fr.set_hot(5, st.hot)
+    with pytest.raises(F.FrugalError):  # one change already pending
+        fr.set_hot(9, st.hot)
+    fr.close()

@@ -13,7 +13,7 @@ from paper_conf_asplos_xiezggl25_b200 import workload as W
 from paper_conf_asplos_xiezggl25_b200.harness import make_context
 
 SLEEP = float(os.environ.get("TL_SLEEP", "0"))
-cfg = W.config("criteo_kaggle", world=1)
+cfg = W.config("criteo_kaggle", world=1, **({"opt": os.environ["TL_OPT"], "lr": 1.0} if os.environ.get("TL_OPT") else {}))
 S, L = int(os.environ.get("TL_STEPS", "60")), cfg.lookahead
 st = W.gen_stream(cfg, S + L + 2)
 fr = make_context(st, flags=F.F_TIMERS)
