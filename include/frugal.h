@@ -152,8 +152,11 @@ frugal_status frugal_backward_update(frugal_ctx* ctx, int64_t s, const float* d_
    one change may be pending.  At the start of frugal_step(t0) the owner flushes every row
    whose hotness changes and whose host copy is not current (the transition set, on the
    critical path, like the urgent bucket), then evicts and admits rows.  Results (tables,
-   losses) do not depend on the hot sets.  FRUGAL_EINVAL: the owned share exceeds the slot
-   capacity (1.25x the initial share + 64); FRUGAL_ESTATE: too late / one already pending. */
+   losses) do not depend on the hot sets.  hot_ids is copied to the device asynchronously
+   (duplicates are ignored): a pageable buffer may be reused on return, a pinned one once
+   frugal_step(t0) has returned.  Ids are validated on the device: an id >= n_rows, or an
+   owned share beyond the slot capacity (1.25x the initial share + 64), fails the next call
+   with FRUGAL_EINVAL.  FRUGAL_ESTATE: too late, or a change is already pending. */
 frugal_status frugal_set_hot(frugal_ctx* ctx, int64_t t0, const int64_t* hot_ids, int64_t n_hot);
 
 /* End of training (L1082-1083): every dirty owned row (w and G) and the G of every

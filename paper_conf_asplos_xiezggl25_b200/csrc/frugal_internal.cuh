@@ -139,14 +139,15 @@ struct frugal_ctx {
     // boundaries t0; cap_slots >= cap_hot leaves room for the owned share to grow
     bool dyn = false;
     int64_t cap_slots = 0;
-    uint8_t* hot_map[2] = {nullptr, nullptr};  // [No] hotness used by the ingest of a step
+    uint32_t* hot_map[2] = {nullptr, nullptr}; // [(No+31)/32] hot bits used by the ingest of a step
     int hot_cur = 0;                           // map of the epoch in force
     bool hot_pending = false;                  // a frugal_set_hot waits for its t0
     int64_t hot_t0 = -1;                       // first step of the pending epoch
     int32_t* new_lk = nullptr;                 // [cap_slots] owned share of the pending hot set
-    int64_t n_new = 0;
+    int64_t* hot_stage = nullptr;              // device copy of the ids passed to frugal_set_hot
+    int64_t hot_stage_cap = 0;
     int32_t* free_slots = nullptr;             // [cap_slots] stack of free slots
-    int32_t* tr_cnt = nullptr;                 // [2]: free-stack size, transition-list size
+    int32_t* tr_cnt = nullptr;                 // [3]: free-stack size, transition-list size, |new_lk|
     int32_t* tr_rows = nullptr;                // [capT + cap_slots] rows flushed by the transition
     cudaEvent_t ev_hot = nullptr;              // pending map / list uploaded
     std::vector<int32_t> rec_transition;
@@ -244,7 +245,8 @@ void launch_convert_ids(frugal_ctx* c, QueueSlot& q, cudaStream_t st);
 void launch_dedup(frugal_ctx* c, QueueSlot& q, cudaStream_t st);
 void launch_owner_side(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st);
 void launch_cache_transition(frugal_ctx* c, int64_t s, int par, cudaStream_t st);
-void launch_hot_map(frugal_ctx* c, int which, const int32_t* lks, int64_t n, cudaStream_t st);
+void launch_hot_map(frugal_ctx* c, int which, const int64_t* ids64, const int32_t* lks, int64_t n, bool list,
+                    cudaStream_t st);
 void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, int32_t* adj_rows, int32_t* adj_p,
                         int32_t* adj_cnt, cudaStream_t st);
 void launch_schedule(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStream_t st);

@@ -504,7 +504,7 @@ __device__ __forceinline__ void nb_append(int32_t* rows, int32_t* ps, int32_t* c
 // a1: set read-ring bits of step t for the owned rows read at t; AdjustPriority inf -> t
 __global__ void k_ingest_bits(const int32_t* __restrict__ T, const uint32_t* __restrict__ Tmask,
                               const int32_t* d_nT, int world, int g, int bit, int32_t t, int adjust,
-                              const int32_t* __restrict__ slot, const uint8_t* __restrict__ hmap,
+                              const int32_t* __restrict__ slot, const uint32_t* __restrict__ hmap,
                               uint64_t* __restrict__ rbits,
                               int32_t* __restrict__ state, int32_t* nb_rows, int32_t* nb_p, int32_t* nb_cnt) {
     int n = *d_nT;
@@ -518,7 +518,7 @@ __global__ void k_ingest_bits(const int32_t* __restrict__ T, const uint32_t* __r
             uint32_t mask = (world > 1) ? Tmask[j] : 1u;
             // host-reader (R7): any other rank, or the owner itself when the row is not
             // hot at step t (hmap: the hot set of t's epoch, N3; else the static cache)
-            const bool hot = hmap ? hmap[lk] != 0 : slot[lk] >= 0;
+            const bool hot = hmap ? ((hmap[lk >> 5] >> (lk & 31)) & 1u) != 0u : slot[lk] >= 0;
             bool host = (mask & ~(1u << g)) != 0u || !hot;
             uint64_t b = (1ull << bit) | (host ? (1ull << (32 + bit)) : 0ull);
             atomicOr((unsigned long long*)&rbits[lk], (unsigned long long)b);  // races with k_optimizer's clear
@@ -609,7 +609,7 @@ __global__ void k_schedule(const int32_t* __restrict__ T, const int32_t* d_nT, c
 
 void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, int32_t* adj_rows, int32_t* adj_p,
                         int32_t* adj_cnt, cudaStream_t st) {
-    const uint8_t* hmap = nullptr;
+    const uint32_t* hmap = nullptr;
     if (c->dyn) hmap = c->hot_map[(c->hot_pending && t >= c->hot_t0) ? (c->hot_cur ^ 1) : c->hot_cur];
     k_ingest_bits<<<grid_for(c->capT, 256), 256, 0, st>>>(q.T, q.Tmask, q.nT, c->n, c->g, (int)(t & 31), (int32_t)t,
                                                            adjust, c->slot, hmap, c->rbits, c->state, adj_rows, adj_p,
@@ -636,6 +636,9 @@ void launch_schedule(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStr
 // but not yet drained -- is flushed now (the transition set X(t0)) and marked clean; then
 // evicted rows release their slots and admitted rows take free slots, loaded from the pool
 // (recently updated) or the host table.  G never moves (HBM-resident for every owned row).
+__device__ __forceinline__ bool hot_bit(const uint32_t* __restrict__ m, int32_t lk) {
+    return ((m[lk >> 5] >> (lk & 31)) & 1u) != 0u;
+}
 __device__ __forceinline__ void tr_append(int32_t* xl, int32_t* xcnt, bool pred, int32_t lk) {
     const unsigned m = __ballot_sync(__activemask(), pred);
     if (!pred) return;
@@ -647,25 +650,25 @@ __device__ __forceinline__ void tr_append(int32_t* xl, int32_t* xcnt, bool pred,
 }
 // (1) pending AdjustPriority entries of t0 whose row changes hotness: into X, cancelled
 __global__ void k_tr_adjust(int32_t* __restrict__ adj_rows, const int32_t* adj_cnt, const int32_t* __restrict__ slot,
-                            const uint8_t* __restrict__ hnew, int32_t* xl, int32_t* xcnt) {
+                            const uint32_t* __restrict__ hnew, int32_t* xl, int32_t* xcnt) {
     const int n = *adj_cnt;
     for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
         const int32_t lk = adj_rows[i];
-        const bool x = lk >= 0 && ((slot[lk] >= 0) != (hnew[lk] != 0));
+        const bool x = lk >= 0 && ((slot[lk] >= 0) != hot_bit(hnew, lk));
         if (x) adj_rows[i] = -1;
         tr_append(xl, xcnt, x, lk);
     }
 }
 // (2) dirty rows among the evicted (old slots not in the new set) and the admitted
 __global__ void k_tr_dirty(const int32_t* __restrict__ hot_lk, int64_t cap_slots, const int32_t* __restrict__ new_lk,
-                           int64_t n_new, const int32_t* __restrict__ slot, const uint8_t* __restrict__ hnew,
+                           const int32_t* d_nnew, const int32_t* __restrict__ slot, const uint32_t* __restrict__ hnew,
                            int32_t* __restrict__ state, int32_t* xl, int32_t* xcnt) {
-    const int64_t n = cap_slots + n_new;
+    const int64_t n = cap_slots + min((int64_t)*d_nnew, cap_slots);
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         int32_t lk = -1;
         if (i < cap_slots) {
             lk = hot_lk[i];
-            if (lk >= 0 && hnew[lk]) lk = -1;  // stays hot
+            if (lk >= 0 && hot_bit(hnew, lk)) lk = -1;  // stays hot
         } else {
             lk = new_lk[i - cap_slots];
             if (slot[lk] >= 0) lk = -1;  // already hot
@@ -677,12 +680,12 @@ __global__ void k_tr_dirty(const int32_t* __restrict__ hot_lk, int64_t cap_slots
 }
 // (3) evict: release the slot; no pool copy of the row is live any more (its value is on
 // the host), so the gather and the flushes read it from the host table
-__global__ void k_tr_evict(int32_t* __restrict__ hot_lk, int64_t cap_slots, const uint8_t* __restrict__ hnew,
+__global__ void k_tr_evict(int32_t* __restrict__ hot_lk, int64_t cap_slots, const uint32_t* __restrict__ hnew,
                            int32_t* __restrict__ slot, int32_t* __restrict__ last_upd, int32_t* free_slots,
                            int32_t* nfree) {
     for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < cap_slots; j += (int64_t)gridDim.x * blockDim.x) {
         const int32_t lk = hot_lk[j];
-        if (lk < 0 || hnew[lk]) continue;
+        if (lk < 0 || hot_bit(hnew, lk)) continue;
         slot[lk] = -1;
         last_upd[lk] = -1;
         hot_lk[j] = -1;
@@ -692,7 +695,7 @@ __global__ void k_tr_evict(int32_t* __restrict__ hot_lk, int64_t cap_slots, cons
 // (4) admit: take a free slot, load the current value (pool when updated within the
 // window, else the host table -- current: X flushed every dirty admitted row)
 template <int GS>
-__global__ void k_tr_admit(const int32_t* __restrict__ new_lk, int64_t n_new, int world, int g, int d4,
+__global__ void k_tr_admit(const int32_t* __restrict__ new_lk, const int32_t* d_nnew, int64_t cap, int world, int g, int d4,
                            int32_t* __restrict__ slot, int32_t* __restrict__ hot_lk, const int32_t* __restrict__ free_slots,
                            int32_t* nfree, const int32_t* __restrict__ last_upd, const int32_t* __restrict__ pool_idx,
                            const float4* __restrict__ pw, int P, int64_t capT, int32_t pool_min, const float4* hw,
@@ -700,6 +703,7 @@ __global__ void k_tr_admit(const int32_t* __restrict__ new_lk, int64_t n_new, in
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
+    const int64_t n_new = min((int64_t)*d_nnew, cap);
     for (int64_t i = gid; i < n_new; i += gs) {
         const int32_t lk = new_lk[i];
         if (slot[lk] >= 0) continue;
@@ -724,13 +728,40 @@ __global__ void k_tr_admit(const int32_t* __restrict__ new_lk, int64_t n_new, in
         }
     }
 }
-__global__ void k_hot_map(uint8_t* __restrict__ map, const int32_t* __restrict__ lks, int64_t n) {
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-        map[lks[i]] = 1;
+// hot bit array of an epoch from a hot set: global ids (ids64, validated, foreign ones
+// skipped) or owned local ids (lks); the distinct owned rows are appended to new_lk
+__global__ void k_hot_build(uint32_t* __restrict__ map, const int64_t* __restrict__ ids64,
+                            const int32_t* __restrict__ lks, int64_t n, int64_t N, int world, int g,
+                            int32_t* __restrict__ new_lk, int32_t* d_nnew, int64_t cap, int32_t* err) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        int32_t lk;
+        if (ids64) {
+            const int64_t k = ids64[i];
+            if (k < 0 || k >= N) {
+                atomicExch(err, 1);
+                continue;
+            }
+            if (k % world != g) continue;
+            lk = (int32_t)(k / world);
+        } else {
+            lk = lks[i];
+        }
+        const uint32_t bit = 1u << (lk & 31);
+        if (atomicOr(&map[lk >> 5], bit) & bit) continue;  // duplicate
+        if (!new_lk) continue;
+        const int at = atomicAdd(d_nnew, 1);
+        if (at < cap) new_lk[at] = lk;
+        else atomicExch(err, 3);
+    }
 }
-void launch_hot_map(frugal_ctx* c, int which, const int32_t* lks, int64_t n, cudaStream_t st) {
-    cudaMemsetAsync(c->hot_map[which], 0, (size_t)c->No, st);
-    if (n > 0) k_hot_map<<<grid_for(n, 256, 4), 256, 0, st>>>(c->hot_map[which], lks, n);
+void launch_hot_map(frugal_ctx* c, int which, const int64_t* ids64, const int32_t* lks, int64_t n, bool list,
+                    cudaStream_t st) {
+    cudaMemsetAsync(c->hot_map[which], 0, (size_t)((c->No + 31) / 32) * 4, st);
+    if (list) cudaMemsetAsync(c->tr_cnt + 2, 0, 4, st);
+    if (n > 0)
+        k_hot_build<<<grid_for(n, 256, 4), 256, 0, st>>>(c->hot_map[which], ids64, lks, n, c->N, c->n, c->g,
+                                                          list ? c->new_lk : nullptr, c->tr_cnt + 2, c->cap_slots,
+                                                          c->err);
     c->launches++;
 }
 
@@ -738,21 +769,21 @@ void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begi
                        int max_blocks, int counter, cudaStream_t st);
 
 void launch_cache_transition(frugal_ctx* c, int64_t s, int par, cudaStream_t st) {
-    const uint8_t* hnew = c->hot_map[c->hot_cur ^ 1];
+    const uint32_t* hnew = c->hot_map[c->hot_cur ^ 1];
     int32_t* xcnt = c->tr_cnt + 1;
     cudaMemsetAsync(xcnt, 0, 4, st);
     k_tr_adjust<<<grid_for(c->capT, 256, 4), 256, 0, st>>>(c->adj_rows[par], c->adj_cnt[par], c->slot, hnew,
                                                             c->tr_rows, xcnt);
-    k_tr_dirty<<<grid_for(c->cap_slots + c->n_new, 256, 4), 256, 0, st>>>(c->hot_lk, c->cap_slots, c->new_lk, c->n_new,
-                                                                          c->slot, hnew, c->state, c->tr_rows, xcnt);
+    k_tr_dirty<<<grid_for(2 * c->cap_slots, 256, 4), 256, 0, st>>>(c->hot_lk, c->cap_slots, c->new_lk, c->tr_cnt + 2,
+                                                                   c->slot, hnew, c->state, c->tr_rows, xcnt);
     launch_flush_rows(c, c->tr_rows, nullptr, xcnt, 1 << 30, FRUGAL_C_TRANSITION_HOT, st);
     k_tr_evict<<<grid_for(c->cap_slots, 256, 4), 256, 0, st>>>(c->hot_lk, c->cap_slots, hnew, c->slot, c->last_upd,
                                                                 c->free_slots, c->tr_cnt);
     const int d4 = c->d / 4, gs = group_size(d4);
     // no optimizer runs concurrently with the transition: segment u % P is intact for u >= s-P+1
     const int32_t pool_min = (int32_t)std::max<int64_t>(0, s - c->P + 1);
-    DISPATCH_GS(gs, (k_tr_admit<GS><<<grid_for(std::max<int64_t>(1, c->n_new) * gs, 256, 8), 256, 0, st>>>(
-                        c->new_lk, c->n_new, c->n, c->g, d4, c->slot, c->hot_lk, c->free_slots, c->tr_cnt,
+    DISPATCH_GS(gs, (k_tr_admit<GS><<<grid_for(c->cap_slots * gs, 256, 8), 256, 0, st>>>(
+                        c->new_lk, c->tr_cnt + 2, c->cap_slots, c->n, c->g, d4, c->slot, c->hot_lk, c->free_slots, c->tr_cnt,
                         c->last_upd, c->pool_idx, (const float4*)c->pw, c->P, c->capT, pool_min,
                         (const float4*)c->dh_w, (float4*)c->cw, c->err)));
     c->launches += 4;

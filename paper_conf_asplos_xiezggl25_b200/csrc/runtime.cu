@@ -162,7 +162,7 @@ static void free_ctx(frugal_ctx* c) {
     };
     F(c->slot); F(c->state); F(c->last_upd); F(c->pool_idx); F(c->rbits);
     F(c->cw); F(c->Gd); F(c->hot_lk); F(c->pw); F(c->pkey); F(c->pcount);
-    F(c->hot_map[0]); F(c->hot_map[1]); F(c->new_lk); F(c->free_slots); F(c->tr_cnt); F(c->tr_rows);
+    F(c->hot_map[0]); F(c->hot_map[1]); F(c->new_lk); F(c->free_slots); F(c->tr_cnt); F(c->tr_rows); F(c->hot_stage);
     for (auto& q : c->q) {
         F(q.eidx); F(q.lidx); F(q.elcnt);
         F(q.ids); F(q.counts); F(q.m); F(q.uniq); F(q.inv); F(q.off); F(q.pos); F(q.n_uniq);
@@ -437,11 +437,11 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     DMALLOC(c->hot_lk, c->cap_slots * 4);
     DMALLOC(c->cw, c->cap_slots * rowb);
     if (c->dyn) {
-        DMALLOC(c->hot_map[0], c->No);
-        DMALLOC(c->hot_map[1], c->No);
+        DMALLOC(c->hot_map[0], (size_t)((c->No + 31) / 32) * 4);
+        DMALLOC(c->hot_map[1], (size_t)((c->No + 31) / 32) * 4);
         DMALLOC(c->new_lk, c->cap_slots * 4);
         DMALLOC(c->free_slots, c->cap_slots * 4);
-        DMALLOC(c->tr_cnt, 8);
+        DMALLOC(c->tr_cnt, 12);
         DMALLOC(c->tr_rows, ((size_t)c->capT + 2 * c->cap_slots) * 4);
     }
     if (adag) DMALLOC(c->Gd, (size_t)c->No * rowb);
@@ -548,9 +548,9 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     if (c->dyn) {
         std::vector<int32_t> fr;
         for (int64_t j = c->cap_slots - 1; j >= c->cap_hot; j--) fr.push_back((int32_t)j);
-        const int32_t cnt2[2] = {(int32_t)fr.size(), 0};
+        const int32_t cnt3[3] = {(int32_t)fr.size(), 0, 0};
         cudaMemcpy(c->free_slots, fr.data(), fr.size() * 4, cudaMemcpyHostToDevice);
-        cudaMemcpy(c->tr_cnt, cnt2, 8, cudaMemcpyHostToDevice);
+        cudaMemcpy(c->tr_cnt, cnt3, 12, cudaMemcpyHostToDevice);
         CK(cudaEventCreateWithFlags(&c->ev_hot, cudaEventDisableTiming));
     }
     if (cudaMemcpy(c->hot_lk, hot.data(), hot.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) {
@@ -559,7 +559,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         return FRUGAL_ECUDA;
     }
     launch_init_meta(c, nullptr, 0, st);
-    if (c->dyn) launch_hot_map(c, 0, c->hot_lk, c->cap_hot, st);
+    if (c->dyn) launch_hot_map(c, 0, nullptr, c->hot_lk, c->cap_hot, false, st);
     cudaMemset(c->pcount, 0, (size_t)c->P * 4);
     cudaMemset(c->pkey, 0xff, (size_t)c->P * c->capT * 4);
     if (c->g == 0 || !k.shm_name) {
@@ -1144,25 +1144,27 @@ extern "C" frugal_status frugal_set_hot(frugal_ctx* c, int64_t t0, const int64_t
                 (long long)c->next_prefetch);
         return FRUGAL_ESTATE;
     }
-    std::vector<int32_t> own;
-    for (int64_t i = 0; i < n_hot; i++) {
-        if (hot_ids[i] < 0 || hot_ids[i] >= c->N) { set_err("hot id out of range"); return FRUGAL_EINVAL; }
-        if (hot_ids[i] % c->n == c->g) own.push_back((int32_t)(hot_ids[i] / c->n));
+    cudaStream_t is = c->istream;
+    if (n_hot > c->hot_stage_cap) {  // rare: grow the device staging of the id list
+        CK(cudaStreamSynchronize(is));
+        if (c->hot_stage) cudaFree(c->hot_stage);
+        c->hot_stage = nullptr;
+        c->hot_stage_cap = 0;
+        if (cudaMalloc(&c->hot_stage, (size_t)n_hot * 8) != cudaSuccess) {
+            cudaGetLastError();
+            set_err("set_hot: staging allocation failed");
+            return FRUGAL_ENOMEM;
+        }
+        c->hot_stage_cap = n_hot;
     }
-    std::sort(own.begin(), own.end());
-    own.erase(std::unique(own.begin(), own.end()), own.end());
-    if ((int64_t)own.size() > c->cap_slots) {
-        set_err("set_hot: owned share %zu exceeds the %lld cache slots", own.size(), (long long)c->cap_slots);
-        return FRUGAL_EINVAL;
-    }
-    // the map of the previous epoch is free: every ingest that read it precedes this on the
-    // in-order ingest stream; the pinned staging keeps the upload asynchronous
-    CK(cudaStreamSynchronize(c->istream));
-    CK(cudaEventSynchronize(c->ev_hot));  // the previous transition has read new_lk
-    if (!own.empty()) CK(cudaMemcpy(c->new_lk, own.data(), own.size() * 4, cudaMemcpyHostToDevice));
-    c->n_new = (int64_t)own.size();
-    launch_hot_map(c, c->hot_cur ^ 1, c->new_lk, c->n_new, c->istream);
-    CK(cudaEventRecord(c->ev_hot, c->istream));
+    // everything on the ingest stream, in order after every ingest that read the other map,
+    // and after the previous transition (it read new_lk); ids are validated and filtered to
+    // the owned share on the device (an id >= n_rows or a share beyond the slots fails the
+    // next call)
+    CK(cudaStreamWaitEvent(is, c->ev_hot, 0));
+    if (n_hot) CK(cudaMemcpyAsync(c->hot_stage, hot_ids, (size_t)n_hot * 8, cudaMemcpyDefault, is));
+    launch_hot_map(c, c->hot_cur ^ 1, c->hot_stage, nullptr, n_hot, true, is);
+    CK(cudaEventRecord(c->ev_hot, is));
     CKL();
     c->hot_t0 = t0;
     c->hot_pending = true;

@@ -322,7 +322,7 @@ def test_dynamic_cache_random_sets(seed):
 
 def test_dynamic_cache_capacity_and_order_errors():
     F = _F()
-    from paper_conf_asplos_xiezggl25_b200.harness import make_context
+    from paper_conf_asplos_xiezggl25_b200.harness import Trainer, make_context
     cfg = tiny1(lookahead=3)
     st = W.gen_stream(cfg, 10)
     fr = make_context(st)  # static cache: set_hot is refused
@@ -330,9 +330,14 @@ def test_dynamic_cache_capacity_and_order_errors():
         fr.set_hot(5, st.hot)
     fr.close()
     fr = make_context(st, flags=F.F_DYNAMIC_CACHE)
-    with pytest.raises(F.FrugalError):  # far more rows than slots
-        fr.set_hot(5, np.arange(cfg.n_rows))
     fr.set_hot(5, st.hot)
     with pytest.raises(F.FrugalError):  # one change already pending
         fr.set_hot(9, st.hot)
+    fr.close()
+    # far more rows than slots: detected on the device, reported by a following call
+    big = dataclasses.replace(st, hot_schedule=[(5, np.arange(cfg.n_rows))])
+    fr = make_context(big)
+    tr = Trainer(fr, big)
+    with pytest.raises(F.FrugalError, match="slots"):
+        tr.run()
     fr.close()
