@@ -57,6 +57,9 @@ def parse():
     ap.add_argument("--peer", action="store_true",
                     help="N4 NVLink-native variant: non-owned rows held in the owner's HBM are loaded "
                          "over peer memory instead of from the host table (N > 1)")
+    ap.add_argument("--cache-refresh", type=int, default=0,
+                    help="N3 dynamic cache: recompute the hot set every E steps (LFU over the previous E "
+                         "steps, per-table top cache_ratio); 0 = static hot set")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for barriers / the max-over-ranks timing only")
     return ap.parse_args()
@@ -265,8 +268,25 @@ def main():
         sys.exit("--exchange a2a needs N > 1")
     fr = make_context(st, rank=rank, device=local, shm_name=shm,
                       flags=F.F_TIMERS | (F.F_NO_HOST_STATE if no_host_state else 0) | (F.F_A2A if a2a else 0)
-                      | (F.F_PEER if (args.peer and world > 1) else 0),
+                      | (F.F_PEER if (args.peer and world > 1) else 0)
+                      | (F.F_DYNAMIC_CACHE if args.cache_refresh > 0 else 0),
                       mode=F.MODE_WRITE_THROUGH if args.mode == "write_through" else F.MODE_P2F)
+    # N3: the hot set of every epoch start t0 (bench step numbering; step t reads generated
+    # step t % SG), from the E bench steps before t0 -- inputs, computed before any timing,
+    # pinned so that frugal_set_hot copies them asynchronously
+    hot_at = {}
+    E = args.cache_refresh
+    if E > 0:
+        if E <= L:
+            sys.exit("--cache-refresh must exceed the lookahead")
+        for t0 in range(E, S, E):
+            win = np.stack([st.ids[t % SG] for t in range(t0 - E, t0)])
+            cw = np.stack([st.counts[t % SG] for t in range(t0 - E, t0)])
+            hot_at[t0] = torch.from_numpy(W.hot_set(cfg, win, cw, window=E)).pin_memory()
+
+    def set_hot_before_ingest(t):
+        if t in hot_at:
+            fr.set_hot(t, hot_at[t].numpy())
     barrier()
     stream = torch.cuda.current_stream(dev)
 
@@ -285,6 +305,7 @@ def main():
     counts = st.counts
 
     for t in range(L):
+        set_hot_before_ingest(t)
         fr.prefetch(t, ids_d[t % SG], counts[t % SG])
 
     kg = cfg.model == "transe"
@@ -329,6 +350,7 @@ def main():
 
     def step_dev(s):
         t = s + L
+        set_hot_before_ingest(t)
         fr.step(s, ids_d[t % SG], counts[t % SG])
         lookup(s)
         if kg:
@@ -354,6 +376,7 @@ def main():
     def step_e2e(s):
         t = s + L
         b = s & 1
+        set_hot_before_ingest(t)
         fr.step(s, ids_h[t % SG], counts[t % SG])  # ids copied from pinned host inside the call
         load_xy(s + 1)
         lookup(s)
@@ -493,7 +516,9 @@ def main():
                                                len(st.hot) * r / 1e6, SG, st.ids.nbytes / 1e6),
                    "hot_set": "top cache_ratio of each table by frequency over the %d generated steps before "
                               "the bench's first step (never over timed steps)" % HOT_WINDOW,
-                   "host_state": "w only (G HBM-resident, no host copy)" if no_host_state else "w (+G at final flush)"},
+                   "host_state": "w only (G HBM-resident, no host copy)" if no_host_state else "w (+G at final flush)",
+                   "cache": ("dynamic (N3): hot set recomputed every %d steps, per-table top cache_ratio by "
+                             "frequency over the previous %d steps" % (E, E)) if E > 0 else "static"},
         "e2e": {"value": e2e, "unit": "samples/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": 8},
         "gpu_launches": int(launches),
         "roofline": roofline,
