@@ -467,6 +467,13 @@ def main():
     per["optimizer"] = dict(bound="hbm", bytes=touched * (5 * r + 28) / K,
                             link_bytes=(cnt["opt_cold"] * r + cnt["mail_in"] * r) / K if world > 1 else 0.0,
                             ms=ph["optimizer"], peak=hbm_peak)
+    if world == 1 and ph["optimizer"] == 0.0 and ph["segred"] > 0.0:
+        # world 1: the optimizer is fused into the segment-reduce (one pass, no partials buffer):
+        # per position r + 4 B (grad row, pos); per touched row w r, G r + r, w out r, 28 B metadata
+        per["segred"] = dict(bound="hbm", kernel="k_segreduce / k_segred_combine (a6 + a8 fused)",
+                             bytes=(cnt["positions"] * (r + 4) + touched * (4 * r + 28)) / K,
+                             ms=ph["segred"], peak=hbm_peak)
+        per["optimizer"]["bytes"] = 0.0
     # a5 glue: read r per position (embeddings, register-cached), write r (grads), x per sample
     per["model"] = dict(bound="hbm", bytes=(cnt["positions"] * 2 * r + B * (r + 4)) / K, ms=ph["model"],
                         peak=hbm_peak)

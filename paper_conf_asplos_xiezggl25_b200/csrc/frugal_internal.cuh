@@ -99,7 +99,8 @@ struct frugal_ctx {
     int64_t N, No;               // rows, owned rows
     int P;                       // pool segments = D + 3
     int QN;                      // sample-queue slots = L + 2 (steps s-1 .. s+L)
-    int side_blocks = 32;        // grid cap of the side-stream drain
+    int side_blocks = 20;        // grid cap of the side-stream drain: its zero-copy D2H stores slow the concurrent backward kernels, 16-24 CTAs balance the two (profiles/r1_sweep15.txt)
+    bool fuse_opt = true;        // world 1: a8 fused into a6 (k_segreduce / k_segred_combine)
     int gather_blocks = 74;      // grid cap of the zero-copy gathers (74 CTAs fill the link: profiles/r1_zc_probe_async.txt)
     bool side_inline = false;    // experiment: drain on the caller stream
     bool drain_after_gather = true;  // side drain after the step's gather (FRUGAL_DRAIN_AT=sched: after the scheduler)
@@ -262,7 +263,7 @@ void launch_transe_model(frugal_ctx* c, QueueSlot& q, const float* emb, int C, d
                          double* loss, int64_t nb, double* Wm, double* A, cudaStream_t st);
 void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const float* x, const float* y,
                       float* grad, double* loss, int64_t nb, cudaStream_t st);
-void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, float* dest, cudaStream_t st);
+void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, float* dest, cudaStream_t st, int64_t fused_step = -1);
 void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, const float* recv, const int32_t* roff,
                       cudaStream_t st);
 void launch_a2a_ids(frugal_ctx* c, QueueSlot& q, int32_t* ids, cudaStream_t st);

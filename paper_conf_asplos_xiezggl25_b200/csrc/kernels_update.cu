@@ -14,6 +14,75 @@ __device__ __forceinline__ float4 add4(float4 a, float4 b) {
     return make_float4(__fadd_rn(a.x, b.x), __fadd_rn(a.y, b.y), __fadd_rn(a.z, b.z), __fadd_rn(a.w, b.w));
 }
 
+// a8 elementwise optimizer on one float4 (reading R13; every op rounded separately, R22):
+// Adagrad G += g*g; w -= (lr*g) / (sqrt(G) + eps), or SGD w -= lr*g
+__device__ __forceinline__ void opt4(float4& w, float4& G, const float4& acc, int adagrad, float lr, float eps) {
+    float* wp = &w.x;
+    float* Gp = &G.x;
+    const float* gp = &acc.x;
+#pragma unroll
+    for (int c = 0; c < 4; c++) {
+        if (adagrad) {
+            Gp[c] = __fadd_rn(Gp[c], __fmul_rn(gp[c], gp[c]));
+            float num = __fmul_rn(lr, gp[c]);
+            float den = __fadd_rn(__fsqrt_rn(Gp[c]), eps);
+            wp[c] = __fsub_rn(wp[c], __fdiv_rn(num, den));
+        } else {
+            wp[c] = __fsub_rn(wp[c], __fmul_rn(lr, gp[c]));
+        }
+    }
+}
+
+// World 1: the owner's optimizer fused into the segment-reduce (T(s) == uniq(s), every
+// partial is this rank's own) -- the reduced gradient of unique row j goes straight from
+// registers into the update instead of through a partials buffer and a second kernel.
+struct FusedOpt {
+    int on;  // 0: write partials (world > 1, comparison path)
+    int32_t s;
+    int adagrad;
+    float lr, eps;
+    const int32_t* uniq;
+    const float4* rows_w;  // this step's gathered rows (w of the cold rows)
+    const int32_t* slot;
+    int32_t* state;
+    int32_t* last_upd;
+    int32_t* pool_idx;
+    uint64_t* rbits;
+    float4* cw;
+    float4* Gd;
+    float4* pw;  // pool segment s % P
+    int32_t* pkey;
+    int32_t* pcount;
+};
+
+// row j of the fused update: lane l's columns from sum(v), then the row's metadata
+template <int GS, typename SumF>
+__device__ __forceinline__ void fused_update_row(const FusedOpt& fo, int j, int d4, int l, SumF sum, unsigned& nhot,
+                                                 unsigned& ncold) {
+    const int32_t lk = fo.uniq[j];
+    const int sl = fo.slot[lk];
+    for (int v = l; v < d4; v += GS) {
+        const float4 acc = sum(v);
+        float4 w = sl >= 0 ? fo.cw[(int64_t)sl * d4 + v] : fo.rows_w[(int64_t)j * d4 + v];
+        float4 G = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (fo.adagrad) G = fo.Gd[(int64_t)lk * d4 + v];
+        opt4(w, G, acc, fo.adagrad, fo.lr, fo.eps);
+        if (sl >= 0) fo.cw[(int64_t)sl * d4 + v] = w;
+        else fo.pw[(int64_t)j * d4 + v] = w;
+        if (fo.adagrad) fo.Gd[(int64_t)lk * d4 + v] = G;
+    }
+    if (l == 0) {
+        if (sl >= 0) nhot++;
+        else ncold++;
+        fo.state[lk] = ST_UPDATED;
+        fo.last_upd[lk] = fo.s;
+        const uint64_t clear = ~((1ull << (fo.s & 31)) | (1ull << (32 + (fo.s & 31))));
+        atomicAnd((unsigned long long*)&fo.rbits[lk], (unsigned long long)clear);  // races with k_ingest_bits
+        if (sl < 0) fo.pool_idx[lk] = j;
+        fo.pkey[j] = sl < 0 ? lk : -1;
+    }
+}
+
 // ============================================================================ a6 segment-reduce
 // P[q] = sum over the occurrences of unique row u in the canonical fixed order
 // (reading R23): positions ascending, cut into chunks of kChunk; each chunk summed
@@ -56,11 +125,12 @@ __global__ void __launch_bounds__(256) k_segreduce(const int32_t* __restrict__ o
                             const int32_t* d_nu, const int32_t* __restrict__ gl, const int32_t* __restrict__ goff,
                             int g, int d4, const float4* __restrict__ grad, float4* __restrict__ Pp, float4* mail,
                             int32_t* long_q, int32_t* long_cnt, int2* tasks, int32_t* task_cnt,
-                            unsigned long long* stats) {
+                            unsigned long long* stats, const FusedOpt fo) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
     const int n = *d_nu;
+    unsigned nhot = 0, ncold = 0;
     int own_lo = 0, own_hi = n;
     if (gl) {
         own_lo = goff[g];
@@ -81,12 +151,21 @@ __global__ void __launch_bounds__(256) k_segreduce(const int32_t* __restrict__ o
             }
             continue;
         }
+        if (fo.on) {
+            fused_update_row<GS>(fo, u, d4, l, [&](int v) { return chunk_sum<GS>(grad, pos, b, e, d4, v); }, nhot, ncold);
+            continue;
+        }
         float4* dst = (q >= own_lo && q < own_hi) ? (Pp + q * d4) : (mail + q * d4);
         for (int v = l; v < d4; v += GS) dst[v] = chunk_sum<GS>(grad, pos, b, e, d4, v);
     }
     if (gl) block_fence_system();
     block_count(stats + FRUGAL_C_LONG_SEGMENTS, nlong);
     block_count(stats + FRUGAL_C_MAIL_OUT, nout);
+    if (fo.on) {
+        if (blockIdx.x == 0 && threadIdx.x == 0) *fo.pcount = n;
+        block_count(stats + FRUGAL_C_OPT_HOT, nhot);
+        block_count(stats + FRUGAL_C_OPT_COLD, ncold);
+    }
 }
 
 // Ordered sum of n rows (row(0) first, then row(1), ...) of src, column v, with the row
@@ -162,12 +241,14 @@ __global__ void __launch_bounds__(256) k_segred_combine(const int32_t* __restric
                                                         const int32_t* __restrict__ goff, int g, int d4,
                                                         float4* __restrict__ Pp, float4* mail,
                                                         const int32_t* __restrict__ long_q, const int32_t* long_cnt,
-                                                        const float4* __restrict__ scratch) {
+                                                        const float4* __restrict__ scratch, unsigned long long* stats,
+                                                        const FusedOpt fo) {
     extern __shared__ float4 smem[];
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
     const int nl = *long_cnt;
+    unsigned nhot = 0, ncold = 0;
     int own_lo = 0, own_hi = 0x7fffffff;
     if (gl) {
         own_lo = goff[g];
@@ -180,15 +261,46 @@ __global__ void __launch_bounds__(256) k_segred_combine(const int32_t* __restric
         const int u = gl ? gl[q] : q;
         const int b = off[u], e = off[u + 1];
         const int nch = (e - b + kChunk - 1) / kChunk;
+        if (fo.on) {  // ordered_sum is per-thread with a uniform trip count: every lane calls it
+            fused_update_row<GS>(fo, u, d4, l, [&](int v) {
+                return ordered_sum([&](int c) { return b + c * kChunk; }, nch, scratch, d4, v, smem); }, nhot, ncold);
+            continue;
+        }
         float4* dst = (q >= own_lo && q < own_hi) ? (Pp + (int64_t)q * d4) : (mail + (int64_t)q * d4);
         for (int v = l; v < d4; v += GS)
             dst[v] = ordered_sum([&](int c) { return b + c * kChunk; }, nch, scratch, d4, v, smem);
     }
     if (gl) block_fence_system();
+    if (fo.on) {
+        block_count(stats + FRUGAL_C_OPT_HOT, nhot);
+        block_count(stats + FRUGAL_C_OPT_COLD, ncold);
+    }
 }
 
-void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, float* dest, cudaStream_t st) {
+void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, float* dest, cudaStream_t st,
+                      int64_t fused_step) {
     const int d4 = c->d / 4, gs = group_size(d4);
+    FusedOpt fo{};
+    if (fused_step >= 0) {  // world 1: a6 + a8 in one pass (launch_optimizer is not called)
+        const int seg = (int)(fused_step % c->P);
+        fo.on = 1;
+        fo.s = (int32_t)fused_step;
+        fo.adagrad = c->cfg.opt == FRUGAL_ADAGRAD;
+        fo.lr = c->cfg.lr;
+        fo.eps = c->cfg.eps;
+        fo.uniq = q.uniq;
+        fo.rows_w = (const float4*)c->rows_buf[fused_step & 1];
+        fo.slot = c->slot;
+        fo.state = c->state;
+        fo.last_upd = c->last_upd;
+        fo.pool_idx = c->pool_idx;
+        fo.rbits = c->rbits;
+        fo.cw = (float4*)c->cw;
+        fo.Gd = (float4*)c->Gd;
+        fo.pw = (float4*)c->pw + (size_t)seg * c->capT * d4;
+        fo.pkey = c->pkey + (size_t)seg * c->capT;
+        fo.pcount = c->pcount + seg;
+    }
     int grid = grid_for((int64_t)c->M * gs, 256, 8);
     const bool multi = c->n > 1;
     // dest (comparison path): every partial, own or not, to one device buffer in grouped order
@@ -199,7 +311,7 @@ void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, f
     DISPATCH_GS(gs, (k_segreduce<GS><<<grid, 256, 0, st>>>(q.off, q.pos, q.n_uniq, multi ? q.gl : nullptr, q.goff,
                                                            c->g, d4, (const float4*)grad, (float4*)Pp, mail,
                                                            c->long_q, c->long_cnt, c->long_tasks, c->long_cnt + 1,
-                                                           c->dstats)));
+                                                           c->dstats, fo)));
     static unsigned attr_mask = 0;
     if (!(attr_mask & gs)) {
         DISPATCH_GS(gs, (cudaFuncSetAttribute(k_segred_chunks<GS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -214,7 +326,8 @@ void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, f
     DISPATCH_GS(gs, (k_segred_combine<GS><<<kSMs, 256, kOrderedSmem, st>>>(q.off, multi ? q.gl : nullptr, q.goff, c->g,
                                                                            d4, (float4*)Pp, mail, c->long_q,
                                                                            c->long_cnt,
-                                                                           (const float4*)c->chunk_scratch)));
+                                                                           (const float4*)c->chunk_scratch, c->dstats,
+                                                                           fo)));
     c->launches += 3;
 }
 
@@ -296,20 +409,7 @@ __global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, 
             else if (rows_w) w = rows_w[j * d4 + v];  // world 1: staged by this step's gather
             else w = prow >= 0 ? pw_all[prow * d4 + v] : hw[k * d4 + v];
             if (adagrad) G = Gd[(int64_t)lk * d4 + v];
-            float* wp = &w.x;
-            float* Gp = &G.x;
-            const float* gp = &acc.x;
-#pragma unroll
-            for (int c = 0; c < 4; c++) {
-                if (adagrad) {
-                    Gp[c] = __fadd_rn(Gp[c], __fmul_rn(gp[c], gp[c]));
-                    float num = __fmul_rn(lr, gp[c]);
-                    float den = __fadd_rn(__fsqrt_rn(Gp[c]), eps);
-                    wp[c] = __fsub_rn(wp[c], __fdiv_rn(num, den));
-                } else {
-                    wp[c] = __fsub_rn(wp[c], __fmul_rn(lr, gp[c]));
-                }
-            }
+            opt4(w, G, acc, adagrad, lr, eps);
             if (sl >= 0) cw[(int64_t)sl * d4 + v] = w;
             else pw[j * d4 + v] = w;
             if (adagrad) Gd[(int64_t)lk * d4 + v] = G;

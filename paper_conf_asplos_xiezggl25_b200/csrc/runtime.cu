@@ -328,7 +328,9 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->dyn = (k.flags & FRUGAL_F_DYNAMIC_CACHE) != 0;
     if (c->dyn) c->early = false;
     c->xhost = c->n > 1 && !c->a2a;
-    c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 32;
+    // world 1: optimizer fused into the segment-reduce (FRUGAL_FUSE_OPT=0: two kernels)
+    c->fuse_opt = !(getenv("FRUGAL_FUSE_OPT") && !atoi(getenv("FRUGAL_FUSE_OPT")));
+    c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 20;
     c->gather_blocks = getenv("FRUGAL_GATHER_BLOCKS") ? atoi(getenv("FRUGAL_GATHER_BLOCKS")) : 74;
     c->side_inline = getenv("FRUGAL_SIDE_INLINE") && atoi(getenv("FRUGAL_SIDE_INLINE"));
     c->drain_after_gather = !(getenv("FRUGAL_DRAIN_AT") && !strcmp(getenv("FRUGAL_DRAIN_AT"), "sched"));
@@ -956,7 +958,11 @@ extern "C" frugal_status frugal_backward_update(frugal_ctx* c, int64_t s, const 
     cudaStream_t st = (cudaStream_t)stream;
     QueueSlot& q = c->q[s % c->QN];
     const int par = (int)(s & 1);
-    {
+    if (c->n == 1 && c->fuse_opt) {
+        // world 1: every partial is this rank's own -- segment-reduce and optimizer in one pass
+        Timer tm(c, PH_SEGRED, st);
+        launch_segreduce(c, q, d_grad, par, nullptr, st, s);
+    } else {
         Timer tm(c, PH_SEGRED, st);
         launch_segreduce(c, q, d_grad, par, nullptr, st);
     }
@@ -968,7 +974,7 @@ extern "C" frugal_status frugal_backward_update(frugal_ctx* c, int64_t s, const 
         launch_set_flag(c, FLAG_MAIL, (uint32_t)(s + 1), st);
         launch_wait_flags(c, FLAG_MAIL, (uint32_t)(s + 1), st);
     }
-    {
+    if (!(c->n == 1 && c->fuse_opt)) {
         Timer tm(c, PH_OPT, st);
         launch_optimizer(c, q, s, par, nullptr, nullptr, st);
     }

@@ -218,7 +218,7 @@ def test_call_order_enforced():
 
 @pytest.mark.parametrize("env", [{"FRUGAL_EARLY": "1"}, {"FRUGAL_DRAIN_AT": "sched"},
                                  {"FRUGAL_EARLY": "1", "FRUGAL_DRAIN_AT": "sched"}, {"FRUGAL_SIDE_INLINE": "1"},
-                                 {"FRUGAL_NO_POOL_HITS": "1"}])
+                                 {"FRUGAL_NO_POOL_HITS": "1"}, {"FRUGAL_FUSE_OPT": "0"}])
 def test_pipeline_modes_parity(env):
     """The optional schedules (early gather of the next step, drain after the gather,
     inline drain) keep every artefact bit-exact (run in a subprocess: the knobs are read
