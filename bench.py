@@ -484,13 +484,14 @@ def main():
     dom = max(("gather", "urgent", "expand", "segred", "optimizer", "model"), key=lambda k: per[k]["ms"])
     top = max(main_ms, key=main_ms.get)
     D = per[dom]
-    traffic, tnote = None, None
-    try:  # committed ncu --set full capture (profiles/, tools/ncu_summary.py)
+    traffic, tnote, htraffic = None, None, None
+    try:  # committed ncu --set full capture (profiles/, tools/ncu_summary.py, tools/profile_round.sh)
         prof = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json"))).get(dom, {})
         traffic = prof.get("traffic_bytes_per_launch")
+        htraffic = prof.get("host_link_bytes_per_launch")
         if traffic is not None:
-            tnote = (f"{prof['traffic_kind']} per launch of {prof['kernel']} in profiles/r1_ncu_full_summary.txt "
-                     f"(a warm-up-phase launch; its own algorithmic sysmem bytes: {prof['sysmem_bytes_per_launch']:.0f})")
+            tnote = (f"dram read+write per launch of {prof['kernel']} in profiles/r1_ncu_full_summary.txt (one "
+                     f"steady-state launch, ncu --set full); host_link_traffic = its sysmem sectors through L2")
     except Exception:
         pass
     roofline = {"bound": "hbm" if D["bound"] == "hbm" else "host-link", "kernel": dom,
@@ -498,7 +499,7 @@ def main():
                 "random_row_ceiling": link["random_rows_h2d"] if D["bound"] != "hbm" else None,
                 "frac_of_random_row_ceiling": (D["achieved_gbs"] / link["random_rows_h2d"])
                 if D["bound"] != "hbm" and D["achieved_gbs"] else None,
-                "traffic": traffic, "traffic_note": tnote,
+                "traffic": traffic, "host_link_traffic": htraffic, "traffic_note": tnote,
                 "peak_source": ("measured pinned cudaMemcpy (256 MiB, best of 5) in this run; random 128-B rows "
                                 "measure 12-33 GB/s on this box (profiles/r1_zc_probe_*.txt)" if D["bound"] != "hbm"
                                 else "MEASURED_PEAKS.json hbm_gbs (burst)")}

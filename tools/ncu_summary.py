@@ -2,7 +2,8 @@
 launch the duration, DRAM bytes, PCIe bytes (rate x duration), sysmem sectors, occupancy
 and the top stall reasons; also writes profiles/ncu_traffic.json (per kernel family, the
 mean measured traffic per launch: DRAM bytes for HBM-bound kernels, PCIe bytes for the
-host-link-bound gather/flush) which bench.py reports as roofline.traffic."""
+host-link-bound gather/flush: the sysmem sectors, next to their DRAM bytes) which bench.py
+reports as roofline.traffic / roofline.host_link_traffic."""
 import collections
 import csv
 import json
@@ -52,8 +53,10 @@ def main(raw_csv, out_txt, out_json):
                         "dram_bytes_per_launch": sum(x["dram"] for x in v) / len(v),
                         "pcie_bytes_per_launch": sum(x["pcie"] for x in v) / len(v),
                         "sysmem_bytes_per_launch": sum(x["sys"] for x in v) / len(v),
-                        "traffic_bytes_per_launch": sum((x["pcie"] if host else x["dram"]) for x in v) / len(v),
-                        "traffic_kind": "pcie (read+write)" if host else "dram (read+write)"}
+                        "traffic_bytes_per_launch": sum(x["dram"] for x in v) / len(v),
+                        "traffic_kind": "dram (read+write)",
+                        "host_link_bytes_per_launch": sum(x["sys"] for x in v) / len(v) if host else None,
+                        "host_link_kind": "sysmem sectors through L2 (read+write)" if host else None}
     open(out_txt, "w").write("\n".join(lines) + "\n")
     json.dump(traffic, open(out_json, "w"), indent=1)
     print("\n".join(lines))
