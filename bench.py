@@ -60,6 +60,9 @@ def parse():
     ap.add_argument("--cache-refresh", type=int, default=0,
                     help="N3 dynamic cache: recompute the hot set every E steps (LFU over the previous E "
                          "steps, per-table top cache_ratio); 0 = static hot set")
+    ap.add_argument("--host-layout", default="id", choices=["id", "freq"],
+                    help="host-table layout: id order, or frequency order over the hot-set window "
+                         "(frugal_config.host_order)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for barriers / the max-over-ranks timing only")
     return ap.parse_args()
@@ -150,15 +153,17 @@ def measured_peaks():
         return {}
 
 
-def gen_bench_stream(W, cfg, steps):
+def gen_bench_stream(W, cfg, steps, layout="id"):
     """The seeded stream, minus the hot-set window: the static hot set is computed from the
     first HOT_WINDOW generated steps (reading R10), and the bench then trains on the steps
     AFTER them -- the cache is warmed from past traffic, never from the batches it times
     (timing those would credit the cache with a perfect forecast of its own steps)."""
     import dataclasses
     full = W.gen_stream(cfg, HOT_WINDOW + steps)
+    # host-table layout from the same past window (frequency order, DESIGN.md §7)
+    order = W.host_order(cfg, full.ids[:HOT_WINDOW], full.counts[:HOT_WINDOW]) if layout == "freq" else None
     return dataclasses.replace(full, ids=full.ids[HOT_WINDOW:], counts=full.counts[HOT_WINDOW:],
-                               x=full.x[HOT_WINDOW:], y=full.y[HOT_WINDOW:])
+                               x=full.x[HOT_WINDOW:], y=full.y[HOT_WINDOW:], host_order=order)
 
 
 HOT_WINDOW = 50
@@ -257,7 +262,7 @@ def main():
     # still exceed the 126 MB L2
     SG = min(S, 256)
     t_gen = time.time()
-    st = gen_bench_stream(W, cfg, SG)  # every rank generates the same seeded stream of all ranks
+    st = gen_bench_stream(W, cfg, SG, args.host_layout)  # every rank generates the same seeded stream of all ranks
     t_gen = time.time() - t_gen
     B, Fs, d = cfg.batch, cfg.slots, cfg.dim
     shm = f"/frugal_bench_{os.environ.get('MASTER_PORT', '0')}" if world > 1 else None
@@ -522,6 +527,8 @@ def main():
                    "l2": "inputs larger than L2: host table %.1f GB, HBM cache %.0f MB, %d distinct id batches "
                          "(%.0f MB) cycled" % (cfg.n_rows * r * (1 if (no_host_state or not adag) else 2) / 1e9,
                                                len(st.hot) * r / 1e6, SG, st.ids.nbytes / 1e6),
+                   "host_layout": ("frequency order over the %d generated steps before the bench's first step "
+                                   "(frugal_config.host_order)" % HOT_WINDOW) if args.host_layout == "freq" else "id order",
                    "hot_set": "top cache_ratio of each table by frequency over the %d generated steps before "
                               "the bench's first step (never over timed steps)" % HOT_WINDOW,
                    "host_state": "w only (G HBM-resident, no host copy)" if no_host_state else "w (+G at final flush)",

@@ -101,6 +101,14 @@ typedef struct {
                                private pinned table (world must be 1)                     */
     int32_t mode;           /* frugal_mode                                                 */
     int32_t flags;          /* FRUGAL_F_*                                                  */
+    const int64_t* host_order; /* optional host array of distinct global ids: the host-table
+                               layout.  Row host_order[i] lives in host row slot i; the rows
+                               not listed follow in ascending id.  NULL: slot = id.  Every
+                               rank of a shared table must pass the same list.  A layout
+                               only moves bytes: no result depends on it.  Meant for a
+                               frequency order (random host writes and reads
+                               over a compact footprint run faster on the host link)      */
+    int64_t n_order;
 } frugal_config;
 
 /* Create the context of this rank: validates cfg, maps (and for rank 0 creates and

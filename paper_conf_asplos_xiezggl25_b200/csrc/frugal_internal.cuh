@@ -100,6 +100,8 @@ struct frugal_ctx {
     int P;                       // pool segments = D + 3
     int QN;                      // sample-queue slots = L + 2 (steps s-1 .. s+L)
     int side_blocks = 20;        // grid cap of the side-stream drain: its zero-copy D2H stores slow the concurrent backward kernels, 16-24 CTAs balance the two (profiles/r1_sweep15.txt)
+    int32_t* hs = nullptr;           // [N] host-table slot of every global row (host_order), or null
+    std::vector<int32_t> hs_host;    // host copy (frugal_read_host)
     bool fuse_opt = true;        // world 1: a8 fused into a6 (k_segreduce / k_segred_combine)
     int gather_blocks = 74;      // grid cap of the zero-copy gathers (74 CTAs fill the link: profiles/r1_zc_probe_async.txt)
     bool side_inline = false;    // experiment: drain on the caller stream

@@ -699,7 +699,7 @@ __global__ void k_tr_admit(const int32_t* __restrict__ new_lk, const int32_t* d_
                            int32_t* __restrict__ slot, int32_t* __restrict__ hot_lk, const int32_t* __restrict__ free_slots,
                            int32_t* nfree, const int32_t* __restrict__ last_upd, const int32_t* __restrict__ pool_idx,
                            const float4* __restrict__ pw, int P, int64_t capT, int32_t pool_min, const float4* hw,
-                           float4* __restrict__ cw, int32_t* err) {
+                           const int32_t* __restrict__ hs, float4* __restrict__ cw, int32_t* err) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
@@ -720,7 +720,7 @@ __global__ void k_tr_admit(const int32_t* __restrict__ new_lk, const int32_t* d_
         }
         const int32_t lu = last_upd[lk];
         const float4* src = (lu >= 0 && lu >= pool_min) ? pw + ((int64_t)(lu % P) * capT + pool_idx[lk]) * d4
-                                                         : hw + ((int64_t)lk * world + g) * d4;
+                                                         : hw + host_row(hs, (int64_t)lk * world + g) * d4;
         for (int v = l; v < d4; v += GS) cw[(int64_t)j * d4 + v] = src[v];
         if (l == 0) {
             slot[lk] = j;
@@ -785,7 +785,7 @@ void launch_cache_transition(frugal_ctx* c, int64_t s, int par, cudaStream_t st)
     DISPATCH_GS(gs, (k_tr_admit<GS><<<grid_for(c->cap_slots * gs, 256, 8), 256, 0, st>>>(
                         c->new_lk, c->tr_cnt + 2, c->cap_slots, c->n, c->g, d4, c->slot, c->hot_lk, c->free_slots, c->tr_cnt,
                         c->last_upd, c->pool_idx, (const float4*)c->pw, c->P, c->capT, pool_min,
-                        (const float4*)c->dh_w, (float4*)c->cw, c->err)));
+                        (const float4*)c->dh_w, c->hs, (float4*)c->cw, c->err)));
     c->launches += 4;
 }
 
@@ -799,7 +799,7 @@ __global__ void k_flush_rows(const int32_t* __restrict__ rows, const int32_t* d_
                              int world, int g, int d4, const int32_t* __restrict__ slot,
                              const int32_t* __restrict__ last_upd, const int32_t* __restrict__ pool_idx, int P,
                              int64_t capT, const float4* __restrict__ cw, const float4* __restrict__ pw, float4* hw,
-                             unsigned long long* stats, int sysfence) {
+                             const int32_t* __restrict__ hs, unsigned long long* stats, int sysfence) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
@@ -817,7 +817,8 @@ __global__ void k_flush_rows(const int32_t* __restrict__ rows, const int32_t* d_
             src = pw + ((int64_t)(last_upd[lk] % P) * capT + pool_idx[lk]) * d4;
             nc += (l == 0);
         }
-        for (int v = l; v < d4; v += GS) hw[k * d4 + v] = src[v];
+        float4* dst = hw + host_row(hs, k) * d4;
+        for (int v = l; v < d4; v += GS) dst[v] = src[v];
     }
     if (sysfence) block_fence_system();
     if (stats) {
@@ -832,7 +833,7 @@ void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begi
     int grid = std::min(grid_for(c->capT * (int64_t)gs, 256, 4), max_blocks);
     DISPATCH_GS(gs, (k_flush_rows<GS><<<grid, 256, 0, st>>>(
                         rows, d_begin, d_end, c->n, c->g, d4, c->slot, c->last_upd, c->pool_idx, c->P, c->capT,
-                        (const float4*)c->cw, (const float4*)c->pw, (float4*)c->dh_w,
+                        (const float4*)c->cw, (const float4*)c->pw, (float4*)c->dh_w, c->hs,
                         counter >= 0 ? c->dstats + counter : nullptr, c->n > 1)));
     c->launches++;
 }
@@ -852,7 +853,7 @@ __global__ void k_gather_uniq(const int32_t* __restrict__ uniq, const int32_t* _
                               const int32_t* __restrict__ last_upd, const int32_t* __restrict__ pool_idx,
                               const float4* __restrict__ pw, int P, int64_t capT, int32_t pool_min,
                               const int32_t* __restrict__ gslot, const PeerTab* __restrict__ pt,
-                              unsigned long long* stats) {
+                              const int32_t* __restrict__ hs, unsigned long long* stats) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
@@ -861,7 +862,7 @@ __global__ void k_gather_uniq(const int32_t* __restrict__ uniq, const int32_t* _
     for (int64_t a = gid; a < n; a += gs) {
         const int u = list ? list[a] : (int)a;
         int32_t k = uniq[u];
-        const float4* src = hw + (int64_t)k * d4;
+        const float4* src = nullptr;
         int kind = 0;  // 0 host, 1 cache, 2 pool
         if (k % world == g) {
             const int32_t lk = k / world;
@@ -895,6 +896,7 @@ __global__ void k_gather_uniq(const int32_t* __restrict__ uniq, const int32_t* _
                 }
             }
         }
+        if (kind == 0) src = hw + host_row(hs, k) * d4;
         if (l == 0) {
             nh += kind == 0;
             nc += kind == 1;
@@ -934,7 +936,8 @@ void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32
                                                              (const float4*)c->cw, (const float4*)c->dh_w,
                                                              (float4*)rows, c->last_upd, c->pool_idx,
                                                              c->pool_hits ? (const float4*)c->pw : nullptr, c->P,
-                                                             c->capT, pool_min, c->gslot, c->peer_tab, c->dstats)));
+                                                             c->capT, pool_min, c->gslot, c->peer_tab, c->hs,
+                                                             c->dstats)));
     c->launches++;
 }
 // host-link calibration: n pseudo-random rows of the host table (hash of i and seed) read

@@ -359,7 +359,7 @@ __global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, 
                             float4* __restrict__ pw, int32_t* __restrict__ pkey, int32_t* pcount, const float4* hw,
                             const float4* __restrict__ pw_all, int P, int32_t pool_min,
                             const float4* __restrict__ recv, const int32_t* __restrict__ roff,
-                            unsigned long long* stats) {
+                            const int32_t* __restrict__ hs, unsigned long long* stats) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
@@ -375,6 +375,7 @@ __global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, 
         const int32_t lu = last_upd[lk];
         const int64_t prow = (sl < 0 && !rows_w && lu >= 0 && lu >= pool_min)
                                  ? ((int64_t)(lu % P) * capT + pool_idx[lk]) : -1;
+        const int64_t hrow = (sl < 0 && !rows_w && prow < 0) ? host_row(hs, k) : 0;
         {  // the group's lanes all read `lu` before its lane 0 rewrites last_upd below
             const unsigned gmask = GS == 32 ? 0xffffffffu : (((1u << GS) - 1u) << ((threadIdx.x & 31) & ~(GS - 1)));
             __syncwarp(gmask);
@@ -407,7 +408,7 @@ __global__ void k_optimizer(const int32_t* __restrict__ T, const int32_t* d_nT, 
             float4 w, G = make_float4(0.f, 0.f, 0.f, 0.f);
             if (sl >= 0) w = cw[(int64_t)sl * d4 + v];
             else if (rows_w) w = rows_w[j * d4 + v];  // world 1: staged by this step's gather
-            else w = prow >= 0 ? pw_all[prow * d4 + v] : hw[k * d4 + v];
+            else w = prow >= 0 ? pw_all[prow * d4 + v] : hw[hrow * d4 + v];
             if (adagrad) G = Gd[(int64_t)lk * d4 + v];
             opt4(w, G, acc, adagrad, lr, eps);
             if (sl >= 0) cw[(int64_t)sl * d4 + v] = w;
@@ -449,7 +450,7 @@ void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, const flo
                         c->last_upd, c->pool_idx, c->rbits, (float4*)c->cw, (float4*)c->Gd, (float4*)c->pw + pofs,
                         c->pkey + (size_t)seg * c->capT, c->pcount + seg, (const float4*)c->dh_w,
                         (const float4*)c->pw, c->P, (int32_t)std::max<int64_t>(0, s - c->P + 2),
-                        (const float4*)recv, roff, c->dstats)));
+                        (const float4*)recv, roff, c->hs, c->dstats)));
     c->launches++;
 }
 
@@ -470,13 +471,14 @@ __global__ void k_final_collect(int64_t No, int32_t* __restrict__ state, int32_t
 }
 // G of every owned row (HBM) to the host table, once, at the end of training
 template <int GS>
-__global__ void k_g_push(int64_t No, int world, int g, int d4, const float4* __restrict__ Gd, float4* hG) {
+__global__ void k_g_push(int64_t No, int world, int g, int d4, const float4* __restrict__ Gd, float4* hG,
+                         const int32_t* __restrict__ hs) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
     for (int64_t lk = gid; lk < No; lk += gs) {
-        int64_t k = lk * world + g;
-        for (int v = l; v < d4; v += GS) hG[k * d4 + v] = Gd[lk * d4 + v];
+        const int64_t hk = host_row(hs, lk * world + g);
+        for (int v = l; v < d4; v += GS) hG[hk * d4 + v] = Gd[lk * d4 + v];
     }
     block_fence_system();
 }
@@ -490,7 +492,7 @@ void launch_final_flush(frugal_ctx* c, cudaStream_t st) {
         const int d4 = c->d / 4, gs = group_size(d4);
         int grid = grid_for(c->No * gs, 256, 8);
         DISPATCH_GS(gs, (k_g_push<GS><<<grid, 256, 0, st>>>(c->No, c->n, c->g, d4, (const float4*)c->Gd,
-                                                            (float4*)c->dh_G)));
+                                                            (float4*)c->dh_G, c->hs)));
         c->launches++;
     }
 }
@@ -509,12 +511,14 @@ __device__ __forceinline__ float w0(uint64_t seed, int64_t k, int d, int j, floa
     return __fmul_rn(scale, __fsub_rn(__fmul_rn(2.0f, u), 1.0f));
 }
 
-__global__ void k_init_table(float4* hw, float4* hG, int64_t N, int d, uint64_t seed, float scale, float accum) {
+__global__ void k_init_table(float4* hw, float4* hG, int64_t N, int d, uint64_t seed, float scale, float accum,
+                             const int32_t* __restrict__ hs) {
     const int d4 = d / 4;
     const int64_t total = N * d4;
-    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
-        int64_t k = e / d4;
-        int j = (int)(e - k * d4) * 4;
+    for (int64_t e0 = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e0 < total; e0 += (int64_t)gridDim.x * blockDim.x) {
+        int64_t k = e0 / d4;
+        int j = (int)(e0 - k * d4) * 4;
+        const int64_t e = host_row(hs, k) * d4 + j / 4;  // row k lives in host slot hs[k]
         hw[e] = make_float4(w0(seed, k, d, j, scale), w0(seed, k, d, j + 1, scale), w0(seed, k, d, j + 2, scale),
                             w0(seed, k, d, j + 3, scale));
         if (hG) hG[e] = make_float4(accum, accum, accum, accum);
@@ -522,7 +526,7 @@ __global__ void k_init_table(float4* hw, float4* hG, int64_t N, int d, uint64_t 
 }
 void launch_init_table(frugal_ctx* c, cudaStream_t st) {
     k_init_table<<<kSMs * 8, 256, 0, st>>>((float4*)c->dh_w, (float4*)c->dh_G, c->N, c->d,
-                                           c->cfg.init_seed, c->cfg.init_scale, c->cfg.init_accum);
+                                           c->cfg.init_seed, c->cfg.init_scale, c->cfg.init_accum, c->hs);
     c->launches++;
 }
 
@@ -617,14 +621,14 @@ __global__ void k_serve_rows(const int32_t* __restrict__ ids, int64_t n, int wor
                              const int32_t* __restrict__ slot, const float4* __restrict__ cw, const float4* hw,
                              const int32_t* __restrict__ last_upd, const int32_t* __restrict__ pool_idx,
                              const float4* __restrict__ pw, int P, int64_t capT, int32_t pool_min,
-                             float4* __restrict__ out, unsigned long long* stats) {
+                             const int32_t* __restrict__ hs, float4* __restrict__ out, unsigned long long* stats) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
     unsigned nh = 0, nc = 0, np = 0;
     for (int64_t a = gid; a < n; a += gs) {
         const int32_t k = ids[a], lk = k / world;
-        const float4* src = hw + (int64_t)k * d4;
+        const float4* src = nullptr;
         const int sl = slot[lk];
         int kind = 0;
         if (sl >= 0) {
@@ -637,6 +641,7 @@ __global__ void k_serve_rows(const int32_t* __restrict__ ids, int64_t n, int wor
                 kind = 2;
             }
         }
+        if (kind == 0) src = hw + host_row(hs, k) * d4;
         if (l == 0) {
             nh += kind == 0;
             nc += kind == 1;
@@ -670,7 +675,7 @@ void launch_serve_rows(frugal_ctx* c, const int32_t* ids, int64_t n, int64_t s, 
     const int32_t pool_min = (int32_t)std::max<int64_t>(0, s - c->P + 2);
     DISPATCH_GS(gs, (k_serve_rows<GS><<<grid, 256, 0, st>>>(ids, n, c->n, d4, c->slot, (const float4*)c->cw,
                                                             (const float4*)c->dh_w, c->last_upd, c->pool_idx,
-                                                            (const float4*)c->pw, c->P, c->capT, pool_min,
+                                                            (const float4*)c->pw, c->P, c->capT, pool_min, c->hs,
                                                             (float4*)out, c->dstats)));
     c->launches++;
 }
@@ -686,7 +691,7 @@ void launch_a2a_place(frugal_ctx* c, QueueSlot& q, const float* in, float* rows,
 __global__ void k_read_rows(const int32_t* __restrict__ lks, int64_t n, int world, int g, int d, int P, int64_t capT,
                             const int32_t* slot, const int32_t* state, const int32_t* last_upd,
                             const int32_t* pool_idx, const float* cw, const float* Gd, const float* pw,
-                            const float* hw, float* ow, float* oG) {
+                            const float* hw, const int32_t* __restrict__ hs, float* ow, float* oG) {
     for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < n * d; e += (int64_t)gridDim.x * blockDim.x) {
         int64_t a = e / d;
         int j = (int)(e - a * d);
@@ -700,7 +705,7 @@ __global__ void k_read_rows(const int32_t* __restrict__ lks, int64_t n, int worl
             int64_t pr = (int64_t)(last_upd[lk] % P) * capT + pool_idx[lk];
             w = pw[pr * d + j];
         } else {
-            w = hw[k * d + j];
+            w = hw[host_row(hs, k) * d + j];
         }
         float G = Gd ? Gd[(int64_t)lk * d + j] : 0.f;
         ow[e] = w;
@@ -711,20 +716,21 @@ void launch_read_rows(frugal_ctx* c, const int32_t* d_lk, int64_t n, float* d_w,
     const bool ad = c->cfg.opt == FRUGAL_ADAGRAD;
     k_read_rows<<<grid_for(n * c->d, 256, 8), 256, 0, st>>>(d_lk, n, c->n, c->g, c->d, c->P, c->capT, c->slot,
                                                              c->state, c->last_upd, c->pool_idx, c->cw,
-                                                             ad ? c->Gd : nullptr, c->pw, c->dh_w, d_w, d_G);
+                                                             ad ? c->Gd : nullptr, c->pw, c->dh_w, c->hs, d_w, d_G);
     c->launches++;
 }
 __global__ void k_read_host(const int64_t* __restrict__ ks, int64_t n, int d, const float* hw, const float* hG,
-                            float* ow, float* oG) {
+                            const int32_t* __restrict__ hs, float* ow, float* oG) {
     for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < n * d; e += (int64_t)gridDim.x * blockDim.x) {
         int64_t a = e / d;
         int j = (int)(e - a * d);
-        ow[e] = hw[ks[a] * d + j];
-        oG[e] = hG ? hG[ks[a] * d + j] : 0.f;
+        const int64_t hk = host_row(hs, ks[a]);
+        ow[e] = hw[hk * d + j];
+        oG[e] = hG ? hG[hk * d + j] : 0.f;
     }
 }
 void launch_read_host(frugal_ctx* c, const int64_t* d_k, int64_t n, float* d_w, float* d_G, cudaStream_t st) {
-    k_read_host<<<grid_for(n * c->d, 256, 8), 256, 0, st>>>(d_k, n, c->d, c->dh_w, c->dh_G, d_w, d_G);
+    k_read_host<<<grid_for(n * c->d, 256, 8), 256, 0, st>>>(d_k, n, c->d, c->dh_w, c->dh_G, c->hs, d_w, d_G);
     c->launches++;
 }
 

@@ -62,6 +62,11 @@ __device__ __forceinline__ void block_fence_system() {
     if (threadIdx.x == 0) __threadfence_system();
 }
 
+// host-table row slot of global row k (frugal_config.host_order); hs == nullptr: slot = k
+__device__ __forceinline__ int64_t host_row(const int32_t* __restrict__ hs, int64_t k) {
+    return hs ? (int64_t)hs[k] : k;
+}
+
 static inline int group_size(int d4) {
     int gs = 1;
     while (gs < d4 && gs < 32) gs <<= 1;

@@ -168,7 +168,7 @@ static void free_ctx(frugal_ctx* c) {
         F(q.ids); F(q.counts); F(q.m); F(q.uniq); F(q.inv); F(q.off); F(q.pos); F(q.n_uniq);
         if (c->n > 1) { F(q.T); F(q.Tmask); F(q.Tidx); F(q.nT); F(q.gl); F(q.goff); }
     }
-    F(c->rows_buf[0]); F(c->rows_buf[1]); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->long_tasks); F(c->owned_cnt);
+    F(c->hs); F(c->rows_buf[0]); F(c->rows_buf[1]); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->long_tasks); F(c->owned_cnt);
     for (int i = 0; i < 2; i++) { F(c->adj_rows[i]); F(c->adj_p[i]); F(c->adj_cnt[i]); }
     for (int i = 0; i < 2; i++) { F(c->sl_rows[i]); F(c->sl_p[i]); F(c->sl_cnt[i]); }
     F(c->dstats); F(c->kg_W); F(c->kg_A); F(c->a2a_roff); F(c->peer_tab); F(c->gslot);
@@ -294,6 +294,10 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         return FRUGAL_EINVAL;
     }
     if (k.n_hot < 0 || (k.n_hot > 0 && !k.hot_ids)) { set_err("bad hot set"); return FRUGAL_EINVAL; }
+    if (k.n_order < 0 || k.n_order > k.n_rows || (k.n_order > 0 && !k.host_order)) {
+        set_err("bad host_order");
+        return FRUGAL_EINVAL;
+    }
     for (int64_t i = 0; i < k.n_hot; i++)
         if (k.hot_ids[i] < 0 || k.hot_ids[i] >= k.n_rows) { set_err("hot id out of range"); return FRUGAL_EINVAL; }
     if (cudaSetDevice(k.device) != cudaSuccess) { set_err("cudaSetDevice(%d) failed", k.device); return FRUGAL_ECUDA; }
@@ -303,6 +307,22 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     frugal_ctx* c = new frugal_ctx();
     c->cfg = k;
     c->cfg.hot_ids = nullptr;
+    c->cfg.host_order = nullptr;
+    if (k.n_order > 0) {  // host-table layout: slot of row host_order[i] = i, the rest in id order
+        c->hs_host.assign((size_t)k.n_rows, -1);
+        for (int64_t i = 0; i < k.n_order; i++) {
+            const int64_t id = k.host_order[i];
+            if (id < 0 || id >= k.n_rows || c->hs_host[id] >= 0) {
+                set_err("host_order: id out of range or repeated at %lld", (long long)i);
+                free_ctx(c);
+                return FRUGAL_EINVAL;
+            }
+            c->hs_host[id] = (int32_t)i;
+        }
+        int32_t next = (int32_t)k.n_order;
+        for (auto& v : c->hs_host)
+            if (v < 0) v = next++;
+    }
     c->n = k.world; c->g = k.rank; c->d = k.dim; c->F = k.slots; c->B = k.batch;
     c->L = k.lookahead; c->D = k.age_out; c->M = k.batch * k.slots; c->N = k.n_rows;
     c->No = c->g < c->N ? (c->N - c->g + c->n - 1) / c->n : 0;
@@ -421,6 +441,14 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     cudaHostGetDevicePointer((void**)&c->err, c->herr, 0);
 
     // ---------------------------------------------------------------- device state
+    if (!c->hs_host.empty()) {
+        DMALLOC(c->hs, (size_t)c->N * 4);
+        if (cudaMemcpy(c->hs, c->hs_host.data(), (size_t)c->N * 4, cudaMemcpyHostToDevice) != cudaSuccess) {
+            set_err("host_order upload failed");
+            free_ctx(c);
+            return FRUGAL_ECUDA;
+        }
+    }
     DMALLOC(c->slot, c->No * 4);
     DMALLOC(c->state, c->No * 4);
     DMALLOC(c->last_upd, c->No * 4);
@@ -1227,9 +1255,10 @@ extern "C" frugal_status frugal_read_host(frugal_ctx* c, const int64_t* ids, int
     CK(cudaDeviceSynchronize());
     for (int64_t i = 0; i < n; i++) {
         if (ids[i] < 0 || ids[i] >= c->N) { set_err("read_host: id out of range"); return FRUGAL_EINVAL; }
-        memcpy(w + i * c->d, c->h_w + ids[i] * c->d, c->d * 4);
+        const int64_t hk = c->hs_host.empty() ? ids[i] : c->hs_host[ids[i]];  // host_order layout
+        memcpy(w + i * c->d, c->h_w + hk * c->d, c->d * 4);
         if (G) {
-            if (c->h_G) memcpy(G + i * c->d, c->h_G + ids[i] * c->d, c->d * 4);
+            if (c->h_G) memcpy(G + i * c->d, c->h_G + hk * c->d, c->d * 4);
             else memset(G + i * c->d, 0, c->d * 4);
         }
     }

@@ -23,6 +23,8 @@ def make_context(st, rank=0, device=0, shm_name=None, flags=0, hot=None, mode=F.
               flags=flags)
     if getattr(st, "hot_schedule", None):
         kw["flags"] |= F.F_DYNAMIC_CACHE  # N3: the stream carries hot-set changes
+    if getattr(st, "host_order", None) is not None:
+        kw["host_order"] = st.host_order  # host-table layout (frugal_config.host_order)
     kw.update(over)
     return F.Frugal(**kw)
 

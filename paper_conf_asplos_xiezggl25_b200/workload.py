@@ -217,6 +217,8 @@ class Stream:
     hot: np.ndarray
     # N3 dynamic cache (reading R27): [(t0, hot ids)], the hot set in force from step t0 on
     hot_schedule: list = dataclasses.field(default_factory=list)
+    # host-table layout (frugal_config.host_order): global ids in host-slot order, or None
+    host_order: Optional[np.ndarray] = None
 
     @property
     def steps(self) -> int:
@@ -263,6 +265,20 @@ def hot_set(cfg: WorkloadConfig, ids: np.ndarray, counts: Optional[np.ndarray] =
     if not hot:
         return np.zeros(0, dtype=np.int64)
     return np.sort(np.concatenate(hot)).astype(np.int64)
+
+
+def host_order(cfg: WorkloadConfig, ids: np.ndarray, counts: Optional[np.ndarray] = None) -> np.ndarray:
+    """Host-table layout from past traffic: every row read in `ids` (steps of
+    all ranks), most frequent first, ties by smaller id.  Rows never read are left to the
+    library (they follow in id order).  A layout only moves bytes; no result depends on it."""
+    S, world = ids.shape[0], ids.shape[1]
+    F, B = cfg.slots, ids.shape[2] // cfg.slots
+    sub = ids.reshape(S, world, B, F)
+    if counts is not None:
+        sub = sub[np.arange(B)[None, None, :] < counts[:, :, None]]
+    freq = np.bincount(sub.ravel(), minlength=cfg.n_rows)
+    seen = np.flatnonzero(freq)
+    return seen[np.argsort(-freq[seen], kind="stable")].astype(np.int64)
 
 
 def gen_stream(cfg: WorkloadConfig, steps: int, world: Optional[int] = None,

@@ -82,15 +82,20 @@ def run_two_ranks(st, timeout=600, a2a=False, peer=False):
     return out
 
 
-@pytest.mark.parametrize("opt,a2a,peer,dyn", [("adagrad", False, False, False), ("sgd", False, False, False),
-                                              ("adagrad", True, False, False), ("adagrad", False, True, False),
-                                              ("adagrad", False, False, True)])
-def test_two_ranks_one_gpu_parity(opt, a2a, peer, dyn):
+@pytest.mark.parametrize("opt,a2a,peer,dyn,layout", [("adagrad", False, False, False, False),
+                                                     ("sgd", False, False, False, False),
+                                                     ("adagrad", True, False, False, False),
+                                                     ("adagrad", False, True, False, False),
+                                                     ("adagrad", False, False, True, False),
+                                                     ("adagrad", False, False, False, True)])
+def test_two_ranks_one_gpu_parity(opt, a2a, peer, dyn, layout):
     """a2a=True: the comparison path (§8(e)) -- ids, rows and partials move by all-to-all
     (gloo with host staging here; NCCL over NVLink on a multi-GPU box) instead of the host
     table and mailbox; every artefact and table must be identical.  peer=True: the N4
     variant -- non-owned rows the owner holds in HBM are loaded from the owner's device
-    memory (CUDA IPC; NVLink on a multi-GPU box); every artefact and table identical."""
+    memory (CUDA IPC; NVLink on a multi-GPU box); every artefact and table identical.
+    layout=True: both ranks share a host table laid out by a random partial host_order
+    (frugal_config.host_order); every artefact and table identical."""
     from oracle.oracle import Oracle
     cfg = W.config("tiny", world=2, batch=64, lookahead=4, age_out=3, opt=opt,
                    lr=0.05 if opt == "adagrad" else 1.0)
@@ -100,6 +105,9 @@ def test_two_ranks_one_gpu_parity(opt, a2a, peer, dyn):
     st = W.gen_stream(cfg, 24, counts=counts)
     if dyn:  # N3: hot set recomputed every 6 steps (each owner moves its own share)
         st = W.with_dynamic_hot(st, epoch=6)
+    if layout:  # a random half of the rows first, in random order; the rest in id order
+        order = np.random.default_rng(11).permutation(cfg.n_rows)[:cfg.n_rows // 2]
+        st = W.dataclasses.replace(st, host_order=order.astype(np.int64))
     out = run_two_ranks(st, a2a=a2a, peer=peer)
     if peer:  # the variant actually served rows from the other rank's HBM
         assert out[0]["stats"]["gather_peer"] > 0 and out[1]["stats"]["gather_peer"] > 0

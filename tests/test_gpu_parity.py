@@ -216,6 +216,33 @@ def test_call_order_enforced():
     fr.close()
 
 
+@pytest.mark.parametrize("kind", ["freq", "random_partial", "random_full"])
+def test_host_layout_parity(kind):
+    """frugal_config.host_order only moves bytes in the host table: every
+    artefact, and the host table read back through the layout, match the oracle (which has
+    no layout) exactly."""
+    cfg = tiny1(batch=128, lookahead=4, age_out=2)
+    st = W.gen_stream(cfg, 40)
+    N = cfg.n_rows
+    rng = np.random.default_rng(17)
+    order = {"freq": lambda: W.host_order(cfg, st.ids[:10], st.counts[:10]),
+             "random_partial": lambda: rng.permutation(N)[: N // 3],
+             "random_full": lambda: rng.permutation(N)}[kind]().astype(np.int64)
+    r = run_parity(dataclasses.replace(st, host_order=order))
+    assert r["exact"]
+    r["fr"].close()
+
+
+def test_host_layout_errors():
+    F = _F()
+    from paper_conf_asplos_xiezggl25_b200.harness import make_context
+    st = W.gen_stream(tiny1(batch=32, lookahead=3), 6)
+    for bad in (np.array([3, 5, 3], np.int64), np.array([0, st.cfg.n_rows], np.int64)):
+        with pytest.raises(F.FrugalError) as e:
+            make_context(dataclasses.replace(st, host_order=bad))
+        assert e.value.status == -1
+
+
 @pytest.mark.parametrize("env", [{"FRUGAL_EARLY": "1"}, {"FRUGAL_DRAIN_AT": "sched"},
                                  {"FRUGAL_EARLY": "1", "FRUGAL_DRAIN_AT": "sched"}, {"FRUGAL_SIDE_INLINE": "1"},
                                  {"FRUGAL_NO_POOL_HITS": "1"}, {"FRUGAL_FUSE_OPT": "0"}])
