@@ -506,7 +506,8 @@ def main():
                 if D["bound"] != "hbm" and D["achieved_gbs"] else None,
                 "traffic": traffic, "host_link_traffic": htraffic, "traffic_note": tnote,
                 "peak_source": ("measured pinned cudaMemcpy (256 MiB, best of 5) in this run; random 128-B rows "
-                                "measure 12-33 GB/s on this box (profiles/r1_zc_probe_*.txt)" if D["bound"] != "hbm"
+                                "measure 12-33 GB/s on this box (profiles/r1_zc_probe_*.txt), the step's exact host-row "
+                                "list replayed alone 25-27 GB/s (profiles/r1_exact_replay.txt)" if D["bound"] != "hbm"
                                 else "MEASURED_PEAKS.json hbm_gbs (burst)")}
     launches = st1["kernel_launches"] - st0["kernel_launches"]
     cpu = None

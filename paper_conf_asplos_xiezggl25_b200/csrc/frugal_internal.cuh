@@ -102,6 +102,7 @@ struct frugal_ctx {
     int side_blocks = 20;        // grid cap of the side-stream drain: its zero-copy D2H stores slow the concurrent backward kernels, 16-24 CTAs balance the two (profiles/r1_sweep15.txt)
     int32_t* hs = nullptr;           // [N] host-table slot of every global row (host_order), or null
     std::vector<int32_t> hs_host;    // host copy (frugal_read_host)
+    int flush_tma = 0;               // flushes by TMA bulk stores: 0 none, 1 side drain, 2 all (FRUGAL_FLUSH_TMA; measured no gain: profiles/r1_sweep21_flush_tma.txt)
     bool fuse_opt = true;        // world 1: a8 fused into a6 (k_segreduce / k_segred_combine)
     int gather_blocks = 74;      // grid cap of the zero-copy gathers (74 CTAs fill the link: profiles/r1_zc_probe_async.txt)
     bool side_inline = false;    // experiment: drain on the caller stream
@@ -254,7 +255,7 @@ void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, int3
                         int32_t* adj_cnt, cudaStream_t st);
 void launch_schedule(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStream_t st);
 void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begin, const int32_t* d_end,
-                       int max_blocks, int counter, cudaStream_t st);
+                       int max_blocks, int counter, cudaStream_t st, bool side = false);
 void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32_t* cnt, float* rows, int64_t step,
                    cudaStream_t st);
 void launch_expand(frugal_ctx* c, QueueSlot& q, const float* rows, float* out, cudaStream_t st);

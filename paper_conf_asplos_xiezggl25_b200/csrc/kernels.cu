@@ -765,8 +765,6 @@ void launch_hot_map(frugal_ctx* c, int which, const int64_t* ids64, const int32_
     c->launches++;
 }
 
-void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begin, const int32_t* d_end,
-                       int max_blocks, int counter, cudaStream_t st);
 
 void launch_cache_transition(frugal_ctx* c, int64_t s, int par, cudaStream_t st) {
     const uint32_t* hnew = c->hot_map[c->hot_cur ^ 1];
@@ -794,7 +792,12 @@ void launch_cache_transition(frugal_ctx* c, int64_t s, int par, cudaStream_t st)
 // cache, w of cold rows from the dirty pool.  Zero-copy stores to host memory.  (The
 // owner's Adagrad state G never leaves HBM during training -- no other rank reads it;
 // frugal_flush writes it back once, reading R8.)
-template <int GS>
+// TMA=true: each row is staged in shared memory and written to the host by one bulk
+// async copy (cp.async.bulk.global.shared::cta) instead of the group's zero-copy stores --
+// the same link rate, but the outstanding host writes sit in the TMA unit instead of the
+// SM's store path, which slows the concurrent HBM kernels about half as much
+// (profiles/r1_interference_probe.txt).  smem: (blockDim / GS) * d4 float4.
+template <int GS, bool TMA>
 __global__ void k_flush_rows(const int32_t* __restrict__ rows, const int32_t* d_begin, const int32_t* d_end,
                              int world, int g, int d4, const int32_t* __restrict__ slot,
                              const int32_t* __restrict__ last_upd, const int32_t* __restrict__ pool_idx, int P,
@@ -805,6 +808,9 @@ __global__ void k_flush_rows(const int32_t* __restrict__ rows, const int32_t* d_
     RowGroup<GS>::ids(gid, gs, l);
     const int b = d_begin ? *d_begin : 0, e = *d_end;
     unsigned nh = 0, nc = 0;
+    extern __shared__ __align__(128) float4 fsm[];
+    float4* my = TMA ? fsm + (threadIdx.x / GS) * d4 : nullptr;
+    const unsigned gmask = GS == 32 ? 0xffffffffu : (((1u << GS) - 1u) << ((threadIdx.x & 31) & ~(GS - 1)));
     for (int64_t a = b + gid; a < e; a += gs) {
         int32_t lk = rows[a];
         int64_t k = (int64_t)lk * world + g;
@@ -818,8 +824,24 @@ __global__ void k_flush_rows(const int32_t* __restrict__ rows, const int32_t* d_
             nc += (l == 0);
         }
         float4* dst = hw + host_row(hs, k) * d4;
-        for (int v = l; v < d4; v += GS) dst[v] = src[v];
+        if (TMA) {
+            for (int v = l; v < d4; v += GS) my[v] = src[v];
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            __syncwarp(gmask);
+            if (l == 0) {
+                const unsigned sa = (unsigned)__cvta_generic_to_shared(my);
+                asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(sa),
+                             "r"(d4 * 16)
+                             : "memory");
+                asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+                asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // smem reusable
+            }
+            __syncwarp(gmask);
+        } else {
+            for (int v = l; v < d4; v += GS) dst[v] = src[v];
+        }
     }
+    if (TMA && l == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // writes complete
     if (sysfence) block_fence_system();
     if (stats) {
         block_count(stats, nh);
@@ -828,13 +850,20 @@ __global__ void k_flush_rows(const int32_t* __restrict__ rows, const int32_t* d_
 }
 
 void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begin, const int32_t* d_end,
-                       int max_blocks, int counter, cudaStream_t st) {
+                       int max_blocks, int counter, cudaStream_t st, bool side) {
     const int d4 = c->d / 4, gs = group_size(d4);
     int grid = std::min(grid_for(c->capT * (int64_t)gs, 256, 4), max_blocks);
-    DISPATCH_GS(gs, (k_flush_rows<GS><<<grid, 256, 0, st>>>(
-                        rows, d_begin, d_end, c->n, c->g, d4, c->slot, c->last_upd, c->pool_idx, c->P, c->capT,
-                        (const float4*)c->cw, (const float4*)c->pw, (float4*)c->dh_w, c->hs,
-                        counter >= 0 ? c->dstats + counter : nullptr, c->n > 1)));
+    const bool tma = c->flush_tma == 2 || (c->flush_tma == 1 && side);
+#define FLUSH_ARGS                                                                                                \
+    rows, d_begin, d_end, c->n, c->g, d4, c->slot, c->last_upd, c->pool_idx, c->P, c->capT, (const float4*)c->cw, \
+        (const float4*)c->pw, (float4*)c->dh_w, c->hs, counter >= 0 ? c->dstats + counter : nullptr, c->n > 1
+    if (tma) {
+        const size_t smem = (size_t)(256 / gs) * d4 * 16;
+        DISPATCH_GS(gs, (k_flush_rows<GS, true><<<grid, 256, smem, st>>>(FLUSH_ARGS)));
+    } else {
+        DISPATCH_GS(gs, (k_flush_rows<GS, false><<<grid, 256, 0, st>>>(FLUSH_ARGS)));
+    }
+#undef FLUSH_ARGS
     c->launches++;
 }
 

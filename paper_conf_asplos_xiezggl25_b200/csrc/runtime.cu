@@ -348,6 +348,8 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->dyn = (k.flags & FRUGAL_F_DYNAMIC_CACHE) != 0;
     if (c->dyn) c->early = false;
     c->xhost = c->n > 1 && !c->a2a;
+    // side-drain flushes by TMA bulk stores (FRUGAL_FLUSH_TMA=0 none, 1 side, 2 all)
+    if (getenv("FRUGAL_FLUSH_TMA")) c->flush_tma = atoi(getenv("FRUGAL_FLUSH_TMA"));
     // world 1: optimizer fused into the segment-reduce (FRUGAL_FUSE_OPT=0: two kernels)
     c->fuse_opt = !(getenv("FRUGAL_FUSE_OPT") && !atoi(getenv("FRUGAL_FUSE_OPT")));
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 20;
@@ -773,13 +775,13 @@ static frugal_status launch_drain(frugal_ctx* c, int64_t s, cudaStream_t st, cud
     if (!no_drain) {
         Timer tm(c, PH_SIDE, sd);
         launch_flush_rows(c, c->sl_rows[par] + c->sl_cap, nullptr, c->sl_cnt[par] + 1, c->side_blocks,
-                          FRUGAL_C_SIDE_HOT, sd);
+                          FRUGAL_C_SIDE_HOT, sd, true);
         CK(cudaEventRecord(c->ev_side_first[par], sd));
         if (c->xhost) launch_set_flag(c, FLAG_SIDE_FIRST, (uint32_t)(s + 1), sd);
         launch_flush_rows(c, c->sl_rows[par] + 2 * c->sl_cap, nullptr, c->sl_cnt[par] + 2, c->side_blocks,
-                          FRUGAL_C_SIDE_HOT, sd);
+                          FRUGAL_C_SIDE_HOT, sd, true);
         launch_flush_rows(c, c->sl_rows[par] + 3 * c->sl_cap, nullptr, c->sl_cnt[par] + 3, c->side_blocks,
-                          FRUGAL_C_SIDE_HOT, sd);
+                          FRUGAL_C_SIDE_HOT, sd, true);
         if (c->xhost) launch_set_flag(c, FLAG_SIDE, (uint32_t)(s + 1), sd);
         CKL();
     }
