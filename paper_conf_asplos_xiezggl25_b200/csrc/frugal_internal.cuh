@@ -102,6 +102,7 @@ struct frugal_ctx {
     int side_blocks = 20;        // grid cap of the side-stream drain: its zero-copy D2H stores slow the concurrent backward kernels, 16-24 CTAs balance the two (profiles/r1_sweep15.txt)
     int32_t* hs = nullptr;           // [N] host-table slot of every global row (host_order), or null
     std::vector<int32_t> hs_host;    // host copy (frugal_read_host)
+    int side_first_blocks = 20;      // grid cap of the drain's deadline-(s+1) part
     int flush_tma = 0;               // flushes by TMA bulk stores: 0 none, 1 side drain, 2 all (FRUGAL_FLUSH_TMA; measured no gain: profiles/r1_sweep21_flush_tma.txt)
     bool fuse_opt = true;        // world 1: a8 fused into a6 (k_segreduce / k_segred_combine)
     int gather_blocks = 74;      // grid cap of the zero-copy gathers (74 CTAs fill the link: profiles/r1_zc_probe_async.txt)

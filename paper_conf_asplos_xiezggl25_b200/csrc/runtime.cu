@@ -353,6 +353,9 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     // world 1: optimizer fused into the segment-reduce (FRUGAL_FUSE_OPT=0: two kernels)
     c->fuse_opt = !(getenv("FRUGAL_FUSE_OPT") && !atoi(getenv("FRUGAL_FUSE_OPT")));
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 20;
+    // the deadline-(s+1) part of the drain (the next gate waits for it) may run wider
+    c->side_first_blocks = getenv("FRUGAL_SIDE_FIRST_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_FIRST_BLOCKS"))
+                                                               : c->side_blocks;
     c->gather_blocks = getenv("FRUGAL_GATHER_BLOCKS") ? atoi(getenv("FRUGAL_GATHER_BLOCKS")) : 74;
     c->side_inline = getenv("FRUGAL_SIDE_INLINE") && atoi(getenv("FRUGAL_SIDE_INLINE"));
     c->drain_after_gather = !(getenv("FRUGAL_DRAIN_AT") && !strcmp(getenv("FRUGAL_DRAIN_AT"), "sched"));
@@ -774,7 +777,7 @@ static frugal_status launch_drain(frugal_ctx* c, int64_t s, cudaStream_t st, cud
     static const bool no_drain = getenv("FRUGAL_EXPERIMENT_NO_DRAIN") != nullptr;  // WRONG RESULTS: upper bound only
     if (!no_drain) {
         Timer tm(c, PH_SIDE, sd);
-        launch_flush_rows(c, c->sl_rows[par] + c->sl_cap, nullptr, c->sl_cnt[par] + 1, c->side_blocks,
+        launch_flush_rows(c, c->sl_rows[par] + c->sl_cap, nullptr, c->sl_cnt[par] + 1, c->side_first_blocks,
                           FRUGAL_C_SIDE_HOT, sd, true);
         CK(cudaEventRecord(c->ev_side_first[par], sd));
         if (c->xhost) launch_set_flag(c, FLAG_SIDE_FIRST, (uint32_t)(s + 1), sd);
