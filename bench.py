@@ -482,7 +482,23 @@ def main():
     # a5 glue: read r per position (embeddings, register-cached), write r (grads), x per sample
     per["model"] = dict(bound="hbm", bytes=(cnt["positions"] * 2 * r + B * (r + 4)) / K, ms=ph["model"],
                         peak=hbm_peak)
+    if kg:
+        # a5 KG glue (TransE, R26): fp64 ALU-bound, not HBM.  Algorithmic ops per chunk of C
+        # triples with C shared negatives: distances C*C*d*3 (sub, mul, add), the two gradient
+        # reductions 2*C*C*d*3; positives d*4 per triple.  Every op is a separately rounded
+        # DADD/DSUB/DMUL (no FMA), so the peak is the fp64 instruction rate: half the guide's
+        # 45 TFLOP/s B200 FP64 (FMA = 2 flops) -> 22.5 TFLOP/s.
+        cnt_b = B  # triples per rank per step (full batches in the bench)
+        C_ = cfg.neg_chunk
+        nch, last = cnt_b // C_, cnt_b % C_
+        pairs = nch * C_ * C_ + last * last
+        flops = pairs * d * 9 + cnt_b * d * 4
+        per["model"] = dict(bound="alu", flops=flops, ms=ph["model"], peak_tflops=22.5,
+                            achieved_tflops=flops / (ph["model"] * 1e-3) / 1e12 if ph["model"] > 0 else None)
+        per["model"]["frac"] = (per["model"]["achieved_tflops"] / 22.5) if per["model"]["achieved_tflops"] else None
     for k, v in per.items():
+        if v.get("bound") == "alu":
+            continue
         v["achieved_gbs"] = gbs(v["bytes"], v["ms"])
         v["frac"] = v["achieved_gbs"] / v["peak"] if v["achieved_gbs"] else None
     main_ms = {k: v for k, v in ph.items() if k != "side"}
@@ -499,16 +515,23 @@ def main():
                      f"steady-state launch, ncu --set full); host_link_traffic = its sysmem sectors through L2")
     except Exception:
         pass
-    roofline = {"bound": "hbm" if D["bound"] == "hbm" else "host-link", "kernel": dom,
-                "achieved": D["achieved_gbs"], "peak": D["peak"], "unit": "GB/s", "frac": D["frac"],
-                "random_row_ceiling": link["random_rows_h2d"] if D["bound"] != "hbm" else None,
-                "frac_of_random_row_ceiling": (D["achieved_gbs"] / link["random_rows_h2d"])
-                if D["bound"] != "hbm" and D["achieved_gbs"] else None,
-                "traffic": traffic, "host_link_traffic": htraffic, "traffic_note": tnote,
-                "peak_source": ("measured pinned cudaMemcpy (256 MiB, best of 5) in this run; random 128-B rows "
-                                "measure 12-33 GB/s on this box (profiles/r1_zc_probe_*.txt), the step's exact host-row "
-                                "list replayed alone 25-27 GB/s (profiles/r1_exact_replay.txt)" if D["bound"] != "hbm"
-                                else "MEASURED_PEAKS.json hbm_gbs (burst)")}
+    if D.get("bound") != "alu":
+        roofline = {"bound": "hbm" if D["bound"] == "hbm" else "host-link", "kernel": dom,
+                    "achieved": D["achieved_gbs"], "peak": D["peak"], "unit": "GB/s", "frac": D["frac"],
+                    "random_row_ceiling": link["random_rows_h2d"] if D["bound"] != "hbm" else None,
+                    "frac_of_random_row_ceiling": (D["achieved_gbs"] / link["random_rows_h2d"])
+                    if D["bound"] != "hbm" and D["achieved_gbs"] else None,
+                    "traffic": traffic, "host_link_traffic": htraffic, "traffic_note": tnote,
+                    "peak_source": ("measured pinned cudaMemcpy (256 MiB, best of 5) in this run; random 128-B rows "
+                                    "measure 12-33 GB/s on this box (profiles/r1_zc_probe_*.txt), the step's exact host-row "
+                                    "list replayed alone 25-27 GB/s (profiles/r1_exact_replay.txt)" if D["bound"] != "hbm"
+                                    else "MEASURED_PEAKS.json hbm_gbs (burst)")}
+    else:  # KG glue dominates: fp64 ALU roofline
+        roofline = {"bound": "alu", "kernel": dom + " (k_transe_pos / _pairs_tiled / _grads_tiled)",
+                    "achieved": D["achieved_tflops"], "peak": D["peak_tflops"], "unit": "TFLOP/s", "frac": D["frac"],
+                    "traffic": None,
+                    "peak_source": "fp64 non-FMA instruction rate: half the 45 TFLOP/s B200 FP64 figure of "
+                                   "/opt/skills/guides/blackwell_cuda_programming.md (DESIGN.md §7)"}
     launches = st1["kernel_launches"] - st0["kernel_launches"]
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

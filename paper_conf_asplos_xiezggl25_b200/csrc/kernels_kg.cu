@@ -98,26 +98,34 @@ __global__ void k_transe_grads(const float* __restrict__ emb, int count, int C, 
     }
 }
 
-// ---- tiled versions (default): 32x32 output tiles per CTA of 256 threads, each thread 2x2
-// outputs; operand tiles of 32 (k, j or b) staged in shared memory as fp64.  Every output
-// still accumulates in the written order (k / j / b ascending), so the results equal the
-// loops above bit for bit.
+// ---- tiled versions (default): 32x32 output tiles per CTA; each thread RI x CQ outputs,
+// rows ty + TY*i and columns tx + TX*q (interleaved: with a row stride of 33 doubles the
+// shared-memory reads of a warp hit distinct bank pairs); operand tiles of 32 (k, j or b)
+// staged in shared memory as fp64.  Every output still accumulates in the written order
+// (k / j / b ascending), so the results equal the loops above bit for bit.
 constexpr int TT = 32;
 
 // distances of all (b, j) pairs of a chunk: W[b][j] = sigma(gamma - dist)/dist/nC, loss
-__global__ void __launch_bounds__(256) k_transe_pairs_tiled(const float* __restrict__ emb, int count, int C, int d,
-                                                            double gamma, double* __restrict__ Wm, double* loss,
-                                                            double nb) {
+template <int RI, int CQ>
+__global__ void __launch_bounds__((TT / RI) * (TT / CQ)) k_transe_pairs_tiled(const float* __restrict__ emb, int count,
+                                                                             int C, int d, double gamma,
+                                                                             double* __restrict__ Wm, double* loss,
+                                                                             double nb) {
+    constexpr int TX = TT / CQ, TY = TT / RI, NT = TX * TY;
     __shared__ double Ps[TT][TT + 1];
     __shared__ double Ns[TT][TT + 1];
     const int tiles = (C + TT - 1) / TT;
     const int c = blockIdx.x / (tiles * tiles), tb = (blockIdx.x / tiles) % tiles, tj = blockIdx.x % tiles;
     const int b0 = c * C, nC = min(C, count - b0);
     if (tb * TT >= nC || tj * TT >= nC) return;
-    const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;  // thread owns b = ty*2+{0,1}, j = tx*2+{0,1}
-    double acc[2][2] = {{0.0, 0.0}, {0.0, 0.0}};
+    const int tx = threadIdx.x % TX, ty = threadIdx.x / TX;  // thread owns b = ty + TY*i, j = tx + TX*q
+    double acc[RI][CQ];
+#pragma unroll
+    for (int i = 0; i < RI; i++)
+#pragma unroll
+        for (int q = 0; q < CQ; q++) acc[i][q] = 0.0;
     for (int k0 = 0; k0 < d; k0 += TT) {
-        for (int e = threadIdx.x; e < TT * TT; e += 256) {
+        for (int e = threadIdx.x; e < TT * TT; e += NT) {
             const int r = e / TT, kk = e % TT, k = k0 + kk;
             const int bl = tb * TT + r, jl = tj * TT + r;
             double pv = 0.0, nv = 0.0;
@@ -132,11 +140,16 @@ __global__ void __launch_bounds__(256) k_transe_pairs_tiled(const float* __restr
         __syncthreads();
         const int kend = min(TT, d - k0);
         for (int kk = 0; kk < kend; kk++) {
+            double pv[RI], nv[CQ];
 #pragma unroll
-            for (int i = 0; i < 2; i++)
+            for (int i = 0; i < RI; i++) pv[i] = Ps[ty + TY * i][kk];
 #pragma unroll
-                for (int q = 0; q < 2; q++) {
-                    const double u = __dsub_rn(Ps[ty * 2 + i][kk], Ns[tx * 2 + q][kk]);
+            for (int q = 0; q < CQ; q++) nv[q] = Ns[tx + TX * q][kk];
+#pragma unroll
+            for (int i = 0; i < RI; i++)
+#pragma unroll
+                for (int q = 0; q < CQ; q++) {
+                    const double u = __dsub_rn(pv[i], nv[q]);
                     acc[i][q] = __dadd_rn(acc[i][q], __dmul_rn(u, u));
                 }
         }
@@ -144,10 +157,10 @@ __global__ void __launch_bounds__(256) k_transe_pairs_tiled(const float* __restr
     }
     double lsum = 0.0;
 #pragma unroll
-    for (int i = 0; i < 2; i++)
+    for (int i = 0; i < RI; i++)
 #pragma unroll
-        for (int q = 0; q < 2; q++) {
-            const int bl = tb * TT + ty * 2 + i, jl = tj * TT + tx * 2 + q;
+        for (int q = 0; q < CQ; q++) {
+            const int bl = tb * TT + ty + TY * i, jl = tj * TT + tx + TX * q;
             if (bl < nC && jl < nC) {
                 const double dist = __dsqrt_rn(acc[i][q]);
                 const double sc = __dsub_rn(gamma, dist);
@@ -155,13 +168,13 @@ __global__ void __launch_bounds__(256) k_transe_pairs_tiled(const float* __restr
                 Wm[(int64_t)(b0 + bl) * C + jl] = dist > 0.0 ? __ddiv_rn(__ddiv_rn(sigm(sc), dist), (double)nC) : 0.0;
             }
         }
-    __shared__ double sl[8];
+    __shared__ double sl[NT / 32];
     for (int o = 16; o; o >>= 1) lsum += __shfl_xor_sync(FULL, lsum, o);
     if ((threadIdx.x & 31) == 0) sl[threadIdx.x >> 5] = lsum;
     __syncthreads();
     if (threadIdx.x == 0) {
         double t = 0.0;
-        for (int i = 0; i < 8; i++) t += sl[i];
+        for (int i = 0; i < NT / 32; i++) t += sl[i];
         if (t != 0.0) atomicAdd(loss, t / nb);
     }
 }
@@ -202,24 +215,26 @@ __global__ void k_transe_pos(const float* __restrict__ emb, int count, int d, do
 
 // gradients: MODE 0: (h, r, t) rows, output tile (b, k), reduction over j ascending;
 //            MODE 1: negative rows,  output tile (j, k), reduction over b ascending.
-template <int MODE>
-__global__ void __launch_bounds__(256) k_transe_grads_tiled(const float* __restrict__ emb, int count, int C, int d,
-                                                            const double* __restrict__ Wm,
-                                                            const double* __restrict__ A, float* __restrict__ grad,
-                                                            double nb) {
+template <int MODE, int RI, int CQ>
+__global__ void __launch_bounds__((TT / RI) * (TT / CQ)) k_transe_grads_tiled(const float* __restrict__ emb, int count,
+                                                                             int C, int d,
+                                                                             const double* __restrict__ Wm,
+                                                                             const double* __restrict__ A,
+                                                                             float* __restrict__ grad, double nb) {
+    constexpr int TX = TT / CQ, TY = TT / RI, NT = TX * TY;
     __shared__ double Ws[TT][TT + 1];  // [out row][red]
     __shared__ double Xs[TT][TT + 1];  // [red][k]: N (mode 0) or P (mode 1)
     const int rtiles = (C + TT - 1) / TT, ktiles = (d + TT - 1) / TT;
     const int c = blockIdx.x / (rtiles * ktiles), tr = (blockIdx.x / ktiles) % rtiles, tk = blockIdx.x % ktiles;
     const int b0 = c * C, nC = min(C, count - b0);
     if (tr * TT >= nC) return;
-    const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;  // outputs rows ty*2+{0,1}, k tx*2+{0,1}
-    double own[2][2], accv[2][2];
+    const int tx = threadIdx.x % TX, ty = threadIdx.x / TX;  // outputs rows ty + TY*i, k = tx + TX*q
+    double own[RI][CQ], accv[RI][CQ];
 #pragma unroll
-    for (int i = 0; i < 2; i++)
+    for (int i = 0; i < RI; i++)
 #pragma unroll
-        for (int q = 0; q < 2; q++) {
-            const int rl = tr * TT + ty * 2 + i, k = tk * TT + tx * 2 + q;
+        for (int q = 0; q < CQ; q++) {
+            const int rl = tr * TT + ty + TY * i, k = tk * TT + tx + TX * q;
             own[i][q] = 0.0;
             accv[i][q] = 0.0;
             if (rl < nC && k < d) {
@@ -233,9 +248,13 @@ __global__ void __launch_bounds__(256) k_transe_grads_tiled(const float* __restr
                 }
             }
         }
-    const double keep[2][2] = {{accv[0][0], accv[0][1]}, {accv[1][0], accv[1][1]}};  // a_b v (mode 0)
+    double keep[RI][CQ];  // a_b v (mode 0)
+#pragma unroll
+    for (int i = 0; i < RI; i++)
+#pragma unroll
+        for (int q = 0; q < CQ; q++) keep[i][q] = accv[i][q];
     for (int r0 = 0; r0 < nC; r0 += TT) {
-        for (int e = threadIdx.x; e < TT * TT; e += 256) {
+        for (int e = threadIdx.x; e < TT * TT; e += NT) {
             const int x = e / TT, y = e % TT;
             // Ws[x][y] = W[out row x][red y]   (mode 0: W[b][j]; mode 1: W[b=red][j=out])
             const int ol = tr * TT + x, rl = r0 + y;
@@ -255,26 +274,29 @@ __global__ void __launch_bounds__(256) k_transe_grads_tiled(const float* __restr
         __syncthreads();
         const int rend = min(TT, nC - r0);
         for (int y = 0; y < rend; y++) {
+            double wv[RI], xv[CQ];
 #pragma unroll
-            for (int i = 0; i < 2; i++)
+            for (int i = 0; i < RI; i++) wv[i] = Ws[ty + TY * i][y];
 #pragma unroll
-                for (int q = 0; q < 2; q++) {
-                    const double w = Ws[ty * 2 + i][y];
-                    const double x = Xs[y][tx * 2 + q];
+            for (int q = 0; q < CQ; q++) xv[q] = Xs[y][tx + TX * q];
+#pragma unroll
+            for (int i = 0; i < RI; i++)
+#pragma unroll
+                for (int q = 0; q < CQ; q++) {
                     if (MODE == 0) {  // gh -= W_bj (P_b - n_j)
-                        accv[i][q] = __dsub_rn(accv[i][q], __dmul_rn(w, __dsub_rn(own[i][q], x)));
+                        accv[i][q] = __dsub_rn(accv[i][q], __dmul_rn(wv[i], __dsub_rn(own[i][q], xv[q])));
                     } else {          // gn += W_bj (P_b - n_j)
-                        accv[i][q] = __dadd_rn(accv[i][q], __dmul_rn(w, __dsub_rn(x, own[i][q])));
+                        accv[i][q] = __dadd_rn(accv[i][q], __dmul_rn(wv[i], __dsub_rn(xv[q], own[i][q])));
                     }
                 }
         }
         __syncthreads();
     }
 #pragma unroll
-    for (int i = 0; i < 2; i++)
+    for (int i = 0; i < RI; i++)
 #pragma unroll
-        for (int q = 0; q < 2; q++) {
-            const int rl = tr * TT + ty * 2 + i, k = tk * TT + tx * 2 + q;
+        for (int q = 0; q < CQ; q++) {
+            const int rl = tr * TT + ty + TY * i, k = tk * TT + tx + TX * q;
             if (rl < nC && k < d) {
                 const int64_t b = b0 + rl;
                 if (MODE == 0) {
@@ -306,9 +328,15 @@ void launch_transe_model(frugal_ctx* c, QueueSlot& q, const float* emb, int C, d
     const int tiles = (C + TT - 1) / TT, ktiles = (c->d + TT - 1) / TT;
     k_transe_pos<<<grid_for((int64_t)count * 32, 128, 4), 128, (size_t)4 * c->d * sizeof(double), st>>>(
         emb, count, c->d, gamma, A, loss, (double)nb);
-    k_transe_pairs_tiled<<<nchunks * tiles * tiles, 256, 0, st>>>(emb, count, C, c->d, gamma, Wm, loss, (double)nb);
-    k_transe_grads_tiled<0><<<nchunks * tiles * ktiles, 256, 0, st>>>(emb, count, C, c->d, Wm, A, grad, (double)nb);
-    k_transe_grads_tiled<1><<<nchunks * tiles * ktiles, 256, 0, st>>>(emb, count, C, c->d, Wm, A, grad, (double)nb);
+    // 2x2 outputs per thread, 256 threads per 32x32 tile: 4x4 / 2x4 / 1x2 / 2x1 measured slower at
+    // C = 200 (profiles/r1_sweep23_kg_tile.txt, r1_sweep24_kg_tile.txt)
+    constexpr int RI = 2, CQ = 2, nt = (TT / RI) * (TT / CQ);
+    k_transe_pairs_tiled<RI, CQ><<<nchunks * tiles * tiles, nt, 0, st>>>(emb, count, C, c->d, gamma, Wm, loss,
+                                                                         (double)nb);
+    k_transe_grads_tiled<0, RI, CQ><<<nchunks * tiles * ktiles, nt, 0, st>>>(emb, count, C, c->d, Wm, A, grad,
+                                                                             (double)nb);
+    k_transe_grads_tiled<1, RI, CQ><<<nchunks * tiles * ktiles, nt, 0, st>>>(emb, count, C, c->d, Wm, A, grad,
+                                                                             (double)nb);
     c->launches += 4;
 }
 
