@@ -113,6 +113,11 @@ __global__ void k_radix_scan_rows(int32_t* __restrict__ hist, int nblk, int32_t*
     if (threadIdx.x == 0) tot[blockIdx.x] = run;
 }
 
+// Super-tiles of kSub * 256 keys: warp w ranks its kSub consecutive 32-key sub-tiles in
+// order with __match_any_sync and a running per-warp digit count, then one block-wide
+// prefix over the 8 warps per digit places all of them -- the digit-count zeroing and
+// prefix (8 x 512 counters) are paid once per 1024 keys instead of once per 256.
+constexpr int kSub = 4;
 __global__ void __launch_bounds__(256) k_radix_scatter(const uint32_t* __restrict__ kin, const int32_t* __restrict__ vin,
                                 uint32_t* __restrict__ kout, int32_t* __restrict__ vout, const int32_t* d_n,
                                 int shift, const int32_t* __restrict__ hist, const int32_t* __restrict__ dtot,
@@ -130,24 +135,37 @@ __global__ void __launch_bounds__(256) k_radix_scatter(const uint32_t* __restric
     }
     int lo, hi;
     chunk_range(*d_n, nblk, blockIdx.x, lo, hi);
-    for (int base = lo; base < hi; base += kTile) {
+    for (int base = lo; base < hi; base += kTile * kSub) {
 #pragma unroll
         for (int i = 0; i < 8; i++) {
             wcnt[i][tid] = 0;
             wcnt[i][tid + 256] = 0;
         }
         __syncthreads();
-        const int i = base + tid;
-        const bool valid = i < hi;
-        uint32_t key = valid ? kin[i] : 0u;
-        int32_t val = valid ? vin[i] : 0;
-        int dg = valid ? (int)((key >> shift) & (kDigits - 1)) : -1;
-        unsigned peers = __match_any_sync(FULL, dg);
-        int rank = __popc(peers & lanemask_lt());
-        if (valid && rank == 0) wcnt[w][dg] = __popc(peers);
+        // warp w: keys [base + w*32*kSub, +32*kSub), sub-tile j = 32 consecutive keys
+        uint32_t key[kSub];
+        int32_t val[kSub];
+        int dg[kSub], loc[kSub];
+#pragma unroll
+        for (int j = 0; j < kSub; j++) {
+            const int i = base + (w * kSub + j) * 32 + lane;
+            const bool valid = i < hi;
+            key[j] = valid ? kin[i] : 0u;
+            val[j] = valid ? vin[i] : 0;
+            dg[j] = valid ? (int)((key[j] >> shift) & (kDigits - 1)) : -1;
+        }
+#pragma unroll
+        for (int j = 0; j < kSub; j++) {
+            const unsigned peers = __match_any_sync(FULL, dg[j]);
+            const int rank = __popc(peers & lanemask_lt());
+            loc[j] = dg[j] >= 0 ? wcnt[w][dg[j]] + rank : 0;  // keys of this digit in earlier sub-tiles
+            __syncwarp();
+            if (dg[j] >= 0 && rank == 0) wcnt[w][dg[j]] += __popc(peers);
+            __syncwarp();
+        }
         __syncthreads();
 #pragma unroll
-        for (int h = 0; h < 2; h++) {
+        for (int h = 0; h < 2; h++) {  // per digit: exclusive prefix over the warps
             const int d = tid + h * 256;
             int acc = 0;
 #pragma unroll
@@ -159,10 +177,13 @@ __global__ void __launch_bounds__(256) k_radix_scatter(const uint32_t* __restric
             tot[d] = acc;
         }
         __syncthreads();
-        if (valid) {
-            int dst = run[dg] + wcnt[w][dg] + rank;
-            kout[dst] = key;
-            vout[dst] = val;
+#pragma unroll
+        for (int j = 0; j < kSub; j++) {
+            if (dg[j] >= 0) {
+                const int dst = run[dg[j]] + wcnt[w][dg[j]] + loc[j];
+                kout[dst] = key[j];
+                vout[dst] = val[j];
+            }
         }
         __syncthreads();
         run[tid] += tot[tid];

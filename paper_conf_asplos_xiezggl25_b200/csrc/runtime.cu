@@ -774,8 +774,7 @@ static frugal_status launch_drain(frugal_ctx* c, int64_t s, cudaStream_t st, cud
     const int par = (int)(s & 1);
     cudaStream_t sd = c->side_inline ? st : c->side;
     if (!c->side_inline) CK(cudaStreamWaitEvent(c->side, after, 0));
-    static const bool no_drain = getenv("FRUGAL_EXPERIMENT_NO_DRAIN") != nullptr;  // WRONG RESULTS: upper bound only
-    if (!no_drain) {
+    {
         Timer tm(c, PH_SIDE, sd);
         launch_flush_rows(c, c->sl_rows[par] + c->sl_cap, nullptr, c->sl_cnt[par] + 1, c->side_first_blocks,
                           FRUGAL_C_SIDE_HOT, sd, true);

@@ -1,4 +1,4 @@
 #!/bin/bash
 run() { env "$@" python bench.py --no-cpu-baseline --steps 150 --warmup 20 2>/dev/null | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('$*', round(d['value']/1e6,2), 'e2e', round(d['e2e']['value']/1e6,2), {k: round(v,3) for k,v in d['phases_ms_per_step'].items()})"; }
-run FRUGAL_EXPERIMENT_NO_DRAIN=1
-run FRUGAL_EXPERIMENT_NO_DRAIN=1 FRUGAL_NO_EARLY=1
+# (FRUGAL_EXPERIMENT_NO_DRAIN was removed; see profiles/r1_no_drain_upper_bound.txt)
+# (FRUGAL_EXPERIMENT_NO_DRAIN was removed; see profiles/r1_no_drain_upper_bound.txt)
