@@ -12,3 +12,9 @@ for k in k_gather_uniq k_segreduce k_flush_rows k_dot_model k_expand k_segred_co
     ncu --set full --import-source on --clock-control none -k regex:$k --launch-skip 30 -c 1 \
         -o gpurun_out/$k -f $B > gpurun_out/prof_$k.log 2>&1
 done
+# KG glue (FB15k-shaped bench)
+BK="python bench.py --config fb15k --steps 40 --warmup 3 --no-cpu-baseline"
+for k in k_transe_pos k_transe_pairs_tiled k_transe_grads_tiled; do
+    ncu --set full --import-source on --clock-control none -k regex:$k --launch-skip 30 -c 1 \
+        -o gpurun_out/$k -f $BK > gpurun_out/prof_$k.log 2>&1
+done
