@@ -91,3 +91,29 @@ def test_bench_module_imports_and_parses():
     a = b.parse()
     assert a.gpus == 1 and a.warmup >= 3 and a.exchange == "host"
     assert b.dist_max(3.0, 1) == 3.0
+
+
+@pytest.mark.parametrize("n_order", [-1, 5, 101])
+def test_host_order_validation(n_order):
+    """frugal_config.host_order: a negative or too long count, or a count without a list,
+    is rejected before any device work."""
+    F = _lib()
+    cfg = F.Config(world=1, rank=0, device=0, dim=16, n_rows=100, slots=1, batch=4, lookahead=4, age_out=2,
+                   opt=1, lr=0.1, eps=1e-10, init_accum=0.0, init_scale=0.05, init_seed=3, hot_ids=None,
+                   n_hot=0, shm_name=None, mode=0, flags=0, host_order=None, n_order=n_order)
+    h = C.c_void_p()
+    assert F.lib().frugal_init(C.byref(cfg), C.byref(h)) == -1
+    assert not h.value
+
+
+def test_workload_host_order():
+    """The frequency layout of past traffic: distinct seen rows, most frequent first, ties by id."""
+    import numpy as np
+    from paper_conf_asplos_xiezggl25_b200 import workload as W
+    cfg = W.config("tiny", world=2, batch=64)
+    st = W.gen_stream(cfg, 8)
+    o = W.host_order(cfg, st.ids, st.counts)
+    freq = np.bincount(st.ids.ravel(), minlength=cfg.n_rows)
+    assert len(set(o.tolist())) == len(o) == int((freq > 0).sum())
+    key = [(-int(freq[k]), int(k)) for k in o]
+    assert key == sorted(key)
