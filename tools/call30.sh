@@ -1,4 +1,5 @@
 timeout 1200 python -m pytest tests -m gpu -x -q > gpurun_out/gputests30.log 2>&1
+# NOTE: historical sweep (results in profiles/); some knobs it sets were removed after the measurement
 run() {
     local cfg=$1; shift
     env "$@" python bench.py --config "$cfg" --no-cpu-baseline --steps 200 --warmup 20 2>/dev/null |

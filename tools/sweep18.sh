@@ -1,4 +1,5 @@
 #!/bin/bash
+# NOTE: historical sweep (results in profiles/); some knobs it sets were removed after the measurement
 # ingest kernels after the scheduler (default) vs after the gather, configs[1]/[2], one B200
 run() {
     local cfg=$1; shift

@@ -1,4 +1,5 @@
 #!/bin/bash
+# NOTE: historical sweep (results in profiles/); some knobs it sets were removed after the measurement
 # KG glue outputs per thread (FRUGAL_KG_TILE), FB15k / Freebase shapes, one B200
 run() {
     local cfg=$1; shift

@@ -1,4 +1,5 @@
 #!/bin/bash
+# NOTE: historical sweep (results in profiles/); some knobs it sets were removed after the measurement
 # split gather (HBM rows on a full grid + host rows on the zero-copy grid) vs one kernel, configs[1]/[2], one B200
 run() {
     local cfg=$1; shift
