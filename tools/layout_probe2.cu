@@ -20,6 +20,17 @@ __global__ void g_scatter(const int32_t* idx, int n, float4* h, const float4* in
     int l = threadIdx.x & 7;
     for (int64_t u = t / 8; u < n; u += gs) h[(int64_t)idx[u] * 8 + l] = in[u * 8 + l];
 }
+// HBM state touched like one step of the library: n random 128-B row RMWs over a big device
+// array (Adagrad G / cache / pool) -- does it slow the next zero-copy host gather?
+__global__ void g_noise(float4* big, int64_t rows, int n, uint64_t seed) {
+    int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x, gs = ((int64_t)gridDim.x * blockDim.x) / 8;
+    int l = threadIdx.x & 7;
+    for (int64_t u = t / 8; u < n; u += gs) {
+        uint64_t x = (u + 1) * 0x9E3779B97F4A7C15ull ^ seed; x ^= x >> 31; x *= 0xBF58476D1CE4E5B9ull; x ^= x >> 29;
+        float4* p = big + (int64_t)(x % rows) * 8 + l;
+        float4 v = *p; v.x += 1.f; *p = v;
+    }
+}
 typedef std::vector<std::vector<int32_t>> Lists;
 static Lists load(const char* p) {
     FILE* f = fopen(p, "rb"); if (!f) { printf("no %s\n", p); exit(1); }
@@ -49,6 +60,9 @@ int main() {
                     {"exact reads only", &empty, &ex_r, &empty}, {"freq urgent>reads>drain", &fx_u, &fx_r, &fx_d},
                     {"freq reads only", &empty, &fx_r, &empty}};
     cudaEvent_t ev[4]; for (auto& x : ev) cudaEventCreate(&x);
+    const int64_t big_rows = (5ll << 30) / 128;
+    float4* big; CK(cudaMalloc(&big, big_rows * 128)); CK(cudaMemset(big, 0, big_rows * 128));
+    for (int noise : {0, 65000, 200000})
     for (int alloc = 0; alloc < 1; alloc++)
     for (auto& cs : cases) {
         float4* dh = alloc ? dB : dA;
@@ -57,6 +71,7 @@ int main() {
         for (size_t s = 0; s < S; s++) {
             Lists* L3[3] = {cs.a, cs.b, cs.c};
             for (int k = 0; k < 3; k++) if ((*L3[k])[s].size()) CK(cudaMemcpy(didx + (size_t)k * (4 << 20), (*L3[k])[s].data(), (*L3[k])[s].size() * 4, cudaMemcpyHostToDevice));
+            if (noise) g_noise<<<1184, 256>>>(big, big_rows, noise, s * 7919);
             cudaEventRecord(ev[0]);
             if ((*L3[0])[s].size()) g_scatter<<<74, 256>>>(didx, (int)(*L3[0])[s].size(), dh, buf);
             cudaEventRecord(ev[1]);
@@ -69,7 +84,7 @@ int main() {
                 cnt++;
             }
         }
-        printf("%-14s %-26s", alloc ? "mmap+register" : "cudaHostAlloc", cs.nm);
+        printf("noise %6d %-14s %-26s", noise, alloc ? "mmap+register" : "cudaHostAlloc", cs.nm);
         const char* nm[3] = {"first", "reads", "last"};
         for (int k = 0; k < 3; k++) printf("  %s %6.0f rows %.3f ms %5.1f GB/s", nm[k], nr[k] / cnt, t[k] / cnt, t[k] > 0 ? nr[k] * 128 / (t[k] * 1e6) : 0.0);
         printf("\n");
