@@ -968,9 +968,23 @@ __global__ void k_expand(const int32_t* __restrict__ inv, const int32_t* d_m, in
     int l;
     RowGroup<GS>::ids(gid, gs, l);
     const int m = *d_m;
-    for (int64_t i = gid; i < m; i += gs) {
-        const float4* src = rows + (int64_t)inv[i] * d4;
-        for (int v = l; v < d4; v += GS) out[i * d4 + v] = src[v];
+    // 4 positions per row group in flight: their inv loads, then their row loads, are
+    // issued together (latency-bound dependent pairs otherwise)
+    constexpr int R = 4;
+    for (int64_t i0 = gid; i0 < m; i0 += gs * R) {
+        int32_t iv[R];
+#pragma unroll
+        for (int r = 0; r < R; r++) iv[r] = i0 + (int64_t)r * gs < m ? inv[i0 + (int64_t)r * gs] : -1;
+        for (int v0 = 0; v0 < d4; v0 += GS) {
+            const int v = v0 + l;
+            float4 x[R];
+#pragma unroll
+            for (int r = 0; r < R; r++)
+                if (iv[r] >= 0 && v < d4) x[r] = rows[(int64_t)iv[r] * d4 + v];
+#pragma unroll
+            for (int r = 0; r < R; r++)
+                if (iv[r] >= 0 && v < d4) out[(i0 + (int64_t)r * gs) * d4 + v] = x[r];
+        }
     }
 }
 
