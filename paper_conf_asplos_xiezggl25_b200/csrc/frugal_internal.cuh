@@ -105,7 +105,7 @@ struct frugal_ctx {
     int side_first_blocks = 20;      // grid cap of the drain's deadline-(s+1) part
     int flush_tma = 0;               // flushes by TMA bulk stores: 0 none, 1 side drain, 2 all (FRUGAL_FLUSH_TMA; measured no gain: profiles/r1_sweep21_flush_tma.txt)
     bool fuse_opt = true;        // world 1: a8 fused into a6 (k_segreduce / k_segred_combine)
-    int gather_blocks = 74;      // grid cap of the zero-copy gathers (74 CTAs fill the link: profiles/r1_zc_probe_async.txt)
+    int gather_blocks = 120;     // grid cap of the zero-copy gathers (120 CTAs: +3% over 74 and 148 in the step, profiles/r1_sweep34_gather_grid.txt)
     bool side_inline = false;    // experiment: drain on the caller stream
     bool drain_after_gather = true;  // side drain after the step's gather (FRUGAL_DRAIN_AT=sched: after the scheduler)
     int64_t capT;                // max owned rows touched per step

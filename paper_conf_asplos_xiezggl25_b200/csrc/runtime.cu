@@ -356,7 +356,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     // the deadline-(s+1) part of the drain (the next gate waits for it) may run wider
     c->side_first_blocks = getenv("FRUGAL_SIDE_FIRST_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_FIRST_BLOCKS"))
                                                                : c->side_blocks;
-    c->gather_blocks = getenv("FRUGAL_GATHER_BLOCKS") ? atoi(getenv("FRUGAL_GATHER_BLOCKS")) : 74;
+    c->gather_blocks = getenv("FRUGAL_GATHER_BLOCKS") ? atoi(getenv("FRUGAL_GATHER_BLOCKS")) : 120;
     c->side_inline = getenv("FRUGAL_SIDE_INLINE") && atoi(getenv("FRUGAL_SIDE_INLINE"));
     c->drain_after_gather = !(getenv("FRUGAL_DRAIN_AT") && !strcmp(getenv("FRUGAL_DRAIN_AT"), "sched"));
     c->capT = std::max<int64_t>(1, std::min<int64_t>((int64_t)c->n * c->M, c->No));
