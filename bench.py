@@ -63,6 +63,11 @@ def parse():
     ap.add_argument("--host-layout", default="id", choices=["id", "freq"],
                     help="host-table layout: id order, or frequency order over the hot-set window "
                          "(frugal_config.host_order)")
+    ap.add_argument("--no-fused-lookup", dest="fused_lookup", action="store_false",
+                    help="expand the gathered rows to [B*F][d] in frugal_lookup and hand them to the glue; "
+                         "default: the REC glue reads the gathered distinct rows through the inverse index "
+                         "(frugal_lookup / frugal_dot_model with NULL emb, no expand; "
+                         "profiles/r1_sweep32_fused_lookup.txt)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for barriers / the max-over-ranks timing only")
     return ap.parse_args()
@@ -328,9 +333,12 @@ def main():
         dist.all_to_all_single(out, src, rc, sc)
         return out.to(dev, non_blocking=True)
 
+    fused = args.fused_lookup and not kg and not a2a
+    emb_arg = None if fused else emb
+
     def lookup(s):
         if not a2a:
-            fr.lookup(s, emb)
+            fr.lookup(s, emb_arg)
             return
         sc = fr.a2a_requests(s, ids_send)
         sct = torch.tensor(sc, dtype=torch.int64, device=coll_dev)
@@ -361,7 +369,7 @@ def main():
         if kg:
             fr.transe_model(s, emb, cfg.neg_chunk, cfg.gamma, grad, loss[s:s + 1])
         else:
-            fr.dot_model(s, emb, x_d[s % SG], y_d[s % SG], grad, loss[s:s + 1])
+            fr.dot_model(s, emb_arg, x_d[s % SG], y_d[s % SG], grad, loss[s:s + 1])
         backward(s)
 
     copy_stream = torch.cuda.Stream(dev)
@@ -389,7 +397,7 @@ def main():
         if kg:
             fr.transe_model(s, emb, cfg.neg_chunk, cfg.gamma, grad, loss[s:s + 1])
         else:
-            fr.dot_model(s, emb, x_e[b], y_e[b], grad, loss[s:s + 1])
+            fr.dot_model(s, emb_arg, x_e[b], y_e[b], grad, loss[s:s + 1])
         xy_free[b].record(stream)
         backward(s)
         loss_h[s:s + 1].copy_(loss[s:s + 1], non_blocking=True)  # the step's result back to the host
@@ -462,7 +470,8 @@ def main():
     for nm, h, c_ in [("urgent", "urgent_hot", "urgent_cold"), ("side", "side_hot", "side_cold")]:
         per[nm] = dict(bound="host-link d2h", bytes=(cnt[h] + cnt[c_]) * r / K, ms=ph[nm], peak=link["d2h"])
     # a4 expand: out[i] = rows[inv[i]]: write r + read r + 4 B index per position
-    per["expand"] = dict(bound="hbm", bytes=(cnt["positions"] * (2 * r + 4)) / K, ms=ph["expand"], peak=hbm_peak)
+    per["expand"] = dict(bound="hbm", bytes=0.0 if fused else (cnt["positions"] * (2 * r + 4)) / K,
+                         ms=ph["expand"], peak=hbm_peak)
     # a6 segment-reduce: read r + 4 B per position, write r + 4 B per unique row
     per["segred"] = dict(bound="hbm", bytes=(cnt["positions"] * (r + 4) + cnt["unique"] * (r + 4)) / K,
                          ms=ph["segred"], peak=hbm_peak)
@@ -547,6 +556,7 @@ def main():
                    "flush_mode": args.mode, "exchange": "host table + mailbox (P2F)" if not a2a else
                    "all-to-all over the process group (comparison path)",
                    "peer_reads": bool(args.peer and world > 1),
+                   "lookup": "fused into the glue (no expand)" if fused else "expanded [B*F][d]",
                    "parallelism": f"dp{world} (owner-sharded rows, shared pinned host table)",
                    "l2": "inputs larger than L2: host table %.1f GB, HBM cache %.0f MB, %d distinct id batches "
                          "(%.0f MB) cycled" % (cfg.n_rows * r * (1 if (no_host_state or not adag) else 2) / 1e9,

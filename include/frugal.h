@@ -141,7 +141,11 @@ frugal_status frugal_step(frugal_ctx* ctx, int64_t s, const int64_t* ids_next_al
 /* Forward query (§3.2): d_out[i] = current value of row ids[rank][i], for
    i < counts[rank]*slots, row-major fp32 [count*slots][dim] in device memory.  Owned
    hot rows come from the HBM cache, all others from the host table by zero-copy
-   loads (CPU bypass, §3.1). */
+   loads (CPU bypass, §3.1).  d_out == NULL (fused lookup, REC glue only):
+   the expand is skipped and the gathered distinct rows stay in the library's step
+   buffer; frugal_dot_model(s) must then be called with d_emb == NULL and reads row
+   ids[rank][i] through the dedup's inverse index (same values, no [count*slots][dim]
+   round trip through HBM).  frugal_transe_model returns FRUGAL_EINVAL after it. */
 frugal_status frugal_lookup(frugal_ctx* ctx, int64_t s, float* d_out, frugal_stream stream);
 
 /* Backward update (§3.2, §3.3): d_grad has d_out's shape.
@@ -180,7 +184,9 @@ const char* frugal_last_error(void);
    per sample b: S = sum_f e_f (f ascending, fp32), z = 0.5(|S|^2 - sum_f |e_f|^2)
    + <x_b,S> (fp64), p = sigmoid(z); loss += softplus(z) - y z (fp64, into *d_loss);
    grad_f = c*((S - e_f) + x_b), c = (float)((p - y)/nb), nb = samples of step s over
-   all ranks.  d_emb/d_grad: [count*slots][dim]; x: [count][dim]; y: [count] (device). */
+   all ranks.  d_emb/d_grad: [count*slots][dim]; x: [count][dim]; y: [count] (device).
+   d_emb == NULL exactly when lookup(s) ran with d_out == NULL (fused lookup), else
+   FRUGAL_EINVAL. */
 frugal_status frugal_dot_model(frugal_ctx* ctx, int64_t s, const float* d_emb, const float* d_x,
                                const float* d_y, float* d_grad, double* d_loss,
                                frugal_stream stream);

@@ -224,6 +224,7 @@ struct frugal_ctx {
     int64_t next_prefetch = 0;  // next t expected by prefetch/step
     int64_t cur_step = -1;
     int phase_in_step = 0;  // 0 = need step, 1 = need lookup, 2 = need backward
+    bool lookup_fused = false;  // lookup(s) ran with d_out == NULL: the glue reads rows_buf through inv
     bool ids_exhausted = false;
 
     // KG glue scratch (allocated on first use): W [batch][C] and A [batch] (fp64)
@@ -265,8 +266,8 @@ void launch_split_early(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st)
 void launch_mail_header(frugal_ctx* c, QueueSlot& q, int par, cudaStream_t st);
 void launch_transe_model(frugal_ctx* c, QueueSlot& q, const float* emb, int C, double gamma, float* grad,
                          double* loss, int64_t nb, double* Wm, double* A, cudaStream_t st);
-void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const float* x, const float* y,
-                      float* grad, double* loss, int64_t nb, cudaStream_t st);
+void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const int32_t* inv, const float* x,
+                      const float* y, float* grad, double* loss, int64_t nb, cudaStream_t st);
 void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, float* dest, cudaStream_t st, int64_t fused_step = -1);
 void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, const float* recv, const int32_t* roff,
                       cudaStream_t st);

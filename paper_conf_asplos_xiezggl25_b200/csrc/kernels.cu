@@ -1068,11 +1068,18 @@ void launch_split_early(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st)
 }
 
 // ============================================================================ model glue
+// row f of sample b: the expanded [count*F][d] array, or (fused lookup, inv != NULL) the
+// gathered unique row inv[b*F + f] -- the expand folded into the glue's loads
+template <bool FUSED>
+__device__ __forceinline__ const float* glue_row(const float* emb, const int32_t* inv, int64_t b, int F, int f, int d) {
+    return FUSED ? emb + (int64_t)__ldg(inv + b * F + f) * d : emb + (b * F + f) * d;
+}
 // warp per sample; lane j holds element j (+32q) of S and, when F <= FC, of every e_f
 // in registers (one HBM read of the embeddings); the loss is block-reduced, one atomic
 // per block.
-template <int J, int FC>
-__global__ void __launch_bounds__(256) k_dot_model(const float* __restrict__ emb, const float* __restrict__ x,
+template <int J, int FC, bool FUSED>
+__global__ void __launch_bounds__(256) k_dot_model(const float* __restrict__ emb, const int32_t* __restrict__ inv,
+                                                   const float* __restrict__ x,
                                                    const float* __restrict__ y, float* __restrict__ grad,
                                                    double* loss, int count, int F, int d, double nb) {
     __shared__ double sl[8];
@@ -1081,7 +1088,6 @@ __global__ void __launch_bounds__(256) k_dot_model(const float* __restrict__ emb
     const int nw = (gridDim.x * blockDim.x) >> 5;
     double lsum = 0.0;
     for (int b = wid; b < count; b += nw) {
-        const float* e0 = emb + (int64_t)b * F * d;
         float S[J];
         float ec[FC > 0 ? FC : 1][J];
 #pragma unroll
@@ -1093,7 +1099,7 @@ __global__ void __launch_bounds__(256) k_dot_model(const float* __restrict__ emb
 #pragma unroll
                 for (int q = 0; q < J; q++) {
                     int j = lane + 32 * q;
-                    ec[f][q] = (f < F && j < d) ? e0[f * d + j] : 0.0f;
+                    ec[f][q] = (f < F && j < d) ? glue_row<FUSED>(emb, inv, b, F, f, d)[j] : 0.0f;
                 }
             }
 #pragma unroll
@@ -1108,11 +1114,12 @@ __global__ void __launch_bounds__(256) k_dot_model(const float* __restrict__ emb
             }
         } else {
             for (int f = 0; f < F; f++) {
+                const float* ef = glue_row<FUSED>(emb, inv, b, F, f, d);
 #pragma unroll
                 for (int q = 0; q < J; q++) {
                     int j = lane + 32 * q;
                     if (j < d) {
-                        float v = e0[f * d + j];
+                        float v = ef[j];
                         S[q] = __fadd_rn(S[q], v);
                         ee += (double)v * (double)v;
                     }
@@ -1154,10 +1161,11 @@ __global__ void __launch_bounds__(256) k_dot_model(const float* __restrict__ emb
             }
         } else {
             for (int f = 0; f < F; f++) {
+                const float* ef = glue_row<FUSED>(emb, inv, b, F, f, d);
 #pragma unroll
                 for (int q = 0; q < J; q++) {
                     int j = lane + 32 * q;
-                    if (j < d) g0[f * d + j] = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[q], e0[f * d + j]), xv[q]));
+                    if (j < d) g0[f * d + j] = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[q], ef[j]), xv[q]));
                 }
             }
         }
@@ -1171,15 +1179,19 @@ __global__ void __launch_bounds__(256) k_dot_model(const float* __restrict__ emb
     }
 }
 
-void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const float* x, const float* y, float* grad,
-                      double* loss, int64_t nb, cudaStream_t st) {
+void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const int32_t* inv, const float* x,
+                      const float* y, float* grad, double* loss, int64_t nb, cudaStream_t st) {
     int count = q.h_counts[c->g];
     if (count <= 0) return;
     int J = (c->d + 31) / 32;
     int grid = grid_for((int64_t)count * 32, 256, 4);
     const double nbd = (double)nb;
     const bool cache = c->F <= 32;
-#define DM(JJ, FC) k_dot_model<JJ, FC><<<grid, 256, 0, st>>>(emb, x, y, grad, loss, count, c->F, c->d, nbd)
+#define DM(JJ, FC)                                                                                     \
+    do {                                                                                               \
+        if (inv) k_dot_model<JJ, FC, true><<<grid, 256, 0, st>>>(emb, inv, x, y, grad, loss, count, c->F, c->d, nbd); \
+        else k_dot_model<JJ, FC, false><<<grid, 256, 0, st>>>(emb, inv, x, y, grad, loss, count, c->F, c->d, nbd);    \
+    } while (0)
     if (J <= 1) { if (cache) DM(1, 32); else DM(1, 0); }
     else if (J <= 2) { if (cache) DM(2, 32); else DM(2, 0); }
     else if (J <= 4) DM(4, 0);

@@ -900,7 +900,7 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
 }
 
 extern "C" frugal_status frugal_lookup(frugal_ctx* c, int64_t s, float* d_out, frugal_stream stream) {
-    if (!c || !d_out) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    if (!c) { set_err("NULL argument"); return FRUGAL_EINVAL; }
     if (c->a2a) { set_err("context uses FRUGAL_F_A2A: use frugal_a2a_requests/serve/lookup"); return FRUGAL_ESTATE; }
     if (c->phase_in_step != 1 || s != c->cur_step) {
         set_err("lookup(%lld) out of order", (long long)s);
@@ -927,7 +927,8 @@ extern "C" frugal_status frugal_lookup(frugal_ctx* c, int64_t s, float* d_out, f
             if (r) return r;
         }
     }
-    {
+    c->lookup_fused = d_out == nullptr;
+    if (d_out) {
         Timer tm(c, PH_EXPAND, st);
         launch_expand(c, q, rows, d_out, st);
     }
@@ -938,17 +939,22 @@ extern "C" frugal_status frugal_lookup(frugal_ctx* c, int64_t s, float* d_out, f
 
 extern "C" frugal_status frugal_dot_model(frugal_ctx* c, int64_t s, const float* d_emb, const float* d_x,
                                           const float* d_y, float* d_grad, double* d_loss, frugal_stream stream) {
-    if (!c || !d_emb || !d_x || !d_y || !d_grad || !d_loss) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    if (!c || !d_x || !d_y || !d_grad || !d_loss) { set_err("NULL argument"); return FRUGAL_EINVAL; }
     if (c->phase_in_step != 2 || s != c->cur_step) {
         set_err("dot_model(%lld) must follow lookup(%lld)", (long long)s, (long long)s);
         return FRUGAL_ESTATE;
+    }
+    if ((d_emb == nullptr) != c->lookup_fused) {
+        set_err("dot_model: d_emb must be NULL exactly when lookup(%lld) ran with d_out == NULL", (long long)s);
+        return FRUGAL_EINVAL;
     }
     cudaStream_t st = (cudaStream_t)stream;
     QueueSlot& q = c->q[s % c->QN];
     int64_t nb = 0;
     for (int r = 0; r < c->n; r++) nb += q.h_counts[r];
     Timer tm(c, PH_MODEL, st);
-    launch_dot_model(c, q, d_emb, d_x, d_y, d_grad, d_loss, nb, st);
+    if (d_emb) launch_dot_model(c, q, d_emb, nullptr, d_x, d_y, d_grad, d_loss, nb, st);
+    else launch_dot_model(c, q, c->rows_buf[s & 1], q.inv, d_x, d_y, d_grad, d_loss, nb, st);
     CKL();
     return FRUGAL_OK;
 }
@@ -962,6 +968,7 @@ extern "C" frugal_status frugal_transe_model(frugal_ctx* c, int64_t s, const flo
         set_err("transe_model(%lld) must follow lookup(%lld)", (long long)s, (long long)s);
         return FRUGAL_ESTATE;
     }
+    if (c->lookup_fused) { set_err("transe_model needs the expanded rows: lookup with d_out != NULL"); return FRUGAL_EINVAL; }
     if (c->kg_C != chunk) {
         cudaFree(c->kg_W);
         cudaFree(c->kg_A);
@@ -1072,6 +1079,7 @@ extern "C" frugal_status frugal_a2a_lookup(frugal_ctx* c, int64_t s, const float
         if (r) return r;
     }
     CKL();
+    c->lookup_fused = false;
     c->phase_in_step = 2;
     return check_err_word(c);
 }

@@ -32,8 +32,11 @@ def make_context(st, rank=0, device=0, shm_name=None, flags=0, hot=None, mode=F.
 class Trainer:
     """Runs the stream on one rank.  Inputs are uploaded per step from host arrays."""
 
-    def __init__(self, fr: F.Frugal, st, rank=0, device=0):
+    def __init__(self, fr: F.Frugal, st, rank=0, device=0, fused_lookup=False):
         self.fr, self.st, self.rank = fr, st, rank
+        # fused lookup (REC glue only): lookup(s, None) + dot_model(s, None, ...) -- the
+        # glue reads the gathered distinct rows through the inverse index, no expand
+        self.fused = fused_lookup and st.cfg.model != "transe"
         self.dev = torch.device("cuda", device)
         B, Fs, d = st.ids.shape[2] // st.cfg.slots, st.cfg.slots, st.cfg.dim
         self.emb = torch.empty(B * Fs, d, device=self.dev)
@@ -61,13 +64,13 @@ class Trainer:
             fr.step(s)
         if on_schedule:
             on_schedule(s)
-        fr.lookup(s, self.emb)
+        fr.lookup(s, None if self.fused else self.emb)
         if st.cfg.model == "transe":
             fr.transe_model(s, self.emb, st.cfg.neg_chunk, st.cfg.gamma, self.grad, self.loss[s:s + 1])
         else:
             x = torch.from_numpy(st.x[s, self.rank]).to(self.dev, non_blocking=False)
             y = torch.from_numpy(st.y[s, self.rank]).to(self.dev, non_blocking=False)
-            fr.dot_model(s, self.emb, x, y, self.grad, self.loss[s:s + 1])
+            fr.dot_model(s, None if self.fused else self.emb, x, y, self.grad, self.loss[s:s + 1])
         fr.backward_update(s, self.grad)
         self.s += 1
 

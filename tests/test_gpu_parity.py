@@ -23,7 +23,7 @@ def _F():
 
 
 def run_parity(st, *, flags=None, mode=None, hot=None, check_dedup=True, check_sched=True, steps=None,
-               sample_rows=None, oracle_kw=None):
+               sample_rows=None, oracle_kw=None, fused=False):
     """Run the stream on cuda:0 (world 1) and on the oracle; assert the bars."""
     F = _F()
     from paper_conf_asplos_xiezggl25_b200.harness import Trainer, make_context
@@ -32,7 +32,7 @@ def run_parity(st, *, flags=None, mode=None, hot=None, check_dedup=True, check_s
     hot = st.hot if hot is None else hot
     fr = make_context(st, flags=flags, mode=mode, hot=hot)
     o = Oracle(st, hot=hot, write_through=(mode == F.MODE_WRITE_THROUGH), **(oracle_kw or {}))
-    tr = Trainer(fr, st)
+    tr = Trainer(fr, st, fused_lookup=fused)
     S = st.steps if steps is None else steps
     L = st.cfg.lookahead
     if check_dedup:
@@ -186,6 +186,62 @@ def test_criteo_kaggle_full_size_sampled():
     r["fr"].close()
 
 
+def test_fused_lookup_parity():
+    """Fused lookup (lookup/dot_model with NULL emb: the glue reads the gathered distinct
+    rows through inv, no expand): tables, losses and sets bit-exact as with the expand."""
+    st = W.gen_stream(tiny1(), 60)
+    r = run_parity(st, fused=True)
+    assert r["exact"]
+    r["fr"].close()
+
+
+@pytest.mark.parametrize("dim,tables", [(8, 3), (64, 5), (32, 40), (400, 3)])
+def test_fused_lookup_shapes(dim, tables):
+    """Every glue variant (J = 1..13 lanes per row, F <= 32 register-cached or F > 32)
+    and ragged / empty batches with the fused lookup."""
+    cfg = W.WorkloadConfig("fz", [500 + 37 * i for i in range(tables)], dim=dim, batch=64, world=1,
+                           lookahead=4, age_out=3)
+    rng = np.random.default_rng(dim + tables)
+    counts = rng.integers(0, 65, size=(20, 1)).astype(np.int32)
+    counts[5] = 0
+    st = W.gen_stream(cfg, 20, counts=counts)
+    run_parity(st, fused=True)["fr"].close()
+
+
+def test_fused_lookup_criteo_full_size_sampled():
+    cfg = W.config("criteo_kaggle", world=1)
+    st = W.gen_stream(cfg, 14)
+    rng = np.random.default_rng(1)
+    touched = np.unique(st.ids[:6, 0].ravel())
+    sample = np.sort(rng.choice(touched, size=20000, replace=False))
+    run_parity(st, steps=6, sample_rows=sample, fused=True)["fr"].close()
+
+
+def test_fused_lookup_errors():
+    """dot_model's emb must be NULL exactly when lookup's out was."""
+    F = _F()
+    import torch
+    from paper_conf_asplos_xiezggl25_b200.harness import make_context
+    st = W.gen_stream(tiny1(batch=32, lookahead=3), 6)
+    fr = make_context(st)
+    for t in range(3):
+        fr.prefetch(t, st.ids[t], st.counts[t])
+    fr.step(0, st.ids[3], st.counts[3])
+    fr.lookup(0, None)
+    B, d = 32, st.cfg.dim
+    emb = torch.empty(B * st.cfg.slots, d, device="cuda")
+    x = torch.from_numpy(st.x[0, 0]).cuda()
+    y = torch.from_numpy(st.y[0, 0]).cuda()
+    loss = torch.zeros(1, dtype=torch.float64, device="cuda")
+    with pytest.raises(F.FrugalError) as e:
+        fr.dot_model(0, emb, x, y, emb, loss)
+    assert e.value.status == -1
+    with pytest.raises(F.FrugalError):
+        fr.transe_model(0, None, 4, 1.0, emb, loss)
+    fr.dot_model(0, None, x, y, emb, loss)
+    fr.close()
+
+
 def test_invalid_id_fails_loudly():
     F = _F()
     from paper_conf_asplos_xiezggl25_b200.harness import Trainer, make_context
@@ -245,7 +301,8 @@ def test_host_layout_errors():
 
 @pytest.mark.parametrize("env", [{"FRUGAL_EARLY": "1"}, {"FRUGAL_DRAIN_AT": "sched"},
                                  {"FRUGAL_EARLY": "1", "FRUGAL_DRAIN_AT": "sched"}, {"FRUGAL_SIDE_INLINE": "1"},
-                                 {"FRUGAL_NO_POOL_HITS": "1"}, {"FRUGAL_FUSE_OPT": "0"}, {"FRUGAL_FLUSH_TMA": "2"}])
+                                 {"FRUGAL_NO_POOL_HITS": "1"}, {"FRUGAL_FUSE_OPT": "0"}, {"FRUGAL_FLUSH_TMA": "2"},
+                                 {"FRUGAL_EARLY": "1", "FUSED": "1"}])
 def test_pipeline_modes_parity(env):
     """The optional schedules (early gather of the next step, drain after the gather,
     inline drain) keep every artefact bit-exact (run in a subprocess: the knobs are read
@@ -254,7 +311,8 @@ def test_pipeline_modes_parity(env):
     import sys
     code = ("import sys; sys.path.insert(0, '.');"
             "from tests.test_gpu_parity import run_parity, tiny1; from paper_conf_asplos_xiezggl25_b200 import workload as W;"
-            "st = W.gen_stream(tiny1(batch=128, lookahead=4, age_out=2), 40); r = run_parity(st); r['fr'].close();"
+            "import os; st = W.gen_stream(tiny1(batch=128, lookahead=4, age_out=2), 40);"
+            "r = run_parity(st, fused=bool(os.environ.get('FUSED'))); r['fr'].close();"
             "print('OK', r['exact'])")
     e = dict(os.environ)
     e.update(env)
