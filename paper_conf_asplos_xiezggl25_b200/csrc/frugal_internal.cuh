@@ -104,6 +104,7 @@ struct frugal_ctx {
     std::vector<int32_t> hs_host;    // host copy (frugal_read_host)
     int side_first_blocks = 20;      // grid cap of the drain's deadline-(s+1) part
     int flush_tma = 0;               // flushes by TMA bulk stores: 0 none, 1 side drain, 2 all (FRUGAL_FLUSH_TMA; measured no gain: profiles/r1_sweep21_flush_tma.txt)
+    int glue_cache = -1;         // REC glue keeps a sample's rows in registers (F <= 32): -1 auto, 0 never, 1 always
     bool fuse_opt = true;        // world 1: a8 fused into a6 (k_segreduce / k_segred_combine)
     int gather_blocks = 120;     // grid cap of the zero-copy gathers (120 CTAs: +3% over 74 and 148 in the step, profiles/r1_sweep34_gather_grid.txt)
     bool side_inline = false;    // experiment: drain on the caller stream

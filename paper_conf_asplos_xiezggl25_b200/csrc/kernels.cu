@@ -1094,12 +1094,17 @@ __global__ void __launch_bounds__(256) k_dot_model(const float* __restrict__ emb
         for (int q = 0; q < J; q++) S[q] = 0.0f;
         double ee = 0.0;
         if (FC > 0) {
+            // fused lookup: one coalesced load of the sample's F (<= 32) row indices, then
+            // broadcast by shuffle (instead of F same-address loads per warp)
+            const int32_t myiv = (FUSED && lane < F) ? __ldg(inv + b * F + lane) : 0;
 #pragma unroll
             for (int f = 0; f < FC; f++) {
+                const int32_t rf = FUSED ? __shfl_sync(FULL, myiv, f) : 0;
+                const float* ef = FUSED ? emb + (int64_t)rf * d : emb + (b * F + f) * d;
 #pragma unroll
                 for (int q = 0; q < J; q++) {
                     int j = lane + 32 * q;
-                    ec[f][q] = (f < F && j < d) ? glue_row<FUSED>(emb, inv, b, F, f, d)[j] : 0.0f;
+                    ec[f][q] = (f < F && j < d) ? ef[j] : 0.0f;
                 }
             }
 #pragma unroll
@@ -1186,7 +1191,9 @@ void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const int32
     int J = (c->d + 31) / 32;
     int grid = grid_for((int64_t)count * 32, 256, 4);
     const double nbd = (double)nb;
-    const bool cache = c->F <= 32;
+    // register-cached rows: one read per row, but ~180 registers/thread (8 warps/SM); the
+    // uncached variant re-reads each row for the gradient (54 registers)
+    const bool cache = c->F <= 32 && (c->glue_cache < 0 ? true : c->glue_cache != 0);
 #define DM(JJ, FC)                                                                                     \
     do {                                                                                               \
         if (inv) k_dot_model<JJ, FC, true><<<grid, 256, 0, st>>>(emb, inv, x, y, grad, loss, count, c->F, c->d, nbd); \

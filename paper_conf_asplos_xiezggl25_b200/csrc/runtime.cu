@@ -351,6 +351,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     // side-drain flushes by TMA bulk stores (FRUGAL_FLUSH_TMA=0 none, 1 side, 2 all)
     if (getenv("FRUGAL_FLUSH_TMA")) c->flush_tma = atoi(getenv("FRUGAL_FLUSH_TMA"));
     // world 1: optimizer fused into the segment-reduce (FRUGAL_FUSE_OPT=0: two kernels)
+    if (getenv("FRUGAL_GLUE_CACHE")) c->glue_cache = atoi(getenv("FRUGAL_GLUE_CACHE"));
     c->fuse_opt = !(getenv("FRUGAL_FUSE_OPT") && !atoi(getenv("FRUGAL_FUSE_OPT")));
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 20;
     // the deadline-(s+1) part of the drain (the next gate waits for it) may run wider
