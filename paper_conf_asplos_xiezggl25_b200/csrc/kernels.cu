@@ -1191,9 +1191,12 @@ void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const int32
     int J = (c->d + 31) / 32;
     int grid = grid_for((int64_t)count * 32, 256, 4);
     const double nbd = (double)nb;
-    // register-cached rows: one read per row, but ~180 registers/thread (8 warps/SM); the
-    // uncached variant re-reads each row for the gradient (54 registers)
-    const bool cache = c->F <= 32 && (c->glue_cache < 0 ? true : c->glue_cache != 0);
+    // register-cached rows: one read per row, but 180-250 registers/thread (8 warps/SM); the
+    // uncached variant re-reads each row for the gradient (48-54 registers).  With the fused
+    // lookup the re-reads hit the L2-resident distinct rows: uncached wins from d > 32 on
+    // (Avazu d 64: glue 134 -> 51 us, +23 % samples/s), cached stays at d <= 32
+    // (Criteo: within noise; profiles/r1_sweep35_glue.txt)
+    const bool cache = c->F <= 32 && (c->glue_cache < 0 ? (J <= 1 || inv == nullptr) : c->glue_cache != 0);
 #define DM(JJ, FC)                                                                                     \
     do {                                                                                               \
         if (inv) k_dot_model<JJ, FC, true><<<grid, 256, 0, st>>>(emb, inv, x, y, grad, loss, count, c->F, c->d, nbd); \

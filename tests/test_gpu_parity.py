@@ -302,7 +302,8 @@ def test_host_layout_errors():
 @pytest.mark.parametrize("env", [{"FRUGAL_EARLY": "1"}, {"FRUGAL_DRAIN_AT": "sched"},
                                  {"FRUGAL_EARLY": "1", "FRUGAL_DRAIN_AT": "sched"}, {"FRUGAL_SIDE_INLINE": "1"},
                                  {"FRUGAL_NO_POOL_HITS": "1"}, {"FRUGAL_FUSE_OPT": "0"}, {"FRUGAL_FLUSH_TMA": "2"},
-                                 {"FRUGAL_EARLY": "1", "FUSED": "1"}])
+                                 {"FRUGAL_EARLY": "1", "FUSED": "1"}, {"FRUGAL_GLUE_CACHE": "0", "FUSED": "1"},
+                                 {"FRUGAL_GLUE_CACHE": "0"}])
 def test_pipeline_modes_parity(env):
     """The optional schedules (early gather of the next step, drain after the gather,
     inline drain) keep every artefact bit-exact (run in a subprocess: the knobs are read
