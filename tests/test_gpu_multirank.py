@@ -14,7 +14,7 @@ from paper_conf_asplos_xiezggl25_b200 import workload as W
 pytestmark = pytest.mark.gpu
 
 
-def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False):
+def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False, fused=False):
     try:
         import torch
         from paper_conf_asplos_xiezggl25_b200 import frugal as F
@@ -29,7 +29,7 @@ def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False):
             dist.init_process_group("gloo", rank=rank, world_size=2)
             tr = A2ATrainer(fr, st, rank=rank, dist=dist, host_staging=True)
         else:
-            tr = Trainer(fr, st, rank=rank)
+            tr = Trainer(fr, st, rank=rank, fused_lookup=fused)
         sched = []
         for s in range(st.steps):
             got = {}
@@ -54,7 +54,7 @@ def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False):
         q.put((rank, traceback.format_exc()))
 
 
-def run_two_ranks(st, timeout=600, a2a=False, peer=False):
+def run_two_ranks(st, timeout=600, a2a=False, peer=False, fused=False):
     import socket
     ctx = mp.get_context("spawn")
     barrier = ctx.Barrier(2)
@@ -64,7 +64,7 @@ def run_two_ranks(st, timeout=600, a2a=False, peer=False):
     sk.bind(("127.0.0.1", 0))
     port = sk.getsockname()[1]
     sk.close()
-    ps = [ctx.Process(target=_rank_main, args=(r, st, shm, barrier, q, a2a, port, peer)) for r in range(2)]
+    ps = [ctx.Process(target=_rank_main, args=(r, st, shm, barrier, q, a2a, port, peer, fused)) for r in range(2)]
     for p in ps:
         p.start()
     out = {}
@@ -138,13 +138,15 @@ def test_two_ranks_one_gpu_parity(opt, a2a, peer, dyn, layout):
 
 
 
-def test_configs0_two_ranks_exact_shape():
+@pytest.mark.parametrize("fused", [False, True])
+def test_configs0_two_ranks_exact_shape(fused):
     """BASELINE.json configs[0] as stated: 1 table 10^4 x 16, batch 256, 20 steps, 2 GPUs
-    (here: 2 rank processes sharing one B200), Zipf ids."""
+    (here: 2 rank processes sharing one B200), Zipf ids.  fused: the bench's default fused
+    lookup (glue reads each rank's gathered distinct rows through its inverse index)."""
     from oracle.oracle import Oracle
     cfg = W.config("tiny")  # world 2, batch 256
     st = W.gen_stream(cfg, 20)
-    out = run_two_ranks(st)
+    out = run_two_ranks(st, fused=fused)
     o = Oracle(st)
     for s in range(st.steps):
         o.step()
