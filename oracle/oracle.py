@@ -16,6 +16,8 @@ import numpy as np
 HERE = os.path.dirname(os.path.abspath(__file__))
 SRC = os.path.join(HERE, "frugal_oracle.c")
 LIB = os.path.join(HERE, "liboracle.so")
+# tools/oracle_mutants.py points this at a deliberately broken build (mutation testing of the pins)
+LIB_OVERRIDE = os.environ.get("FRUGAL_ORACLE_LIB")
 
 INF = 2**31 - 1
 L_URGENT, L_DEFERRED, L_DEFERRED_P, L_AGEOUT, L_FINAL, L_UPDATED, L_INF, L_EXEMPT, L_TRANSITION = range(9)
@@ -34,6 +36,8 @@ class _Cfg(C.Structure):
 
 def build(force: bool = False) -> str:
     """Compile the oracle (plain C, -O2, no FMA contraction, no fast-math)."""
+    if LIB_OVERRIDE:
+        return LIB_OVERRIDE
     if force or not os.path.exists(LIB) or os.path.getmtime(LIB) < os.path.getmtime(SRC):
         subprocess.check_call(["gcc", "-O2", "-std=c11", "-ffp-contract=off", "-fno-fast-math",
                                "-fPIC", "-shared", "-o", LIB, SRC, "-lm"])

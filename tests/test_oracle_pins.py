@@ -386,3 +386,165 @@ def test_transe_glue_vs_torch_fp64():
             np.add.at(acc, st.ids[s, g, :cnt * F], o.grad(g)[:cnt * F].astype(np.float64))
         ref = E.grad.numpy()
         assert np.abs(acc - ref).max() <= 1e-6 * max(1e-3, np.abs(ref).max())
+
+
+# ----------------------------------------------------------------------------- long segments (R23)
+def _const_stream(seq, dim=4, world=1):
+    """One step, one rank, slot 0 = row seq[b] for sample b; model 'const' makes the glue
+    gradient of position b exactly x_b (oracle OR_MODEL_CONST: linear loss <x_b, e>)."""
+    cfg = W.WorkloadConfig("seg", [max(seq) + 1], dim=dim, batch=len(seq), world=world,
+                           lookahead=2, age_out=1, cache_ratio=0.0)
+    return W.stream_from_lists(cfg, [[list(seq)]])
+
+
+@pytest.mark.parametrize("n", [1, 63, 64, 65, 127, 128, 129, 1000, 1537])
+def test_partials_long_segments_exact_integers(n):
+    """Partial of a row with n occurrences (up to 1537: 25 chunks of the R23 chunked
+    order, ragged last chunk) when every gradient is a small integer: the fp32 sum is
+    then exact in ANY order, so the oracle's partial must equal the integer sum bit for
+    bit (a dropped, repeated or mis-indexed occurrence anywhere changes it).  Rows with
+    1 and 2 occurrences sit beside it (neighbouring segments must not bleed in)."""
+    rng = np.random.default_rng(n)
+    seq = [0] * n + [1] + [2, 2]
+    rng.shuffle(seq)
+    st = _const_stream(seq)
+    x = rng.integers(-4, 5, size=(len(seq), 4)).astype(np.float32)
+    x[x == 0] = 3.0                    # no zero term: every dropped occurrence shows
+    st.x[0, 0, :len(seq)] = x
+    o = Oracle(st, model="const")
+    o.step()
+    keys, P = o.partial(0)
+    assert keys.tolist() == [0, 1, 2]
+    for r in range(3):
+        exact = x[np.array(seq) == r].astype(np.int64).sum(0)
+        assert np.array_equal(P[r], exact.astype(np.float32)), (r, P[r], exact)
+
+
+def test_partials_long_segment_error_bound():
+    """Random fp32 gradients, 1500 occurrences of one row: |P - exact| <= (64 + n/64) u sum|g|
+    (the textbook bound of a two-level sequential sum with chunks of 64, u = 2^-24; the exact
+    value is the fp64 sum of the same fp32 terms)."""
+    rng = np.random.default_rng(7)
+    n = 1500
+    seq = [0] * n + [1] * 5
+    rng.shuffle(seq)
+    st = _const_stream(seq)
+    x = rng.normal(0, 1, size=(len(seq), 4)).astype(np.float32)
+    st.x[0, 0, :len(seq)] = x
+    o = Oracle(st, model="const")
+    o.step()
+    keys, P = o.partial(0)
+    g = x[np.array(seq) == 0].astype(np.float64)
+    exact = g.sum(0)
+    bound = (64 + n / 64 + 2) * 2.0 ** -24 * np.abs(g).sum(0)
+    assert np.all(np.abs(P[0] - exact) <= bound), (np.abs(P[0] - exact), bound)
+
+
+def test_partials_chunk_order_R23_hand_value():
+    """Reading R23 fixed by a hand-derived value.  Row 0 occurs 128 times: position 0
+    carries 1.0, the other 127 carry 2^-25 = half an ulp of 1.0, so each is lost when added to
+    1.0 (round to nearest, ties to even) but sums exactly with its peers.  Chunks of 64:
+    chunk 0 = 1.0 (its 63 small terms round away one by one), chunk 1 = 64 * 2^-25 = 2^-19
+    (exact), total 1 + 2^-19.  A plain sequential sum would give 1.0, chunks of 32 give
+    1 + 3*2^-20, chunks of 128 or 256 give 1.0."""
+    seq = [0] * 128
+    st = _const_stream(seq, dim=4)
+    x = np.full((128, 4), 2.0 ** -25, dtype=np.float32)
+    x[0] = 1.0
+    st.x[0, 0, :128] = x
+    o = Oracle(st, model="const")
+    o.step()
+    _, P = o.partial(0)
+    assert np.all(P[0] == np.float32(1.0 + 2.0 ** -19)), P[0]
+
+
+# ----------------------------------------------------------------------------- age-out (R9)
+def _trace(per_step, L, D, hot=()):
+    cfg = W.WorkloadConfig("age", [64], dim=4, batch=4, world=1, lookahead=L, age_out=D, cache_ratio=0.0)
+    st = W.stream_from_lists(cfg, per_step)
+    o = Oracle(st, hot=np.array(sorted(hot), dtype=np.int64))
+    out = []
+    for s in range(st.steps):
+        o.step()
+        sch = o.schedule()
+        out.append(dict(age=sch["ageout"].tolist(), urgent=sch["urgent"].tolist(),
+                        deferred=sorted(zip(sch["deferred"].tolist(), sch["deferred_p"].tolist())),
+                        inf=sch["inf"].tolist()))
+    assert o.violations == 0
+    return out, o
+
+
+@pytest.mark.parametrize("D", [1, 2, 3, 5])
+def test_ageout_hand_trace(D):
+    """Reading R9 (a row with no read in sight is held, then
+    flushed by the lazy flushers): a cold row updated at step u and never read again gets
+    priority INF from the scheduler of u+1 and is flushed by the age-out of step u+1+D --
+    exactly D steps after the scheduler that found no read in its window.  Row 10+u is read
+    only at step u (one filler row per step), so the age-out set of step s is exactly
+    {10 + (s-1-D)} for s >= 1+D and empty before; the INF set of step s holds the rows
+    updated at s-1-D+1 .. s-1."""
+    S, L = 12, 3
+    per_step = [[[10 + s]] for s in range(S)]
+    out, o = _trace(per_step, L, D)
+    for s in range(S):
+        exp_age = [10 + (s - 1 - D)] if s >= 1 + D else []
+        assert out[s]["age"] == exp_age, (s, out[s]["age"], exp_age)
+        assert out[s]["urgent"] == [] and out[s]["deferred"] == []
+        exp_inf = [10 + u for u in range(max(0, s - D), s)]
+        assert out[s]["inf"] == exp_inf, (s, out[s]["inf"], exp_inf)
+    # the last scheduler (step S-1) ages out u <= S-2-D: rows updated at S-1-D .. S-1 are
+    # still dirty and go out with the final flush
+    assert o.final_flush().tolist() == [10 + u for u in range(S - 1 - D, S)]
+
+
+def test_ageout_vs_adjust_priority_hand_trace():
+    """Hand trace of the two ways an INF row leaves INF (R9 vs Fig. 6 step 4, L1074-1077).
+    L = 3.  Row 7 is read at steps 0 and 5; rows 20+s fill every step.
+      D = 10: step 1 buckets row 7 INF (no read in [1, 3]); the ingest of step 3+3-1 = 5
+      (AdjustPriority, made by frugal_step(3)) gives it deadline 5: D(3) = {(7, 5)}; never
+      aged out.
+      D = 1: row 7 is aged out by step 0+1+1 = 2, before the read of step 5 enters the
+      window; at step 3 it is clean, so no AdjustPriority, no deferred entry."""
+    per_step = [[[20, 7]], [[21]], [[22]], [[23]], [[24]], [[25, 7]], [[26]], [[27]]]
+    out, _ = _trace(per_step, 3, 10)
+    assert (7, 5) in out[3]["deferred"]
+    assert all(7 not in out[s]["age"] for s in range(len(per_step)))
+    assert all((7, 5) not in out[s]["deferred"] for s in range(len(per_step)) if s != 3)
+    out, _ = _trace(per_step, 3, 1)
+    assert 7 in out[2]["age"]
+    assert all(k != 7 for s in range(len(per_step)) for k, _ in out[s]["deferred"])
+    assert [s for s in range(len(per_step)) if 7 in out[s]["age"]] == [2, 7]  # then re-aged after the update at 5
+
+
+def test_ageout_skips_hot_rows():
+    """R9: hot (cached) rows with no host-reader are never aged out (they stay dirty until a
+    host-reader appears or the final flush).  Row 3 hot, read at step 0 only, D = 1."""
+    per_step = [[[3, 30]], [[31]], [[32]], [[33]], [[34]]]
+    out, o = _trace(per_step, 2, 1, hot={3})
+    assert all(3 not in out[s]["age"] for s in range(5))
+    assert 3 in o.final_flush().tolist()
+
+
+def test_hot_flush_moves_w_only_R8():
+    """Reading R8 by hand: an owner's hot row flushed during training for another rank's read
+    moves w only (its Adagrad state G stays with the owner until the final flush); a cold row
+    moves w and G.  world 2, no age-out in sight (D = 10), L = 2; rows 0 (hot) and 2 (cold)
+    are owned by rank 0.  Step 0: rank 0 reads 0 and 2.  Step 1: rank 1 reads 0 and 2, so
+    both are urgent at step 1 (U(1) = {0, 2}) and the host copies hold their post-step-0
+    values.  G of row 0 on the host is then still G0 = 0; G of row 2 is g0^2 != 0."""
+    cfg = W.WorkloadConfig("r8", [8], dim=4, batch=2, world=2, lookahead=2, age_out=10, cache_ratio=0.0)
+    st = W.stream_from_lists(cfg, [[[0, 2], []], [[], [0, 2]], [[], []]])
+    o = Oracle(st, hot=np.array([0], dtype=np.int64))
+    o.step()
+    w0, G0 = o.read_rows([0, 2])  # values after step 0
+    o.step()
+    assert o.schedule()["urgent"].tolist() == [0, 2]
+    hw, hG = o.host_rows([0, 2])
+    assert np.array_equal(hw, w0)
+    assert np.all(G0 > 0)
+    assert np.all(hG[0] == 0.0) and np.array_equal(hG[1], G0[1])
+    o.step()
+    o.final_flush()
+    w, G = o.read_rows([0, 2])
+    hw, hG = o.host_rows([0, 2])
+    assert np.array_equal(hw, w) and np.array_equal(hG, G)
