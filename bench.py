@@ -276,7 +276,13 @@ def main():
     a2a = args.exchange == "a2a"
     if a2a and world == 1:
         sys.exit("--exchange a2a needs N > 1")
-    fr = make_context(st, rank=rank, device=local, shm_name=shm,
+    nonce = 0
+    if world > 1:  # one run id for the shared segment, drawn by rank 0 (frugal_config.run_nonce)
+        t = torch.tensor([int.from_bytes(os.urandom(7), "little") | 1 if rank == 0 else 0], dtype=torch.int64,
+                         device=coll_dev)
+        dist.broadcast(t, 0)
+        nonce = int(t.item())
+    fr = make_context(st, rank=rank, device=local, shm_name=shm, run_nonce=nonce,
                       flags=F.F_TIMERS | (F.F_NO_HOST_STATE if no_host_state else 0) | (F.F_A2A if a2a else 0)
                       | (F.F_PEER if (args.peer and world > 1) else 0)
                       | (F.F_DYNAMIC_CACHE if args.cache_refresh > 0 else 0),

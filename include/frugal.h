@@ -109,13 +109,19 @@ typedef struct {
                                frequency order (random host writes and reads
                                over a compact footprint run faster on the host link)      */
     int64_t n_order;
+    uint64_t run_nonce;     /* identifies this training run (world > 1 with shm_name: required,
+                               != 0, the same on every rank, e.g. drawn by rank 0 and broadcast
+                               through the process group).  Rank 0 stamps it into the segment
+                               header; other ranks attach only to a segment carrying it, so a
+                               stale segment of a crashed run under the same name is never
+                               used (they re-open the name until rank 0's new one appears).  */
 } frugal_config;
 
 /* Create the context of this rank: validates cfg, maps (and for rank 0 creates and
    initialises) the host table w[N][d] (+ G[N][d] for Adagrad), registers it with
    CUDA (mapped, portable), allocates the HBM cache of the owned hot rows, per-row
-   metadata, sample-queue ring, dirty-row pool and scratch.  Ranks > 0 wait (bounded)
-   for rank 0's table.  On error *out is NULL. */
+   metadata, sample-queue ring, dirty-row pool and scratch.  Ranks > 0 wait (bounded,
+   600 s) for rank 0's table stamped with cfg->run_nonce.  On error *out is NULL. */
 frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out);
 
 /* Sample queue (§3.2, §3.3): enqueue the ids of step t of ALL

@@ -282,4 +282,5 @@ void launch_wait_flags(frugal_ctx* c, int which, uint32_t value, cudaStream_t st
 void launch_set_flag(frugal_ctx* c, int which, uint32_t value, cudaStream_t st);
 void launch_read_rows(frugal_ctx* c, const int32_t* d_lk, int64_t n, float* d_w, float* d_G, cudaStream_t st);
 void launch_read_host(frugal_ctx* c, const int64_t* d_k, int64_t n, float* d_w, float* d_G, cudaStream_t st);
+cudaError_t setup_kernel_attrs();
 }  // namespace frugal

@@ -312,14 +312,6 @@ void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, f
                                                            c->g, d4, (const float4*)grad, (float4*)Pp, mail,
                                                            c->long_q, c->long_cnt, c->long_tasks, c->long_cnt + 1,
                                                            c->dstats, fo)));
-    static unsigned attr_mask = 0;
-    if (!(attr_mask & gs)) {
-        DISPATCH_GS(gs, (cudaFuncSetAttribute(k_segred_chunks<GS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                              (int)kOrderedSmem),
-                         cudaFuncSetAttribute(k_segred_combine<GS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                              (int)kOrderedSmem)));
-        attr_mask |= gs;
-    }
     DISPATCH_GS(gs, (k_segred_chunks<GS><<<kSMs, 256, kOrderedSmem, st>>>(q.pos, d4, (const float4*)grad,
                                                                           (float4*)c->chunk_scratch, c->long_tasks,
                                                                           c->long_cnt + 1)));
@@ -329,6 +321,21 @@ void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, f
                                                                            (const float4*)c->chunk_scratch, c->dstats,
                                                                            fo)));
     c->launches += 3;
+}
+
+// per-device kernel attributes (cudaFuncSetAttribute applies to the current device): called
+// by frugal_init after cudaSetDevice, for every row-group width
+cudaError_t setup_kernel_attrs() {
+    cudaError_t e = cudaSuccess;
+    for (int gs = 1; gs <= 32; gs <<= 1) {
+        DISPATCH_GS(gs, (e = cudaFuncSetAttribute(k_segred_chunks<GS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                  (int)kOrderedSmem)));
+        if (e != cudaSuccess) return e;
+        DISPATCH_GS(gs, (e = cudaFuncSetAttribute(k_segred_combine<GS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                  (int)kOrderedSmem)));
+        if (e != cudaSuccess) return e;
+    }
+    return e;
 }
 
 // mailbox header of (parity, this sender): goff[0..world]

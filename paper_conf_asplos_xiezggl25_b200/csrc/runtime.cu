@@ -78,6 +78,7 @@ struct ShmHeader {
     uint64_t total_bytes;
     int64_t n_rows;
     int32_t dim, world, opt, pad;
+    volatile uint64_t nonce;  // frugal_config.run_nonce of the run that created the segment
 };
 
 size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
@@ -284,6 +285,10 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     if (k.opt != FRUGAL_SGD && k.opt != FRUGAL_ADAGRAD) { set_err("bad opt"); return FRUGAL_EINVAL; }
     if (k.mode != FRUGAL_MODE_P2F && k.mode != FRUGAL_MODE_WRITE_THROUGH) { set_err("bad mode"); return FRUGAL_EINVAL; }
     if (!k.shm_name && k.world != 1) { set_err("world > 1 needs shm_name"); return FRUGAL_EINVAL; }
+    if (k.shm_name && k.world > 1 && k.run_nonce == 0) {
+        set_err("world > 1 needs a run_nonce != 0 (the same on every rank)");
+        return FRUGAL_EINVAL;
+    }
     if ((k.flags & FRUGAL_F_A2A) && k.world < 2) { set_err("FRUGAL_F_A2A needs world > 1"); return FRUGAL_EINVAL; }
     if ((k.flags & FRUGAL_F_PEER) && (k.world < 2 || (k.flags & FRUGAL_F_A2A))) {
         set_err("FRUGAL_F_PEER needs world > 1 and the host-bounced exchange");
@@ -301,8 +306,10 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     for (int64_t i = 0; i < k.n_hot; i++)
         if (k.hot_ids[i] < 0 || k.hot_ids[i] >= k.n_rows) { set_err("hot id out of range"); return FRUGAL_EINVAL; }
     if (cudaSetDevice(k.device) != cudaSuccess) { set_err("cudaSetDevice(%d) failed", k.device); return FRUGAL_ECUDA; }
-    int dev_major = 0;
-    cudaDeviceGetAttribute(&dev_major, cudaDevAttrComputeCapabilityMajor, k.device);
+    if (cudaError_t e = setup_kernel_attrs(); e != cudaSuccess) {
+        set_err("kernel attributes on device %d: %s", k.device, cudaGetErrorString(e));
+        return FRUGAL_ECUDA;
+    }
 
     frugal_ctx* c = new frugal_ctx();
     c->cfg = k;
@@ -388,18 +395,38 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
                 return FRUGAL_ESHM;
             }
             c->shm_owner = true;
+            c->shm_base = mmap(nullptr, total, PROT_READ | PROT_WRITE, MAP_SHARED, c->shm_fd, 0);
         } else {
+            // attach only to the segment of THIS run: rank 0 stamps run_nonce into the header
+            // once the table is initialised; a stale segment left under the same name by a
+            // crashed run (other nonce) is closed and the name re-opened until rank 0's new
+            // segment (created after it unlinked the old one) carries our nonce
             double t0 = now_s();
             while (true) {
                 c->shm_fd = shm_open(k.shm_name, O_RDWR, 0600);
                 struct stat sb;
-                if (c->shm_fd >= 0 && fstat(c->shm_fd, &sb) == 0 && (size_t)sb.st_size == total) break;
+                if (c->shm_fd >= 0 && fstat(c->shm_fd, &sb) == 0 && (size_t)sb.st_size == total) {
+                    void* m = mmap(nullptr, total, PROT_READ | PROT_WRITE, MAP_SHARED, c->shm_fd, 0);
+                    if (m != MAP_FAILED) {
+                        const ShmHeader* h = (const ShmHeader*)m;
+                        if (h->ready == kMagic && h->nonce == k.run_nonce) {
+                            __sync_synchronize();
+                            c->shm_base = m;
+                            break;
+                        }
+                        munmap(m, total);
+                    }
+                }
                 if (c->shm_fd >= 0) { close(c->shm_fd); c->shm_fd = -1; }
-                if (now_s() - t0 > 600) { set_err("timed out attaching shm %s", k.shm_name); delete c; return FRUGAL_ESHM; }
+                if (now_s() - t0 > 600) {
+                    set_err("timed out attaching shm %s (no segment of run %llx)", k.shm_name,
+                            (unsigned long long)k.run_nonce);
+                    delete c;
+                    return FRUGAL_ESHM;
+                }
                 usleep(20000);
             }
         }
-        c->shm_base = mmap(nullptr, total, PROT_READ | PROT_WRITE, MAP_SHARED, c->shm_fd, 0);
     } else {
         c->shm_base = mmap(nullptr, total, PROT_READ | PROT_WRITE, MAP_SHARED | MAP_ANONYMOUS, -1, 0);
     }
@@ -612,18 +639,11 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         hdr->dim = c->d;
         hdr->world = c->n;
         hdr->opt = k.opt;
+        hdr->nonce = k.run_nonce;
         __sync_synchronize();
         hdr->ready = kMagic;
     } else {
-        double t0 = now_s();
-        while (hdr->ready != kMagic) {
-            if (now_s() - t0 > 600) {
-                        set_err("timed out waiting for rank 0's table");
-                free_ctx(c);
-                return FRUGAL_ETIMEOUT;
-            }
-            usleep(20000);
-        }
+        // attached above to a segment whose header is ready and carries this run's nonce
         if (hdr->n_rows != c->N || hdr->dim != c->d || hdr->world != c->n || hdr->opt != k.opt) {
                 set_err("shm table config mismatch with rank 0");
             free_ctx(c);
@@ -643,7 +663,6 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         }
     }
     *out = c;
-    (void)dev_major;
     return FRUGAL_OK;
 }
 

@@ -37,7 +37,8 @@ class Config(C.Structure):
                 ("age_out", C.c_int32), ("opt", C.c_int32), ("lr", C.c_float), ("eps", C.c_float),
                 ("init_accum", C.c_float), ("init_scale", C.c_float), ("init_seed", C.c_uint64),
                 ("hot_ids", C.c_void_p), ("n_hot", C.c_int64), ("shm_name", C.c_char_p), ("mode", C.c_int32),
-                ("flags", C.c_int32), ("host_order", C.c_void_p), ("n_order", C.c_int64)]
+                ("flags", C.c_int32), ("host_order", C.c_void_p), ("n_order", C.c_int64),
+                ("run_nonce", C.c_uint64)]
 
 
 class ScheduleInfo(C.Structure):
@@ -146,7 +147,7 @@ class Frugal:
 
     def __init__(self, *, world, rank, device, dim, n_rows, slots, batch, lookahead=10, age_out=10,
                  opt="adagrad", lr=0.05, eps=1e-10, init_accum=0.0, init_scale=0.05, init_seed=3, hot_ids=None,
-                 shm_name=None, mode=MODE_P2F, flags=0, host_order=None):
+                 shm_name=None, mode=MODE_P2F, flags=0, host_order=None, run_nonce=0):
         self.world, self.rank, self.dim, self.slots, self.batch = world, rank, dim, slots, batch
         self.lookahead = lookahead
         hot = np.ascontiguousarray(np.zeros(0, np.int64) if hot_ids is None else hot_ids, dtype=np.int64)
@@ -158,7 +159,8 @@ class Frugal:
                    lookahead=lookahead, age_out=age_out, opt=ADAGRAD if opt == "adagrad" else SGD, lr=lr, eps=eps,
                    init_accum=init_accum, init_scale=init_scale, init_seed=init_seed,
                    hot_ids=hot.ctypes.data if hot.size else None, n_hot=hot.size, shm_name=self._shm, mode=mode,
-                   flags=flags, host_order=order.ctypes.data if order.size else None, n_order=order.size)
+                   flags=flags, host_order=order.ctypes.data if order.size else None, n_order=order.size,
+                   run_nonce=run_nonce)
         self._cfg = c
         h = C.c_void_p()
         _check(lib().frugal_init(C.byref(c), C.byref(h)))

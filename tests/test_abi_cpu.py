@@ -64,6 +64,18 @@ def test_world_gt1_needs_shm():
     assert b"shm" in F.lib().frugal_last_error()
 
 
+def test_world_gt1_needs_run_nonce():
+    """A shared table needs a run nonce (ranks > 0 attach only to their run's segment)."""
+    F = _lib()
+    cfg = F.Config(world=2, rank=1, device=0, dim=16, n_rows=100, slots=1, batch=4, lookahead=4, age_out=2,
+                   opt=1, lr=0.1, eps=1e-10, init_accum=0.0, init_scale=0.05, init_seed=3, hot_ids=None,
+                   n_hot=0, shm_name=b"/frugal_nonce_test", mode=0, flags=0, run_nonce=0)
+    h = C.c_void_p()
+    assert F.lib().frugal_init(C.byref(cfg), C.byref(h)) == -1
+    assert b"run_nonce" in F.lib().frugal_last_error()
+    assert not h.value
+
+
 def test_null_ctx_calls_fail_cleanly():
     F = _lib()
     L = F.lib()

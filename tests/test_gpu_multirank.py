@@ -14,13 +14,13 @@ from paper_conf_asplos_xiezggl25_b200 import workload as W
 pytestmark = pytest.mark.gpu
 
 
-def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False, fused=False):
+def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False, fused=False, nonce=1):
     try:
         import torch
         from paper_conf_asplos_xiezggl25_b200 import frugal as F
         from paper_conf_asplos_xiezggl25_b200.harness import A2ATrainer, Trainer, make_context
         torch.cuda.set_device(0)
-        fr = make_context(st, rank=rank, device=0, shm_name=shm,
+        fr = make_context(st, rank=rank, device=0, shm_name=shm, run_nonce=nonce,
                           flags=F.F_RECORD | (F.F_A2A if a2a else 0) | (F.F_PEER if peer else 0))
         barrier.wait()
         if a2a:
@@ -64,7 +64,9 @@ def run_two_ranks(st, timeout=600, a2a=False, peer=False, fused=False):
     sk.bind(("127.0.0.1", 0))
     port = sk.getsockname()[1]
     sk.close()
-    ps = [ctx.Process(target=_rank_main, args=(r, st, shm, barrier, q, a2a, port, peer, fused)) for r in range(2)]
+    nonce = int.from_bytes(os.urandom(8), "little") | 1
+    ps = [ctx.Process(target=_rank_main, args=(r, st, shm, barrier, q, a2a, port, peer, fused, nonce))
+          for r in range(2)]
     for p in ps:
         p.start()
     out = {}
