@@ -477,6 +477,13 @@ static void train(oracle* o, int64_t s) {
     int64_t nb = 0;
     for (int g = 0; g < n; g++) nb += o->counts[s * n + g];
     double loss = 0.0;
+    /* materialise every row this step reads first: row() may grow (realloc) W, and the glue
+       below holds pointers into W across several row() calls (TransE: h, r, t while looking
+       up the negatives) */
+    for (int g = 0; g < n; g++) {
+        const int64_t* id = step_ids(o, s, g);
+        for (int64_t i = 0; i < step_len(o, s, g); i++) row(o, id[i]);
+    }
     float* S = malloc(d * sizeof(float));
     /* (f) forward + glue backward, all reads before any update */
     for (int g = 0; g < n; g++) {
