@@ -68,9 +68,28 @@ def parse():
                          "default: the REC glue reads the gathered distinct rows through the inverse index "
                          "(frugal_lookup / frugal_dot_model with NULL emb, no expand; "
                          "profiles/r1_sweep32_fused_lookup.txt)")
+    ap.add_argument("--drain", default="gpu", choices=["gpu", "host"],
+                    help="deferred drain (a11): gpu = zero-copy scatter kernel on the side stream; host = packed "
+                         "into a staging queue, copied into the table by the library's flushing threads "
+                         "(FRUGAL_F_HOST_FLUSH)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for barriers / the max-over-ranks timing only")
     return ap.parse_args()
+
+
+kSMs = 148
+
+
+def source_sha():
+    """Hash of the CUDA sources and the ABI header: ties a committed ncu capture to the code it measured."""
+    import hashlib
+    h = hashlib.sha256()
+    csrc = os.path.join(ROOT, "paper_conf_asplos_xiezggl25_b200", "csrc")
+    for f in sorted(os.listdir(csrc)):
+        if f.endswith((".cu", ".cuh")):
+            h.update(open(os.path.join(csrc, f), "rb").read())
+    h.update(open(os.path.join(ROOT, "include", "frugal.h"), "rb").read())
+    return h.hexdigest()[:12]
 
 
 def dist_max(x, world, dist=None, device="cpu"):
@@ -285,7 +304,8 @@ def main():
     fr = make_context(st, rank=rank, device=local, shm_name=shm, run_nonce=nonce,
                       flags=F.F_TIMERS | (F.F_NO_HOST_STATE if no_host_state else 0) | (F.F_A2A if a2a else 0)
                       | (F.F_PEER if (args.peer and world > 1) else 0)
-                      | (F.F_DYNAMIC_CACHE if args.cache_refresh > 0 else 0),
+                      | (F.F_DYNAMIC_CACHE if args.cache_refresh > 0 else 0)
+                      | (F.F_HOST_FLUSH if args.drain == "host" else 0),
                       mode=F.MODE_WRITE_THROUGH if args.mode == "write_through" else F.MODE_P2F)
     # N3: the hot set of every epoch start t0 (bench step numbering; step t reads generated
     # step t % SG), from the E bench steps before t0 -- inputs, computed before any timing,
@@ -423,6 +443,7 @@ def main():
     e0.record(stream)
     for s in range(Wm, Wm + K):
         step_dev(s)
+    fr.join(stream)  # the last steps' ingest (s+L) and side drain belong to the timed work
     e1.record(stream)
     torch.cuda.synchronize()
     barrier()
@@ -441,6 +462,7 @@ def main():
     load_xy(Wm + K)
     for s in range(Wm + K, Wm + 2 * K):
         step_e2e(s)
+    fr.join(stream)
     f1.record(stream)
     torch.cuda.synchronize()
     wall = time.perf_counter() - t0
@@ -501,35 +523,47 @@ def main():
         # a5 KG glue (TransE, R26): fp64 ALU-bound, not HBM.  Algorithmic ops per chunk of C
         # triples with C shared negatives: distances C*C*d*3 (sub, mul, add), the two gradient
         # reductions 2*C*C*d*3; positives d*4 per triple.  Every op is a separately rounded
-        # DADD/DSUB/DMUL (no FMA), so the peak is the fp64 instruction rate: half the guide's
-        # 45 TFLOP/s B200 FP64 (FMA = 2 flops) -> 22.5 TFLOP/s.
+        # DADD/DSUB/DMUL (no FMA), so the peak is the fp64 instruction rate, measured in this run
+        # by frugal_probe_fp64 (all SMs, independent DADD/DMUL chains) next to its derivation
+        # SMs x fp64 lanes per SM x clock.
         cnt_b = B  # triples per rank per step (full batches in the bench)
         C_ = cfg.neg_chunk
         nch, last = cnt_b // C_, cnt_b % C_
         pairs = nch * C_ * C_ + last * last
         flops = pairs * d * 9 + cnt_b * d * 4
-        per["model"] = dict(bound="alu", flops=flops, ms=ph["model"], peak_tflops=22.5,
+        fp64_peak = F.probe_fp64(local) / 1e12
+        per["model"] = dict(bound="alu", flops=flops, ms=ph["model"], peak_tflops=fp64_peak,
                             achieved_tflops=flops / (ph["model"] * 1e-3) / 1e12 if ph["model"] > 0 else None)
-        per["model"]["frac"] = (per["model"]["achieved_tflops"] / 22.5) if per["model"]["achieved_tflops"] else None
+        per["model"]["frac"] = (per["model"]["achieved_tflops"] / fp64_peak) if per["model"]["achieved_tflops"] else None
     for k, v in per.items():
         if v.get("bound") == "alu":
             continue
         v["achieved_gbs"] = gbs(v["bytes"], v["ms"])
         v["frac"] = v["achieved_gbs"] / v["peak"] if v["achieved_gbs"] else None
-    main_ms = {k: v for k, v in ph.items() if k != "side"}
+    # phases on the caller's (main) stream; ingest, side drain and early gather run on library streams
+    main_ms = {k: v for k, v in ph.items() if k not in ("side", "ingest", "prefetch")}
     dom = max(("gather", "urgent", "expand", "segred", "optimizer", "model"), key=lambda k: per[k]["ms"])
     top = max(main_ms, key=main_ms.get)
     D = per[dom]
     traffic, tnote, htraffic = None, None, None
-    try:  # committed ncu --set full capture (profiles/, tools/ncu_summary.py, tools/profile_round.sh)
-        prof = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json"))).get(dom, {})
-        traffic = prof.get("traffic_bytes_per_launch")
-        htraffic = prof.get("host_link_bytes_per_launch")
-        if traffic is not None:
-            tnote = (f"dram read+write per launch of {prof['kernel']} in profiles/r1_ncu_full_summary.txt (one "
-                     f"steady-state launch, ncu --set full); host_link_traffic = its sysmem sectors through L2")
-    except Exception:
-        pass
+    try:  # committed ncu --set full capture (tools/profile_round.sh -> tools/ncu_summary.py)
+        cap = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json"))).get(cfg.name, {})
+        prof = cap.get("kernels", {}).get(dom, {})
+        if prof:
+            if cap.get("source_sha") == source_sha():
+                traffic = prof.get("traffic_bytes_per_launch")
+                htraffic = prof.get("host_link_bytes_per_launch")
+                tnote = (f"dram read+write per launch of {prof['kernel']}: mean of {prof['launches_profiled']} "
+                         f"steady-state launches, ncu --set full of this config on this source "
+                         f"(sha {cap['source_sha']}, {cap.get('file', 'profiles/')}); host_link_traffic = its "
+                         f"sysmem sectors through L2")
+            else:
+                tnote = (f"null: the committed ncu capture of {cfg.name} (source sha {cap.get('source_sha')}) "
+                         f"predates this source (sha {source_sha()})")
+        else:
+            tnote = f"null: no committed ncu capture of {dom} for {cfg.name}"
+    except Exception as e:
+        tnote = f"null: {e}"
     if D.get("bound") != "alu":
         roofline = {"bound": "hbm" if D["bound"] == "hbm" else "host-link", "kernel": dom,
                     "achieved": D["achieved_gbs"], "peak": D["peak"], "unit": "GB/s", "frac": D["frac"],
@@ -545,8 +579,10 @@ def main():
         roofline = {"bound": "alu", "kernel": dom + " (k_transe_pos / _pairs_tiled / _grads_tiled)",
                     "achieved": D["achieved_tflops"], "peak": D["peak_tflops"], "unit": "TFLOP/s", "frac": D["frac"],
                     "traffic": None,
-                    "peak_source": "fp64 non-FMA instruction rate: half the 45 TFLOP/s B200 FP64 figure of "
-                                   "/opt/skills/guides/blackwell_cuda_programming.md (DESIGN.md §7)"}
+                    "peak_source": "fp64 add/mul instruction rate measured in this run by frugal_probe_fp64 "
+                                   "(every op of the KG glue is one such instruction, DESIGN.md §7)",
+                    "peak_derived": kSMs * 64 * (clk.get("sm_max_mhz") or 1965.0) * 1e6 / 1e12,
+                    "peak_derived_note": "148 SMs x 64 fp64 lanes x max SM clock (1 op per lane per clock)"}
     launches = st1["kernel_launches"] - st0["kernel_launches"]
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -559,7 +595,10 @@ def main():
         "config": {"workload": f"{cfg.name} ({CONFIG_NAMES.get(cfg.name, '')})", "global_batch": world * B,
                    "batch_per_gpu": B, "tables": Fs, "rows": cfg.n_rows, "dim": d, "alpha": cfg.alpha,
                    "lookahead": L, "age_out": cfg.age_out, "cache_ratio": cfg.cache_ratio, "opt": cfg.opt,
-                   "flush_mode": args.mode, "exchange": "host table + mailbox (P2F)" if not a2a else
+                   "flush_mode": args.mode,
+                   "drain": "side-stream zero-copy scatter kernel" if args.drain == "gpu" else
+                            "packed staging queue + library flushing threads (FRUGAL_F_HOST_FLUSH)",
+                   "exchange": "host table + mailbox (P2F)" if not a2a else
                    "all-to-all over the process group (comparison path)",
                    "peer_reads": bool(args.peer and world > 1),
                    "lookup": "fused into the glue (no expand)" if fused else "expanded [B*F][d]",

@@ -68,6 +68,14 @@ enum {
     FRUGAL_F_DYNAMIC_CACHE = 32,/* N3: the hot set may change at epoch
                                    boundaries (frugal_set_hot); the cache gets 25% spare
                                    slots; not with FRUGAL_F_PEER or the early gather      */
+    FRUGAL_F_HOST_FLUSH = 64,   /* the side-stream drain (a11) packs its rows into a pinned
+                                   staging queue as one contiguous run and the library's
+                                   background flushing threads (§3.2,
+                                   L1055-1059) copy them into the host table; the gate of
+                                   s+1 waits for the threads' progress word.  Random 128-B
+                                   zero-copy stores from the GPU over the whole table stall
+                                   the concurrent HBM kernels; the staging
+                                   run is sequential.  Threads: FRUGAL_FLUSH_THREADS (env) */
     FRUGAL_F_A2A = 8            /* comparison path (the message pipeline of
                                    PAPER.md Fig. 2b): rows and gradients move between
                                    ranks by the caller's all-to-all (NCCL over NVLink) through
@@ -310,6 +318,18 @@ frugal_status frugal_get_timeline(frugal_ctx* ctx, int32_t* phase, double* t0, d
    table with the gather's access pattern and grid (read-only; between steps) -- the
    random-row ceiling of this machine's host link, next to the sequential pinned-copy peak */
 frugal_status frugal_probe_host_reads(frugal_ctx* ctx, int64_t n, uint64_t seed, double* ms);
+
+/* make `stream` wait for every piece of work the library has enqueued on its own streams so
+   far (the ingest of the sample queue, the side-stream drain, the early gather): a timing
+   event recorded on `stream` after this call covers all of the steps' device work.  The
+   bench joins before its closing event; training loops never need it (the library orders
+   its streams itself). */
+frugal_status frugal_join(frugal_ctx* ctx, frugal_stream stream);
+
+/* fp64 calibration (bench only, no context): *ops_per_s = separately rounded fp64 add/mul
+   instructions per second of a full-device kernel of independent DADD/DMUL chains (the
+   peak of the KG glue, whose every op is such an instruction, reading R26) */
+frugal_status frugal_probe_fp64(int32_t device, double* ops_per_s);
 
 /* number of owned rows / hot slots of this rank */
 int64_t frugal_owned_rows(frugal_ctx* ctx);

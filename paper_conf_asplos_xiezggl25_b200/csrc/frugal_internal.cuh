@@ -69,6 +69,13 @@ struct QueueSlot {
     int32_t* eidx = nullptr;   // [M]
     int32_t* lidx = nullptr;   // [M]
     int32_t* elcnt = nullptr;  // [2] early, late counts
+    // world 1, fused update: the long segments (> 64 occurrences, Zipf head) of this step,
+    // found at ingest: per long row {u, first task, chunks}, one task per 64-chunk
+    // {begin, end, long row, chunk}, arrival counters, counts {long rows, tasks}
+    int4* linfo = nullptr;     // [M/65 + 1]
+    int4* ltask = nullptr;     // [M/64 + M/65 + 2]
+    int32_t* lcnt = nullptr;   // [M/65 + 1]
+    int32_t* lnum = nullptr;   // [2]
     // sender side grouping (world > 1): uniq positions grouped by owner
     int32_t* gl = nullptr;     // [M] grouped position -> uniq index
     int32_t* goff = nullptr;   // [world+1]
@@ -80,6 +87,10 @@ struct PhaseEv {
 };
 
 struct HostShared;  // shm segment layout (runtime.cu)
+struct Flushers;    // host flushing threads (runtime.cu)
+// control words of the drain staging queue (uint32, host memory): the device writes READY
+// (job seq of each parity buffer) and the part sizes; the flushing threads write APPLIED_*
+enum { CTL_READY = 0, CTL_N1 = 2, CTL_NTOT = 4, CTL_APPLIED_FIRST = 16, CTL_APPLIED_ALL = 32 };
 
 // NVLink-native variant (FRUGAL_F_PEER): every rank's HBM cache / pool / metadata, opened
 // through CUDA IPC (device pointers valid in this process)
@@ -106,6 +117,7 @@ struct frugal_ctx {
     int flush_tma = 0;               // flushes by TMA bulk stores: 0 none, 1 side drain, 2 all (FRUGAL_FLUSH_TMA; measured no gain: profiles/r1_sweep21_flush_tma.txt)
     int glue_cache = -1;         // REC glue keeps a sample's rows in registers (F <= 32): -1 auto, 0 never, 1 always
     bool fuse_opt = true;        // world 1: a8 fused into a6 (k_segreduce / k_segred_combine)
+    bool update1 = true;         // world 1 fused: one-launch k_update1 (FRUGAL_UPDATE1=0: the 3-kernel path)
     int gather_blocks = 120;     // grid cap of the zero-copy gathers (120 CTAs: +3% over 74 and 148 in the step, profiles/r1_sweep34_gather_grid.txt)
     bool side_inline = false;    // experiment: drain on the caller stream
     bool drain_after_gather = true;  // side drain after the step's gather (FRUGAL_DRAIN_AT=sched: after the scheduler)
@@ -233,6 +245,19 @@ struct frugal_ctx {
     double* kg_A = nullptr;
     int kg_C = 0;
 
+    // host flushing threads (FRUGAL_F_HOST_FLUSH): the side drain is packed into a pinned staging
+    // queue (2 buffers, by step parity) and copied into the host table by these threads
+    bool host_flush = false;
+    int n_flushers = 0;
+    frugal::Flushers* flushers = nullptr;
+    float* hfl_rows[2] = {nullptr, nullptr};     // host pointers of the staging rows [cap][d]
+    int64_t* hfl_keys[2] = {nullptr, nullptr};   // host-table row slot of each staged row
+    float* dfl_rows[2] = {nullptr, nullptr};     // device aliases
+    int64_t* dfl_keys[2] = {nullptr, nullptr};
+    uint32_t* hfl_ctl = nullptr;                 // control words (host): ready[2], n1[2], ntot[2], ...
+    uint32_t* dfl_ctl = nullptr;                 // device alias
+    int64_t drains_issued = 0;                   // drain jobs published so far (job s = drain of step s)
+
     // instrumentation
     int64_t launches = 0;
     std::vector<frugal::PhaseEv> evs;
@@ -259,6 +284,8 @@ void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, int3
 void launch_schedule(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStream_t st);
 void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begin, const int32_t* d_end,
                        int max_blocks, int counter, cudaStream_t st, bool side = false);
+void launch_pack_drain(frugal_ctx* c, int par, uint32_t seq, int max_blocks, cudaStream_t st);
+void launch_wait_word(frugal_ctx* c, const uint32_t* dflag, uint32_t value, cudaStream_t st);
 void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32_t* cnt, float* rows, int64_t step,
                    cudaStream_t st);
 void launch_expand(frugal_ctx* c, QueueSlot& q, const float* rows, float* out, cudaStream_t st);
@@ -270,6 +297,8 @@ void launch_transe_model(frugal_ctx* c, QueueSlot& q, const float* emb, int C, d
 void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const int32_t* inv, const float* x,
                       const float* y, float* grad, double* loss, int64_t nb, cudaStream_t st);
 void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, float* dest, cudaStream_t st, int64_t fused_step = -1);
+void launch_long_tasks(frugal_ctx* c, QueueSlot& q, cudaStream_t st);
+void launch_update1(frugal_ctx* c, QueueSlot& q, const float* grad, int64_t s, cudaStream_t st);
 void launch_optimizer(frugal_ctx* c, QueueSlot& q, int64_t s, int par, const float* recv, const int32_t* roff,
                       cudaStream_t st);
 void launch_a2a_ids(frugal_ctx* c, QueueSlot& q, int32_t* ids, cudaStream_t st);
@@ -283,4 +312,5 @@ void launch_set_flag(frugal_ctx* c, int which, uint32_t value, cudaStream_t st);
 void launch_read_rows(frugal_ctx* c, const int32_t* d_lk, int64_t n, float* d_w, float* d_G, cudaStream_t st);
 void launch_read_host(frugal_ctx* c, const int64_t* d_k, int64_t n, float* d_w, float* d_G, cudaStream_t st);
 cudaError_t setup_kernel_attrs();
+void launch_probe_fp64(double* out, int iters, int64_t* ops, cudaStream_t st);
 }  // namespace frugal

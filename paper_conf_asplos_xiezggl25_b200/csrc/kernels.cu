@@ -888,6 +888,65 @@ void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begi
     c->launches++;
 }
 
+// a11 with host flushing threads (FRUGAL_F_HOST_FLUSH; §3.2:
+// "background flushing threads ... flush the parameter updates ... to host memory"): the
+// drain's rows -- list 1 (deadline s+1) first, then list 2 (later deadlines) and list 3
+// (age-outs) -- are packed into a host staging queue as ONE contiguous run (coalesced
+// zero-copy stores over a few MB that are reused every other step, instead of scattered
+// 128-B stores over the whole table), with the host-table slot of every row; the library's
+// flushing threads then copy them into the table.  The rows are untouched until their
+// deadline (> s), so packing them at any point of step s reads their post-(s-1) values.
+// The publish kernel that follows tells the threads how many rows each part has.
+template <int GS>
+__global__ void k_pack_drain(const int32_t* __restrict__ lists, const int32_t* __restrict__ cnt, int64_t cap, int world,
+                             int g, int d4, const int32_t* __restrict__ slot, const int32_t* __restrict__ last_upd,
+                             const int32_t* __restrict__ pool_idx, int P, int64_t capT, const float4* __restrict__ cw,
+                             const float4* __restrict__ pw, const int32_t* __restrict__ hs, float4* hrows,
+                             int64_t* hkeys, unsigned long long* stats) {
+    int64_t gid, gs;
+    int l;
+    RowGroup<GS>::ids(gid, gs, l);
+    const int n1 = cnt[1], n2 = cnt[2], n3 = cnt[3];
+    const int n = n1 + n2 + n3;
+    unsigned nh = 0, nc = 0;
+    for (int64_t a = gid; a < n; a += gs) {
+        const int64_t at = a < n1 ? cap + a : a < n1 + n2 ? 2 * cap + (a - n1) : 3 * cap + (a - n1 - n2);
+        const int32_t lk = lists[at];
+        const int sl = slot[lk];
+        const float4* src;
+        if (sl >= 0) {
+            src = cw + (int64_t)sl * d4;
+            nh += (l == 0);
+        } else {
+            src = pw + ((int64_t)(last_upd[lk] % P) * capT + pool_idx[lk]) * d4;
+            nc += (l == 0);
+        }
+        for (int v = l; v < d4; v += GS) hrows[a * d4 + v] = src[v];
+        if (l == 0) hkeys[a] = host_row(hs, (int64_t)lk * world + g);
+    }
+    block_fence_system();  // rows and keys reach host memory before the publish kernel's flag
+    block_count(stats, nh);
+    block_count(stats + 1, nc);
+}
+// publish job `seq` (= s+1) of staging buffer `par`: part sizes, then the flag (release)
+__global__ void k_publish_drain(const int32_t* __restrict__ cnt, uint32_t* ctl, int par, uint32_t seq) {
+    // ctl layout (uint32 words): [0..1] ready[par], [2..3] n1[par], [4..5] ntot[par]
+    ctl[2 + par] = (uint32_t)cnt[1];
+    ctl[4 + par] = (uint32_t)(cnt[1] + cnt[2] + cnt[3]);
+    __threadfence_system();
+    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(ctl + par), "r"(seq) : "memory");
+}
+void launch_pack_drain(frugal_ctx* c, int par, uint32_t seq, int max_blocks, cudaStream_t st) {
+    const int d4 = c->d / 4, gs = group_size(d4);
+    int grid = std::min(grid_for(3 * c->sl_cap * (int64_t)gs, 256, 4), max_blocks);
+    DISPATCH_GS(gs, (k_pack_drain<GS><<<grid, 256, 0, st>>>(
+                        c->sl_rows[par], c->sl_cnt[par], c->sl_cap, c->n, c->g, d4, c->slot, c->last_upd, c->pool_idx,
+                        c->P, c->capT, (const float4*)c->cw, (const float4*)c->pw, c->hs,
+                        (float4*)c->dfl_rows[par], c->dfl_keys[par], c->dstats + FRUGAL_C_SIDE_HOT)));
+    k_publish_drain<<<1, 1, 0, st>>>(c->sl_cnt[par], c->dfl_ctl, par, seq);
+    c->launches += 2;
+}
+
 // a4 gather: unique rows -> staging (owned hot: HBM cache; else host, zero-copy).
 // list: the uniq indices to gather (early or late part), cnt: its device count.
 // An owned cold row whose latest update is still in the dirty pool is read from the pool

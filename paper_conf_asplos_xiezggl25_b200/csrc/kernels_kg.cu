@@ -340,4 +340,31 @@ void launch_transe_model(frugal_ctx* c, QueueSlot& q, const float* emb, int C, d
     c->launches += 4;
 }
 
+// fp64 instruction-rate probe (frugal_probe_fp64): per thread 8 independent chains of
+// dependent DADD/DMUL pairs (the KG glue's instruction mix, no FMA contraction), all SMs,
+// 32 warps per SM; 2 ops per chain step
+constexpr int kProbeChains = 8, kProbeInner = 256;
+__global__ void __launch_bounds__(256) k_probe_fp64(double* out, int iters) {
+    double x[kProbeChains];
+#pragma unroll
+    for (int c = 0; c < kProbeChains; c++) x[c] = 1.0 + 1e-3 * (threadIdx.x + c);
+    const double a = 1.0000001, m = 0.9999999;
+    for (int it = 0; it < iters; it++) {
+#pragma unroll 4
+        for (int i = 0; i < kProbeInner; i++) {
+#pragma unroll
+            for (int c = 0; c < kProbeChains; c++) x[c] = __dmul_rn(__dadd_rn(x[c], a), m);
+        }
+    }
+    double acc = 0.0;
+#pragma unroll
+    for (int c = 0; c < kProbeChains; c++) acc += x[c];
+    if (acc == 12345.678) out[threadIdx.x] = acc;  // keeps the chains live
+}
+void launch_probe_fp64(double* out, int iters, int64_t* ops, cudaStream_t st) {
+    const int grid = kSMs * 8, block = 256;
+    k_probe_fp64<<<grid, block, 0, st>>>(out, iters);
+    *ops = (int64_t)grid * block * iters * kProbeInner * kProbeChains * 2;
+}
+
 }  // namespace frugal

@@ -338,6 +338,175 @@ cudaError_t setup_kernel_attrs() {
     return e;
 }
 
+// ============================================================================ a6 + a8, world 1, one launch
+// Long segments of a step (> kChunk occurrences), listed at ingest (one step ahead, off the
+// critical path): per long row {u, first task, chunks}; per 64-chunk a task {b, e, row, c}.
+// The order of the lists is irrelevant to the results: chunk c of a row always lands in
+// scratch slot t0 + c and the chunk sums are added in c order.
+__global__ void k_long_tasks(const int32_t* __restrict__ off, const int32_t* d_nu, int4* __restrict__ linfo,
+                             int4* __restrict__ ltask, int32_t* __restrict__ lcnt, int32_t* lnum,
+                             unsigned long long* stats) {
+    const int n = *d_nu;
+    unsigned nl = 0;
+    for (int u = blockIdx.x * blockDim.x + threadIdx.x; u < n; u += gridDim.x * blockDim.x) {
+        const int b = off[u], e = off[u + 1];
+        if (e - b <= kChunk) continue;
+        const int nch = (e - b + kChunk - 1) / kChunk;
+        const int L = atomicAdd(&lnum[0], 1);
+        const int t0 = atomicAdd(&lnum[1], nch);
+        linfo[L] = make_int4(u, t0, nch, 0);
+        lcnt[L] = 0;
+        for (int c = 0; c < nch; c++) ltask[t0 + c] = make_int4(b + c * kChunk, min(e, b + (c + 1) * kChunk), L, c);
+        nl++;
+    }
+    block_count(stats + FRUGAL_C_LONG_SEGMENTS, nl);
+}
+void launch_long_tasks(frugal_ctx* c, QueueSlot& q, cudaStream_t st) {
+    cudaMemsetAsync(q.lnum, 0, 8, st);
+    k_long_tasks<<<grid_for(c->M, 256, 2), 256, 0, st>>>(q.off, q.n_uniq, q.linfo, q.ltask, q.lcnt, q.lnum, c->dstats);
+    c->launches++;
+}
+
+// ordered sum of n rows base[0], base[d4], ... (row 0 first), 16 loads in flight; L1 bypassed
+// (the rows were written by other CTAs of this launch)
+__device__ __forceinline__ float4 ordered_rows_cg(const float4* base, int d4, int n) {
+    float4 acc = __ldcg(base);
+    int c = 1;
+    for (; c + 16 <= n; c += 16) {
+        float4 x[16];
+#pragma unroll
+        for (int q = 0; q < 16; q++) x[q] = __ldcg(base + (int64_t)(c + q) * d4);
+#pragma unroll
+        for (int q = 0; q < 16; q++) acc = add4(acc, x[q]);
+    }
+    for (; c < n; c++) acc = add4(acc, __ldcg(base + (int64_t)c * d4));
+    return acc;
+}
+
+// the fused update of unique row j with the row's w and G loaded BEFORE its gradient sum (they
+// do not depend on it): lane l owns columns v = l + k*GS, k < VPL
+template <int GS, int VPL, typename SumF>
+__device__ __forceinline__ void update_row_pf(const FusedOpt& fo, int j, int d4, int l, SumF sum, unsigned& nhot,
+                                              unsigned& ncold) {
+    const int32_t lk = fo.uniq[j];
+    const int sl = fo.slot[lk];
+    const float4* wsrc = sl >= 0 ? fo.cw + (int64_t)sl * d4 : fo.rows_w + (int64_t)j * d4;
+    float4 w[VPL], G[VPL];
+#pragma unroll
+    for (int k = 0; k < VPL; k++) {
+        const int v = l + k * GS;
+        G[k] = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (v < d4) {
+            w[k] = wsrc[v];
+            if (fo.adagrad) G[k] = fo.Gd[(int64_t)lk * d4 + v];
+        }
+    }
+#pragma unroll
+    for (int k = 0; k < VPL; k++) {
+        const int v = l + k * GS;
+        if (v < d4) {
+            const float4 acc = sum(v);
+            opt4(w[k], G[k], acc, fo.adagrad, fo.lr, fo.eps);
+            if (sl >= 0) fo.cw[(int64_t)sl * d4 + v] = w[k];
+            else fo.pw[(int64_t)j * d4 + v] = w[k];
+            if (fo.adagrad) fo.Gd[(int64_t)lk * d4 + v] = G[k];
+        }
+    }
+    if (l == 0) {
+        if (sl >= 0) nhot++;
+        else ncold++;
+        fo.state[lk] = ST_UPDATED;
+        fo.last_upd[lk] = fo.s;
+        const uint64_t clear = ~((1ull << (fo.s & 31)) | (1ull << (32 + (fo.s & 31))));
+        atomicAnd((unsigned long long*)&fo.rbits[lk], (unsigned long long)clear);  // races with k_ingest_bits
+        if (sl < 0) fo.pool_idx[lk] = j;
+        fo.pkey[j] = sl < 0 ? lk : -1;
+    }
+}
+
+// One launch for the whole world-1 backward (a6 + a8): work items [0, nt) are the 64-chunks
+// of the long rows (summed in order into scratch[item]; the group that completes a row's last
+// chunk adds the row's chunk sums in chunk order and applies the optimizer), items
+// [nt, nt + nu) the unique rows, of which the short ones (<= 64 occurrences) are reduced
+// and updated directly.  Same arithmetic, same order as k_segreduce + k_segred_chunks +
+// k_segred_combine (reading R23), without their serialisation.
+template <int GS, int VPL>
+__global__ void __launch_bounds__(256) k_update1(const int32_t* __restrict__ off, const int32_t* __restrict__ pos,
+                                                 const int32_t* d_nu, const int4* __restrict__ ltask,
+                                                 const int4* __restrict__ linfo, int32_t* lcnt,
+                                                 const int32_t* lnum, int d4, const float4* __restrict__ grad,
+                                                 float4* scratch, unsigned long long* stats, const FusedOpt fo) {
+    int64_t gid, gs;
+    int l;
+    RowGroup<GS>::ids(gid, gs, l);
+    const unsigned gmask = GS == 32 ? 0xffffffffu : (((1u << GS) - 1u) << ((threadIdx.x & 31) & ~(GS - 1)));
+    const int leader = (threadIdx.x & 31) & ~(GS - 1);
+    const int nt = lnum[1], nu = *d_nu;
+    unsigned nhot = 0, ncold = 0;
+    for (int64_t w = gid; w < (int64_t)nt + nu; w += gs) {
+        if (w < nt) {
+            const int4 tk = ltask[w];
+            for (int v = l; v < d4; v += GS) __stcg(scratch + w * d4 + v, chunk_sum<GS>(grad, pos, tk.x, tk.y, d4, v));
+            __threadfence();
+            __syncwarp(gmask);
+            const int4 li = linfo[tk.z];
+            int last = 0;
+            if (l == 0) last = atomicAdd(&lcnt[tk.z], 1) == li.z - 1;
+            last = __shfl_sync(gmask, last, leader);
+            if (!last) continue;
+            __threadfence();  // every chunk of the row is in scratch
+            update_row_pf<GS, VPL>(fo, li.x, d4, l, [&](int v) {
+                return ordered_rows_cg(scratch + (int64_t)li.y * d4 + v, d4, li.z); }, nhot, ncold);
+        } else {
+            const int u = (int)(w - nt);
+            const int b = off[u], e = off[u + 1];
+            if (e - b > kChunk) continue;  // a long row: its last chunk task updates it
+            update_row_pf<GS, VPL>(fo, u, d4, l, [&](int v) { return chunk_sum<GS>(grad, pos, b, e, d4, v); },
+                                   nhot, ncold);
+        }
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) *fo.pcount = nu;
+    block_count(stats + FRUGAL_C_OPT_HOT, nhot);
+    block_count(stats + FRUGAL_C_OPT_COLD, ncold);
+}
+
+void launch_update1(frugal_ctx* c, QueueSlot& q, const float* grad, int64_t s, cudaStream_t st) {
+    const int d4 = c->d / 4, gs = group_size(d4);
+    const int vpl = (d4 + gs - 1) / gs;
+    const int seg = (int)(s % c->P);
+    FusedOpt fo{};
+    fo.on = 1;
+    fo.s = (int32_t)s;
+    fo.adagrad = c->cfg.opt == FRUGAL_ADAGRAD;
+    fo.lr = c->cfg.lr;
+    fo.eps = c->cfg.eps;
+    fo.uniq = q.uniq;
+    fo.rows_w = (const float4*)c->rows_buf[s & 1];
+    fo.slot = c->slot;
+    fo.state = c->state;
+    fo.last_upd = c->last_upd;
+    fo.pool_idx = c->pool_idx;
+    fo.rbits = c->rbits;
+    fo.cw = (float4*)c->cw;
+    fo.Gd = (float4*)c->Gd;
+    fo.pw = (float4*)c->pw + (size_t)seg * c->capT * d4;
+    fo.pkey = c->pkey + (size_t)seg * c->capT;
+    fo.pcount = c->pcount + seg;
+    const int grid = grid_for((int64_t)c->M * gs, 256, 8);
+#define U1(V)                                                                                                     \
+    do {                                                                                                          \
+        DISPATCH_GS(gs, (k_update1<GS, V><<<grid, 256, 0, st>>>(q.off, q.pos, q.n_uniq, q.ltask, q.linfo, q.lcnt, \
+                                                                 q.lnum, d4, (const float4*)grad,                  \
+                                                                 (float4*)c->chunk_scratch, c->dstats, fo)));      \
+    } while (0)
+    if (vpl <= 1) U1(1);
+    else if (vpl <= 2) U1(2);
+    else if (vpl <= 4) U1(4);
+    else U1(8);
+#undef U1
+    c->launches++;
+}
+
 // mailbox header of (parity, this sender): goff[0..world]
 __global__ void k_mail_header(const int32_t* __restrict__ goff, int world, int32_t* hdr) {
     if (threadIdx.x <= world) hdr[threadIdx.x] = goff[threadIdx.x];
@@ -606,6 +775,11 @@ __global__ void k_wait_flags(const uint32_t* f, int world, uint32_t v, int32_t* 
     }
     __syncwarp();
     __threadfence_system();
+}
+// wait (device side) until one host word reaches `value` (wrap-around compare)
+void launch_wait_word(frugal_ctx* c, const uint32_t* dflag, uint32_t value, cudaStream_t st) {
+    k_wait_flags<<<1, 32, 0, st>>>(dflag, 1, value, c->err);
+    c->launches++;
 }
 void launch_set_flag(frugal_ctx* c, int which, uint32_t value, cudaStream_t st) {
     k_set_flag<<<1, 1, 0, st>>>(c->dh_flags + (which * 32 + c->g) * 16, value);

@@ -19,8 +19,12 @@
 #include <unistd.h>
 #include <stdlib.h>
 
+#include <immintrin.h>
+
 #include <algorithm>
+#include <atomic>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "frugal_internal.cuh"
@@ -122,6 +126,92 @@ struct Timer {
 
 }  // namespace
 
+// ================================================================================ flushing threads
+// PAPER.md §3.2 (L794-797) and §3.3 (L1055-1059): "background flushing threads ... flush the
+// parameter updates ... to host memory".  With FRUGAL_F_HOST_FLUSH the side-stream drain of
+// step s packs its rows into staging buffer s&1 and publishes job s (READY[s&1] = s+1); the
+// threads copy part 1 (deadline s+1) into the table, publish APPLIED_FIRST = s+1 (and, with a
+// shared table, this rank's FLAG_SIDE_FIRST), then part 2 (later deadlines, age-outs) and
+// APPLIED_ALL = s+1 (FLAG_SIDE).  Jobs are applied strictly in order, so APPLIED_FIRST >= s+1
+// also covers every earlier job.  Each thread copies a contiguous share of the part with
+// non-temporal stores (the rows are not read back by the CPU).
+struct frugal::Flushers {
+    std::vector<std::thread> th;
+    std::atomic<bool> stop{false};
+    std::atomic<int> done[2][2];  // [parity][part]: threads finished
+};
+
+static inline uint32_t ctl_load(const uint32_t* p) { return __atomic_load_n(p, __ATOMIC_ACQUIRE); }
+static inline void ctl_store(uint32_t* p, uint32_t v) { __atomic_store_n(p, v, __ATOMIC_RELEASE); }
+static inline bool seq_reached(uint32_t x, uint32_t v) { return (int32_t)(x - v) >= 0; }
+
+static void copy_rows_nt(float* table, const float* rows, const int64_t* keys, int64_t lo, int64_t hi, int d) {
+    const int n16 = d / 4;  // 16-byte chunks per row (d is a multiple of 4)
+    for (int64_t i = lo; i < hi; i++) {
+        __m128i* dst = (__m128i*)(table + keys[i] * d);
+        const __m128i* src = (const __m128i*)(rows + i * d);
+        for (int q = 0; q < n16; q++) _mm_stream_si128(dst + q, _mm_load_si128(src + q));
+    }
+    _mm_sfence();
+}
+
+static void flusher_main(frugal_ctx* c, int t) {
+    frugal::Flushers* F = c->flushers;
+    const int T = c->n_flushers;
+    uint32_t* ctl = c->hfl_ctl;
+    double idle_since = 0.0;
+    for (int64_t job = 0;; job++) {
+        const int par = (int)(job & 1);
+        const uint32_t seq = (uint32_t)(job + 1);
+        // wait for the device to publish the job: spin while jobs keep coming, then poll gently
+        while (!seq_reached(ctl_load(ctl + CTL_READY + par), seq)) {
+            if (F->stop.load(std::memory_order_relaxed)) return;
+            timespec ts;
+            clock_gettime(CLOCK_MONOTONIC, &ts);
+            const double now = ts.tv_sec + 1e-9 * ts.tv_nsec;
+            if (idle_since == 0.0) idle_since = now;
+            if (now - idle_since < 2e-3) {
+                for (int k = 0; k < 64; k++) _mm_pause();
+            } else {
+                usleep(20);
+            }
+        }
+        idle_since = 0.0;
+        const int64_t n1 = ctl_load(ctl + CTL_N1 + par), nt = ctl_load(ctl + CTL_NTOT + par);
+        const float* rows = c->hfl_rows[par];
+        const int64_t* keys = c->hfl_keys[par];
+        for (int part = 0; part < 2; part++) {
+            const int64_t b = part == 0 ? 0 : n1, e = part == 0 ? n1 : nt;
+            copy_rows_nt(c->h_w, rows, keys, b + (e - b) * t / T, b + (e - b) * (t + 1) / T, c->d);
+            if (F->done[par][part].fetch_add(1, std::memory_order_acq_rel) + 1 == T) {
+                F->done[par][part].store(0, std::memory_order_relaxed);
+                ctl_store(ctl + (part == 0 ? CTL_APPLIED_FIRST : CTL_APPLIED_ALL), seq);
+                if (c->xhost) {  // readers on other GPUs wait for this owner's flags
+                    const int which = part == 0 ? 3 /* FLAG_SIDE_FIRST */ : 1 /* FLAG_SIDE */;
+                    ctl_store((uint32_t*)(c->h_flags + (which * 32 + c->g) * 16), seq);
+                }
+            }
+        }
+    }
+}
+
+// host side: every published drain job applied (frugal_flush, introspection); 120 s bound
+static frugal_status wait_flushers(frugal_ctx* c) {
+    if (!c->host_flush || c->drains_issued == 0) return FRUGAL_OK;
+    const uint32_t want = (uint32_t)c->drains_issued;
+    timespec t0, t1;
+    clock_gettime(CLOCK_MONOTONIC, &t0);
+    while (!seq_reached(ctl_load(c->hfl_ctl + CTL_APPLIED_ALL), want)) {
+        usleep(10);
+        clock_gettime(CLOCK_MONOTONIC, &t1);
+        if (t1.tv_sec - t0.tv_sec > 120) {
+            set_err("flushing threads did not apply drain %u within 120 s", want);
+            return FRUGAL_ETIMEOUT;
+        }
+    }
+    return FRUGAL_OK;
+}
+
 // ================================================================================ helpers
 // Spread the host table over every NUMA node (best effort, before the pages are first
 // touched): on a two-socket host each GPU then finds half the rows behind its own root
@@ -158,6 +248,17 @@ static void free_ctx(frugal_ctx* c) {
     if (!c) return;
     cudaSetDevice(c->cfg.device);
     cudaDeviceSynchronize();
+    if (c->flushers) {
+        c->flushers->stop.store(true);
+        for (auto& t : c->flushers->th) t.join();
+        delete c->flushers;
+        c->flushers = nullptr;
+    }
+    for (int i = 0; i < 2; i++) {
+        if (c->hfl_rows[i]) cudaFreeHost(c->hfl_rows[i]);
+        if (c->hfl_keys[i]) cudaFreeHost(c->hfl_keys[i]);
+    }
+    if (c->hfl_ctl) cudaFreeHost(c->hfl_ctl);
     auto F = [](void* p) {
         if (p) cudaFree(p);
     };
@@ -167,6 +268,7 @@ static void free_ctx(frugal_ctx* c) {
     for (auto& q : c->q) {
         F(q.eidx); F(q.lidx); F(q.elcnt);
         F(q.ids); F(q.counts); F(q.m); F(q.uniq); F(q.inv); F(q.off); F(q.pos); F(q.n_uniq);
+        F(q.linfo); F(q.ltask); F(q.lcnt); F(q.lnum);
         if (c->n > 1) { F(q.T); F(q.Tmask); F(q.Tidx); F(q.nT); F(q.gl); F(q.goff); }
     }
     F(c->hs); F(c->rows_buf[0]); F(c->rows_buf[1]); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->long_tasks); F(c->owned_cnt);
@@ -354,12 +456,17 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->peer = (k.flags & FRUGAL_F_PEER) != 0;
     c->dyn = (k.flags & FRUGAL_F_DYNAMIC_CACHE) != 0;
     if (c->dyn) c->early = false;
+    // host flushing threads: the config flag, or FRUGAL_HOST_FLUSH=0/1 (experiments) overriding it
+    c->host_flush = (k.flags & FRUGAL_F_HOST_FLUSH) != 0;
+    if (getenv("FRUGAL_HOST_FLUSH")) c->host_flush = atoi(getenv("FRUGAL_HOST_FLUSH")) != 0;
+    if (c->host_flush) c->early = false;  // the early gather synchronises on the GPU drain's events
     c->xhost = c->n > 1 && !c->a2a;
     // side-drain flushes by TMA bulk stores (FRUGAL_FLUSH_TMA=0 none, 1 side, 2 all)
     if (getenv("FRUGAL_FLUSH_TMA")) c->flush_tma = atoi(getenv("FRUGAL_FLUSH_TMA"));
     // world 1: optimizer fused into the segment-reduce (FRUGAL_FUSE_OPT=0: two kernels)
     if (getenv("FRUGAL_GLUE_CACHE")) c->glue_cache = atoi(getenv("FRUGAL_GLUE_CACHE"));
     c->fuse_opt = !(getenv("FRUGAL_FUSE_OPT") && !atoi(getenv("FRUGAL_FUSE_OPT")));
+    c->update1 = !(getenv("FRUGAL_UPDATE1") && !atoi(getenv("FRUGAL_UPDATE1")));
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 20;
     // the deadline-(s+1) part of the drain (the next gate waits for it) may run wider
     c->side_first_blocks = getenv("FRUGAL_SIDE_FIRST_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_FIRST_BLOCKS"))
@@ -524,6 +631,12 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         DMALLOC(q.eidx, (size_t)c->M * 4);
         DMALLOC(q.lidx, (size_t)c->M * 4);
         DMALLOC(q.elcnt, 8);
+        if (c->n == 1) {
+            DMALLOC(q.linfo, ((size_t)c->M / 65 + 1) * sizeof(int4));
+            DMALLOC(q.ltask, ((size_t)c->M / 64 + c->M / 65 + 2) * sizeof(int4));
+            DMALLOC(q.lcnt, ((size_t)c->M / 65 + 1) * 4);
+            DMALLOC(q.lnum, 8);
+        }
         if (c->n > 1) {
             DMALLOC(q.T, c->capT * 4);
             DMALLOC(q.Tmask, c->capT * 4);
@@ -655,6 +768,36 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         free_ctx(c);
         return FRUGAL_ECUDA;
     }
+    if (c->host_flush) {
+        const int64_t cap = std::max<int64_t>(1, std::min<int64_t>(3 * c->sl_cap, c->No));
+        bool ok = cudaHostAlloc((void**)&c->hfl_ctl, 4096, cudaHostAllocMapped | cudaHostAllocPortable) == cudaSuccess;
+        for (int i = 0; ok && i < 2; i++) {
+            ok = cudaHostAlloc((void**)&c->hfl_rows[i], (size_t)cap * rowb, cudaHostAllocMapped | cudaHostAllocPortable) ==
+                     cudaSuccess &&
+                 cudaHostAlloc((void**)&c->hfl_keys[i], (size_t)cap * 8, cudaHostAllocMapped | cudaHostAllocPortable) ==
+                     cudaSuccess;
+            if (ok) {
+                cudaHostGetDevicePointer((void**)&c->dfl_rows[i], c->hfl_rows[i], 0);
+                cudaHostGetDevicePointer((void**)&c->dfl_keys[i], c->hfl_keys[i], 0);
+            }
+        }
+        if (!ok) {
+            cudaGetLastError();
+            set_err("cudaHostAlloc of the drain staging queue failed");
+            free_ctx(c);
+            return FRUGAL_ENOMEM;
+        }
+        memset(c->hfl_ctl, 0, 4096);
+        cudaHostGetDevicePointer((void**)&c->dfl_ctl, c->hfl_ctl, 0);
+        const long ncpu = sysconf(_SC_NPROCESSORS_ONLN);
+        c->n_flushers = getenv("FRUGAL_FLUSH_THREADS") ? atoi(getenv("FRUGAL_FLUSH_THREADS"))
+                                                       : (int)std::max(2L, std::min(8L, ncpu / 4));
+        c->n_flushers = std::max(1, c->n_flushers);
+        c->flushers = new frugal::Flushers();
+        for (int i = 0; i < 2; i++)
+            for (int j = 0; j < 2; j++) c->flushers->done[i][j].store(0);
+        for (int t = 0; t < c->n_flushers; t++) c->flushers->th.emplace_back(flusher_main, c, t);
+    }
     if (c->peer) {
         frugal_status r = setup_peers(c, hbase + off_ipc, hot_global);
         if (r) {
@@ -704,6 +847,7 @@ static frugal_status ingest(frugal_ctx* c, int64_t t, const int64_t* ids_all, co
         Timer tm(c, PH_INGEST, is);
         launch_convert_ids(c, q, is);
         launch_dedup(c, q, is);
+        if (c->n == 1) launch_long_tasks(c, q, is);
         if (c->n > 1) launch_owner_side(c, q, t, is);
         const int apar = (int)((t - c->L + 1) & 1);  // consumed by frugal_step(t - L + 1)
         CK(cudaMemsetAsync(c->adj_cnt[apar], 0, 4, is));
@@ -794,7 +938,14 @@ static frugal_status launch_drain(frugal_ctx* c, int64_t s, cudaStream_t st, cud
     const int par = (int)(s & 1);
     cudaStream_t sd = c->side_inline ? st : c->side;
     if (!c->side_inline) CK(cudaStreamWaitEvent(c->side, after, 0));
-    {
+    if (c->host_flush) {
+        // host flushing threads: staging buffer `par` was last used by job s-2
+        Timer tm(c, PH_SIDE, sd);
+        if (s >= 2) launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_ALL, (uint32_t)(s - 1), sd);
+        launch_pack_drain(c, par, (uint32_t)(s + 1), c->side_blocks, sd);
+        CK(cudaEventRecord(c->ev_side_first[par], sd));  // the lists of this parity were read
+        CKL();
+    } else {
         Timer tm(c, PH_SIDE, sd);
         launch_flush_rows(c, c->sl_rows[par] + c->sl_cap, nullptr, c->sl_cnt[par] + 1, c->side_first_blocks,
                           FRUGAL_C_SIDE_HOT, sd, true);
@@ -809,6 +960,7 @@ static frugal_status launch_drain(frugal_ctx* c, int64_t s, cudaStream_t st, cud
     }
     CK(cudaEventRecord(c->ev_side[par], sd));
     c->side_pending[par] = true;
+    c->drains_issued = s + 1;
     return FRUGAL_OK;
 }
 
@@ -846,6 +998,8 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
         // of the new set precede the transition; it runs on the critical path
         Timer tm(c, PH_URGENT, st);
         if (s >= 1 && c->side_pending[par ^ 1]) CK(cudaStreamWaitEvent(st, c->ev_side[par ^ 1], 0));
+        if (s >= 1 && c->host_flush && c->side_pending[par ^ 1])  // ... and applied by the flushing threads
+            launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_ALL, (uint32_t)s, st);
         CK(cudaStreamWaitEvent(st, c->ev_hot, 0));
         launch_cache_transition(c, s, par, st);
         CK(cudaEventRecord(c->ev_hot, st));  // the next frugal_set_hot reuses new_lk after it
@@ -907,7 +1061,10 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
         // (deadline-s rows are the first part of drain s-1; the side stream is FIFO, so that
         // event also covers every earlier drain)
         if (!c->xhost) {  // world 1, or the comparison path: only this rank reads its host rows
-            if (s >= 1 && c->side_pending[par ^ 1]) CK(cudaStreamWaitEvent(st, c->ev_side_first[par ^ 1], 0));
+            if (s >= 1 && c->side_pending[par ^ 1]) {
+                if (c->host_flush) launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_FIRST, (uint32_t)s, st);
+                else CK(cudaStreamWaitEvent(st, c->ev_side_first[par ^ 1], 0));
+            }
         } else {
             launch_wait_flags(c, FLAG_URGENT, (uint32_t)(s + 1), st);
             if (s >= 1) launch_wait_flags(c, FLAG_SIDE_FIRST, (uint32_t)s, st);
@@ -1017,8 +1174,12 @@ extern "C" frugal_status frugal_backward_update(frugal_ctx* c, int64_t s, const 
     cudaStream_t st = (cudaStream_t)stream;
     QueueSlot& q = c->q[s % c->QN];
     const int par = (int)(s & 1);
-    if (c->n == 1 && c->fuse_opt) {
-        // world 1: every partial is this rank's own -- segment-reduce and optimizer in one pass
+    if (c->n == 1 && c->fuse_opt && c->update1) {
+        // world 1: every partial is this rank's own -- segment-reduce (short rows and the long
+        // rows' chunks) and optimizer in one launch
+        Timer tm(c, PH_SEGRED, st);
+        launch_update1(c, q, d_grad, s, st);
+    } else if (c->n == 1 && c->fuse_opt) {
         Timer tm(c, PH_SEGRED, st);
         launch_segreduce(c, q, d_grad, par, nullptr, st, s);
     } else {
@@ -1148,6 +1309,10 @@ extern "C" frugal_status frugal_flush(frugal_ctx* c, int32_t what, frugal_stream
     cudaStream_t st = (cudaStream_t)stream;
     for (int i = 0; i < 2; i++)
         if (c->side_pending[i]) CK(cudaStreamWaitEvent(st, c->ev_side[i], 0));
+    if (c->host_flush) {  // every drain job applied by the flushing threads before the final flush
+        CK(cudaStreamSynchronize(c->side));
+        if (frugal_status r = wait_flushers(c)) return r;
+    }
     launch_final_flush(c, st);
     CKL();
     CK(cudaStreamSynchronize(st));
@@ -1263,6 +1428,7 @@ extern "C" frugal_status frugal_read_rows(frugal_ctx* c, const int64_t* ids, int
         lk[i] = (int32_t)(ids[i] / c->n);
     }
     CK(cudaDeviceSynchronize());
+    if (frugal_status r = wait_flushers(c)) return r;
     int32_t* d_lk;
     float *d_w, *d_G;
     CK(cudaMalloc(&d_lk, n * 4));
@@ -1285,6 +1451,7 @@ extern "C" frugal_status frugal_read_rows(frugal_ctx* c, const int64_t* ids, int
 extern "C" frugal_status frugal_read_host(frugal_ctx* c, const int64_t* ids, int64_t n, float* w, float* G) {
     if (!c || (n && (!ids || !w))) { set_err("NULL argument"); return FRUGAL_EINVAL; }
     CK(cudaDeviceSynchronize());
+    if (frugal_status r = wait_flushers(c)) return r;
     for (int64_t i = 0; i < n; i++) {
         if (ids[i] < 0 || ids[i] >= c->N) { set_err("read_host: id out of range"); return FRUGAL_EINVAL; }
         const int64_t hk = c->hs_host.empty() ? ids[i] : c->hs_host[ids[i]];  // host_order layout
@@ -1360,6 +1527,50 @@ extern "C" frugal_status frugal_probe_host_reads(frugal_ctx* c, int64_t n, uint6
     cudaEventDestroy(b);
     *ms = f;
     CKL();
+    return FRUGAL_OK;
+}
+
+extern "C" frugal_status frugal_join(frugal_ctx* c, frugal_stream stream) {
+    if (!c) { set_err("NULL ctx"); return FRUGAL_EINVAL; }
+    cudaStream_t st = (cudaStream_t)stream;
+    for (cudaStream_t s : {c->istream, c->side, c->pstream}) {
+        if (!s) continue;
+        cudaEvent_t e;
+        CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        cudaError_t r1 = cudaEventRecord(e, s);
+        cudaError_t r2 = r1 == cudaSuccess ? cudaStreamWaitEvent(st, e, 0) : r1;
+        cudaEventDestroy(e);  // released once the wait resolves
+        if (r2 != cudaSuccess) { set_err("join: %s", cudaGetErrorString(r2)); return FRUGAL_ECUDA; }
+    }
+    // host flushing threads: every drain job issued so far applied to the host table
+    if (c->host_flush && c->drains_issued > 0) {
+        launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_ALL, (uint32_t)c->drains_issued, st);
+        CKL();
+    }
+    return FRUGAL_OK;
+}
+
+extern "C" frugal_status frugal_probe_fp64(int32_t device, double* ops_per_s) {
+    if (!ops_per_s) { set_err("NULL argument"); return FRUGAL_EINVAL; }
+    CK(cudaSetDevice(device));
+    cudaEvent_t a, b;
+    CK(cudaEventCreate(&a));
+    CK(cudaEventCreate(&b));
+    double* out = nullptr;
+    CK(cudaMalloc(&out, 1 << 20));
+    int64_t ops = 0;
+    launch_probe_fp64(out, 1, &ops, 0);  // warm-up
+    CK(cudaEventRecord(a, 0));
+    launch_probe_fp64(out, 64, &ops, 0);
+    CK(cudaEventRecord(b, 0));
+    CK(cudaEventSynchronize(b));
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, a, b);
+    cudaEventDestroy(a);
+    cudaEventDestroy(b);
+    cudaFree(out);
+    CKL();
+    *ops_per_s = ms > 0 ? (double)ops / (ms * 1e-3) : 0.0;
     return FRUGAL_OK;
 }
 

@@ -17,7 +17,7 @@ LIB_PATH = os.path.join(PKG, "libfrugal.so")
 
 SGD, ADAGRAD = 0, 1
 MODE_P2F, MODE_WRITE_THROUGH = 0, 1
-F_RECORD, F_TIMERS, F_NO_HOST_STATE, F_A2A, F_PEER, F_DYNAMIC_CACHE = 1, 2, 4, 8, 16, 32
+F_RECORD, F_TIMERS, F_NO_HOST_STATE, F_A2A, F_PEER, F_DYNAMIC_CACHE, F_HOST_FLUSH = 1, 2, 4, 8, 16, 32, 64
 FLUSH_ALL = 0
 PHASES = ["ingest", "schedule", "urgent", "gate", "gather", "expand", "model", "segred", "exchange",
           "optimizer", "side", "prefetch"]
@@ -88,6 +88,8 @@ def lib():
             "frugal_get_stats": [P, C.POINTER(Stats)],
             "frugal_get_timeline": [P, P, P, P, I64, C.POINTER(I64)],
             "frugal_probe_host_reads": [P, I64, C.c_uint64, C.POINTER(C.c_double)],
+            "frugal_join": [P, P],
+            "frugal_probe_fp64": [I32, C.POINTER(C.c_double)],
             "frugal_a2a_requests": [P, I64, P, P, P],
             "frugal_a2a_serve": [P, I64, P, I64, P, P],
             "frugal_a2a_lookup": [P, I64, P, P, P],
@@ -114,7 +116,8 @@ EXPORTED = ["frugal_init", "frugal_prefetch", "frugal_step", "frugal_lookup", "f
             "frugal_get_schedule", "frugal_get_final_flush", "frugal_read_rows", "frugal_read_host",
             "frugal_get_stats", "frugal_get_timeline", "frugal_owned_rows", "frugal_hot_slots",
             "frugal_a2a_requests", "frugal_a2a_serve", "frugal_a2a_lookup", "frugal_a2a_pack", "frugal_a2a_update",
-            "frugal_probe_host_reads", "frugal_set_hot", "frugal_get_transition"]
+            "frugal_probe_host_reads", "frugal_set_hot", "frugal_get_transition", "frugal_join",
+            "frugal_probe_fp64"]
 
 
 def _check(status):
@@ -305,6 +308,10 @@ class Frugal:
         _check(lib().frugal_probe_host_reads(self.h, n, seed, C.byref(ms)))
         return ms.value
 
+    def join(self, stream=None):
+        """`stream` waits for all work enqueued on the library's own streams (timing)."""
+        _check(lib().frugal_join(self.h, _stream(stream)))
+
     @property
     def owned_rows(self):
         return lib().frugal_owned_rows(self.h)
@@ -312,3 +319,10 @@ class Frugal:
     @property
     def hot_slots(self):
         return lib().frugal_hot_slots(self.h)
+
+
+def probe_fp64(device=0):
+    """Separately rounded fp64 add/mul instructions per second of the device (calibration)."""
+    r = C.c_double()
+    _check(lib().frugal_probe_fp64(device, C.byref(r)))
+    return r.value

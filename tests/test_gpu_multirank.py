@@ -1,5 +1,7 @@
-"""world = 2 on ONE B200: two rank processes share device 0 and one POSIX-shm host
-table; mailboxes, flags and gates go through host memory exactly as across GPUs.
+"""world = 2: two rank processes and one POSIX-shm host table; mailboxes, flags and gates go
+through host memory.  With >= 2 visible GPUs rank r runs on device r (the distinct-device
+path: cross-GPU visibility of zero-copy host writes, NVLink peer loads, NCCL all-to-all);
+the `same_device` variants put both ranks on device 0 (the only choice on a one-GPU box).
 Compared against the oracle run with world 2: per-rank schedule sets (each rank owns
 k mod 2 == rank), final flush, host table (w, G) and the global loss."""
 import multiprocessing as mp
@@ -14,22 +16,33 @@ from paper_conf_asplos_xiezggl25_b200 import workload as W
 pytestmark = pytest.mark.gpu
 
 
-def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False, fused=False, nonce=1):
+def n_gpus():
+    import torch
+    return torch.cuda.device_count()
+
+
+def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False, fused=False, nonce=1, device=0,
+               record=True, backend="gloo", host_flush=False):
     try:
         import torch
         from paper_conf_asplos_xiezggl25_b200 import frugal as F
         from paper_conf_asplos_xiezggl25_b200.harness import A2ATrainer, Trainer, make_context
-        torch.cuda.set_device(0)
-        fr = make_context(st, rank=rank, device=0, shm_name=shm, run_nonce=nonce,
-                          flags=F.F_RECORD | (F.F_A2A if a2a else 0) | (F.F_PEER if peer else 0))
+        torch.cuda.set_device(device)
+        flags = (F.F_RECORD if record else F.F_TIMERS) | (F.F_A2A if a2a else 0) | (F.F_PEER if peer else 0) \
+            | (F.F_HOST_FLUSH if host_flush else 0)
+        fr = make_context(st, rank=rank, device=device, shm_name=shm, run_nonce=nonce, flags=flags)
         barrier.wait()
         if a2a:
             import torch.distributed as dist
             os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
-            dist.init_process_group("gloo", rank=rank, world_size=2)
-            tr = A2ATrainer(fr, st, rank=rank, dist=dist, host_staging=True)
+            if backend == "nccl":
+                dist.init_process_group("nccl", rank=rank, world_size=2, device_id=torch.device("cuda", device))
+            else:
+                dist.init_process_group("gloo", rank=rank, world_size=2)
+            tr = A2ATrainer(fr, st, rank=rank, device=device, dist=dist, host_staging=backend == "gloo")
         else:
-            tr = Trainer(fr, st, rank=rank, fused_lookup=fused)
+            # record=False: the bench's configuration -- no per-step synchronisation, inputs in HBM
+            tr = Trainer(fr, st, rank=rank, device=device, fused_lookup=fused, device_inputs=not record)
         sched = []
         for s in range(st.steps):
             got = {}
@@ -37,7 +50,7 @@ def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False, fused=F
             def cb(s_):
                 got.update(fr.get_schedule())
                 got["transition"] = fr.get_transition()
-            tr.step(on_schedule=cb)
+            tr.step(on_schedule=cb if record else None)
             sched.append(got)
         fr.flush()
         ff = fr.get_final_flush()
@@ -54,7 +67,8 @@ def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False, fused=F
         q.put((rank, traceback.format_exc()))
 
 
-def run_two_ranks(st, timeout=600, a2a=False, peer=False, fused=False):
+def run_two_ranks(st, timeout=600, a2a=False, peer=False, fused=False, same_device=True, record=True,
+                  backend="gloo", host_flush=False):
     import socket
     ctx = mp.get_context("spawn")
     barrier = ctx.Barrier(2)
@@ -65,7 +79,10 @@ def run_two_ranks(st, timeout=600, a2a=False, peer=False, fused=False):
     port = sk.getsockname()[1]
     sk.close()
     nonce = int.from_bytes(os.urandom(8), "little") | 1
-    ps = [ctx.Process(target=_rank_main, args=(r, st, shm, barrier, q, a2a, port, peer, fused, nonce))
+    if not same_device and n_gpus() < 2:
+        pytest.skip("needs 2 GPUs (rank r on device r)")
+    ps = [ctx.Process(target=_rank_main, args=(r, st, shm, barrier, q, a2a, port, peer, fused, nonce,
+                                               0 if same_device else r, record, backend, host_flush))
           for r in range(2)]
     for p in ps:
         p.start()
@@ -84,13 +101,14 @@ def run_two_ranks(st, timeout=600, a2a=False, peer=False, fused=False):
     return out
 
 
+@pytest.mark.parametrize("same_device", [True, False])
 @pytest.mark.parametrize("opt,a2a,peer,dyn,layout", [("adagrad", False, False, False, False),
                                                      ("sgd", False, False, False, False),
                                                      ("adagrad", True, False, False, False),
                                                      ("adagrad", False, True, False, False),
                                                      ("adagrad", False, False, True, False),
                                                      ("adagrad", False, False, False, True)])
-def test_two_ranks_one_gpu_parity(opt, a2a, peer, dyn, layout):
+def test_two_ranks_parity(opt, a2a, peer, dyn, layout, same_device):
     """a2a=True: the comparison path (§8(e)) -- ids, rows and partials move by all-to-all
     (gloo with host staging here; NCCL over NVLink on a multi-GPU box) instead of the host
     table and mailbox; every artefact and table must be identical.  peer=True: the N4
@@ -110,7 +128,7 @@ def test_two_ranks_one_gpu_parity(opt, a2a, peer, dyn, layout):
     if layout:  # a random half of the rows first, in random order; the rest in id order
         order = np.random.default_rng(11).permutation(cfg.n_rows)[:cfg.n_rows // 2]
         st = W.dataclasses.replace(st, host_order=order.astype(np.int64))
-    out = run_two_ranks(st, a2a=a2a, peer=peer)
+    out = run_two_ranks(st, a2a=a2a, peer=peer, same_device=same_device)
     if peer:  # the variant actually served rows from the other rank's HBM
         assert out[0]["stats"]["gather_peer"] > 0 and out[1]["stats"]["gather_peer"] > 0
     o = Oracle(st)
@@ -140,15 +158,16 @@ def test_two_ranks_one_gpu_parity(opt, a2a, peer, dyn, layout):
 
 
 
+@pytest.mark.parametrize("same_device", [True, False])
 @pytest.mark.parametrize("fused", [False, True])
-def test_configs0_two_ranks_exact_shape(fused):
+def test_configs0_two_ranks_exact_shape(fused, same_device):
     """BASELINE.json configs[0] as stated: 1 table 10^4 x 16, batch 256, 20 steps, 2 GPUs
     (here: 2 rank processes sharing one B200), Zipf ids.  fused: the bench's default fused
     lookup (glue reads each rank's gathered distinct rows through its inverse index)."""
     from oracle.oracle import Oracle
     cfg = W.config("tiny")  # world 2, batch 256
     st = W.gen_stream(cfg, 20)
-    out = run_two_ranks(st, fused=fused)
+    out = run_two_ranks(st, fused=fused, same_device=same_device)
     o = Oracle(st)
     for s in range(st.steps):
         o.step()
@@ -163,3 +182,86 @@ def test_configs0_two_ranks_exact_shape(fused):
     assert np.array_equal(out[0]["w"], wo) and np.array_equal(out[0]["G"], Go)
     lo = np.array([o.loss(s) for s in range(st.steps)])
     assert np.abs(out[0]["losses"] + out[1]["losses"] - lo).max() <= 1e-5
+
+
+def _compare_whole_run(st, out, exact=True):
+    """Values-only comparison (no per-step sets): losses, final flush, host table."""
+    from oracle.oracle import Oracle
+    o = Oracle(st)
+    o.run()
+    assert o.violations == 0
+    lo = np.array([o.loss(s) for s in range(st.steps)])
+    assert np.abs(out[0]["losses"] + out[1]["losses"] - lo).max() <= 1e-5
+    assert sorted(out[0]["ff"].tolist() + out[1]["ff"].tolist()) == o.final_flush().tolist()
+    wo, Go = o.read_rows(np.arange(st.cfg.n_rows))
+    if exact:
+        assert np.array_equal(out[0]["w"], wo) and np.array_equal(out[0]["G"], Go)
+    assert np.abs(out[0]["w"] - wo).max() <= 1e-5 and np.abs(out[0]["G"] - Go).max() <= 1e-5
+
+
+@pytest.mark.parametrize("same_device", [True, False])
+@pytest.mark.parametrize("fused", [False, True])
+def test_two_ranks_overlapped_pipeline(fused, same_device):
+    """world 2 in the bench's configuration (F_TIMERS only, device-resident inputs,
+    no per-step callbacks, so ingest, drain, mailbox exchange and gates overlap freely);
+    losses, final-flush set and the whole host table against the oracle."""
+    cfg = W.config("tiny", world=2, batch=128, lookahead=4, age_out=3)
+    st = W.gen_stream(cfg, 60)
+    out = run_two_ranks(st, fused=fused, same_device=same_device, record=False)
+    _compare_whole_run(st, out)
+
+
+@pytest.mark.parametrize("variant", ["p2f", "peer", "a2a_gloo", "a2a_nccl"])
+@pytest.mark.parametrize("same_device", [True, False])
+def test_two_ranks_100_step_stress(variant, same_device):
+    """100 steps of configs[0] (world 2, batch 256, L 10, D 10) for the host-bounced P2F path,
+    the N4 peer variant and the a2a comparison path (gloo with host staging, or NCCL -- over
+    NVLink when the ranks sit on distinct GPUs; NCCL needs distinct devices).  Every schedule
+    set per step, the oracle's invariant (2), losses, final flush and the whole table."""
+    if variant == "a2a_nccl" and same_device:
+        pytest.skip("NCCL needs one device per rank")
+    from oracle.oracle import Oracle
+    cfg = W.config("tiny")
+    st = W.gen_stream(cfg, 100)
+    out = run_two_ranks(st, a2a=variant.startswith("a2a"), peer=variant == "peer", same_device=same_device,
+                        backend="nccl" if variant == "a2a_nccl" else "gloo", timeout=1200)
+    o = Oracle(st)
+    for s in range(st.steps):
+        o.step()
+        ref = o.schedule()
+        urg = sorted(sum((out[r]["sched"][s]["urgent"].tolist() for r in range(2)), []))
+        assert urg == ref["urgent"].tolist(), f"urgent differs at {s}"
+        dfr = sorted(sum((list(zip(out[r]["sched"][s]["deferred"].tolist(),
+                                   out[r]["sched"][s]["deferred_p"].tolist())) for r in range(2)), []))
+        assert dfr == sorted(zip(ref["deferred"].tolist(), ref["deferred_p"].tolist())), f"deferred differs at {s}"
+        age = sorted(sum((out[r]["sched"][s]["ageout"].tolist() for r in range(2)), []))
+        assert age == ref["ageout"].tolist(), f"age-out differs at {s}"
+        assert any(out[r]["sched"][s]["gate_wait"] for r in range(2)) == ref["gate_wait"]
+    assert o.violations == 0
+    assert sorted(out[0]["ff"].tolist() + out[1]["ff"].tolist()) == o.final_flush().tolist()
+    lo = np.array([o.loss(s) for s in range(st.steps)])
+    assert np.abs(out[0]["losses"] + out[1]["losses"] - lo).max() <= 1e-5
+    wo, Go = o.read_rows(np.arange(cfg.n_rows))
+    assert np.array_equal(out[0]["w"], wo) and np.array_equal(out[0]["G"], Go)
+    if variant == "peer":
+        assert out[0]["stats"]["gather_peer"] > 0 and out[1]["stats"]["gather_peer"] > 0
+
+
+@pytest.mark.parametrize("record", [True, False])
+@pytest.mark.parametrize("same_device", [True, False])
+def test_two_ranks_host_flush(record, same_device):
+    """FRUGAL_F_HOST_FLUSH at world 2: each owner's flushing threads publish its FLAG_SIDE_FIRST;
+    the other rank's gate waits for it before reading the owner's drained rows."""
+    from oracle.oracle import Oracle
+    cfg = W.config("tiny", world=2, batch=128, lookahead=4, age_out=3)
+    st = W.gen_stream(cfg, 50)
+    out = run_two_ranks(st, same_device=same_device, record=record, host_flush=True, fused=True)
+    if record:
+        o = Oracle(st)
+        for s in range(st.steps):
+            o.step()
+            ref = o.schedule()
+            dfr = sorted(sum((list(zip(out[r]["sched"][s]["deferred"].tolist(),
+                                       out[r]["sched"][s]["deferred_p"].tolist())) for r in range(2)), []))
+            assert dfr == sorted(zip(ref["deferred"].tolist(), ref["deferred_p"].tolist())), f"deferred differs at {s}"
+    _compare_whole_run(st, out)

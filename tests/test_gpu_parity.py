@@ -23,7 +23,7 @@ def _F():
 
 
 def run_parity(st, *, flags=None, mode=None, hot=None, check_dedup=True, check_sched=True, steps=None,
-               sample_rows=None, oracle_kw=None, fused=False):
+               sample_rows=None, oracle_kw=None, fused=False, on_step=None):
     """Run the stream on cuda:0 (world 1) and on the oracle; assert the bars."""
     F = _F()
     from paper_conf_asplos_xiezggl25_b200.harness import Trainer, make_context
@@ -66,6 +66,8 @@ def run_parity(st, *, flags=None, mode=None, hot=None, check_dedup=True, check_s
             assert sorted(got["transition"].tolist()) == ref["transition"].tolist(), f"transition differs at {s}"
             assert got["gate_wait"] == ref["gate_wait"]
             gate_waits += ref["gate_wait"]
+            if on_step:
+                on_step(s, got)
     assert o.violations == 0
     lo = np.array([o.loss(s) for s in range(S)])
     lg = tr.losses()[:S]
@@ -88,6 +90,45 @@ def run_parity(st, *, flags=None, mode=None, hot=None, check_dedup=True, check_s
         out.update(dw=float(np.abs(w - wo).max()), dG=float(np.abs(G - Go).max()))
         assert out["dw"] <= TOL and out["dG"] <= TOL, (out["dw"], out["dG"])
     return out
+
+
+def run_overlapped(st, *, fused=True, flags=None, sample_rows=None, hot=None, exact=None):
+    """The bench's launch configuration: FRUGAL_F_TIMERS only (no F_RECORD, so no
+    per-step synchronisation), no per-step callbacks, ids / x / y resident in HBM and passed
+    as device pointers -- the ingest of s+L, the side drain and the main stream overlap as in
+    bench.py.  After frugal_flush: per-step losses, the final-flush set and the host table
+    (w, G; all rows or `sample_rows`) against the oracle run to the end."""
+    F = _F()
+    from paper_conf_asplos_xiezggl25_b200.harness import Trainer, make_context
+    flags = F.F_TIMERS if flags is None else flags
+    hot = st.hot if hot is None else hot
+    fr = make_context(st, flags=flags, hot=hot)
+    tr = Trainer(fr, st, fused_lookup=fused, device_inputs=True)
+    tr.run()
+    fr.flush()
+    lg = tr.losses()
+    o = Oracle(st, hot=hot)
+    o.run()
+    assert o.violations == 0
+    lo = np.array([o.loss(s) for s in range(st.steps)])
+    assert np.abs(lg - lo).max() <= TOL, f"loss differs by {np.abs(lg - lo).max()}"
+    assert sorted(fr.get_final_flush().tolist()) == o.final_flush().tolist(), "final flush set differs"
+    ks = np.arange(st.cfg.n_rows) if sample_rows is None else sample_rows
+    w, G = fr.read_host(ks)
+    wo, Go = o.read_rows(ks)
+    dw, dG = float(np.abs(w - wo).max()), float(np.abs(G - Go).max())
+    assert dw <= TOL and dG <= TOL, (dw, dG)
+    if exact:
+        assert np.array_equal(w, wo) and np.array_equal(G, Go), "tables are expected bit-exact"
+    stats = fr.get_stats()
+    fr.close()
+    return dict(stats=stats, w=w, wo=wo)
+
+
+def _touched_sample(st, steps, size, seed):
+    rng = np.random.default_rng(seed)
+    touched = np.unique(st.ids[:steps, 0].ravel())
+    return np.sort(rng.choice(touched, size=min(size, len(touched)), replace=False))
 
 
 def tiny1(**over):
@@ -173,19 +214,6 @@ def test_write_through_flushes_every_update():
     r["fr"].close()
 
 
-def test_criteo_kaggle_full_size_sampled():
-    """configs[1] shape (26 tables, 33.8M rows, d=32, batch 8192) at world 1, the launch
-    configuration bench.py times: dedup and schedule sets bit-exact every step, sampled
-    touched rows within 1e-5 (oracle materialises rows lazily)."""
-    cfg = W.config("criteo_kaggle", world=1)
-    st = W.gen_stream(cfg, 14)
-    rng = np.random.default_rng(0)
-    touched = np.unique(st.ids[:6, 0].ravel())
-    sample = np.sort(rng.choice(touched, size=20000, replace=False))
-    r = run_parity(st, steps=6, sample_rows=sample)
-    r["fr"].close()
-
-
 def test_fused_lookup_parity():
     """Fused lookup (lookup/dot_model with NULL emb: the glue reads the gathered distinct
     rows through inv, no expand): tables, losses and sets bit-exact as with the expand."""
@@ -206,15 +234,6 @@ def test_fused_lookup_shapes(dim, tables):
     counts[5] = 0
     st = W.gen_stream(cfg, 20, counts=counts)
     run_parity(st, fused=True)["fr"].close()
-
-
-def test_fused_lookup_criteo_full_size_sampled():
-    cfg = W.config("criteo_kaggle", world=1)
-    st = W.gen_stream(cfg, 14)
-    rng = np.random.default_rng(1)
-    touched = np.unique(st.ids[:6, 0].ravel())
-    sample = np.sort(rng.choice(touched, size=20000, replace=False))
-    run_parity(st, steps=6, sample_rows=sample, fused=True)["fr"].close()
 
 
 def test_fused_lookup_errors():
@@ -347,18 +366,6 @@ def test_kg_transe_tiles_ragged():
 
 
 
-def test_avazu_full_size_sampled():
-    """configs[2] shape (22 tables, 9.4e6 rows, d=64, batch 16384, cache 10 %) at world 1:
-    dedup and schedule sets bit-exact every step, sampled touched rows within 1e-5."""
-    cfg = W.config("avazu", world=1)
-    st = W.gen_stream(cfg, 12)
-    rng = np.random.default_rng(1)
-    touched = np.unique(st.ids[:5, 0].ravel())
-    sample = np.sort(rng.choice(touched, size=min(20000, len(touched)), replace=False))
-    r = run_parity(st, steps=5, sample_rows=sample)
-    r["fr"].close()
-
-
 def test_fb15k_kg_full_size():
     """FB15k-shaped KG at full size (14,951 entities + 1,345 relations, d=400, batch 1200,
     chunks of 200 negatives): every artefact and the whole table against the oracle."""
@@ -427,3 +434,122 @@ def test_dynamic_cache_capacity_and_order_errors():
     with pytest.raises(F.FrugalError, match="slots"):
         tr.run()
     fr.close()
+
+
+# ----------------------------------------------------------------------------- overlapped pipeline
+@pytest.mark.parametrize("fused", [False, True])
+def test_overlapped_pipeline_tiny_100_steps(fused):
+    """the exact-parity runs above record the schedule (F_RECORD synchronises
+    after every scheduler), so they never overlap the ingest of s+L with the gather and the
+    backward of s.  Here: the bench's configuration (F_TIMERS only, device-resident inputs,
+    no callbacks), world 1, 100 steps; tables bit-exact."""
+    st = W.gen_stream(tiny1(), 100)
+    run_overlapped(st, fused=fused, exact=True)
+
+
+@pytest.mark.parametrize("env", [{"FRUGAL_EARLY": "1"}, {"FRUGAL_DRAIN_AT": "sched"}, {"FRUGAL_FUSE_OPT": "0"}])
+def test_overlapped_pipeline_knobs(env):
+    """The optional schedules of DESIGN.md §10 in the overlapped configuration (subprocess:
+    the knobs are read at context creation)."""
+    import subprocess
+    import sys
+    code = ("import sys; sys.path.insert(0, '.');"
+            "from tests.test_gpu_parity import run_overlapped, tiny1; from paper_conf_asplos_xiezggl25_b200 import workload as W;"
+            "st = W.gen_stream(tiny1(batch=128, lookahead=4, age_out=2), 60);"
+            "run_overlapped(st, fused=True, exact=True); print('OK')")
+    e = dict(os.environ)
+    e.update(env)
+    out = subprocess.run([sys.executable, "-c", code], env=e, capture_output=True, text=True,
+                         cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=600)
+    assert "OK" in out.stdout, out.stdout + out.stderr
+
+
+# ----------------------------------------------------------------------------- full size, 100 steps
+def test_criteo_kaggle_100_steps_recorded():
+    """configs[1] at full size (26 tables, 33.8M rows, d 32, batch 8192, cache 5 %, L 10,
+    D 10), 100 steps (the north_star bar): dedup, every schedule set and the gate bit-exact
+    at every step; losses within 1e-5; final-flush set exact; 20k sampled touched rows of
+    the host table (w, G) within 1e-5 after the final flush.  Past step 11 rows are aged
+    out, and 100 steps wrap each of the P = D+3 = 13 dirty-pool segments 7 times."""
+    cfg = W.config("criteo_kaggle", world=1)
+    st = W.gen_stream(cfg, 100)
+    sample = _touched_sample(st, 100, 20000, 0)
+    ages = []
+
+    F = _F()
+    r = run_parity(st, sample_rows=sample, fused=True, flags=F.F_RECORD,
+                   on_step=lambda s, got: ages.append(len(got["ageout"])))
+    c = r["fr"].get_stats()["count"]
+    assert sum(ages[:cfg.age_out + 1]) == 0 and sum(ages) > 0, "age-out never exercised"
+    assert c["gather_pool"] > 0 and st.steps > cfg.age_out + 3 + 1, "dirty pool never wrapped"
+    r["fr"].close()
+
+
+def test_criteo_kaggle_100_steps_overlapped():
+    """configs[1], 100 steps, in the exact launch configuration bench.py times (fused
+    lookup, F_TIMERS, device-resident inputs, overlapped streams)."""
+    cfg = W.config("criteo_kaggle", world=1)
+    st = W.gen_stream(cfg, 100)
+    run_overlapped(st, fused=True, sample_rows=_touched_sample(st, 100, 20000, 1))
+
+
+def test_avazu_100_steps_recorded():
+    """configs[2] (22 tables, 9.4e6 rows, d 64, batch 16384, cache 10 %), 100 steps, every
+    set exact per step, sampled host rows after the final flush."""
+    cfg = W.config("avazu", world=1)
+    st = W.gen_stream(cfg, 100)
+    ages = []
+    r = run_parity(st, sample_rows=_touched_sample(st, 100, 20000, 2), fused=True,
+                   on_step=lambda s, got: ages.append(len(got["ageout"])))
+    assert sum(ages) > 0
+    r["fr"].close()
+
+
+def test_freebase_shape_sampled():
+    """configs[3] at its shape (Freebase: 86.1M entities + 14,824 relations, d 400, TransE,
+    batch 2000, chunks of 200 negatives; host w 138 GB, G in HBM -- FRUGAL_F_NO_HOST_STATE),
+    15 steps: dedup and every schedule set exact per step, losses within 1e-5, 5000 sampled
+    touched rows (w and G, authoritative values) within 1e-5."""
+    F = _F()
+    cfg = W.config("freebase", world=1)
+    st = W.gen_stream(cfg, 16)
+    r = run_parity(st, steps=15, sample_rows=_touched_sample(st, 15, 5000, 3),
+                   flags=F.F_RECORD | F.F_NO_HOST_STATE)
+    r["fr"].close()
+
+
+# ----------------------------------------------------------------------------- host flushing threads
+def test_host_flush_recorded_tiny():
+    """FRUGAL_F_HOST_FLUSH (the side drain packed into a staging queue, copied into the table by
+    the library's flushing threads): every set, the gate, losses and the whole table exact."""
+    F = _F()
+    st = W.gen_stream(tiny1(lookahead=4, age_out=2, batch=128), 80)
+    r = run_parity(st, flags=F.F_RECORD | F.F_HOST_FLUSH, fused=True)
+    assert r["exact"]
+    r["fr"].close()
+
+
+@pytest.mark.parametrize("fused", [False, True])
+def test_host_flush_overlapped_tiny(fused):
+    F = _F()
+    st = W.gen_stream(tiny1(), 100)
+    run_overlapped(st, fused=fused, flags=F.F_TIMERS | F.F_HOST_FLUSH, exact=True)
+
+
+def test_host_flush_dynamic_cache():
+    """N3 transitions wait for the flushing threads (an admitted row may have been drained by the
+    previous step and must be read from the table after the threads applied it)."""
+    F = _F()
+    cfg = tiny1(lookahead=4, age_out=3, cache_ratio=0.05)
+    st = W.with_dynamic_hot(W.gen_stream(cfg, 60), epoch=7)
+    r = run_parity(st, flags=F.F_RECORD | F.F_HOST_FLUSH)
+    assert r["exact"]
+    r["fr"].close()
+
+
+def test_host_flush_criteo_kaggle_100_steps_overlapped():
+    """configs[1] at full size, 100 steps, bench configuration with the flushing threads."""
+    F = _F()
+    cfg = W.config("criteo_kaggle", world=1)
+    st = W.gen_stream(cfg, 100)
+    run_overlapped(st, fused=True, flags=F.F_TIMERS | F.F_HOST_FLUSH, sample_rows=_touched_sample(st, 100, 20000, 4))
