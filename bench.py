@@ -68,10 +68,10 @@ def parse():
                          "default: the REC glue reads the gathered distinct rows through the inverse index "
                          "(frugal_lookup / frugal_dot_model with NULL emb, no expand; "
                          "profiles/r1_sweep32_fused_lookup.txt)")
-    ap.add_argument("--drain", default="gpu", choices=["gpu", "host"],
-                    help="deferred drain (a11): gpu = zero-copy scatter kernel on the side stream; host = packed "
-                         "into a staging queue, copied into the table by the library's flushing threads "
-                         "(FRUGAL_F_HOST_FLUSH)")
+    ap.add_argument("--drain", default="host", choices=["gpu", "host"],
+                    help="deferred drain (a11): host (default) = packed by a kernel into a staging queue, copied "
+                         "into the table by the library's flushing threads (PAPER.md L1055-1059); gpu = zero-copy "
+                         "scatter kernel on the side stream (FRUGAL_F_GPU_DRAIN)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for barriers / the max-over-ranks timing only")
     return ap.parse_args()
@@ -305,7 +305,7 @@ def main():
                       flags=F.F_TIMERS | (F.F_NO_HOST_STATE if no_host_state else 0) | (F.F_A2A if a2a else 0)
                       | (F.F_PEER if (args.peer and world > 1) else 0)
                       | (F.F_DYNAMIC_CACHE if args.cache_refresh > 0 else 0)
-                      | (F.F_HOST_FLUSH if args.drain == "host" else 0),
+                      | (F.F_GPU_DRAIN if args.drain == "gpu" else 0),
                       mode=F.MODE_WRITE_THROUGH if args.mode == "write_through" else F.MODE_P2F)
     # N3: the hot set of every epoch start t0 (bench step numbering; step t reads generated
     # step t % SG), from the E bench steps before t0 -- inputs, computed before any timing,
@@ -597,7 +597,7 @@ def main():
                    "lookahead": L, "age_out": cfg.age_out, "cache_ratio": cfg.cache_ratio, "opt": cfg.opt,
                    "flush_mode": args.mode,
                    "drain": "side-stream zero-copy scatter kernel" if args.drain == "gpu" else
-                            "packed staging queue + library flushing threads (FRUGAL_F_HOST_FLUSH)",
+                            "packed staging queue + library flushing threads (default)",
                    "exchange": "host table + mailbox (P2F)" if not a2a else
                    "all-to-all over the process group (comparison path)",
                    "peer_reads": bool(args.peer and world > 1),

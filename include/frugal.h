@@ -68,14 +68,16 @@ enum {
     FRUGAL_F_DYNAMIC_CACHE = 32,/* N3: the hot set may change at epoch
                                    boundaries (frugal_set_hot); the cache gets 25% spare
                                    slots; not with FRUGAL_F_PEER or the early gather      */
-    FRUGAL_F_HOST_FLUSH = 64,   /* the side-stream drain (a11) packs its rows into a pinned
-                                   staging queue as one contiguous run and the library's
-                                   background flushing threads (§3.2,
-                                   L1055-1059) copy them into the host table; the gate of
-                                   s+1 waits for the threads' progress word.  Random 128-B
-                                   zero-copy stores from the GPU over the whole table stall
-                                   the concurrent HBM kernels; the staging
-                                   run is sequential.  Threads: FRUGAL_FLUSH_THREADS (env) */
+    FRUGAL_F_GPU_DRAIN = 64,    /* the side-stream drain (a11) scatters its rows into the host
+                                   table with zero-copy stores from a kernel.  Default (flag
+                                   clear): the drain kernel packs the rows into a pinned staging
+                                   queue as one contiguous run and the library's background
+                                   flushing threads (§3.2) copy them
+                                   into the table; the gate of s+1 waits for the threads' progress
+                                   word.  Random 128-B zero-copy stores over the whole table stall
+                                   the concurrent HBM kernels; the staging run is
+                                   sequential.  Threads: FRUGAL_FLUSH_THREADS (env, default
+                                   nproc/4 in [2, 8]) */
     FRUGAL_F_A2A = 8            /* comparison path (the message pipeline of
                                    PAPER.md Fig. 2b): rows and gradients move between
                                    ranks by the caller's all-to-all (NCCL over NVLink) through

@@ -116,6 +116,7 @@ struct frugal_ctx {
     int side_first_blocks = 20;      // grid cap of the drain's deadline-(s+1) part
     int flush_tma = 0;               // flushes by TMA bulk stores: 0 none, 1 side drain, 2 all (FRUGAL_FLUSH_TMA; measured no gain: profiles/r1_sweep21_flush_tma.txt)
     int glue_cache = -1;         // REC glue keeps a sample's rows in registers (F <= 32): -1 auto, 0 never, 1 always
+    bool glue_rg = true;         // REC glue: row-group kernel k_dot_rg (FRUGAL_GLUE_RG=0: the warp-per-sample k_dot_model)
     bool fuse_opt = true;        // world 1: a8 fused into a6 (k_segreduce / k_segred_combine)
     bool update1 = true;         // world 1 fused: one-launch k_update1 (FRUGAL_UPDATE1=0: the 3-kernel path)
     int gather_blocks = 120;     // grid cap of the zero-copy gathers (120 CTAs: +3% over 74 and 148 in the step, profiles/r1_sweep34_gather_grid.txt)
@@ -245,7 +246,7 @@ struct frugal_ctx {
     double* kg_A = nullptr;
     int kg_C = 0;
 
-    // host flushing threads (FRUGAL_F_HOST_FLUSH): the side drain is packed into a pinned staging
+    // host flushing threads (default; FRUGAL_F_GPU_DRAIN: off): the side drain is packed into a pinned staging
     // queue (2 buffers, by step parity) and copied into the host table by these threads
     bool host_flush = false;
     int n_flushers = 0;

@@ -888,7 +888,7 @@ void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begi
     c->launches++;
 }
 
-// a11 with host flushing threads (FRUGAL_F_HOST_FLUSH; §3.2:
+// a11 with host flushing threads (default; FRUGAL_F_GPU_DRAIN: k_flush_rows instead; §3.2:
 // "background flushing threads ... flush the parameter updates ... to host memory"): the
 // drain's rows -- list 1 (deadline s+1) first, then list 2 (later deadlines) and list 3
 // (age-outs) -- are packed into a host staging queue as ONE contiguous run (coalesced
@@ -1243,10 +1243,121 @@ __global__ void __launch_bounds__(256) k_dot_model(const float* __restrict__ emb
     }
 }
 
+// Row-group glue: GS lanes per sample (GS = pow2 >= d/4, <= 32), lane l holds columns
+// v = l + k*GS (float4, k < VPL) of S and x; the sample's F rows are read twice from L2 (the
+// fused lookup's distinct rows, or the expanded rows) -- once for S and |e|^2, once for the
+// gradient -- instead of being kept in registers, so ~40 registers and full occupancy.
+// Same arithmetic as k_dot_model: S in fp32, f ascending; z, p, loss in fp64; c rounded to
+// fp32 once; grad = c*((S - e_f) + x) with each op rounded (R16).
+template <int GS, int VPL, bool FUSED>
+__global__ void __launch_bounds__(256) k_dot_rg(const float4* __restrict__ emb, const int32_t* __restrict__ inv,
+                                                const float4* __restrict__ x, const float* __restrict__ y,
+                                                float4* __restrict__ grad, double* loss, int count, int F, int d4,
+                                                double nb) {
+    __shared__ double sl[8];
+    int64_t gid, gs;
+    int l;
+    RowGroup<GS>::ids(gid, gs, l);
+    double lsum = 0.0;
+    const unsigned gmask = GS == 32 ? FULL : (((1u << GS) - 1u) << ((threadIdx.x & 31) & ~(GS - 1)));
+    auto row = [&](int64_t b, int f) -> const float4* {
+        return FUSED ? emb + (int64_t)__ldg(inv + b * F + f) * d4 : emb + (b * F + f) * d4;
+    };
+    for (int64_t b = gid; b < count; b += gs) {
+        float4 S[VPL], xv[VPL];
+        double ee = 0.0, sq = 0.0, xs = 0.0;
+#pragma unroll
+        for (int k = 0; k < VPL; k++) {
+            S[k] = make_float4(0.f, 0.f, 0.f, 0.f);
+            const int v = l + k * GS;
+            xv[k] = v < d4 ? x[b * d4 + v] : make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+        for (int f = 0; f < F; f++) {
+            const float4* e = row(b, f);
+#pragma unroll
+            for (int k = 0; k < VPL; k++) {
+                const int v = l + k * GS;
+                if (v < d4) {
+                    const float4 a = e[v];
+                    S[k].x = __fadd_rn(S[k].x, a.x);
+                    S[k].y = __fadd_rn(S[k].y, a.y);
+                    S[k].z = __fadd_rn(S[k].z, a.z);
+                    S[k].w = __fadd_rn(S[k].w, a.w);
+                    ee += (double)a.x * a.x + (double)a.y * a.y + (double)a.z * a.z + (double)a.w * a.w;
+                }
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < VPL; k++) {
+            sq += (double)S[k].x * S[k].x + (double)S[k].y * S[k].y + (double)S[k].z * S[k].z + (double)S[k].w * S[k].w;
+            xs += (double)xv[k].x * S[k].x + (double)xv[k].y * S[k].y + (double)xv[k].z * S[k].z +
+                  (double)xv[k].w * S[k].w;
+        }
+#pragma unroll
+        for (int o = GS / 2; o; o >>= 1) {  // within the sample's lane group only
+            sq += __shfl_xor_sync(gmask, sq, o);
+            ee += __shfl_xor_sync(gmask, ee, o);
+            xs += __shfl_xor_sync(gmask, xs, o);
+        }
+        const double z = 0.5 * (sq - ee) + xs;
+        const double p = 1.0 / (1.0 + exp(-z));
+        const double yb = (double)y[b];
+        if (l == 0) lsum += (z > 0 ? z + log1p(exp(-z)) : log1p(exp(z))) - yb * z;
+        const float cc = (float)((p - yb) / nb);  // same rounding as the definition (R16)
+        for (int f = 0; f < F; f++) {
+            const float4* e = row(b, f);
+            float4* g0 = grad + (b * F + f) * d4;
+#pragma unroll
+            for (int k = 0; k < VPL; k++) {
+                const int v = l + k * GS;
+                if (v < d4) {
+                    const float4 a = e[v];
+                    float4 r;
+                    r.x = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[k].x, a.x), xv[k].x));
+                    r.y = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[k].y, a.y), xv[k].y));
+                    r.z = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[k].z, a.z), xv[k].z));
+                    r.w = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[k].w, a.w), xv[k].w));
+                    g0[v] = r;
+                }
+            }
+        }
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) lsum += __shfl_xor_sync(FULL, lsum, o);  // whole warp, after the loop
+    if ((threadIdx.x & 31) == 0) sl[threadIdx.x >> 5] = lsum;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int i = 0; i < 8; i++) t += sl[i];
+        if (t != 0.0) atomicAdd(loss, t / nb);  // mean over the global batch (R17)
+    }
+}
+
 void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const int32_t* inv, const float* x,
                       const float* y, float* grad, double* loss, int64_t nb, cudaStream_t st) {
     int count = q.h_counts[c->g];
     if (count <= 0) return;
+    if (c->glue_rg) {
+        const int d4 = c->d / 4, gs = group_size(d4), vpl = (d4 + gs - 1) / gs;
+        const double nbd = (double)nb;
+#define RG(V)                                                                                                         \
+    do {                                                                                                              \
+        if (inv) {                                                                                                    \
+            DISPATCH_GS(gs, (k_dot_rg<GS, V, true><<<grid_for((int64_t)count * GS, 256, 8), 256, 0, st>>>(           \
+                                (const float4*)emb, inv, (const float4*)x, y, (float4*)grad, loss, count, c->F, d4, nbd))); \
+        } else {                                                                                                      \
+            DISPATCH_GS(gs, (k_dot_rg<GS, V, false><<<grid_for((int64_t)count * GS, 256, 8), 256, 0, st>>>(          \
+                                (const float4*)emb, inv, (const float4*)x, y, (float4*)grad, loss, count, c->F, d4, nbd))); \
+        }                                                                                                             \
+    } while (0)
+        if (vpl <= 1) RG(1);
+        else if (vpl <= 2) RG(2);
+        else if (vpl <= 4) RG(4);
+        else RG(8);
+#undef RG
+        c->launches++;
+        return;
+    }
     int J = (c->d + 31) / 32;
     int grid = grid_for((int64_t)count * 32, 256, 4);
     const double nbd = (double)nb;

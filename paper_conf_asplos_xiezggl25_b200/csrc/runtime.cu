@@ -128,7 +128,7 @@ struct Timer {
 
 // ================================================================================ flushing threads
 // PAPER.md §3.2 (L794-797) and §3.3 (L1055-1059): "background flushing threads ... flush the
-// parameter updates ... to host memory".  With FRUGAL_F_HOST_FLUSH the side-stream drain of
+// parameter updates ... to host memory".  By default (no FRUGAL_F_GPU_DRAIN) the side-stream drain of
 // step s packs its rows into staging buffer s&1 and publishes job s (READY[s&1] = s+1); the
 // threads copy part 1 (deadline s+1) into the table, publish APPLIED_FIRST = s+1 (and, with a
 // shared table, this rank's FLAG_SIDE_FIRST), then part 2 (later deadlines, age-outs) and
@@ -456,8 +456,9 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->peer = (k.flags & FRUGAL_F_PEER) != 0;
     c->dyn = (k.flags & FRUGAL_F_DYNAMIC_CACHE) != 0;
     if (c->dyn) c->early = false;
-    // host flushing threads: the config flag, or FRUGAL_HOST_FLUSH=0/1 (experiments) overriding it
-    c->host_flush = (k.flags & FRUGAL_F_HOST_FLUSH) != 0;
+    // host flushing threads (default), or the GPU scatter drain (FRUGAL_F_GPU_DRAIN);
+    // FRUGAL_HOST_FLUSH=0/1 (experiments) overrides the flag
+    c->host_flush = (k.flags & FRUGAL_F_GPU_DRAIN) == 0;
     if (getenv("FRUGAL_HOST_FLUSH")) c->host_flush = atoi(getenv("FRUGAL_HOST_FLUSH")) != 0;
     if (c->host_flush) c->early = false;  // the early gather synchronises on the GPU drain's events
     c->xhost = c->n > 1 && !c->a2a;
@@ -465,6 +466,8 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     if (getenv("FRUGAL_FLUSH_TMA")) c->flush_tma = atoi(getenv("FRUGAL_FLUSH_TMA"));
     // world 1: optimizer fused into the segment-reduce (FRUGAL_FUSE_OPT=0: two kernels)
     if (getenv("FRUGAL_GLUE_CACHE")) c->glue_cache = atoi(getenv("FRUGAL_GLUE_CACHE"));
+    c->glue_rg = !(getenv("FRUGAL_GLUE_RG") && !atoi(getenv("FRUGAL_GLUE_RG")));
+    if (getenv("FRUGAL_GLUE_CACHE")) c->glue_rg = false;  // the warp-per-sample variants were asked for
     c->fuse_opt = !(getenv("FRUGAL_FUSE_OPT") && !atoi(getenv("FRUGAL_FUSE_OPT")));
     c->update1 = !(getenv("FRUGAL_UPDATE1") && !atoi(getenv("FRUGAL_UPDATE1")));
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 20;

@@ -17,7 +17,7 @@ LIB_PATH = os.path.join(PKG, "libfrugal.so")
 
 SGD, ADAGRAD = 0, 1
 MODE_P2F, MODE_WRITE_THROUGH = 0, 1
-F_RECORD, F_TIMERS, F_NO_HOST_STATE, F_A2A, F_PEER, F_DYNAMIC_CACHE, F_HOST_FLUSH = 1, 2, 4, 8, 16, 32, 64
+F_RECORD, F_TIMERS, F_NO_HOST_STATE, F_A2A, F_PEER, F_DYNAMIC_CACHE, F_GPU_DRAIN = 1, 2, 4, 8, 16, 32, 64
 FLUSH_ALL = 0
 PHASES = ["ingest", "schedule", "urgent", "gate", "gather", "expand", "model", "segred", "exchange",
           "optimizer", "side", "prefetch"]

@@ -22,14 +22,14 @@ def n_gpus():
 
 
 def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False, fused=False, nonce=1, device=0,
-               record=True, backend="gloo", host_flush=False):
+               record=True, backend="gloo", gpu_drain=False):
     try:
         import torch
         from paper_conf_asplos_xiezggl25_b200 import frugal as F
         from paper_conf_asplos_xiezggl25_b200.harness import A2ATrainer, Trainer, make_context
         torch.cuda.set_device(device)
         flags = (F.F_RECORD if record else F.F_TIMERS) | (F.F_A2A if a2a else 0) | (F.F_PEER if peer else 0) \
-            | (F.F_HOST_FLUSH if host_flush else 0)
+            | (F.F_GPU_DRAIN if gpu_drain else 0)
         fr = make_context(st, rank=rank, device=device, shm_name=shm, run_nonce=nonce, flags=flags)
         barrier.wait()
         if a2a:
@@ -68,7 +68,7 @@ def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False, fused=F
 
 
 def run_two_ranks(st, timeout=600, a2a=False, peer=False, fused=False, same_device=True, record=True,
-                  backend="gloo", host_flush=False):
+                  backend="gloo", gpu_drain=False):
     import socket
     ctx = mp.get_context("spawn")
     barrier = ctx.Barrier(2)
@@ -82,7 +82,7 @@ def run_two_ranks(st, timeout=600, a2a=False, peer=False, fused=False, same_devi
     if not same_device and n_gpus() < 2:
         pytest.skip("needs 2 GPUs (rank r on device r)")
     ps = [ctx.Process(target=_rank_main, args=(r, st, shm, barrier, q, a2a, port, peer, fused, nonce,
-                                               0 if same_device else r, record, backend, host_flush))
+                                               0 if same_device else r, record, backend, gpu_drain))
           for r in range(2)]
     for p in ps:
         p.start()
@@ -249,13 +249,13 @@ def test_two_ranks_100_step_stress(variant, same_device):
 
 @pytest.mark.parametrize("record", [True, False])
 @pytest.mark.parametrize("same_device", [True, False])
-def test_two_ranks_host_flush(record, same_device):
-    """FRUGAL_F_HOST_FLUSH at world 2: each owner's flushing threads publish its FLAG_SIDE_FIRST;
-    the other rank's gate waits for it before reading the owner's drained rows."""
+def test_two_ranks_gpu_drain(record, same_device):
+    """FRUGAL_F_GPU_DRAIN at world 2 (the default drain's flushing threads publish each owner's
+    FLAG_SIDE_FIRST from the host; here the drain kernel does, after its zero-copy scatter)."""
     from oracle.oracle import Oracle
     cfg = W.config("tiny", world=2, batch=128, lookahead=4, age_out=3)
     st = W.gen_stream(cfg, 50)
-    out = run_two_ranks(st, same_device=same_device, record=record, host_flush=True, fused=True)
+    out = run_two_ranks(st, same_device=same_device, record=record, gpu_drain=True, fused=True)
     if record:
         o = Oracle(st)
         for s in range(st.steps):

@@ -318,11 +318,14 @@ def test_host_layout_errors():
         assert e.value.status == -1
 
 
-@pytest.mark.parametrize("env", [{"FRUGAL_EARLY": "1"}, {"FRUGAL_DRAIN_AT": "sched"},
-                                 {"FRUGAL_EARLY": "1", "FRUGAL_DRAIN_AT": "sched"}, {"FRUGAL_SIDE_INLINE": "1"},
-                                 {"FRUGAL_NO_POOL_HITS": "1"}, {"FRUGAL_FUSE_OPT": "0"}, {"FRUGAL_FLUSH_TMA": "2"},
-                                 {"FRUGAL_EARLY": "1", "FUSED": "1"}, {"FRUGAL_GLUE_CACHE": "0", "FUSED": "1"},
-                                 {"FRUGAL_GLUE_CACHE": "0"}])
+@pytest.mark.parametrize("env", [{"FRUGAL_EARLY": "1", "FRUGAL_HOST_FLUSH": "0"}, {"FRUGAL_DRAIN_AT": "sched"},
+                                 {"FRUGAL_EARLY": "1", "FRUGAL_DRAIN_AT": "sched", "FRUGAL_HOST_FLUSH": "0"},
+                                 {"FRUGAL_SIDE_INLINE": "1"}, {"FRUGAL_SIDE_INLINE": "1", "FRUGAL_HOST_FLUSH": "0"},
+                                 {"FRUGAL_NO_POOL_HITS": "1"}, {"FRUGAL_FUSE_OPT": "0"}, {"FRUGAL_UPDATE1": "0"},
+                                 {"FRUGAL_FLUSH_TMA": "2", "FRUGAL_HOST_FLUSH": "0"},
+                                 {"FRUGAL_EARLY": "1", "FUSED": "1", "FRUGAL_HOST_FLUSH": "0"},
+                                 {"FRUGAL_GLUE_CACHE": "0", "FUSED": "1"}, {"FRUGAL_GLUE_CACHE": "1", "FUSED": "1"},
+                                 {"FRUGAL_GLUE_CACHE": "0"}, {"FRUGAL_GLUE_RG": "0", "FUSED": "1"}])
 def test_pipeline_modes_parity(env):
     """The optional schedules (early gather of the next step, drain after the gather,
     inline drain) keep every artefact bit-exact (run in a subprocess: the knobs are read
@@ -518,38 +521,54 @@ def test_freebase_shape_sampled():
     r["fr"].close()
 
 
-# ----------------------------------------------------------------------------- host flushing threads
-def test_host_flush_recorded_tiny():
-    """FRUGAL_F_HOST_FLUSH (the side drain packed into a staging queue, copied into the table by
-    the library's flushing threads): every set, the gate, losses and the whole table exact."""
+# ----------------------------------------------------------------------------- GPU scatter drain
+def test_gpu_drain_recorded_tiny():
+    """FRUGAL_F_GPU_DRAIN (the side drain scatters rows into the table from a kernel instead of
+    packing them for the flushing threads): every set, the gate, losses and the whole table exact."""
     F = _F()
     st = W.gen_stream(tiny1(lookahead=4, age_out=2, batch=128), 80)
-    r = run_parity(st, flags=F.F_RECORD | F.F_HOST_FLUSH, fused=True)
+    r = run_parity(st, flags=F.F_RECORD | F.F_GPU_DRAIN, fused=True)
     assert r["exact"]
     r["fr"].close()
 
 
 @pytest.mark.parametrize("fused", [False, True])
-def test_host_flush_overlapped_tiny(fused):
+def test_gpu_drain_overlapped_tiny(fused):
     F = _F()
     st = W.gen_stream(tiny1(), 100)
-    run_overlapped(st, fused=fused, flags=F.F_TIMERS | F.F_HOST_FLUSH, exact=True)
+    run_overlapped(st, fused=fused, flags=F.F_TIMERS | F.F_GPU_DRAIN, exact=True)
 
 
-def test_host_flush_dynamic_cache():
-    """N3 transitions wait for the flushing threads (an admitted row may have been drained by the
-    previous step and must be read from the table after the threads applied it)."""
+def test_gpu_drain_dynamic_cache():
     F = _F()
     cfg = tiny1(lookahead=4, age_out=3, cache_ratio=0.05)
     st = W.with_dynamic_hot(W.gen_stream(cfg, 60), epoch=7)
-    r = run_parity(st, flags=F.F_RECORD | F.F_HOST_FLUSH)
+    r = run_parity(st, flags=F.F_RECORD | F.F_GPU_DRAIN)
     assert r["exact"]
     r["fr"].close()
 
 
-def test_host_flush_criteo_kaggle_100_steps_overlapped():
-    """configs[1] at full size, 100 steps, bench configuration with the flushing threads."""
+def test_gpu_drain_criteo_kaggle_100_steps_overlapped():
+    """configs[1] at full size, 100 steps, overlapped, with the GPU scatter drain."""
     F = _F()
     cfg = W.config("criteo_kaggle", world=1)
     st = W.gen_stream(cfg, 100)
-    run_overlapped(st, fused=True, flags=F.F_TIMERS | F.F_HOST_FLUSH, sample_rows=_touched_sample(st, 100, 20000, 4))
+    run_overlapped(st, fused=True, flags=F.F_TIMERS | F.F_GPU_DRAIN, sample_rows=_touched_sample(st, 100, 20000, 4))
+
+
+def test_flushing_threads_counts_and_env():
+    """The default drain (flushing threads) with 1 and 7 threads (uneven shares) and the
+    N3 transition that waits for them, bit-exact (subprocess: threads are read at init)."""
+    import subprocess
+    import sys
+    for th in ("1", "7"):
+        code = ("import sys; sys.path.insert(0, '.');"
+                "from tests.test_gpu_parity import run_parity, run_overlapped, tiny1; "
+                "from paper_conf_asplos_xiezggl25_b200 import workload as W;"
+                "st = W.gen_stream(tiny1(batch=128, lookahead=4, age_out=2), 50);"
+                "r = run_parity(st); assert r['exact']; r['fr'].close();"
+                "run_overlapped(W.with_dynamic_hot(st, epoch=7), exact=True); print('OK')")
+        e = dict(os.environ, FRUGAL_FLUSH_THREADS=th)
+        out = subprocess.run([sys.executable, "-c", code], env=e, capture_output=True, text=True,
+                             cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=600)
+        assert "OK" in out.stdout, out.stdout + out.stderr

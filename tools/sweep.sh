@@ -9,9 +9,12 @@ cfg=${1:?config}; shift
 REPEAT=${REPEAT:-2}; STEPS=${STEPS:-200}; WARMUP=${WARMUP:-20}
 for i in $(seq "$REPEAT"); do
   for v in "$@"; do
-    envs=(); flags=()
-    for tok in $v; do
-      if [[ $tok == --* ]]; then flags+=("$tok"); else envs+=("$tok"); fi
+    envs=(); flags=(); prev=""
+    for tok in $v; do  # --flag [value] go to bench.py, NAME=value to the environment
+      if [[ $tok == --* ]]; then flags+=("$tok"); prev=flag
+      elif [[ $tok == *=* ]]; then envs+=("$tok"); prev=""
+      elif [[ $prev == flag ]]; then flags+=("$tok"); prev=""
+      else envs+=("$tok"); fi
     done
     env "${envs[@]}" python bench.py --config "$cfg" --no-cpu-baseline --steps "$STEPS" --warmup "$WARMUP" \
         "${flags[@]}" 2>/dev/null |
