@@ -72,6 +72,10 @@ def parse():
                     help="deferred drain (a11): host (default) = packed by a kernel into a staging queue, copied "
                          "into the table by the library's flushing threads (PAPER.md L1055-1059); gpu = zero-copy "
                          "scatter kernel on the side stream (FRUGAL_F_GPU_DRAIN)")
+    ap.add_argument("--ingest", default="v2", choices=["v1", "v2"],
+                    help="N > 1: v2 (default) = each rank passes only its own ids, the ranks exchange distinct "
+                         "ids through the host id mailbox (FRUGAL_F_OWN_IDS); v1 = every rank copies and scans "
+                         "all ranks' ids")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for barriers / the max-over-ranks timing only")
     return ap.parse_args()
@@ -305,7 +309,8 @@ def main():
                       flags=F.F_TIMERS | (F.F_NO_HOST_STATE if no_host_state else 0) | (F.F_A2A if a2a else 0)
                       | (F.F_PEER if (args.peer and world > 1) else 0)
                       | (F.F_DYNAMIC_CACHE if args.cache_refresh > 0 else 0)
-                      | (F.F_GPU_DRAIN if args.drain == "gpu" else 0),
+                      | (F.F_GPU_DRAIN if args.drain == "gpu" else 0)
+                      | (F.F_OWN_IDS if (args.ingest == "v2" and world > 1) else 0),
                       mode=F.MODE_WRITE_THROUGH if args.mode == "write_through" else F.MODE_P2F)
     # N3: the hot set of every epoch start t0 (bench step numbering; step t reads generated
     # step t % SG), from the E bench steps before t0 -- inputs, computed before any timing,
@@ -334,7 +339,10 @@ def main():
     grad = torch.empty_like(emb)
     loss = torch.zeros(S, dtype=torch.float64, device=dev)
     # pinned host copies for the e2e leg
-    ids_h = torch.from_numpy(st.ids).pin_memory()
+    own = args.ingest == "v2" and world > 1  # FRUGAL_F_OWN_IDS: the library gets this rank's ids only
+    ids_h = torch.from_numpy(np.ascontiguousarray(st.ids[:, rank] if own else st.ids)).pin_memory()
+    if own:
+        ids_d = ids_d[:, rank].contiguous()
     x_h = torch.from_numpy(np.ascontiguousarray(st.x[:, rank])).pin_memory()
     y_h = torch.from_numpy(np.ascontiguousarray(st.y[:, rank])).pin_memory()
     loss_h = torch.zeros(S, dtype=torch.float64).pin_memory()
@@ -587,7 +595,8 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(cfg, st, args.cpu_seconds)  # the oracle on the first steps of the same stream
-    h2d = int(world * B * Fs * 8 + B * d * 4 + B * 4 + world * 4)  # ids of all ranks, x, y, counts
+    # ids (this rank's with ingest v2, all ranks' with v1), x, y, counts
+    h2d = int((1 if own else world) * B * Fs * 8 + B * d * 4 + B * 4 + world * 4)
     line = {
         "metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": world, "steps": K, "warmup": Wm,
         "ms_per_step": ms_max / K, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
@@ -601,6 +610,8 @@ def main():
                    "exchange": "host table + mailbox (P2F)" if not a2a else
                    "all-to-all over the process group (comparison path)",
                    "peer_reads": bool(args.peer and world > 1),
+                   "ingest": ("v2: own ids, distinct ids exchanged through the host id mailbox" if own else
+                              "v1: every rank scans all ranks' ids") if world > 1 else "world 1",
                    "lookup": "fused into the glue (no expand)" if fused else "expanded [B*F][d]",
                    "parallelism": f"dp{world} (owner-sharded rows, shared pinned host table)",
                    "l2": "inputs larger than L2: host table %.1f GB, HBM cache %.0f MB, %d distinct id batches "

@@ -78,6 +78,13 @@ enum {
                                    the concurrent HBM kernels; the staging run is
                                    sequential.  Threads: FRUGAL_FLUSH_THREADS (env, default
                                    nproc/4 in [2, 8]) */
+    FRUGAL_F_OWN_IDS = 128,     /* world > 1: frugal_prefetch/frugal_step get only THIS rank's
+                                   ids (int64 [batch*slots]) instead of all ranks' ([world][...]);
+                                   every rank publishes its distinct ids, grouped by owner, in a
+                                   host id mailbox and each owner merges the ids it owns from
+                                   all ranks (its read sets) -- per-rank
+                                   ingest bytes and work no longer grow with world.  counts is
+                                   still [world] (the global batch size of the loss mean) */
     FRUGAL_F_A2A = 8            /* comparison path (the message pipeline of
                                    PAPER.md Fig. 2b): rows and gradients move between
                                    ranks by the caller's all-to-all (NCCL over NVLink) through
@@ -135,7 +142,9 @@ typedef struct {
 frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out);
 
 /* Sample queue (§3.2, §3.3): enqueue the ids of step t of ALL
-   ranks.  ids_all: int64 [world][batch*slots], host (pageable or pinned) or device
+   ranks (FRUGAL_F_OWN_IDS: of this rank only, int64 [batch*slots]; the ranks exchange
+   their distinct ids through the host table's id mailbox).
+   ids_all: int64 [world][batch*slots], host (pageable or pinned) or device
    pointer; it is read after the work already on `stream`, asynchronously on a library
    stream: the caller may overwrite it once the next frugal_prefetch/frugal_step call
    has returned (pageable host memory: as soon as this call returns).

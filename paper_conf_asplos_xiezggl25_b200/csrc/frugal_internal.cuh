@@ -231,6 +231,9 @@ struct frugal_ctx {
     void* peer_open[32][4] = {};                        // opened IPC mappings (to close)
     int32_t* gslot = nullptr;                           // [N] owner's cache slot of every hot row
     bool xhost = false;                                 // world > 1 and host-bounced exchange
+    bool own_ids = false;                               // FRUGAL_F_OWN_IDS: ingest v2 (id mailbox)
+    char* dh_idbox = nullptr;                           // device alias of the id mailbox [kIdSlots][world]
+    size_t idbox_stride = 0;                            // bytes per (slot, rank): 256 B header + M int32
     int32_t* a2a_roff = nullptr;                        // [world] receive offsets (device)
     bool side_pending[2] = {false, false};
 
@@ -277,6 +280,9 @@ namespace frugal {
 void launch_convert_ids(frugal_ctx* c, QueueSlot& q, cudaStream_t st);
 void launch_dedup(frugal_ctx* c, QueueSlot& q, cudaStream_t st);
 void launch_owner_side(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st);
+void launch_owner_side_v2(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st);
+constexpr int kIdSlots = 4;  // id-mailbox slots (step t uses slot t % kIdSlots)
+enum { FLAG_IDS_KIND = 4 };  // host flag kind: this rank's distinct ids of step t published (t+1)
 void launch_cache_transition(frugal_ctx* c, int64_t s, int par, cudaStream_t st);
 void launch_hot_map(frugal_ctx* c, int which, const int64_t* ids64, const int32_t* lks, int64_t n, bool list,
                     cudaStream_t st);

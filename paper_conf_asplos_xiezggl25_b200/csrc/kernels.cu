@@ -237,11 +237,13 @@ void scan_free(ScanScratch& s) {
 __global__ void k_convert_ids(const int64_t* __restrict__ ids64, int32_t* __restrict__ ids32,
                               const int32_t* __restrict__ counts, int world, int M, int F, int64_t N,
                               int g, uint32_t* __restrict__ sk, int32_t* __restrict__ sv,
-                              int32_t* __restrict__ d_m, int32_t* err) {
-    // err lives in mapped pinned host memory: the host sees a bad id without a sync
-    const int64_t total = (int64_t)world * M;
-    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total;
-         e += (int64_t)gridDim.x * blockDim.x) {
+                              int32_t* __restrict__ d_m, int32_t* err, int own_only) {
+    // err lives in mapped pinned host memory: the host sees a bad id without a sync.
+    // own_only (ingest v2): only rank g's row of ids64 / ids32 exists and is converted
+    const int64_t total = own_only ? (int64_t)M : (int64_t)world * M;
+    for (int64_t e0 = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e0 < total;
+         e0 += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t e = own_only ? (int64_t)g * M + e0 : e0;
         int r = (int)(e / M), i = (int)(e - (int64_t)r * M);
         if (i >= counts[r] * F) continue;
         int64_t k = ids64[e];
@@ -318,8 +320,10 @@ __global__ void k_dedup_emit(const uint32_t* __restrict__ ks, const int32_t* __r
 
 void launch_convert_ids(frugal_ctx* c, QueueSlot& q, cudaStream_t st) {
     int64_t total = (int64_t)c->n * c->M;
+    if (c->own_ids) total = c->M;
     k_convert_ids<<<grid_for(total, 256), 256, 0, st>>>(c->ids_stage, q.ids, q.counts, c->n, c->M, c->F, c->N,
-                                                         c->g, c->sort.k[0], c->sort.v[0], q.m, c->err);
+                                                         c->g, c->sort.k[0], c->sort.v[0], q.m, c->err,
+                                                         c->own_ids ? 1 : 0);
     c->launches++;
 }
 
@@ -474,6 +478,84 @@ __global__ void k_copy_i32(const int32_t* __restrict__ a, int32_t* __restrict__ 
     for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) b[i] = a[i];
 }
 
+// ---------------------------------------------------------------------------- ingest v2 (FRUGAL_F_OWN_IDS)
+// (1) this rank's distinct ids of step t, grouped by owner (gl, goff), to its id-mailbox slot:
+// [goff[0..world]] in a 256-B header, then the ids (coalesced zero-copy stores, sequential)
+__global__ void k_idbox_write(const int32_t* __restrict__ uniq, const int32_t* __restrict__ gl,
+                              const int32_t* __restrict__ goff, const int32_t* d_nu, int world, char* box) {
+    const int n = *d_nu;
+    int32_t* hdr = (int32_t*)box;
+    int32_t* ids = (int32_t*)(box + 256);
+    if (blockIdx.x == 0 && threadIdx.x <= world) hdr[threadIdx.x] = goff[threadIdx.x];
+    for (int q = blockIdx.x * blockDim.x + threadIdx.x; q < n; q += gridDim.x * blockDim.x) ids[q] = uniq[gl[q]];
+    block_fence_system();
+}
+// (2) every rank r's segment of ids owned by this rank g (ascending), as composite sort keys
+// (lk * world + r) -- the same key set k_owned_emit builds from all ranks' raw ids, minus the
+// duplicates; one block per rank r (segment offsets from the world headers)
+__global__ void k_idbox_gather(const char* boxes, size_t stride, int world, int g, uint32_t* __restrict__ sk,
+                               int32_t* __restrict__ sv, int32_t* d_cnt) {
+    const int r = blockIdx.x;
+    int base = 0, total = 0;
+    for (int q = 0; q < world; q++) {
+        const int32_t* h = (const int32_t*)(boxes + (size_t)q * stride);
+        const int len = h[g + 1] - h[g];
+        if (q < r) base += len;
+        total += len;
+    }
+    const int32_t* h = (const int32_t*)(boxes + (size_t)r * stride);
+    const int b = h[g], len = h[g + 1] - h[g];
+    const int32_t* ids = (const int32_t*)(boxes + (size_t)r * stride + 256);
+    for (int i = threadIdx.x; i < len; i += blockDim.x) {
+        const uint32_t k = (uint32_t)ids[b + i];
+        sk[base + i] = (k / (uint32_t)world) * (uint32_t)world + (uint32_t)r;
+        sv[base + i] = r;
+    }
+    if (r == 0 && threadIdx.x == 0) *d_cnt = total;
+}
+
+static void owner_group(frugal_ctx* c, QueueSlot& q, cudaStream_t st) {
+    // this rank's uniq grouped by owner (stable 1-pass partition): gl, goff
+    const int n = c->n;
+    k_owner_keys<<<grid_for(c->M, 256), 256, 0, st>>>(q.uniq, q.n_uniq, n, c->sort.k[0], c->sort.v[0]);
+    int obits = 1;
+    while ((1 << obits) < n) obits++;
+    int r2 = sort_pairs(c->sort, q.n_uniq, obits, st, &c->launches);
+    k_copy_i32<<<grid_for(c->M, 256), 256, 0, st>>>(c->sort.v[r2], q.gl, q.n_uniq);
+    k_goff<<<1, 64, 0, st>>>(c->sort.k[r2], q.n_uniq, n, q.goff);
+    c->launches += 3;
+}
+static void owner_pairs(frugal_ctx* c, QueueSlot& q, cudaStream_t st) {
+    // composite keys (lk, r) in sort.k[0] (count owned_cnt) -> T, Tmask, Tidx
+    const int n = c->n;
+    const int nb = c->scan.nblk;
+    int bits = 1;
+    while ((((int64_t)1) << bits) < ((c->No + 1) * (int64_t)n)) bits++;
+    int r = sort_pairs(c->sort, c->owned_cnt, bits, st, &c->launches);
+    k_pairs_count<<<nb, 256, 0, st>>>(c->sort.k[r], c->owned_cnt, n, c->scan.part, nb);
+    for (int qq = 0; qq <= n; qq++) {
+        k_scan_small<<<1, 1024, 0, st>>>(c->scan.part + (size_t)qq * nb, nb, nullptr);
+        c->launches++;
+    }
+    k_pairs_emit<<<nb, 256, 0, st>>>(c->sort.k[r], c->owned_cnt, n, c->scan.part, nb, (int)c->capT, q.T, q.Tmask,
+                                     q.Tidx, q.nT);
+    c->launches += 2;
+}
+void launch_owner_side_v2(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st) {
+    const int n = c->n;
+    cudaMemsetAsync(q.Tmask, 0, c->capT * sizeof(uint32_t), st);
+    owner_group(c, q, st);
+    char* slot = c->dh_idbox + (size_t)(t % kIdSlots) * n * c->idbox_stride;
+    k_idbox_write<<<grid_for(c->M, 256, 2), 256, 0, st>>>(q.uniq, q.gl, q.goff, q.n_uniq, n,
+                                                          slot + (size_t)c->g * c->idbox_stride);
+    c->launches++;
+    launch_set_flag(c, FLAG_IDS_KIND, (uint32_t)(t + 1), st);
+    launch_wait_flags(c, FLAG_IDS_KIND, (uint32_t)(t + 1), st);  // every rank's ids of step t are out
+    k_idbox_gather<<<n, 256, 0, st>>>(slot, c->idbox_stride, n, c->g, c->sort.k[0], c->sort.v[0], c->owned_cnt);
+    c->launches++;
+    owner_pairs(c, q, st);
+}
+
 void launch_owner_side(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st) {
     (void)t;
     const int n = c->n;
@@ -485,28 +567,9 @@ void launch_owner_side(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st) 
     k_owned_emit<<<nb, 256, 0, st>>>(q.ids, q.counts, n, c->M, c->F, c->g, c->scan.part, nb, c->sort.k[0],
                                      c->sort.v[0], c->owned_cnt);
     c->launches += 3;
-    int bits = 1;
-    while ((((int64_t)1) << bits) < ((c->No + 1) * (int64_t)n)) bits++;
-    int r = sort_pairs(c->sort, c->owned_cnt, bits, st, &c->launches);
-    // (2) unique pairs -> T, masks, per-rank indices
-    k_pairs_count<<<nb, 256, 0, st>>>(c->sort.k[r], c->owned_cnt, n, c->scan.part, nb);
-    for (int qq = 0; qq <= n; qq++) {
-        k_scan_small<<<1, 1024, 0, st>>>(c->scan.part + (size_t)qq * nb, nb, nullptr);
-        c->launches++;
-    }
-    k_pairs_emit<<<nb, 256, 0, st>>>(c->sort.k[r], c->owned_cnt, n, c->scan.part, nb, (int)c->capT, q.T, q.Tmask,
-                                     q.Tidx, q.nT);
-    c->launches += 2;
-    // (3) this rank's uniq grouped by owner (stable 1-pass partition)
-    k_owner_keys<<<grid_for(c->M, 256), 256, 0, st>>>(q.uniq, q.n_uniq, n, c->sort.k[0], c->sort.v[0]);
-    int obits = 1;
-    while ((1 << obits) < n) obits++;
-    int r2 = sort_pairs(c->sort, q.n_uniq, obits, st, &c->launches);
-    k_copy_i32<<<grid_for(c->M, 256), 256, 0, st>>>(c->sort.v[r2], q.gl, q.n_uniq);
-    k_goff<<<1, 64, 0, st>>>(c->sort.k[r2], q.n_uniq, n, q.goff);
-    c->launches += 3;
+    owner_pairs(c, q, st);
+    owner_group(c, q, st);
 }
-
 // ============================================================================ scheduler (P2F)
 // warp-aggregated append of (row, p) to the newly-bucketed list
 __device__ __forceinline__ void nb_append(int32_t* rows, int32_t* ps, int32_t* cnt, bool pred, int32_t lk,

@@ -63,7 +63,7 @@ namespace {
 
 constexpr uint64_t kMagic = 0x46525547414c3235ULL;  // "FRUGAL25"
 constexpr size_t kHdr = 4096;
-constexpr size_t kFlags = 8192;  // 4 kinds x 32 ranks x 64 B
+constexpr size_t kFlags = 16384;  // 8 kinds x 32 ranks x 64 B (FLAG_* below, FLAG_IDS_KIND)
 constexpr size_t kIpc = 32 * 512;  // per rank: IPC handles of cache / pool / last_upd / pool_idx (PEER)
 
 struct IpcRecord {
@@ -462,6 +462,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     if (getenv("FRUGAL_HOST_FLUSH")) c->host_flush = atoi(getenv("FRUGAL_HOST_FLUSH")) != 0;
     if (c->host_flush) c->early = false;  // the early gather synchronises on the GPU drain's events
     c->xhost = c->n > 1 && !c->a2a;
+    c->own_ids = (k.flags & FRUGAL_F_OWN_IDS) != 0 && c->n > 1;
     // side-drain flushes by TMA bulk stores (FRUGAL_FLUSH_TMA=0 none, 1 side, 2 all)
     if (getenv("FRUGAL_FLUSH_TMA")) c->flush_tma = atoi(getenv("FRUGAL_FLUSH_TMA"));
     // world 1: optimizer fused into the segment-reduce (FRUGAL_FUSE_OPT=0: two kernels)
@@ -488,9 +489,12 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     // ---------------------------------------------------------------- host table (shm)
     c->mail_stride = c->n > 1 ? align_up(256 + (size_t)c->M * rowb, 4096) : 0;
     const size_t mail_bytes = c->n > 1 ? 2 * (size_t)c->n * c->mail_stride : 0;
+    c->idbox_stride = c->own_ids ? align_up(256 + (size_t)c->M * 4, 4096) : 0;
+    const size_t idbox_bytes = c->own_ids ? (size_t)kIdSlots * c->n * c->idbox_stride : 0;
     const size_t off_ipc = kHdr + kFlags;
     const size_t off_mail = off_ipc + kIpc;
-    const size_t off_w = align_up(off_mail + mail_bytes, 2 << 20);
+    const size_t off_idbox = off_mail + mail_bytes;
+    const size_t off_w = align_up(off_idbox + idbox_bytes, 2 << 20);
     const size_t tab = (size_t)c->N * rowb;
     const size_t off_G = align_up(off_w + tab, 2 << 20);
     const size_t total = host_G ? off_G + tab : off_w + tab;
@@ -568,6 +572,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->dh_flags = (uint32_t*)(dbase + kHdr);
     c->h_mail = hbase + off_mail;
     c->dh_mail = dbase + off_mail;
+    if (c->own_ids) c->dh_idbox = dbase + off_idbox;
     c->h_w = (float*)(hbase + off_w);
     c->dh_w = (float*)(dbase + off_w);
     if (host_G) {
@@ -843,7 +848,10 @@ static frugal_status ingest(frugal_ctx* c, int64_t t, const int64_t* ids_all, co
     memcpy(pin, counts, (size_t)c->n * 4);
     CK(cudaMemcpyAsync(q.counts, pin, (size_t)c->n * 4, cudaMemcpyHostToDevice, is));
     CK(cudaEventRecord(c->ev_counts[qi], is));
-    CK(cudaMemcpyAsync(c->ids_stage, ids_all, (size_t)c->n * c->M * 8, cudaMemcpyDefault, is));
+    if (c->own_ids)  // this rank's ids only (ingest v2): into its row of the staging array
+        CK(cudaMemcpyAsync(c->ids_stage + (size_t)c->g * c->M, ids_all, (size_t)c->M * 8, cudaMemcpyDefault, is));
+    else
+        CK(cudaMemcpyAsync(c->ids_stage, ids_all, (size_t)c->n * c->M * 8, cudaMemcpyDefault, is));
     CK(cudaEventRecord(c->ev_copied, is));
     if (after) CK(cudaStreamWaitEvent(is, after, 0));
     {
@@ -851,7 +859,8 @@ static frugal_status ingest(frugal_ctx* c, int64_t t, const int64_t* ids_all, co
         launch_convert_ids(c, q, is);
         launch_dedup(c, q, is);
         if (c->n == 1) launch_long_tasks(c, q, is);
-        if (c->n > 1) launch_owner_side(c, q, t, is);
+        if (c->own_ids) launch_owner_side_v2(c, q, t, is);
+        else if (c->n > 1) launch_owner_side(c, q, t, is);
         const int apar = (int)((t - c->L + 1) & 1);  // consumed by frugal_step(t - L + 1)
         CK(cudaMemsetAsync(c->adj_cnt[apar], 0, 4, is));
         launch_ingest_bits(c, q, t, adjust, c->adj_rows[apar], c->adj_p[apar], c->adj_cnt[apar], is);

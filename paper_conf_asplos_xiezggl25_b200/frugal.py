@@ -17,7 +17,7 @@ LIB_PATH = os.path.join(PKG, "libfrugal.so")
 
 SGD, ADAGRAD = 0, 1
 MODE_P2F, MODE_WRITE_THROUGH = 0, 1
-F_RECORD, F_TIMERS, F_NO_HOST_STATE, F_A2A, F_PEER, F_DYNAMIC_CACHE, F_GPU_DRAIN = 1, 2, 4, 8, 16, 32, 64
+F_RECORD, F_TIMERS, F_NO_HOST_STATE, F_A2A, F_PEER, F_DYNAMIC_CACHE, F_GPU_DRAIN, F_OWN_IDS = 1, 2, 4, 8, 16, 32, 64, 128
 FLUSH_ALL = 0
 PHASES = ["ingest", "schedule", "urgent", "gate", "gather", "expand", "model", "segred", "exchange",
           "optimizer", "side", "prefetch"]
@@ -152,6 +152,7 @@ class Frugal:
                  opt="adagrad", lr=0.05, eps=1e-10, init_accum=0.0, init_scale=0.05, init_seed=3, hot_ids=None,
                  shm_name=None, mode=MODE_P2F, flags=0, host_order=None, run_nonce=0):
         self.world, self.rank, self.dim, self.slots, self.batch = world, rank, dim, slots, batch
+        self.flags = flags
         self.lookahead = lookahead
         hot = np.ascontiguousarray(np.zeros(0, np.int64) if hot_ids is None else hot_ids, dtype=np.int64)
         self._hot = hot

@@ -59,7 +59,9 @@ class Trainer:
             fr.prefetch(t, self._ids(t), st.counts[t])
 
     def _ids(self, t):
-        return self.st.ids[t] if self.d_ids is None else self.d_ids[t]
+        ids = self.st.ids[t] if self.d_ids is None else self.d_ids[t]
+        # FRUGAL_F_OWN_IDS (ingest v2): the library gets this rank's ids only
+        return ids[self.rank] if (self.fr.flags & F.F_OWN_IDS) and self.fr.world > 1 else ids
 
     def _set_hot_before_ingest(self, t):
         if t in self._hot:
@@ -129,7 +131,7 @@ class A2ATrainer(Trainer):
         t = s + fr.lookahead
         if t < st.steps:
             self._set_hot_before_ingest(t)
-            fr.step(s, st.ids[t], st.counts[t])
+            fr.step(s, self._ids(t), st.counts[t])
         else:
             fr.step(s)
         if on_schedule:

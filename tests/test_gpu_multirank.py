@@ -22,14 +22,14 @@ def n_gpus():
 
 
 def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False, fused=False, nonce=1, device=0,
-               record=True, backend="gloo", gpu_drain=False):
+               record=True, backend="gloo", gpu_drain=False, own_ids=False):
     try:
         import torch
         from paper_conf_asplos_xiezggl25_b200 import frugal as F
         from paper_conf_asplos_xiezggl25_b200.harness import A2ATrainer, Trainer, make_context
         torch.cuda.set_device(device)
         flags = (F.F_RECORD if record else F.F_TIMERS) | (F.F_A2A if a2a else 0) | (F.F_PEER if peer else 0) \
-            | (F.F_GPU_DRAIN if gpu_drain else 0)
+            | (F.F_GPU_DRAIN if gpu_drain else 0) | (F.F_OWN_IDS if own_ids else 0)
         fr = make_context(st, rank=rank, device=device, shm_name=shm, run_nonce=nonce, flags=flags)
         barrier.wait()
         if a2a:
@@ -68,7 +68,7 @@ def _rank_main(rank, st, shm, barrier, q, a2a=False, port=0, peer=False, fused=F
 
 
 def run_two_ranks(st, timeout=600, a2a=False, peer=False, fused=False, same_device=True, record=True,
-                  backend="gloo", gpu_drain=False):
+                  backend="gloo", gpu_drain=False, own_ids=False):
     import socket
     ctx = mp.get_context("spawn")
     barrier = ctx.Barrier(2)
@@ -82,7 +82,7 @@ def run_two_ranks(st, timeout=600, a2a=False, peer=False, fused=False, same_devi
     if not same_device and n_gpus() < 2:
         pytest.skip("needs 2 GPUs (rank r on device r)")
     ps = [ctx.Process(target=_rank_main, args=(r, st, shm, barrier, q, a2a, port, peer, fused, nonce,
-                                               0 if same_device else r, record, backend, gpu_drain))
+                                               0 if same_device else r, record, backend, gpu_drain, own_ids))
           for r in range(2)]
     for p in ps:
         p.start()
@@ -264,4 +264,36 @@ def test_two_ranks_gpu_drain(record, same_device):
             dfr = sorted(sum((list(zip(out[r]["sched"][s]["deferred"].tolist(),
                                        out[r]["sched"][s]["deferred_p"].tolist())) for r in range(2)), []))
             assert dfr == sorted(zip(ref["deferred"].tolist(), ref["deferred_p"].tolist())), f"deferred differs at {s}"
+    _compare_whole_run(st, out)
+
+
+@pytest.mark.parametrize("variant", ["p2f", "peer", "a2a", "overlapped", "dyn"])
+def test_two_ranks_own_ids(variant):
+    """Ingest v2 (FRUGAL_F_OWN_IDS): every rank gets only its own ids; the ranks exchange their
+    distinct ids, grouped by owner, through the host id mailbox, and each owner merges the ids
+    it owns into its read sets -- every set per step, losses and the whole table as the oracle."""
+    from oracle.oracle import Oracle
+    cfg = W.config("tiny", world=2, batch=96, lookahead=4, age_out=3)
+    rng = np.random.default_rng(21)
+    counts = rng.integers(0, 97, size=(40, 2)).astype(np.int32)
+    counts[7, 0] = 0
+    counts[9] = 0
+    st = W.gen_stream(cfg, 40, counts=counts)
+    if variant == "dyn":
+        st = W.with_dynamic_hot(st, epoch=6)
+    record = variant != "overlapped"
+    out = run_two_ranks(st, a2a=variant == "a2a", peer=variant == "peer", record=record, own_ids=True,
+                        fused=variant == "overlapped")
+    if record:
+        o = Oracle(st)
+        for s in range(st.steps):
+            o.step()
+            ref = o.schedule()
+            urg = sorted(sum((out[r]["sched"][s]["urgent"].tolist() for r in range(2)), []))
+            assert urg == ref["urgent"].tolist(), f"urgent differs at {s}"
+            dfr = sorted(sum((list(zip(out[r]["sched"][s]["deferred"].tolist(),
+                                       out[r]["sched"][s]["deferred_p"].tolist())) for r in range(2)), []))
+            assert dfr == sorted(zip(ref["deferred"].tolist(), ref["deferred_p"].tolist())), f"deferred differs at {s}"
+            age = sorted(sum((out[r]["sched"][s]["ageout"].tolist() for r in range(2)), []))
+            assert age == ref["ageout"].tolist()
     _compare_whole_run(st, out)
