@@ -372,7 +372,7 @@ def main():
 
     def lookup(s):
         if not a2a:
-            fr.lookup(s, emb_arg)
+            fr.lookup(s, emb_arg, stream=stream.cuda_stream)
             return
         sc = fr.a2a_requests(s, ids_send)
         sct = torch.tensor(sc, dtype=torch.int64, device=coll_dev)
@@ -388,53 +388,50 @@ def main():
 
     def backward(s):
         if not a2a:
-            fr.backward_update(s, grad)
+            fr.backward_update(s, grad, stream=stream.cuda_stream)
             return
         sc, rc = lookup.counts
         fr.a2a_pack(s, grad, part_send)
         part_in = a2a_xchg(part_send, sc, rc, d)
         fr.a2a_update(s, part_in, rc)
 
+    # per-step views and counts made once: the step loop is a handful of C-ABI calls
+    ids_v = [ids_d[t] for t in range(SG)]
+    ids_hv = [ids_h[t] for t in range(SG)]
+    x_v = [x_d[t] for t in range(SG)]
+    y_v = [y_d[t] for t in range(SG)]
+    loss_v = [loss[t:t + 1] for t in range(S)]
+    cnt_v = [np.ascontiguousarray(counts[t], dtype=np.int32) for t in range(SG)]
+    sh = stream.cuda_stream
+
     def step_dev(s):
         t = s + L
         set_hot_before_ingest(t)
-        fr.step(s, ids_d[t % SG], counts[t % SG])
+        fr.step(s, ids_v[t % SG], cnt_v[t % SG], stream=sh)
         lookup(s)
         if kg:
-            fr.transe_model(s, emb, cfg.neg_chunk, cfg.gamma, grad, loss[s:s + 1])
+            fr.transe_model(s, emb, cfg.neg_chunk, cfg.gamma, grad, loss_v[s], stream=sh)
         else:
-            fr.dot_model(s, emb_arg, x_d[s % SG], y_d[s % SG], grad, loss[s:s + 1])
+            fr.dot_model(s, emb_arg, x_v[s % SG], y_v[s % SG], grad, loss_v[s], stream=sh)
         backward(s)
 
-    copy_stream = torch.cuda.Stream(dev)
-    x_e = [torch.empty(B, d, device=dev) for _ in range(2)]
-    y_e = [torch.empty(B, device=dev) for _ in range(2)]
-    xy_ready = [torch.cuda.Event() for _ in range(2)]
-    xy_free = [torch.cuda.Event() for _ in range(2)]
-
-    def load_xy(s):  # H2D of step s's dense inputs on a copy stream, double-buffered
-        b = s & 1
-        with torch.cuda.stream(copy_stream):
-            copy_stream.wait_event(xy_free[b])
-            x_e[b].copy_(x_h[s % SG], non_blocking=True)
-            y_e[b].copy_(y_h[s % SG], non_blocking=True)
-            xy_ready[b].record(copy_stream)
+    x_hv = [x_h[t] for t in range(SG)]
+    y_hv = [y_h[t] for t in range(SG)]
+    loss_hv = [loss_h[t:t + 1] for t in range(S)]
 
     def step_e2e(s):
+        # every input from pinned host memory through the C ABI: ids in frugal_step, x and y in
+        # frugal_dot_model (copied by the library); the step's loss read back to the host
         t = s + L
-        b = s & 1
         set_hot_before_ingest(t)
-        fr.step(s, ids_h[t % SG], counts[t % SG])  # ids copied from pinned host inside the call
-        load_xy(s + 1)
+        fr.step(s, ids_hv[t % SG], cnt_v[t % SG], stream=sh)
         lookup(s)
-        stream.wait_event(xy_ready[b])
         if kg:
-            fr.transe_model(s, emb, cfg.neg_chunk, cfg.gamma, grad, loss[s:s + 1])
+            fr.transe_model(s, emb, cfg.neg_chunk, cfg.gamma, grad, loss_v[s], stream=sh)
         else:
-            fr.dot_model(s, emb_arg, x_e[b], y_e[b], grad, loss[s:s + 1])
-        xy_free[b].record(stream)
+            fr.dot_model(s, emb_arg, x_hv[s % SG], y_hv[s % SG], grad, loss_v[s], stream=sh)
         backward(s)
-        loss_h[s:s + 1].copy_(loss[s:s + 1], non_blocking=True)  # the step's result back to the host
+        loss_hv[s].copy_(loss_v[s], non_blocking=True)  # the step's result back to the host
 
     # ---- warm-up
     for s in range(Wm):
@@ -467,7 +464,6 @@ def main():
     t0 = time.perf_counter()
     f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     f0.record(stream)
-    load_xy(Wm + K)
     for s in range(Wm + K, Wm + 2 * K):
         step_e2e(s)
     fr.join(stream)

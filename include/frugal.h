@@ -209,7 +209,10 @@ const char* frugal_last_error(void);
    per sample b: S = sum_f e_f (f ascending, fp32), z = 0.5(|S|^2 - sum_f |e_f|^2)
    + <x_b,S> (fp64), p = sigmoid(z); loss += softplus(z) - y z (fp64, into *d_loss);
    grad_f = c*((S - e_f) + x_b), c = (float)((p - y)/nb), nb = samples of step s over
-   all ranks.  d_emb/d_grad: [count*slots][dim]; x: [count][dim]; y: [count] (device).
+   all ranks.  d_emb/d_grad: [count*slots][dim] (device); x: [count][dim]; y: [count]: both
+   device pointers, or both host pointers (pinned or pageable: the library copies them to its
+   own device staging on a copy stream as soon as the call is made; a host buffer may be
+   reused once `stream` has passed this call).
    d_emb == NULL exactly when lookup(s) ran with d_out == NULL (fused lookup), else
    FRUGAL_EINVAL. */
 frugal_status frugal_dot_model(frugal_ctx* ctx, int64_t s, const float* d_emb, const float* d_x,

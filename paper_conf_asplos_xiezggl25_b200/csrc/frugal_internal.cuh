@@ -90,7 +90,7 @@ struct HostShared;  // shm segment layout (runtime.cu)
 struct Flushers;    // host flushing threads (runtime.cu)
 // control words of the drain staging queue (uint32, host memory): the device writes READY
 // (job seq of each parity buffer) and the part sizes; the flushing threads write APPLIED_*
-enum { CTL_READY = 0, CTL_N1 = 2, CTL_NTOT = 4, CTL_APPLIED_FIRST = 16, CTL_APPLIED_ALL = 32 };
+enum { CTL_READY = 0, CTL_N1 = 2, CTL_NTOT = 4, CTL_READY1 = 8, CTL_APPLIED_FIRST = 16, CTL_APPLIED_ALL = 32 };
 
 // NVLink-native variant (FRUGAL_F_PEER): every rank's HBM cache / pool / metadata, opened
 // through CUDA IPC (device pointers valid in this process)
@@ -114,6 +114,7 @@ struct frugal_ctx {
     int32_t* hs = nullptr;           // [N] host-table slot of every global row (host_order), or null
     std::vector<int32_t> hs_host;    // host copy (frugal_read_host)
     int side_first_blocks = 20;      // grid cap of the drain's deadline-(s+1) part
+    int pack_blocks = 20;            // grid cap of the drain's pack kernel (flushing-thread drain)
     int flush_tma = 0;               // flushes by TMA bulk stores: 0 none, 1 side drain, 2 all (FRUGAL_FLUSH_TMA; measured no gain: profiles/r1_sweep21_flush_tma.txt)
     int glue_cache = -1;         // REC glue keeps a sample's rows in registers (F <= 32): -1 auto, 0 never, 1 always
     bool glue_rg = true;         // REC glue: row-group kernel k_dot_rg (FRUGAL_GLUE_RG=0: the warp-per-sample k_dot_model)
@@ -122,6 +123,7 @@ struct frugal_ctx {
     int gather_blocks = 120;     // grid cap of the zero-copy gathers (120 CTAs: +3% over 74 and 148 in the step, profiles/r1_sweep34_gather_grid.txt)
     bool side_inline = false;    // experiment: drain on the caller stream
     bool drain_after_gather = true;  // side drain after the step's gather (FRUGAL_DRAIN_AT=sched: after the scheduler)
+    bool urgent_side = false;        // world 1: urgent flush on the side stream (reading R7'), see frugal_step
     int64_t capT;                // max owned rows touched per step
     int key_bits, lk_bits;       // bits of global ids / local ids
 
@@ -262,6 +264,20 @@ struct frugal_ctx {
     uint32_t* dfl_ctl = nullptr;                 // device alias
     int64_t drains_issued = 0;                   // drain jobs published so far (job s = drain of step s)
 
+    // ingest as CUDA graphs (one per queue slot; FRUGAL_GRAPHS=0: direct launches)
+    bool use_graphs = true;
+    cudaStream_t gstream = nullptr;              // capture stream
+    std::vector<cudaGraphExec_t> ingest_exec;    // [QN]
+    std::vector<int64_t> ingest_nodes;           // kernels per graph (launch counter)
+    int32_t* d_iprm = nullptr;                   // [QN][IP_N] device
+    int32_t* h_iprm = nullptr;                   // [QN][IP_N] pinned staging
+
+    // host dense inputs of the REC glue (frugal_dot_model with host x / y): staging by step parity
+    cudaStream_t xstream = nullptr;
+    cudaEvent_t ev_xy = nullptr, ev_glue[2] = {nullptr, nullptr};
+    float* x_stage[2] = {nullptr, nullptr};
+    float* y_stage[2] = {nullptr, nullptr};
+
     // instrumentation
     int64_t launches = 0;
     std::vector<frugal::PhaseEv> evs;
@@ -280,14 +296,20 @@ namespace frugal {
 void launch_convert_ids(frugal_ctx* c, QueueSlot& q, cudaStream_t st);
 void launch_dedup(frugal_ctx* c, QueueSlot& q, cudaStream_t st);
 void launch_owner_side(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st);
-void launch_owner_side_v2(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st);
+void launch_owner_side_v2(frugal_ctx* c, QueueSlot& q, const int32_t* prm, cudaStream_t st);
+void launch_set_flag_prm(frugal_ctx* c, int which, const int32_t* prm, cudaStream_t st);
+void launch_wait_flags_prm(frugal_ctx* c, int which, const int32_t* prm, cudaStream_t st);
 constexpr int kIdSlots = 4;  // id-mailbox slots (step t uses slot t % kIdSlots)
 enum { FLAG_IDS_KIND = 4 };  // host flag kind: this rank's distinct ids of step t published (t+1)
 void launch_cache_transition(frugal_ctx* c, int64_t s, int par, cudaStream_t st);
 void launch_hot_map(frugal_ctx* c, int which, const int64_t* ids64, const int32_t* lks, int64_t n, bool list,
                     cudaStream_t st);
-void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, int32_t* adj_rows, int32_t* adj_p,
-                        int32_t* adj_cnt, cudaStream_t st);
+// per-step parameters of the ingest (device words, one block of IP_N per queue slot): the
+// ingest's kernels read them, so its launch sequence is the same every step and is replayed
+// as one CUDA graph per queue slot
+enum { IP_T = 0, IP_APAR = 1, IP_ADJUST = 2, IP_HMAP = 3, IP_IDSLOT = 4, IP_FLAGV = 5, IP_N = 8 };
+void launch_ingest_prologue(frugal_ctx* c, const int32_t* prm, cudaStream_t st);
+void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, const int32_t* prm, cudaStream_t st);
 void launch_schedule(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStream_t st);
 void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begin, const int32_t* d_end,
                        int max_blocks, int counter, cudaStream_t st, bool side = false);
@@ -297,7 +319,7 @@ void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32
                    cudaStream_t st);
 void launch_expand(frugal_ctx* c, QueueSlot& q, const float* rows, float* out, cudaStream_t st);
 void launch_probe_rows(frugal_ctx* c, int64_t n, uint64_t seed, float* out, int64_t out_rows, cudaStream_t st);
-void launch_split_early(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st);
+void launch_split_early(frugal_ctx* c, QueueSlot& q, const int32_t* prm, cudaStream_t st);
 void launch_mail_header(frugal_ctx* c, QueueSlot& q, int par, cudaStream_t st);
 void launch_transe_model(frugal_ctx* c, QueueSlot& q, const float* emb, int C, double gamma, float* grad,
                          double* loss, int64_t nb, double* Wm, double* A, cudaStream_t st);

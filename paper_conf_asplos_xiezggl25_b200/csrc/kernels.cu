@@ -482,7 +482,9 @@ __global__ void k_copy_i32(const int32_t* __restrict__ a, int32_t* __restrict__ 
 // (1) this rank's distinct ids of step t, grouped by owner (gl, goff), to its id-mailbox slot:
 // [goff[0..world]] in a 256-B header, then the ids (coalesced zero-copy stores, sequential)
 __global__ void k_idbox_write(const int32_t* __restrict__ uniq, const int32_t* __restrict__ gl,
-                              const int32_t* __restrict__ goff, const int32_t* d_nu, int world, char* box) {
+                              const int32_t* __restrict__ goff, const int32_t* d_nu, int world, char* boxes,
+                              size_t stride, int g, const int32_t* __restrict__ prm) {
+    char* box = boxes + ((size_t)prm[IP_IDSLOT] * world + g) * stride;
     const int n = *d_nu;
     int32_t* hdr = (int32_t*)box;
     int32_t* ids = (int32_t*)(box + 256);
@@ -493,8 +495,9 @@ __global__ void k_idbox_write(const int32_t* __restrict__ uniq, const int32_t* _
 // (2) every rank r's segment of ids owned by this rank g (ascending), as composite sort keys
 // (lk * world + r) -- the same key set k_owned_emit builds from all ranks' raw ids, minus the
 // duplicates; one block per rank r (segment offsets from the world headers)
-__global__ void k_idbox_gather(const char* boxes, size_t stride, int world, int g, uint32_t* __restrict__ sk,
-                               int32_t* __restrict__ sv, int32_t* d_cnt) {
+__global__ void k_idbox_gather(const char* boxes0, size_t stride, int world, int g, uint32_t* __restrict__ sk,
+                               int32_t* __restrict__ sv, int32_t* d_cnt, const int32_t* __restrict__ prm) {
+    const char* boxes = boxes0 + (size_t)prm[IP_IDSLOT] * world * stride;
     const int r = blockIdx.x;
     int base = 0, total = 0;
     for (int q = 0; q < world; q++) {
@@ -541,17 +544,17 @@ static void owner_pairs(frugal_ctx* c, QueueSlot& q, cudaStream_t st) {
                                      q.Tidx, q.nT);
     c->launches += 2;
 }
-void launch_owner_side_v2(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st) {
+void launch_owner_side_v2(frugal_ctx* c, QueueSlot& q, const int32_t* prm, cudaStream_t st) {
     const int n = c->n;
     cudaMemsetAsync(q.Tmask, 0, c->capT * sizeof(uint32_t), st);
     owner_group(c, q, st);
-    char* slot = c->dh_idbox + (size_t)(t % kIdSlots) * n * c->idbox_stride;
-    k_idbox_write<<<grid_for(c->M, 256, 2), 256, 0, st>>>(q.uniq, q.gl, q.goff, q.n_uniq, n,
-                                                          slot + (size_t)c->g * c->idbox_stride);
+    k_idbox_write<<<grid_for(c->M, 256, 2), 256, 0, st>>>(q.uniq, q.gl, q.goff, q.n_uniq, n, c->dh_idbox,
+                                                          c->idbox_stride, c->g, prm);
     c->launches++;
-    launch_set_flag(c, FLAG_IDS_KIND, (uint32_t)(t + 1), st);
-    launch_wait_flags(c, FLAG_IDS_KIND, (uint32_t)(t + 1), st);  // every rank's ids of step t are out
-    k_idbox_gather<<<n, 256, 0, st>>>(slot, c->idbox_stride, n, c->g, c->sort.k[0], c->sort.v[0], c->owned_cnt);
+    launch_set_flag_prm(c, FLAG_IDS_KIND, prm, st);
+    launch_wait_flags_prm(c, FLAG_IDS_KIND, prm, st);  // every rank's ids of step t are out
+    k_idbox_gather<<<n, 256, 0, st>>>(c->dh_idbox, c->idbox_stride, n, c->g, c->sort.k[0], c->sort.v[0],
+                                      c->owned_cnt, prm);
     c->launches++;
     owner_pairs(c, q, st);
 }
@@ -585,12 +588,29 @@ __device__ __forceinline__ void nb_append(int32_t* rows, int32_t* ps, int32_t* c
     ps[at] = p;
 }
 
-// a1: set read-ring bits of step t for the owned rows read at t; AdjustPriority inf -> t
+// zero the AdjustPriority list count the ingest of this step appends to (by parity, prm)
+__global__ void k_ingest_prologue(const int32_t* __restrict__ prm, int32_t* cnt0, int32_t* cnt1) {
+    *(prm[IP_APAR] ? cnt1 : cnt0) = 0;
+}
+void launch_ingest_prologue(frugal_ctx* c, const int32_t* prm, cudaStream_t st) {
+    k_ingest_prologue<<<1, 1, 0, st>>>(prm, c->adj_cnt[0], c->adj_cnt[1]);
+    c->launches++;
+}
+
+// a1: set read-ring bits of step t for the owned rows read at t; AdjustPriority inf -> t.
+// t, the adjust switch, the list parity and the hot map of t's epoch come from prm
 __global__ void k_ingest_bits(const int32_t* __restrict__ T, const uint32_t* __restrict__ Tmask,
-                              const int32_t* d_nT, int world, int g, int bit, int32_t t, int adjust,
-                              const int32_t* __restrict__ slot, const uint32_t* __restrict__ hmap,
-                              uint64_t* __restrict__ rbits,
-                              int32_t* __restrict__ state, int32_t* nb_rows, int32_t* nb_p, int32_t* nb_cnt) {
+                              const int32_t* d_nT, int world, int g, const int32_t* __restrict__ prm,
+                              const int32_t* __restrict__ slot, const uint32_t* __restrict__ hmap0,
+                              const uint32_t* __restrict__ hmap1, uint64_t* __restrict__ rbits,
+                              int32_t* __restrict__ state, int32_t* rows0, int32_t* p0, int32_t* cnt0,
+                              int32_t* rows1, int32_t* p1, int32_t* cnt1) {
+    const int32_t t = prm[IP_T];
+    const int bit = t & 31, adjust = prm[IP_ADJUST], par = prm[IP_APAR], hm = prm[IP_HMAP];
+    const uint32_t* hmap = hm < 0 ? nullptr : (hm ? hmap1 : hmap0);
+    int32_t* nb_rows = par ? rows1 : rows0;
+    int32_t* nb_p = par ? p1 : p0;
+    int32_t* nb_cnt = par ? cnt1 : cnt0;
     int n = *d_nT;
     int nloop = (n + blockDim.x * gridDim.x - 1) / (blockDim.x * gridDim.x) * (blockDim.x * gridDim.x);
     for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < nloop; j += gridDim.x * blockDim.x) {
@@ -691,13 +711,11 @@ __global__ void k_schedule(const int32_t* __restrict__ T, const int32_t* d_nT, c
     }
 }
 
-void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, int64_t t, int adjust, int32_t* adj_rows, int32_t* adj_p,
-                        int32_t* adj_cnt, cudaStream_t st) {
-    const uint32_t* hmap = nullptr;
-    if (c->dyn) hmap = c->hot_map[(c->hot_pending && t >= c->hot_t0) ? (c->hot_cur ^ 1) : c->hot_cur];
-    k_ingest_bits<<<grid_for(c->capT, 256), 256, 0, st>>>(q.T, q.Tmask, q.nT, c->n, c->g, (int)(t & 31), (int32_t)t,
-                                                           adjust, c->slot, hmap, c->rbits, c->state, adj_rows, adj_p,
-                                                           adj_cnt);
+void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, const int32_t* prm, cudaStream_t st) {
+    k_ingest_bits<<<grid_for(c->capT, 256), 256, 0, st>>>(q.T, q.Tmask, q.nT, c->n, c->g, prm, c->slot, c->hot_map[0],
+                                                           c->hot_map[1], c->rbits, c->state, c->adj_rows[0],
+                                                           c->adj_p[0], c->adj_cnt[0], c->adj_rows[1], c->adj_p[1],
+                                                           c->adj_cnt[1]);
     c->launches++;
 }
 
@@ -965,14 +983,15 @@ __global__ void k_pack_drain(const int32_t* __restrict__ lists, const int32_t* _
                              int g, int d4, const int32_t* __restrict__ slot, const int32_t* __restrict__ last_upd,
                              const int32_t* __restrict__ pool_idx, int P, int64_t capT, const float4* __restrict__ cw,
                              const float4* __restrict__ pw, const int32_t* __restrict__ hs, float4* hrows,
-                             int64_t* hkeys, unsigned long long* stats) {
+                             int64_t* hkeys, unsigned long long* stats, int part) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
     const int n1 = cnt[1], n2 = cnt[2], n3 = cnt[3];
-    const int n = n1 + n2 + n3;
+    // part 0: list 1 (deadline s+1) -> staging [0, n1); part 1: lists 2, 3 -> [n1, n1+n2+n3)
+    const int lo = part == 0 ? 0 : n1, n = part == 0 ? n1 : n1 + n2 + n3;
     unsigned nh = 0, nc = 0;
-    for (int64_t a = gid; a < n; a += gs) {
+    for (int64_t a = lo + gid; a < n; a += gs) {
         const int64_t at = a < n1 ? cap + a : a < n1 + n2 ? 2 * cap + (a - n1) : 3 * cap + (a - n1 - n2);
         const int32_t lk = lists[at];
         const int sl = slot[lk];
@@ -991,23 +1010,27 @@ __global__ void k_pack_drain(const int32_t* __restrict__ lists, const int32_t* _
     block_count(stats, nh);
     block_count(stats + 1, nc);
 }
-// publish job `seq` (= s+1) of staging buffer `par`: part sizes, then the flag (release)
-__global__ void k_publish_drain(const int32_t* __restrict__ cnt, uint32_t* ctl, int par, uint32_t seq) {
-    // ctl layout (uint32 words): [0..1] ready[par], [2..3] n1[par], [4..5] ntot[par]
-    ctl[2 + par] = (uint32_t)cnt[1];
-    ctl[4 + par] = (uint32_t)(cnt[1] + cnt[2] + cnt[3]);
+// publish part `part` of job `seq` (= s+1) of staging buffer `par`: part sizes, then the part's
+// ready word (release) -- the threads start on part 0 (deadline s+1, the next gate waits for
+// it) while the kernel packs part 1
+__global__ void k_publish_drain(const int32_t* __restrict__ cnt, uint32_t* ctl, int par, uint32_t seq, int part) {
+    ctl[CTL_N1 + par] = (uint32_t)cnt[1];
+    ctl[CTL_NTOT + par] = (uint32_t)(cnt[1] + cnt[2] + cnt[3]);
     __threadfence_system();
-    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(ctl + par), "r"(seq) : "memory");
+    uint32_t* w = ctl + (part == 0 ? CTL_READY1 : CTL_READY) + par;
+    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(w), "r"(seq) : "memory");
 }
 void launch_pack_drain(frugal_ctx* c, int par, uint32_t seq, int max_blocks, cudaStream_t st) {
     const int d4 = c->d / 4, gs = group_size(d4);
     int grid = std::min(grid_for(3 * c->sl_cap * (int64_t)gs, 256, 4), max_blocks);
-    DISPATCH_GS(gs, (k_pack_drain<GS><<<grid, 256, 0, st>>>(
-                        c->sl_rows[par], c->sl_cnt[par], c->sl_cap, c->n, c->g, d4, c->slot, c->last_upd, c->pool_idx,
-                        c->P, c->capT, (const float4*)c->cw, (const float4*)c->pw, c->hs,
-                        (float4*)c->dfl_rows[par], c->dfl_keys[par], c->dstats + FRUGAL_C_SIDE_HOT)));
-    k_publish_drain<<<1, 1, 0, st>>>(c->sl_cnt[par], c->dfl_ctl, par, seq);
-    c->launches += 2;
+    for (int part = 0; part < 2; part++) {
+        DISPATCH_GS(gs, (k_pack_drain<GS><<<grid, 256, 0, st>>>(
+                            c->sl_rows[par], c->sl_cnt[par], c->sl_cap, c->n, c->g, d4, c->slot, c->last_upd,
+                            c->pool_idx, c->P, c->capT, (const float4*)c->cw, (const float4*)c->pw, c->hs,
+                            (float4*)c->dfl_rows[par], c->dfl_keys[par], c->dstats + FRUGAL_C_SIDE_HOT, part)));
+        k_publish_drain<<<1, 1, 0, st>>>(c->sl_cnt[par], c->dfl_ctl, par, seq, part);
+    }
+    c->launches += 4;
 }
 
 // a4 gather: unique rows -> staging (owned hot: HBM cache; else host, zero-copy).
@@ -1161,8 +1184,9 @@ void launch_expand(frugal_ctx* c, QueueSlot& q, const float* rows, float* out, c
 // world 1: split uniq(t) into rows not read at t-1 (early) and rows read at t-1 (late;
 // they are updated at t-1 and may be urgent at t).  Read-ring bit t-1 is still set: it is
 // cleared by the optimizer of step t-1, which runs after this ingest (one step ahead).
-__global__ void k_split_early(const int32_t* __restrict__ uniq, const int32_t* d_nu, int64_t t,
+__global__ void k_split_early(const int32_t* __restrict__ uniq, const int32_t* d_nu, const int32_t* __restrict__ prm,
                               const uint64_t* __restrict__ rbits, int32_t* eidx, int32_t* lidx, int32_t* elcnt) {
+    const int64_t t = prm[IP_T];
     const int n = *d_nu;
     const int nloop = (n + blockDim.x * gridDim.x - 1) / (blockDim.x * gridDim.x) * (blockDim.x * gridDim.x);
     const uint64_t bit = t > 0 ? (1ull << ((t - 1) & 31)) : 0ull;
@@ -1183,9 +1207,9 @@ __global__ void k_split_early(const int32_t* __restrict__ uniq, const int32_t* d
         if (late) lidx[bl + __popc(ml & lanemask_lt())] = u;
     }
 }
-void launch_split_early(frugal_ctx* c, QueueSlot& q, int64_t t, cudaStream_t st) {
+void launch_split_early(frugal_ctx* c, QueueSlot& q, const int32_t* prm, cudaStream_t st) {
     cudaMemsetAsync(q.elcnt, 0, 8, st);
-    k_split_early<<<grid_for(c->M, 256, 4), 256, 0, st>>>(q.uniq, q.n_uniq, t, c->rbits, q.eidx, q.lidx, q.elcnt);
+    k_split_early<<<grid_for(c->M, 256, 4), 256, 0, st>>>(q.uniq, q.n_uniq, prm, c->rbits, q.eidx, q.lidx, q.elcnt);
     c->launches++;
 }
 

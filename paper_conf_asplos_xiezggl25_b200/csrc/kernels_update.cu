@@ -776,6 +776,44 @@ __global__ void k_wait_flags(const uint32_t* f, int world, uint32_t v, int32_t* 
     __syncwarp();
     __threadfence_system();
 }
+// flag value from the ingest's parameter block (graph-replayed launches)
+__global__ void k_set_flag_prm(uint32_t* f, const int32_t* __restrict__ prm) {
+    __threadfence_system();
+    const uint32_t v = (uint32_t)prm[IP_FLAGV];
+    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(f), "r"(v) : "memory");
+}
+__global__ void k_wait_flags_prm(const uint32_t* f, int world, const int32_t* __restrict__ prm, int32_t* err) {
+    const uint32_t v = (uint32_t)prm[IP_FLAGV];
+    int r = threadIdx.x;
+    if (r < world) {
+        const uint32_t* p = f + r * 16;
+        uint64_t t0;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+        while (true) {
+            uint32_t x;
+            asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(x) : "l"(p) : "memory");
+            if ((int32_t)(x - v) >= 0) break;
+            uint64_t t1;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
+            if (t1 - t0 > 120ull * 1000000000ull) {
+                atomicExch(err, 2);
+                break;
+            }
+            __nanosleep(256);
+        }
+    }
+    __syncwarp();
+    __threadfence_system();
+}
+void launch_set_flag_prm(frugal_ctx* c, int which, const int32_t* prm, cudaStream_t st) {
+    k_set_flag_prm<<<1, 1, 0, st>>>(c->dh_flags + (which * 32 + c->g) * 16, prm);
+    c->launches++;
+}
+void launch_wait_flags_prm(frugal_ctx* c, int which, const int32_t* prm, cudaStream_t st) {
+    k_wait_flags_prm<<<1, 32, 0, st>>>(c->dh_flags + which * 32 * 16, c->n, prm, c->err);
+    c->launches++;
+}
+
 // wait (device side) until one host word reaches `value` (wrap-around compare)
 void launch_wait_word(frugal_ctx* c, const uint32_t* dflag, uint32_t value, cudaStream_t st) {
     k_wait_flags<<<1, 32, 0, st>>>(dflag, 1, value, c->err);

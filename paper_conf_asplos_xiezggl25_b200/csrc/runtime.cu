@@ -163,24 +163,25 @@ static void flusher_main(frugal_ctx* c, int t) {
     for (int64_t job = 0;; job++) {
         const int par = (int)(job & 1);
         const uint32_t seq = (uint32_t)(job + 1);
-        // wait for the device to publish the job: spin while jobs keep coming, then poll gently
-        while (!seq_reached(ctl_load(ctl + CTL_READY + par), seq)) {
-            if (F->stop.load(std::memory_order_relaxed)) return;
-            timespec ts;
-            clock_gettime(CLOCK_MONOTONIC, &ts);
-            const double now = ts.tv_sec + 1e-9 * ts.tv_nsec;
-            if (idle_since == 0.0) idle_since = now;
-            if (now - idle_since < 2e-3) {
-                for (int k = 0; k < 64; k++) _mm_pause();
-            } else {
-                usleep(20);
-            }
-        }
-        idle_since = 0.0;
-        const int64_t n1 = ctl_load(ctl + CTL_N1 + par), nt = ctl_load(ctl + CTL_NTOT + par);
         const float* rows = c->hfl_rows[par];
         const int64_t* keys = c->hfl_keys[par];
         for (int part = 0; part < 2; part++) {
+            // wait for the device to publish the part: spin while jobs keep coming, then poll gently
+            const uint32_t* ready = ctl + (part == 0 ? CTL_READY1 : CTL_READY) + par;
+            while (!seq_reached(ctl_load(ready), seq)) {
+                if (F->stop.load(std::memory_order_relaxed)) return;
+                timespec ts;
+                clock_gettime(CLOCK_MONOTONIC, &ts);
+                const double now = ts.tv_sec + 1e-9 * ts.tv_nsec;
+                if (idle_since == 0.0) idle_since = now;
+                if (now - idle_since < 2e-3) {
+                    for (int k = 0; k < 64; k++) _mm_pause();
+                } else {
+                    usleep(20);
+                }
+            }
+            idle_since = 0.0;
+            const int64_t n1 = ctl_load(ctl + CTL_N1 + par), nt = ctl_load(ctl + CTL_NTOT + par);
             const int64_t b = part == 0 ? 0 : n1, e = part == 0 ? n1 : nt;
             copy_rows_nt(c->h_w, rows, keys, b + (e - b) * t / T, b + (e - b) * (t + 1) / T, c->d);
             if (F->done[par][part].fetch_add(1, std::memory_order_acq_rel) + 1 == T) {
@@ -259,6 +260,18 @@ static void free_ctx(frugal_ctx* c) {
         if (c->hfl_keys[i]) cudaFreeHost(c->hfl_keys[i]);
     }
     if (c->hfl_ctl) cudaFreeHost(c->hfl_ctl);
+    for (auto e : c->ingest_exec)
+        if (e) cudaGraphExecDestroy(e);
+    if (c->gstream) cudaStreamDestroy(c->gstream);
+    if (c->xstream) cudaStreamDestroy(c->xstream);
+    if (c->ev_xy) cudaEventDestroy(c->ev_xy);
+    for (int i = 0; i < 2; i++) {
+        if (c->ev_glue[i]) cudaEventDestroy(c->ev_glue[i]);
+        if (c->x_stage[i]) cudaFree(c->x_stage[i]);
+        if (c->y_stage[i]) cudaFree(c->y_stage[i]);
+    }
+    if (c->d_iprm) cudaFree(c->d_iprm);
+    if (c->h_iprm) cudaFreeHost(c->h_iprm);
     auto F = [](void* p) {
         if (p) cudaFree(p);
     };
@@ -472,12 +485,17 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->fuse_opt = !(getenv("FRUGAL_FUSE_OPT") && !atoi(getenv("FRUGAL_FUSE_OPT")));
     c->update1 = !(getenv("FRUGAL_UPDATE1") && !atoi(getenv("FRUGAL_UPDATE1")));
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 20;
+    c->pack_blocks = getenv("FRUGAL_PACK_BLOCKS") ? atoi(getenv("FRUGAL_PACK_BLOCKS")) : c->side_blocks;
     // the deadline-(s+1) part of the drain (the next gate waits for it) may run wider
     c->side_first_blocks = getenv("FRUGAL_SIDE_FIRST_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_FIRST_BLOCKS"))
                                                                : c->side_blocks;
     c->gather_blocks = getenv("FRUGAL_GATHER_BLOCKS") ? atoi(getenv("FRUGAL_GATHER_BLOCKS")) : 120;
     c->side_inline = getenv("FRUGAL_SIDE_INLINE") && atoi(getenv("FRUGAL_SIDE_INLINE"));
     c->drain_after_gather = !(getenv("FRUGAL_DRAIN_AT") && !strcmp(getenv("FRUGAL_DRAIN_AT"), "sched"));
+    // world 1 with pool reads (R7'): the urgent bucket is not read from the host at its step
+    // (FRUGAL_URGENT_SIDE=0: keep it on the critical path)
+    c->urgent_side = c->n == 1 && c->pool_hits && !c->side_inline && !c->early &&
+                     !(getenv("FRUGAL_URGENT_SIDE") && !atoi(getenv("FRUGAL_URGENT_SIDE")));
     c->capT = std::max<int64_t>(1, std::min<int64_t>((int64_t)c->n * c->M, c->No));
     c->sl_cap = 2 * c->capT;
     c->key_bits = bits_for(c->N - 1);
@@ -726,6 +744,19 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     for (auto& e : c->ev_counts) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     c->ev_ingest.resize(c->QN);
     for (auto& e : c->ev_ingest) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    CK(cudaStreamCreateWithFlags(&c->xstream, cudaStreamNonBlocking));
+    CK(cudaEventCreateWithFlags(&c->ev_xy, cudaEventDisableTiming));
+    for (int i = 0; i < 2; i++) CK(cudaEventCreateWithFlags(&c->ev_glue[i], cudaEventDisableTiming));
+    c->use_graphs = !(getenv("FRUGAL_GRAPHS") && !atoi(getenv("FRUGAL_GRAPHS")));
+    c->ingest_exec.assign(c->QN, nullptr);
+    c->ingest_nodes.assign(c->QN, 0);
+    CK(cudaStreamCreateWithFlags(&c->gstream, cudaStreamNonBlocking));
+    DMALLOC(c->d_iprm, (size_t)c->QN * IP_N * 4);
+    if (cudaHostAlloc((void**)&c->h_iprm, (size_t)c->QN * IP_N * 4, cudaHostAllocPortable) != cudaSuccess) {
+        set_err("cudaHostAlloc(ingest parameters) failed");
+        free_ctx(c);
+        return FRUGAL_ENOMEM;
+    }
 
     cudaStream_t st = 0;
     cudaMemset(c->hot_lk, 0xff, c->cap_slots * 4);  // spare slots (N3) are free
@@ -823,6 +854,25 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
 // AdjustPriority inf -> t (into the adjust list consumed by frugal_step(t-L+1)).  The
 // ingest of step s+L runs one step ahead, overlapping step s's gather.
 // `after`: an event the ingest must follow (the scheduler of the current step).
+// The ingest of step t in two parts.  Part A (id conversion, dedup, long-segment tasks,
+// owner side) only needs the ids: it starts as soon as they are copied.  Part B (read-ring
+// bits of t, AdjustPriority inf -> t) must follow the scheduler of t-L (which buckets the rows
+// updated at t-L-1 over the window [t-L, t-1] and marks the inf ones) -- only this small part
+// sits between two schedulers.  Every per-step value is read from the device parameter block
+// prm, so part A's launch sequence is identical every step (graph-captured once per slot).
+static void enqueue_ingest_a(frugal_ctx* c, QueueSlot& q, const int32_t* prm, cudaStream_t is) {
+    launch_convert_ids(c, q, is);
+    launch_dedup(c, q, is);
+    if (c->n == 1) launch_long_tasks(c, q, is);
+    if (c->own_ids) launch_owner_side_v2(c, q, prm, is);
+    else if (c->n > 1) launch_owner_side(c, q, 0, is);
+}
+static void enqueue_ingest_b(frugal_ctx* c, QueueSlot& q, const int32_t* prm, cudaStream_t is) {
+    launch_ingest_prologue(c, prm, is);
+    launch_ingest_bits(c, q, prm, is);
+    if (c->early) launch_split_early(c, q, prm, is);
+}
+
 static frugal_status ingest(frugal_ctx* c, int64_t t, const int64_t* ids_all, const int32_t* counts, int adjust,
                             cudaStream_t caller, cudaEvent_t after) {
     for (int r = 0; r < c->n; r++)
@@ -840,31 +890,54 @@ static frugal_status ingest(frugal_ctx* c, int64_t t, const int64_t* ids_all, co
     // the caller's buffer is read after the caller's prior work on `caller`; the copy of the
     // previous call has finished once this call returns (host wait, normally long done), so
     // the caller may reuse a buffer after the next frugal_step/frugal_prefetch returns
-    CK(cudaEventSynchronize(c->ev_copied));
+    static const bool no_copy_wait = getenv("FRUGAL_NO_COPY_WAIT") && atoi(getenv("FRUGAL_NO_COPY_WAIT"));  // diagnostic
+    if (!no_copy_wait) CK(cudaEventSynchronize(c->ev_copied));
     CK(cudaEventRecord(c->ev_call, caller));
     CK(cudaStreamWaitEvent(is, c->ev_call, 0));
-    CK(cudaEventSynchronize(c->ev_counts[qi]));  // pinned counts staging of this slot is free
+    CK(cudaEventSynchronize(c->ev_counts[qi]));  // pinned counts / parameter staging of this slot is free
     int32_t* pin = c->counts_pin + (size_t)qi * c->n;
     memcpy(pin, counts, (size_t)c->n * 4);
     CK(cudaMemcpyAsync(q.counts, pin, (size_t)c->n * 4, cudaMemcpyHostToDevice, is));
+    // the ingest's per-step parameters (its kernels read them: one graph per slot)
+    int32_t* hp = c->h_iprm + (size_t)qi * IP_N;
+    int32_t* dp = c->d_iprm + (size_t)qi * IP_N;
+    hp[IP_T] = (int32_t)t;
+    hp[IP_APAR] = (int)((t - c->L + 1) & 1);  // adjust list consumed by frugal_step(t - L + 1)
+    hp[IP_ADJUST] = adjust;
+    hp[IP_HMAP] = c->dyn ? ((c->hot_pending && t >= c->hot_t0) ? (c->hot_cur ^ 1) : c->hot_cur) : -1;
+    hp[IP_IDSLOT] = (int)(t % kIdSlots);
+    hp[IP_FLAGV] = (int32_t)(uint32_t)(t + 1);
+    CK(cudaMemcpyAsync(dp, hp, IP_N * 4, cudaMemcpyHostToDevice, is));
     CK(cudaEventRecord(c->ev_counts[qi], is));
     if (c->own_ids)  // this rank's ids only (ingest v2): into its row of the staging array
         CK(cudaMemcpyAsync(c->ids_stage + (size_t)c->g * c->M, ids_all, (size_t)c->M * 8, cudaMemcpyDefault, is));
     else
         CK(cudaMemcpyAsync(c->ids_stage, ids_all, (size_t)c->n * c->M * 8, cudaMemcpyDefault, is));
     CK(cudaEventRecord(c->ev_copied, is));
-    if (after) CK(cudaStreamWaitEvent(is, after, 0));
     {
         Timer tm(c, PH_INGEST, is);
-        launch_convert_ids(c, q, is);
-        launch_dedup(c, q, is);
-        if (c->n == 1) launch_long_tasks(c, q, is);
-        if (c->own_ids) launch_owner_side_v2(c, q, t, is);
-        else if (c->n > 1) launch_owner_side(c, q, t, is);
-        const int apar = (int)((t - c->L + 1) & 1);  // consumed by frugal_step(t - L + 1)
-        CK(cudaMemsetAsync(c->adj_cnt[apar], 0, 4, is));
-        launch_ingest_bits(c, q, t, adjust, c->adj_rows[apar], c->adj_p[apar], c->adj_cnt[apar], is);
-        if (c->early) launch_split_early(c, q, t, is);
+        if (c->use_graphs && !serial) {
+            if (!c->ingest_exec[qi]) {  // first use of this slot: capture its launch sequence once
+                cudaGraph_t g = nullptr;
+                const int64_t l0 = c->launches;
+                CK(cudaStreamBeginCapture(c->gstream, cudaStreamCaptureModeThreadLocal));
+                enqueue_ingest_a(c, q, dp, c->gstream);
+                CK(cudaStreamEndCapture(c->gstream, &g));
+                CK(cudaGraphInstantiate(&c->ingest_exec[qi], g, 0));
+                cudaGraphDestroy(g);
+                c->ingest_nodes[qi] = c->launches - l0;
+                c->launches = l0;
+            }
+            CK(cudaGraphLaunch(c->ingest_exec[qi], is));
+            c->launches += c->ingest_nodes[qi];
+        } else {
+            enqueue_ingest_a(c, q, dp, is);
+        }
+    }
+    if (after) CK(cudaStreamWaitEvent(is, after, 0));  // part B follows the current step's scheduler
+    {
+        Timer tm(c, PH_INGEST, is);
+        enqueue_ingest_b(c, q, dp, is);
     }
     CK(cudaEventRecord(c->ev_ingest[qi], is));
     CKL();
@@ -954,7 +1027,7 @@ static frugal_status launch_drain(frugal_ctx* c, int64_t s, cudaStream_t st, cud
         // host flushing threads: staging buffer `par` was last used by job s-2
         Timer tm(c, PH_SIDE, sd);
         if (s >= 2) launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_ALL, (uint32_t)(s - 1), sd);
-        launch_pack_drain(c, par, (uint32_t)(s + 1), c->side_blocks, sd);
+        launch_pack_drain(c, par, (uint32_t)(s + 1), c->pack_blocks, sd);
         CK(cudaEventRecord(c->ev_side_first[par], sd));  // the lists of this parity were read
         CKL();
     } else {
@@ -1037,7 +1110,18 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
         CKL();
     }
     if (c->cfg.flags & FRUGAL_F_RECORD) record_schedule(c, par, st);
-    {
+    if (c->urgent_side) {
+        // a10 at world 1 (reading R7'): the only reader of step s is this owner, and it reads
+        // every row updated within the pool window -- the whole urgent bucket (updated at s-1)
+        // -- from its dirty pool in HBM, so no read of step s needs the bucket's host copies;
+        // they are written on the side stream ahead of the drain, long before any host read of
+        // those rows (after the pool window, P = D+3 >= 4 steps).  Same set, same bytes.
+        CK(cudaEventRecord(c->ev_sched, st));
+        CK(cudaStreamWaitEvent(c->side, c->ev_sched, 0));
+        Timer tm(c, PH_URGENT, c->side);
+        launch_flush_rows(c, c->sl_rows[par], nullptr, c->sl_cnt[par], 1 << 30, FRUGAL_C_URGENT_HOT, c->side);
+        CKL();
+    } else {
         // a10: urgent bucket (priority == s) to the host table on the critical path
         Timer tm(c, PH_URGENT, st);
         launch_flush_rows(c, c->sl_rows[par], nullptr, c->sl_cnt[par], 1 << 30, FRUGAL_C_URGENT_HOT, st);
@@ -1141,9 +1225,34 @@ extern "C" frugal_status frugal_dot_model(frugal_ctx* c, int64_t s, const float*
     QueueSlot& q = c->q[s % c->QN];
     int64_t nb = 0;
     for (int r = 0; r < c->n; r++) nb += q.h_counts[r];
+    // host x / y (pinned or pageable): copied into a library staging pair (by step parity) on
+    // the copy stream as soon as this call is made -- the host usually runs ahead of the GPU,
+    // so the copy overlaps the step's gather
+    cudaPointerAttributes ax{}, ay{};
+    if (cudaPointerGetAttributes(&ax, d_x) != cudaSuccess) { cudaGetLastError(); ax.type = cudaMemoryTypeUnregistered; }
+    if (cudaPointerGetAttributes(&ay, d_y) != cudaSuccess) { cudaGetLastError(); ay.type = cudaMemoryTypeUnregistered; }
+    if (ax.type != cudaMemoryTypeDevice && ax.type != cudaMemoryTypeManaged) {
+        const int par = (int)(s & 1);
+        if (!c->x_stage[par]) {
+            CK(cudaMalloc(&c->x_stage[par], (size_t)c->B * c->d * 4));
+            CK(cudaMalloc(&c->y_stage[par], (size_t)c->B * 4));
+        }
+        const int cnt = q.h_counts[c->g];
+        CK(cudaStreamWaitEvent(c->xstream, c->ev_glue[par], 0));  // the glue of s-2 read this pair
+        CK(cudaMemcpyAsync(c->x_stage[par], d_x, (size_t)cnt * c->d * 4, cudaMemcpyDefault, c->xstream));
+        CK(cudaMemcpyAsync(c->y_stage[par], d_y, (size_t)cnt * 4, cudaMemcpyDefault, c->xstream));
+        CK(cudaEventRecord(c->ev_xy, c->xstream));
+        CK(cudaStreamWaitEvent(st, c->ev_xy, 0));
+        d_x = c->x_stage[par];
+        d_y = c->y_stage[par];
+    } else if (ay.type != cudaMemoryTypeDevice && ay.type != cudaMemoryTypeManaged) {
+        set_err("dot_model: x and y must both be device or both host pointers");
+        return FRUGAL_EINVAL;
+    }
     Timer tm(c, PH_MODEL, st);
     if (d_emb) launch_dot_model(c, q, d_emb, nullptr, d_x, d_y, d_grad, d_loss, nb, st);
     else launch_dot_model(c, q, c->rows_buf[s & 1], q.inv, d_x, d_y, d_grad, d_loss, nb, st);
+    CK(cudaEventRecord(c->ev_glue[s & 1], st));
     CKL();
     return FRUGAL_OK;
 }

@@ -136,10 +136,23 @@ def _ptr(x):
     return x.ctypes.data
 
 
+_raw_stream = None
+
+
 def _stream(stream):
+    """cudaStream_t of `stream`; None = torch's current stream of the current device (read
+    through torch's raw-stream accessor: no Python Stream object per call)."""
+    global _raw_stream
     if stream is None:
-        import torch
-        return torch.cuda.current_stream().cuda_stream
+        if _raw_stream is None:
+            import torch
+            try:
+                get, dev = torch._C._cuda_getCurrentRawStream, torch._C._cuda_getDevice
+                get(dev())
+                _raw_stream = lambda: get(dev())
+            except Exception:  # older torch: the public (slower) path
+                _raw_stream = lambda: torch.cuda.current_stream().cuda_stream
+        return _raw_stream()
     if isinstance(stream, int):
         return stream
     return stream.cuda_stream

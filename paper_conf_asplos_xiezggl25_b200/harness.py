@@ -32,7 +32,8 @@ def make_context(st, rank=0, device=0, shm_name=None, flags=0, hot=None, mode=F.
 class Trainer:
     """Runs the stream on one rank.  Inputs are uploaded per step from host arrays."""
 
-    def __init__(self, fr: F.Frugal, st, rank=0, device=0, fused_lookup=False, device_inputs=False):
+    def __init__(self, fr: F.Frugal, st, rank=0, device=0, fused_lookup=False, device_inputs=False,
+                 host_inputs=False):
         self.fr, self.st, self.rank = fr, st, rank
         # fused lookup (REC glue only): lookup(s, None) + dot_model(s, None, ...) -- the
         # glue reads the gathered distinct rows through the inverse index, no expand
@@ -42,6 +43,11 @@ class Trainer:
         # and passed as device pointers -- the bench's value leg; no host copy or host wait
         # inside the step loop, so the library's streams overlap exactly as in bench.py
         self.d_ids = self.d_x = self.d_y = None
+        self.h_x = self.h_y = None
+        if host_inputs:  # pinned host ids, x, y handed to the C ABI as host pointers (the e2e path)
+            self.d_ids = torch.from_numpy(np.ascontiguousarray(st.ids)).pin_memory()
+            self.h_x = torch.from_numpy(np.ascontiguousarray(st.x[:, rank])).pin_memory()
+            self.h_y = torch.from_numpy(np.ascontiguousarray(st.y[:, rank])).pin_memory()
         if device_inputs:
             self.d_ids = torch.from_numpy(np.ascontiguousarray(st.ids)).to(self.dev)
             self.d_x = torch.from_numpy(np.ascontiguousarray(st.x[:, rank])).to(self.dev)
@@ -82,6 +88,9 @@ class Trainer:
             fr.transe_model(s, self.emb, st.cfg.neg_chunk, st.cfg.gamma, self.grad, self.loss[s:s + 1])
         elif self.d_x is not None:
             fr.dot_model(s, None if self.fused else self.emb, self.d_x[s], self.d_y[s], self.grad,
+                         self.loss[s:s + 1])
+        elif self.h_x is not None:
+            fr.dot_model(s, None if self.fused else self.emb, self.h_x[s], self.h_y[s], self.grad,
                          self.loss[s:s + 1])
         else:
             x = torch.from_numpy(st.x[s, self.rank]).to(self.dev, non_blocking=False)

@@ -92,7 +92,7 @@ def run_parity(st, *, flags=None, mode=None, hot=None, check_dedup=True, check_s
     return out
 
 
-def run_overlapped(st, *, fused=True, flags=None, sample_rows=None, hot=None, exact=None):
+def run_overlapped(st, *, fused=True, flags=None, sample_rows=None, hot=None, exact=None, host_inputs=False):
     """The bench's launch configuration: FRUGAL_F_TIMERS only (no F_RECORD, so no
     per-step synchronisation), no per-step callbacks, ids / x / y resident in HBM and passed
     as device pointers -- the ingest of s+L, the side drain and the main stream overlap as in
@@ -103,7 +103,7 @@ def run_overlapped(st, *, fused=True, flags=None, sample_rows=None, hot=None, ex
     flags = F.F_TIMERS if flags is None else flags
     hot = st.hot if hot is None else hot
     fr = make_context(st, flags=flags, hot=hot)
-    tr = Trainer(fr, st, fused_lookup=fused, device_inputs=True)
+    tr = Trainer(fr, st, fused_lookup=fused, device_inputs=not host_inputs, host_inputs=host_inputs)
     tr.run()
     fr.flush()
     lg = tr.losses()
@@ -572,3 +572,15 @@ def test_flushing_threads_counts_and_env():
         out = subprocess.run([sys.executable, "-c", code], env=e, capture_output=True, text=True,
                              cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=600)
         assert "OK" in out.stdout, out.stdout + out.stderr
+
+
+@pytest.mark.parametrize("fused", [False, True])
+def test_host_inputs_e2e_path(fused):
+    """The e2e leg's path: ids, x and y from pinned host memory through the C ABI (frugal_step
+    copies the ids, frugal_dot_model copies x and y into its staging), ragged batches."""
+    cfg = tiny1(batch=128, lookahead=4, age_out=2)
+    rng = np.random.default_rng(41)
+    counts = rng.integers(0, 129, size=(50, 1)).astype(np.int32)
+    counts[6] = 0
+    st = W.gen_stream(cfg, 50, counts=counts)
+    run_overlapped(st, fused=fused, exact=True, host_inputs=True)

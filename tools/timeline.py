@@ -26,18 +26,23 @@ grad = torch.empty_like(emb)
 loss = torch.zeros(S + L + 2, dtype=torch.float64, device=dev)
 for t in range(L):
     fr.prefetch(t, ids[t], st.counts[t])
+FUSED = os.environ.get("TL_FUSED", "1") == "1"
+host_ms = []
 for s in range(S):
+    h0 = time.perf_counter()
     fr.step(s, ids[s + L], st.counts[s + L])
     if SLEEP:  # diagnostic: let the step's flushes settle before the gather
         torch.cuda.synchronize()
         time.sleep(SLEEP)
-    fr.lookup(s, emb)
-    fr.dot_model(s, emb, x[s], y[s], grad, loss[s:s + 1])
+    fr.lookup(s, None if FUSED else emb)
+    fr.dot_model(s, None if FUSED else emb, x[s], y[s], grad, loss[s:s + 1])
     fr.backward_update(s, grad)
+    host_ms.append((time.perf_counter() - h0) * 1e3)
     if s == S - 6:
         torch.cuda.synchronize()
         fr.get_stats()
 torch.cuda.synchronize()
+print("host enqueue ms/step (steady state, last 30): %.3f" % (sum(host_ms[-30:]) / 30))
 tl = fr.get_timeline()
 t00 = tl[0][1]
 for name, a, b in tl:
