@@ -115,6 +115,7 @@ struct frugal_ctx {
     std::vector<int32_t> hs_host;    // host copy (frugal_read_host)
     int side_first_blocks = 20;      // grid cap of the drain's deadline-(s+1) part
     int pack_blocks = 20;            // grid cap of the drain's pack kernel (flushing-thread drain)
+    int pack_rows = 1;               // rows in flight per lane group in the pack kernel (FRUGAL_PACK_ROWS=4)
     int flush_tma = 0;               // flushes by TMA bulk stores: 0 none, 1 side drain, 2 all (FRUGAL_FLUSH_TMA; measured no gain: profiles/r1_sweep21_flush_tma.txt)
     int glue_cache = -1;         // REC glue keeps a sample's rows in registers (F <= 32): -1 auto, 0 never, 1 always
     bool glue_rg = true;         // REC glue: row-group kernel k_dot_rg (FRUGAL_GLUE_RG=0: the warp-per-sample k_dot_model)
@@ -195,6 +196,7 @@ struct frugal_ctx {
     int64_t sl_cap = 0;
     int32_t* sl_rows[2] = {nullptr, nullptr};
     int32_t* sl_p[2] = {nullptr, nullptr};
+    int32_t* sl_src[2] = {nullptr, nullptr};  // [4][sl_cap]: each listed row's source at schedule time (-1-slot | pool row)
     int32_t* sl_cnt[2] = {nullptr, nullptr};
     int32_t* adj_rows[2] = {nullptr, nullptr};  // AdjustPriority inf -> t rows, by consuming step parity
     int32_t* adj_p[2] = {nullptr, nullptr};
@@ -312,7 +314,8 @@ void launch_ingest_prologue(frugal_ctx* c, const int32_t* prm, cudaStream_t st);
 void launch_ingest_bits(frugal_ctx* c, QueueSlot& q, const int32_t* prm, cudaStream_t st);
 void launch_schedule(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStream_t st);
 void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begin, const int32_t* d_end,
-                       int max_blocks, int counter, cudaStream_t st, bool side = false);
+                       int max_blocks, int counter, cudaStream_t st, bool side = false,
+                       const int32_t* srcs = nullptr);
 void launch_pack_drain(frugal_ctx* c, int par, uint32_t seq, int max_blocks, cudaStream_t st);
 void launch_wait_word(frugal_ctx* c, const uint32_t* dflag, uint32_t value, cudaStream_t st);
 void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32_t* cnt, float* rows, int64_t step,

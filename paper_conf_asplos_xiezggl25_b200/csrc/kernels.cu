@@ -653,7 +653,9 @@ __global__ void k_schedule(const int32_t* __restrict__ T, const int32_t* d_nT, c
                            const int32_t* __restrict__ pkey, const int32_t* pcount_seg, int32_t u_age, int32_t s,
                            int write_through, const uint64_t* __restrict__ rbits, int32_t* __restrict__ state,
                            const int32_t* __restrict__ last_upd, int32_t* __restrict__ lists,
-                           int32_t* __restrict__ plist, int32_t* cnt, int64_t cap) {
+                           int32_t* __restrict__ plist, int32_t* cnt, int64_t cap, const int32_t* __restrict__ slot,
+                           const int32_t* __restrict__ pool_idx, int P, int64_t capT, int32_t* __restrict__ srcl,
+                           int age_seg) {
     const int nA = d_nT ? *d_nT : 0;
     const int nB = *adj_cnt;
     const int nC = pcount_seg ? *pcount_seg : 0;
@@ -707,6 +709,19 @@ __global__ void k_schedule(const int32_t* __restrict__ T, const int32_t* d_nT, c
             const int64_t at = (int64_t)cls * cap + base + __popc(peers & lanemask_lt());
             lists[at] = lk;
             if (cls < 3) plist[at] = p;
+            // the row's current source -- its cache slot (-1 - slot) or its dirty-pool row -- read
+            // now: the flushes and the drain's pack then need one dependent load per row instead
+            // of three, and an urgent row (read and updated at s, world 1 flushes it off the
+            // critical path) is copied from exactly its post-(s-1) bytes.  Age-outs come from
+            // pool segment age_seg, row i of it.
+            int32_t code;
+            if (cls == 3) {
+                code = (int32_t)((int64_t)age_seg * capT + (i - nA - nB));
+            } else {
+                const int sl = slot[lk];
+                code = sl >= 0 ? -1 - sl : (int32_t)((int64_t)(last_upd[lk] % P) * capT + pool_idx[lk]);
+            }
+            srcl[at] = code;
         }
     }
 }
@@ -727,7 +742,7 @@ void launch_schedule(frugal_ctx* c, QueueSlot* prev, int64_t s, int par, cudaStr
         prev ? prev->T : nullptr, prev ? prev->nT : nullptr, c->adj_rows[par], c->adj_p[par], c->adj_cnt[par],
         c->pkey + (size_t)seg * c->capT, u >= 0 ? c->pcount + seg : nullptr, (int32_t)u, (int32_t)s,
         c->cfg.mode == FRUGAL_MODE_WRITE_THROUGH, c->rbits, c->state, c->last_upd, c->sl_rows[par], c->sl_p[par],
-        c->sl_cnt[par], c->sl_cap);
+        c->sl_cnt[par], c->sl_cap, c->slot, c->pool_idx, c->P, c->capT, c->sl_src[par], seg);
     c->launches++;
 }
 
@@ -904,7 +919,8 @@ __global__ void k_flush_rows(const int32_t* __restrict__ rows, const int32_t* d_
                              int world, int g, int d4, const int32_t* __restrict__ slot,
                              const int32_t* __restrict__ last_upd, const int32_t* __restrict__ pool_idx, int P,
                              int64_t capT, const float4* __restrict__ cw, const float4* __restrict__ pw, float4* hw,
-                             const int32_t* __restrict__ hs, unsigned long long* stats, int sysfence) {
+                             const int32_t* __restrict__ hs, unsigned long long* stats, int sysfence,
+                             const int32_t* __restrict__ srcs) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
@@ -916,13 +932,16 @@ __global__ void k_flush_rows(const int32_t* __restrict__ rows, const int32_t* d_
     for (int64_t a = b + gid; a < e; a += gs) {
         int32_t lk = rows[a];
         int64_t k = (int64_t)lk * world + g;
-        int sl = slot[lk];
+        // source: the location recorded by the scheduler (urgent bucket off the critical path),
+        // else the row's live metadata
+        const int32_t code = srcs ? srcs[a] : 0;
+        int sl = srcs ? (code < 0 ? -1 - code : -1) : slot[lk];
         const float4* src;
         if (sl >= 0) {
             src = cw + (int64_t)sl * d4;
             nh += (l == 0);
         } else {
-            src = pw + ((int64_t)(last_upd[lk] % P) * capT + pool_idx[lk]) * d4;
+            src = pw + (srcs ? (int64_t)code : ((int64_t)(last_upd[lk] % P) * capT + pool_idx[lk])) * d4;
             nc += (l == 0);
         }
         float4* dst = hw + host_row(hs, k) * d4;
@@ -952,13 +971,13 @@ __global__ void k_flush_rows(const int32_t* __restrict__ rows, const int32_t* d_
 }
 
 void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begin, const int32_t* d_end,
-                       int max_blocks, int counter, cudaStream_t st, bool side) {
+                       int max_blocks, int counter, cudaStream_t st, bool side, const int32_t* srcs) {
     const int d4 = c->d / 4, gs = group_size(d4);
     int grid = std::min(grid_for(c->capT * (int64_t)gs, 256, 4), max_blocks);
     const bool tma = c->flush_tma == 2 || (c->flush_tma == 1 && side);
 #define FLUSH_ARGS                                                                                                \
     rows, d_begin, d_end, c->n, c->g, d4, c->slot, c->last_upd, c->pool_idx, c->P, c->capT, (const float4*)c->cw, \
-        (const float4*)c->pw, (float4*)c->dh_w, c->hs, counter >= 0 ? c->dstats + counter : nullptr, c->n > 1
+        (const float4*)c->pw, (float4*)c->dh_w, c->hs, counter >= 0 ? c->dstats + counter : nullptr, c->n > 1, srcs
     if (tma) {
         const size_t smem = (size_t)(256 / gs) * d4 * 16;
         DISPATCH_GS(gs, (k_flush_rows<GS, true><<<grid, 256, smem, st>>>(FLUSH_ARGS)));
@@ -978,44 +997,67 @@ void launch_flush_rows(frugal_ctx* c, const int32_t* rows, const int32_t* d_begi
 // flushing threads then copy them into the table.  The rows are untouched until their
 // deadline (> s), so packing them at any point of step s reads their post-(s-1) values.
 // The publish kernel that follows tells the threads how many rows each part has.
-template <int GS>
-__global__ void k_pack_drain(const int32_t* __restrict__ lists, const int32_t* __restrict__ cnt, int64_t cap, int world,
-                             int g, int d4, const int32_t* __restrict__ slot, const int32_t* __restrict__ last_upd,
-                             const int32_t* __restrict__ pool_idx, int P, int64_t capT, const float4* __restrict__ cw,
-                             const float4* __restrict__ pw, const int32_t* __restrict__ hs, float4* hrows,
-                             int64_t* hkeys, unsigned long long* stats, int part) {
+template <int GS, int R>
+__global__ void k_pack_drain(const int32_t* __restrict__ lists, const int32_t* __restrict__ srcl,
+                             const int32_t* __restrict__ cnt, int64_t cap, int world, int g, int d4,
+                             const float4* __restrict__ cw, const float4* __restrict__ pw,
+                             const int32_t* __restrict__ hs, float4* hrows, int64_t* hkeys,
+                             unsigned long long* stats, unsigned long long* ustats, int part, int with_urgent) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
-    const int n1 = cnt[1], n2 = cnt[2], n3 = cnt[3];
-    // part 0: list 1 (deadline s+1) -> staging [0, n1); part 1: lists 2, 3 -> [n1, n1+n2+n3)
-    const int lo = part == 0 ? 0 : n1, n = part == 0 ? n1 : n1 + n2 + n3;
-    unsigned nh = 0, nc = 0;
-    for (int64_t a = lo + gid; a < n; a += gs) {
-        const int64_t at = a < n1 ? cap + a : a < n1 + n2 ? 2 * cap + (a - n1) : 3 * cap + (a - n1 - n2);
-        const int32_t lk = lists[at];
-        const int sl = slot[lk];
-        const float4* src;
-        if (sl >= 0) {
-            src = cw + (int64_t)sl * d4;
-            nh += (l == 0);
-        } else {
-            src = pw + ((int64_t)(last_upd[lk] % P) * capT + pool_idx[lk]) * d4;
-            nc += (l == 0);
+    const int n1 = cnt[1], n2 = cnt[2], n3 = cnt[3], n0 = with_urgent ? cnt[0] : 0;
+    // part 0: list 1 (deadline s+1) -> staging [0, n1); part 1: lists 2, 3 (and, world 1 with
+    // the urgent bucket off the critical path, list 0) -> [n1, n1+n2+n3+n0)
+    const int lo = part == 0 ? 0 : n1, n = part == 0 ? n1 : n1 + n2 + n3 + n0;
+    unsigned nh = 0, nc = 0, uh = 0, uc = 0;
+    // R rows in flight per lane group: list entry + source (coalesced), then the row
+    for (int64_t a0 = lo + gid; a0 < n; a0 += gs * R) {
+        int64_t at[R];
+        int32_t code[R], lk[R];
+#pragma unroll
+        for (int r = 0; r < R; r++) {
+            const int64_t a = a0 + (int64_t)r * gs;
+            at[r] = a >= n ? -1
+                  : a < n1 ? cap + a : a < n1 + n2 ? 2 * cap + (a - n1)
+                  : a < n1 + n2 + n3 ? 3 * cap + (a - n1 - n2) : (a - n1 - n2 - n3);
+            code[r] = at[r] >= 0 ? srcl[at[r]] : 0;
+            lk[r] = at[r] >= 0 ? lists[at[r]] : 0;
         }
-        for (int v = l; v < d4; v += GS) hrows[a * d4 + v] = src[v];
-        if (l == 0) hkeys[a] = host_row(hs, (int64_t)lk * world + g);
+        for (int v0 = 0; v0 < d4; v0 += GS) {
+            const int v = v0 + l;
+            float4 x[R];
+#pragma unroll
+            for (int r = 0; r < R; r++)
+                if (at[r] >= 0 && v < d4)
+                    x[r] = code[r] < 0 ? cw[(int64_t)(-1 - code[r]) * d4 + v] : pw[(int64_t)code[r] * d4 + v];
+#pragma unroll
+            for (int r = 0; r < R; r++)
+                if (at[r] >= 0 && v < d4) hrows[(a0 + (int64_t)r * gs) * d4 + v] = x[r];
+        }
+#pragma unroll
+        for (int r = 0; r < R; r++) {
+            if (at[r] < 0 || l != 0) continue;
+            const int64_t a = a0 + (int64_t)r * gs;
+            hkeys[a] = host_row(hs, (int64_t)lk[r] * world + g);
+            const bool urg = a >= n1 + n2 + n3;
+            if (code[r] < 0) { if (urg) uh++; else nh++; }
+            else { if (urg) uc++; else nc++; }
+        }
     }
     block_fence_system();  // rows and keys reach host memory before the publish kernel's flag
     block_count(stats, nh);
     block_count(stats + 1, nc);
+    block_count(ustats, uh);
+    block_count(ustats + 1, uc);
 }
 // publish part `part` of job `seq` (= s+1) of staging buffer `par`: part sizes, then the part's
 // ready word (release) -- the threads start on part 0 (deadline s+1, the next gate waits for
 // it) while the kernel packs part 1
-__global__ void k_publish_drain(const int32_t* __restrict__ cnt, uint32_t* ctl, int par, uint32_t seq, int part) {
+__global__ void k_publish_drain(const int32_t* __restrict__ cnt, uint32_t* ctl, int par, uint32_t seq, int part,
+                                int with_urgent) {
     ctl[CTL_N1 + par] = (uint32_t)cnt[1];
-    ctl[CTL_NTOT + par] = (uint32_t)(cnt[1] + cnt[2] + cnt[3]);
+    ctl[CTL_NTOT + par] = (uint32_t)(cnt[1] + cnt[2] + cnt[3] + (with_urgent ? cnt[0] : 0));
     __threadfence_system();
     uint32_t* w = ctl + (part == 0 ? CTL_READY1 : CTL_READY) + par;
     asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(w), "r"(seq) : "memory");
@@ -1023,12 +1065,21 @@ __global__ void k_publish_drain(const int32_t* __restrict__ cnt, uint32_t* ctl, 
 void launch_pack_drain(frugal_ctx* c, int par, uint32_t seq, int max_blocks, cudaStream_t st) {
     const int d4 = c->d / 4, gs = group_size(d4);
     int grid = std::min(grid_for(3 * c->sl_cap * (int64_t)gs, 256, 4), max_blocks);
+    const int wu = c->urgent_side ? 1 : 0;  // world 1: the urgent bucket goes with the drain
     for (int part = 0; part < 2; part++) {
-        DISPATCH_GS(gs, (k_pack_drain<GS><<<grid, 256, 0, st>>>(
-                            c->sl_rows[par], c->sl_cnt[par], c->sl_cap, c->n, c->g, d4, c->slot, c->last_upd,
-                            c->pool_idx, c->P, c->capT, (const float4*)c->cw, (const float4*)c->pw, c->hs,
-                            (float4*)c->dfl_rows[par], c->dfl_keys[par], c->dstats + FRUGAL_C_SIDE_HOT, part)));
-        k_publish_drain<<<1, 1, 0, st>>>(c->sl_cnt[par], c->dfl_ctl, par, seq, part);
+#define PACK(RR)                                                                                              \
+    DISPATCH_GS(gs, (k_pack_drain<GS, RR><<<grid, 256, 0, st>>>(                                              \
+                        c->sl_rows[par], c->sl_src[par], c->sl_cnt[par], c->sl_cap, c->n, c->g, d4,           \
+                        (const float4*)c->cw, (const float4*)c->pw, c->hs, (float4*)c->dfl_rows[par],        \
+                        c->dfl_keys[par], c->dstats + FRUGAL_C_SIDE_HOT, c->dstats + FRUGAL_C_URGENT_HOT, part, \
+                        wu)))
+        if (c->pack_rows >= 4) {
+            PACK(4);
+        } else {
+            PACK(1);
+        }
+#undef PACK
+        k_publish_drain<<<1, 1, 0, st>>>(c->sl_cnt[par], c->dfl_ctl, par, seq, part, wu);
     }
     c->launches += 4;
 }

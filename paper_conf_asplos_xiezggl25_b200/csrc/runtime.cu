@@ -139,7 +139,14 @@ struct frugal::Flushers {
     std::vector<std::thread> th;
     std::atomic<bool> stop{false};
     std::atomic<int> done[2][2];  // [parity][part]: threads finished
+    // instrumentation (thread 0): jobs, ns from its part-0 flag to the job's end, ns waiting
+    std::atomic<int64_t> jobs{0}, busy_ns{0}, wait_ns{0};
 };
+static inline int64_t mono_ns() {
+    timespec ts;
+    clock_gettime(CLOCK_MONOTONIC, &ts);
+    return (int64_t)ts.tv_sec * 1000000000 + ts.tv_nsec;
+}
 
 static inline uint32_t ctl_load(const uint32_t* p) { return __atomic_load_n(p, __ATOMIC_ACQUIRE); }
 static inline void ctl_store(uint32_t* p, uint32_t v) { __atomic_store_n(p, v, __ATOMIC_RELEASE); }
@@ -165,6 +172,7 @@ static void flusher_main(frugal_ctx* c, int t) {
         const uint32_t seq = (uint32_t)(job + 1);
         const float* rows = c->hfl_rows[par];
         const int64_t* keys = c->hfl_keys[par];
+        int64_t t_wait0 = t == 0 ? mono_ns() : 0, t_start = 0;
         for (int part = 0; part < 2; part++) {
             // wait for the device to publish the part: spin while jobs keep coming, then poll gently
             const uint32_t* ready = ctl + (part == 0 ? CTL_READY1 : CTL_READY) + par;
@@ -181,6 +189,10 @@ static void flusher_main(frugal_ctx* c, int t) {
                 }
             }
             idle_since = 0.0;
+            if (t == 0 && part == 0) {
+                t_start = mono_ns();
+                F->wait_ns.fetch_add(t_start - t_wait0, std::memory_order_relaxed);
+            }
             const int64_t n1 = ctl_load(ctl + CTL_N1 + par), nt = ctl_load(ctl + CTL_NTOT + par);
             const int64_t b = part == 0 ? 0 : n1, e = part == 0 ? n1 : nt;
             copy_rows_nt(c->h_w, rows, keys, b + (e - b) * t / T, b + (e - b) * (t + 1) / T, c->d);
@@ -192,6 +204,10 @@ static void flusher_main(frugal_ctx* c, int t) {
                     ctl_store((uint32_t*)(c->h_flags + (which * 32 + c->g) * 16), seq);
                 }
             }
+        }
+        if (t == 0) {
+            F->busy_ns.fetch_add(mono_ns() - t_start, std::memory_order_relaxed);
+            F->jobs.fetch_add(1, std::memory_order_relaxed);
         }
     }
 }
@@ -286,7 +302,7 @@ static void free_ctx(frugal_ctx* c) {
     }
     F(c->hs); F(c->rows_buf[0]); F(c->rows_buf[1]); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->long_tasks); F(c->owned_cnt);
     for (int i = 0; i < 2; i++) { F(c->adj_rows[i]); F(c->adj_p[i]); F(c->adj_cnt[i]); }
-    for (int i = 0; i < 2; i++) { F(c->sl_rows[i]); F(c->sl_p[i]); F(c->sl_cnt[i]); }
+    for (int i = 0; i < 2; i++) { F(c->sl_rows[i]); F(c->sl_p[i]); F(c->sl_src[i]); F(c->sl_cnt[i]); }
     F(c->dstats); F(c->kg_W); F(c->kg_A); F(c->a2a_roff); F(c->peer_tab); F(c->gslot);
     for (int r = 0; r < 32; r++)
         for (int i = 0; i < 4; i++)
@@ -486,6 +502,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->update1 = !(getenv("FRUGAL_UPDATE1") && !atoi(getenv("FRUGAL_UPDATE1")));
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 20;
     c->pack_blocks = getenv("FRUGAL_PACK_BLOCKS") ? atoi(getenv("FRUGAL_PACK_BLOCKS")) : c->side_blocks;
+    c->pack_rows = getenv("FRUGAL_PACK_ROWS") ? atoi(getenv("FRUGAL_PACK_ROWS")) : 1;
     // the deadline-(s+1) part of the drain (the next gate waits for it) may run wider
     c->side_first_blocks = getenv("FRUGAL_SIDE_FIRST_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_FIRST_BLOCKS"))
                                                                : c->side_blocks;
@@ -495,6 +512,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     // world 1 with pool reads (R7'): the urgent bucket is not read from the host at its step
     // (FRUGAL_URGENT_SIDE=0: keep it on the critical path)
     c->urgent_side = c->n == 1 && c->pool_hits && !c->side_inline && !c->early &&
+                     k.mode == FRUGAL_MODE_P2F &&
                      !(getenv("FRUGAL_URGENT_SIDE") && !atoi(getenv("FRUGAL_URGENT_SIDE")));
     c->capT = std::max<int64_t>(1, std::min<int64_t>((int64_t)c->n * c->M, c->No));
     c->sl_cap = 2 * c->capT;
@@ -560,7 +578,9 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
             }
         }
     } else {
-        c->shm_base = mmap(nullptr, total, PROT_READ | PROT_WRITE, MAP_SHARED | MAP_ANONYMOUS, -1, 0);
+        // private anonymous memory: transparent huge pages apply (shmem usually has them off),
+        // so the flushing threads' scattered row stores miss the TLB far less often
+        c->shm_base = mmap(nullptr, total, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
     }
     if (c->shm_base == MAP_FAILED) {
         c->shm_base = nullptr;
@@ -694,6 +714,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     for (int i = 0; i < 2; i++) {
         DMALLOC(c->sl_rows[i], 4 * c->sl_cap * 4);
         DMALLOC(c->sl_p[i], 3 * c->sl_cap * 4);
+        DMALLOC(c->sl_src[i], 4 * c->sl_cap * 4);
         DMALLOC(c->sl_cnt[i], 4 * 4);
         cudaMemset(c->sl_cnt[i], 0, 16);
     }
@@ -808,7 +829,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         return FRUGAL_ECUDA;
     }
     if (c->host_flush) {
-        const int64_t cap = std::max<int64_t>(1, std::min<int64_t>(3 * c->sl_cap, c->No));
+        const int64_t cap = std::max<int64_t>(1, std::min<int64_t>(4 * c->sl_cap, c->No));
         bool ok = cudaHostAlloc((void**)&c->hfl_ctl, 4096, cudaHostAllocMapped | cudaHostAllocPortable) == cudaSuccess;
         for (int i = 0; ok && i < 2; i++) {
             ok = cudaHostAlloc((void**)&c->hfl_rows[i], (size_t)cap * rowb, cudaHostAllocMapped | cudaHostAllocPortable) ==
@@ -1033,13 +1054,13 @@ static frugal_status launch_drain(frugal_ctx* c, int64_t s, cudaStream_t st, cud
     } else {
         Timer tm(c, PH_SIDE, sd);
         launch_flush_rows(c, c->sl_rows[par] + c->sl_cap, nullptr, c->sl_cnt[par] + 1, c->side_first_blocks,
-                          FRUGAL_C_SIDE_HOT, sd, true);
+                          FRUGAL_C_SIDE_HOT, sd, true, c->sl_src[par] + c->sl_cap);
         CK(cudaEventRecord(c->ev_side_first[par], sd));
         if (c->xhost) launch_set_flag(c, FLAG_SIDE_FIRST, (uint32_t)(s + 1), sd);
         launch_flush_rows(c, c->sl_rows[par] + 2 * c->sl_cap, nullptr, c->sl_cnt[par] + 2, c->side_blocks,
-                          FRUGAL_C_SIDE_HOT, sd, true);
+                          FRUGAL_C_SIDE_HOT, sd, true, c->sl_src[par] + 2 * c->sl_cap);
         launch_flush_rows(c, c->sl_rows[par] + 3 * c->sl_cap, nullptr, c->sl_cnt[par] + 3, c->side_blocks,
-                          FRUGAL_C_SIDE_HOT, sd, true);
+                          FRUGAL_C_SIDE_HOT, sd, true, c->sl_src[par] + 3 * c->sl_cap);
         if (c->xhost) launch_set_flag(c, FLAG_SIDE, (uint32_t)(s + 1), sd);
         CKL();
     }
@@ -1114,17 +1135,23 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
         // a10 at world 1 (reading R7'): the only reader of step s is this owner, and it reads
         // every row updated within the pool window -- the whole urgent bucket (updated at s-1)
         // -- from its dirty pool in HBM, so no read of step s needs the bucket's host copies;
-        // they are written on the side stream ahead of the drain, long before any host read of
-        // those rows (after the pool window, P = D+3 >= 4 steps).  Same set, same bytes.
-        CK(cudaEventRecord(c->ev_sched, st));
-        CK(cudaStreamWaitEvent(c->side, c->ev_sched, 0));
-        Timer tm(c, PH_URGENT, c->side);
-        launch_flush_rows(c, c->sl_rows[par], nullptr, c->sl_cnt[par], 1 << 30, FRUGAL_C_URGENT_HOT, c->side);
-        CKL();
+        // they are written off the critical path, long before any host read of those rows
+        // (after the pool window, P = D+3 >= 4 steps): with the flushing threads as the last
+        // part of this step's drain job, else on the side stream ahead of the drain.  Same set,
+        // same bytes.
+        if (!c->host_flush) {
+            CK(cudaEventRecord(c->ev_sched, st));
+            CK(cudaStreamWaitEvent(c->side, c->ev_sched, 0));
+            Timer tm(c, PH_URGENT, c->side);
+            launch_flush_rows(c, c->sl_rows[par], nullptr, c->sl_cnt[par], 1 << 30, FRUGAL_C_URGENT_HOT, c->side,
+                              false, c->sl_src[par] /* sources recorded by the scheduler */);
+            CKL();
+        }
     } else {
         // a10: urgent bucket (priority == s) to the host table on the critical path
         Timer tm(c, PH_URGENT, st);
-        launch_flush_rows(c, c->sl_rows[par], nullptr, c->sl_cnt[par], 1 << 30, FRUGAL_C_URGENT_HOT, st);
+        launch_flush_rows(c, c->sl_rows[par], nullptr, c->sl_cnt[par], 1 << 30, FRUGAL_C_URGENT_HOT, st, false,
+                          c->sl_src[par]);
         if (c->xhost) launch_set_flag(c, FLAG_URGENT, (uint32_t)(s + 1), st);
         CKL();
     }
@@ -1156,7 +1183,20 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
         Timer tm(c, PH_GATE, st);
         // (deadline-s rows are the first part of drain s-1; the side stream is FIFO, so that
         // event also covers every earlier drain)
-        if (!c->xhost) {  // world 1, or the comparison path: only this rank reads its host rows
+        static const bool strict_gate = getenv("FRUGAL_GATE_STRICT") && atoi(getenv("FRUGAL_GATE_STRICT"));
+        if (!c->xhost && c->urgent_side && c->L >= 3 && !strict_gate) {
+            // world 1 reading its dirty pool (R7'): step s reads from the host only rows outside
+            // the pool window (last update < s-D-1, or never).  The deadline-s part of drain s-1
+            // holds rows updated at s-2 -- inside the window -- and, for L >= 3, no
+            // AdjustPriority'd row (those have deadline s-1+L-1 > s); every host-read row of s was
+            // drained at a step <= s-2 (deferred by AdjustPriority at s-L+1, or aged out, and
+            // an aged row read at s had no read in sight at its age-out).  So the gate of s
+            // needs drain s-2 applied in full, one step of slack more than the general rule.
+            if (s >= 2 && c->side_pending[par]) {
+                if (c->host_flush) launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_ALL, (uint32_t)(s - 1), st);
+                else CK(cudaStreamWaitEvent(st, c->ev_side[par], 0));
+            }
+        } else if (!c->xhost) {  // world 1, or the comparison path: only this rank reads its host rows
             if (s >= 1 && c->side_pending[par ^ 1]) {
                 if (c->host_flush) launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_FIRST, (uint32_t)s, st);
                 else CK(cudaStreamWaitEvent(st, c->ev_side_first[par ^ 1], 0));
@@ -1627,6 +1667,13 @@ extern "C" frugal_status frugal_get_stats(frugal_ctx* c, frugal_stats* out) {
     for (int i = 0; i < FRUGAL_N_COUNTERS; i++) out->count[i] = (int64_t)cnt[i];
     for (int i = 0; i < FRUGAL_N_PHASES; i++) c->phase_ms[i] = 0;
     c->timed_steps = 0;
+    out->flush_jobs = 0;
+    out->flush_ms = out->flush_wait_ms = 0.0;
+    if (c->flushers) {
+        out->flush_jobs = c->flushers->jobs.exchange(0);
+        out->flush_ms = c->flushers->busy_ns.exchange(0) * 1e-6;
+        out->flush_wait_ms = c->flushers->wait_ns.exchange(0) * 1e-6;
+    }
     return FRUGAL_OK;
 }
 

@@ -584,3 +584,29 @@ def test_host_inputs_e2e_path(fused):
     counts[6] = 0
     st = W.gen_stream(cfg, 50, counts=counts)
     run_overlapped(st, fused=fused, exact=True, host_inputs=True)
+
+
+@pytest.mark.parametrize("env", [{}, {"FRUGAL_HOST_FLUSH": "0"}, {"FRUGAL_URGENT_SIDE": "0"}])
+def test_host_table_contents_every_step(env):
+    """The flushed BYTES, not only the flushed sets: after every step (all of the step's flushes
+    applied -- urgent bucket, drain, age-outs, by the flushing threads or the GPU), the whole host
+    table equals the oracle's simulated host table (each row = its value at its last flush),
+    bit for bit.  Catches a flush that copies a row after the optimizer moved it (world 1 flushes
+    the urgent bucket off the critical path from the source the scheduler recorded)."""
+    import subprocess
+    import sys
+    code = ("import sys; sys.path.insert(0, '.'); import numpy as np;"
+            "from tests.test_gpu_parity import tiny1; from oracle.oracle import Oracle;"
+            "from paper_conf_asplos_xiezggl25_b200 import workload as W;"
+            "from paper_conf_asplos_xiezggl25_b200.harness import Trainer, make_context;"
+            "st = W.gen_stream(tiny1(batch=128, lookahead=4, age_out=2), 40);"
+            "fr = make_context(st); tr = Trainer(fr, st, fused_lookup=True, device_inputs=True); o = Oracle(st);"
+            "ks = np.arange(st.cfg.n_rows);"
+            "[(tr.step(), o.step(), (lambda a, b: (np.array_equal(a[0], b[0]) or sys.exit(f'host w differs at step {s}')))"
+            "  (fr.read_host(ks), o.host_rows(ks))) for s in range(st.steps)];"
+            "print('OK')")
+    e = dict(os.environ)
+    e.update(env)
+    out = subprocess.run([sys.executable, "-c", code], env=e, capture_output=True, text=True,
+                         cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=600)
+    assert "OK" in out.stdout, out.stdout + out.stderr
