@@ -42,7 +42,9 @@ struct RowGroup {
     }
 };
 
-// block-aggregated counter: every thread passes its count, one atomic per block
+// block-aggregated counter: every thread passes its count, one atomic per block.  The closing
+// barrier keeps thread 0's reset of the next call away from this call's read (the shared word
+// is one per block across calls; compute-sanitizer racecheck flagged the unordered pair)
 __device__ __forceinline__ void block_count(unsigned long long* dst, unsigned v) {
     __shared__ unsigned s_cnt;
     if (threadIdx.x == 0) s_cnt = 0;
@@ -50,7 +52,11 @@ __device__ __forceinline__ void block_count(unsigned long long* dst, unsigned v)
     for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
     if ((threadIdx.x & 31) == 0 && v) atomicAdd(&s_cnt, v);
     __syncthreads();
-    if (threadIdx.x == 0 && s_cnt) atomicAdd(dst, (unsigned long long)s_cnt);
+    if (threadIdx.x == 0) {
+        const unsigned t = s_cnt;
+        if (t) atomicAdd(dst, (unsigned long long)t);
+    }
+    __syncthreads();
 }
 
 // make this block's prior (host-memory) writes visible system-wide before anything the
