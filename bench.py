@@ -76,6 +76,10 @@ def parse():
                     help="N > 1: v2 (default) = each rank passes only its own ids, the ranks exchange distinct "
                          "ids through the host id mailbox (FRUGAL_F_OWN_IDS); v1 = every rank copies and scans "
                          "all ranks' ids")
+    ap.add_argument("--host-gb", type=float, default=0.0,
+                    help="criteo_tb (configs[4]): scale the Kaggle-profile tables to a host table of this many GB "
+                         "(default: the full 8.8e8 rows if they fit in 45%% of this host's memory, else as many "
+                         "rows as do)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for barriers / the max-over-ranks timing only")
     return ap.parse_args()
@@ -282,7 +286,12 @@ def main():
     def max_over_ranks(x):
         return dist_max(x, world, dist, coll_dev)
 
-    cfg = W.config(args.config, world=world, alpha=args.alpha)
+    over = {}
+    if args.config == "criteo_tb":  # configs[4]: 450 GB at full size -- rows scaled to the host's memory
+        mem = os.sysconf("SC_PAGE_SIZE") * os.sysconf("SC_PHYS_PAGES")
+        budget = args.host_gb * 1e9 if args.host_gb > 0 else 0.45 * mem
+        over["rows_total"] = min(8.8e8, budget / (128 * 4))
+    cfg = W.config(args.config, world=world, alpha=args.alpha, **over)
     K, Wm, L = args.steps, args.warmup, cfg.lookahead
     S = Wm + 2 * K + L + 2
     # at most SG distinct generated steps, cycled (step t reads generated step t % SG): the
@@ -599,6 +608,9 @@ def main():
         "dtype": "f32", "data": "synthetic",
         "config": {"workload": f"{cfg.name} ({CONFIG_NAMES.get(cfg.name, '')})", "global_batch": world * B,
                    "batch_per_gpu": B, "tables": Fs, "rows": cfg.n_rows, "dim": d, "alpha": cfg.alpha,
+                   "rows_note": ("the Kaggle profile scaled to %.3g rows (%.0f GB host table) to fit this host's "
+                                 "memory; configs[4] is 8.8e8 rows / 450 GB" % (cfg.n_rows, cfg.n_rows * d * 4 / 1e9))
+                   if cfg.name == "criteo_tb" and cfg.n_rows < 8.7e8 else None,
                    "lookahead": L, "age_out": cfg.age_out, "cache_ratio": cfg.cache_ratio, "opt": cfg.opt,
                    "flush_mode": args.mode,
                    "drain": "side-stream zero-copy scatter kernel" if args.drain == "gpu" else

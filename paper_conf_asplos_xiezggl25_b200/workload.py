@@ -91,8 +91,16 @@ class WorkloadConfig:
         return np.concatenate([[0], np.cumsum(self.table_rows)[:-1]]).astype(np.int64)
 
 
+def criteo_tb_rows(total: float = 8.8e8) -> List[int]:
+    """CriteoTB-shaped tables: the Criteo-Kaggle cardinality profile scaled to `total` rows
+    (Table 2: 882M rows at full size)."""
+    scale = total / sum(CRITEO_KAGGLE_ROWS)
+    return [max(1, int(round(r * scale))) for r in CRITEO_KAGGLE_ROWS]
+
+
 def config(name: str, **over) -> WorkloadConfig:
-    """The BASELINE.json configs restated as synthetic inputs."""
+    """The BASELINE.json configs restated as synthetic inputs.  criteo_tb takes
+    `rows_total` (default 8.8e8) to scale its tables to what the host's memory holds."""
     if name == "tiny":          # configs[0]
         c = WorkloadConfig("tiny", [10_000], dim=16, batch=256, world=2)
     elif name == "criteo_kaggle":  # configs[1]
@@ -109,8 +117,7 @@ def config(name: str, **over) -> WorkloadConfig:
         c = WorkloadConfig("tiny_kg", [5_000, 40], dim=16, batch=96, world=1, slot_tables=[0, 1, 0, 0],
                            model="transe", neg_chunk=32, lookahead=4, age_out=3)
     elif name == "criteo_tb":   # configs[4]
-        scale = 8.8e8 / sum(CRITEO_KAGGLE_ROWS)
-        rows = [max(1, int(round(r * scale))) for r in CRITEO_KAGGLE_ROWS]
+        rows = criteo_tb_rows(over.pop("rows_total", 8.8e8))
         c = WorkloadConfig("criteo_tb", rows, dim=128, batch=8192, world=8, cache_ratio=0.10,
                            opt="sgd", lr=1.0)
     else:
