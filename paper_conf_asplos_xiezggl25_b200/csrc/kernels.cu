@@ -1002,7 +1002,8 @@ __global__ void k_pack_drain(const int32_t* __restrict__ lists, const int32_t* _
                              const int32_t* __restrict__ cnt, int64_t cap, int world, int g, int d4,
                              const float4* __restrict__ cw, const float4* __restrict__ pw,
                              const int32_t* __restrict__ hs, float4* hrows, int64_t* hkeys,
-                             unsigned long long* stats, unsigned long long* ustats, int part, int with_urgent) {
+                             unsigned long long* stats, unsigned long long* ustats, int part, int with_urgent,
+                             int to_host) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
@@ -1045,11 +1046,27 @@ __global__ void k_pack_drain(const int32_t* __restrict__ lists, const int32_t* _
             else { if (urg) uc++; else nc++; }
         }
     }
-    block_fence_system();  // rows and keys reach host memory before the publish kernel's flag
+    if (to_host) block_fence_system();  // rows and keys reach host memory before the publish kernel's flag
     block_count(stats, nh);
     block_count(stats + 1, nc);
     block_count(ustats, uh);
     block_count(ustats + 1, uc);
+}
+
+// second stage of the two-stage pack: one part of the job, already contiguous in HBM, copied to
+// the pinned staging queue by a FEW CTAs as one sequential run (8 CTAs reach ~50 GB/s of
+// zero-copy writes, profiles/r2_zc_write_probe.txt) -- few CTAs keep the queue of posted PCIe
+// writes short, and a PCIe read issued meanwhile (the gather's host rows, a gate's flag) waits
+// behind that queue
+__global__ void __launch_bounds__(256) k_copy_seq(const int32_t* __restrict__ cnt, int part, int with_urgent, int d4,
+                                                  const float4* __restrict__ srows, const int64_t* __restrict__ skeys,
+                                                  float4* hrows, int64_t* hkeys) {
+    const int n1 = cnt[1], nall = cnt[1] + cnt[2] + cnt[3] + (with_urgent ? cnt[0] : 0);
+    const int64_t lo = part == 0 ? 0 : n1, hi = part == 0 ? n1 : nall;
+    const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x, nt = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t e = lo * d4 + t; e < hi * d4; e += nt) hrows[e] = srows[e];
+    for (int64_t a = lo + t; a < hi; a += nt) hkeys[a] = skeys[a];
+    block_fence_system();
 }
 // publish part `part` of job `seq` (= s+1) of staging buffer `par`: part sizes, then the part's
 // ready word (release) -- the threads start on part 0 (deadline s+1, the next gate waits for
@@ -1064,21 +1081,33 @@ __global__ void k_publish_drain(const int32_t* __restrict__ cnt, uint32_t* ctl, 
 }
 void launch_pack_drain(frugal_ctx* c, int par, uint32_t seq, int max_blocks, cudaStream_t st) {
     const int d4 = c->d / 4, gs = group_size(d4);
-    int grid = std::min(grid_for(3 * c->sl_cap * (int64_t)gs, 256, 4), max_blocks);
+    const int nthr = c->pack_threads;
     const int wu = c->urgent_side ? 1 : 0;  // world 1: the urgent bucket goes with the drain
+    // two stages (default): the rows are gathered into a contiguous HBM staging run by a full
+    // grid (HBM-bound, a few us), then copied to the host by k_copy_seq with max_blocks CTAs;
+    // FRUGAL_PACK_2STAGE=0: one kernel gathers straight to the host with max_blocks CTAs
+    const bool two = c->pack_2stage;
+    const int grid = two ? grid_for(3 * c->sl_cap * (int64_t)gs, 256, 2)
+                         : std::min(grid_for(3 * c->sl_cap * (int64_t)gs, nthr, 4), max_blocks);
+    float4* rows_dst = two ? (float4*)c->dst_rows[par] : (float4*)c->dfl_rows[par];
+    int64_t* keys_dst = two ? c->dst_keys[par] : c->dfl_keys[par];
     for (int part = 0; part < 2; part++) {
 #define PACK(RR)                                                                                              \
-    DISPATCH_GS(gs, (k_pack_drain<GS, RR><<<grid, 256, 0, st>>>(                                              \
+    DISPATCH_GS(gs, (k_pack_drain<GS, RR><<<grid, two ? 256 : nthr, 0, st>>>(                                \
                         c->sl_rows[par], c->sl_src[par], c->sl_cnt[par], c->sl_cap, c->n, c->g, d4,           \
-                        (const float4*)c->cw, (const float4*)c->pw, c->hs, (float4*)c->dfl_rows[par],        \
-                        c->dfl_keys[par], c->dstats + FRUGAL_C_SIDE_HOT, c->dstats + FRUGAL_C_URGENT_HOT, part, \
-                        wu)))
+                        (const float4*)c->cw, (const float4*)c->pw, c->hs, rows_dst, keys_dst,                \
+                        c->dstats + FRUGAL_C_SIDE_HOT, c->dstats + FRUGAL_C_URGENT_HOT, part, wu, two ? 0 : 1)))
         if (c->pack_rows >= 4) {
             PACK(4);
         } else {
             PACK(1);
         }
 #undef PACK
+        if (two) {
+            k_copy_seq<<<max_blocks, 256, 0, st>>>(c->sl_cnt[par], part, wu, d4, (const float4*)c->dst_rows[par],
+                                                    c->dst_keys[par], (float4*)c->dfl_rows[par], c->dfl_keys[par]);
+            c->launches++;
+        }
         k_publish_drain<<<1, 1, 0, st>>>(c->sl_cnt[par], c->dfl_ctl, par, seq, part, wu);
     }
     c->launches += 4;

@@ -774,7 +774,10 @@ __global__ void k_wait_flags(const uint32_t* f, int world, uint32_t v, int32_t* 
         }
     }
     __syncwarp();
-    __threadfence_system();
+    // acquire only (each lane already loaded its flag with ld.acquire.sys): a fence.sc.sys here
+    // would wait for every outstanding system-scope access of the GPU -- with the drain's
+    // zero-copy stores in flight on the side stream that cost ~70 us per gate
+    asm volatile("fence.acquire.sys;" ::: "memory");
 }
 // flag value from the ingest's parameter block (graph-replayed launches)
 __global__ void k_set_flag_prm(uint32_t* f, const int32_t* __restrict__ prm) {
@@ -803,7 +806,10 @@ __global__ void k_wait_flags_prm(const uint32_t* f, int world, const int32_t* __
         }
     }
     __syncwarp();
-    __threadfence_system();
+    // acquire only (each lane already loaded its flag with ld.acquire.sys): a fence.sc.sys here
+    // would wait for every outstanding system-scope access of the GPU -- with the drain's
+    // zero-copy stores in flight on the side stream that cost ~70 us per gate
+    asm volatile("fence.acquire.sys;" ::: "memory");
 }
 void launch_set_flag_prm(frugal_ctx* c, int which, const int32_t* prm, cudaStream_t st) {
     k_set_flag_prm<<<1, 1, 0, st>>>(c->dh_flags + (which * 32 + c->g) * 16, prm);

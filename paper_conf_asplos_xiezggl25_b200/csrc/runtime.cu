@@ -272,6 +272,8 @@ static void free_ctx(frugal_ctx* c) {
         c->flushers = nullptr;
     }
     for (int i = 0; i < 2; i++) {
+        if (c->dst_rows[i]) cudaFree(c->dst_rows[i]);
+        if (c->dst_keys[i]) cudaFree(c->dst_keys[i]);
         if (c->hfl_rows[i]) cudaFreeHost(c->hfl_rows[i]);
         if (c->hfl_keys[i]) cudaFreeHost(c->hfl_keys[i]);
     }
@@ -501,8 +503,12 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->fuse_opt = !(getenv("FRUGAL_FUSE_OPT") && !atoi(getenv("FRUGAL_FUSE_OPT")));
     c->update1 = !(getenv("FRUGAL_UPDATE1") && !atoi(getenv("FRUGAL_UPDATE1")));
     c->side_blocks = getenv("FRUGAL_SIDE_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_BLOCKS")) : 20;
-    c->pack_blocks = getenv("FRUGAL_PACK_BLOCKS") ? atoi(getenv("FRUGAL_PACK_BLOCKS")) : c->side_blocks;
+    // few CTAs for the zero-copy writes of the pack: 8 reach the link rate, and a short queue of
+    // posted writes keeps concurrent PCIe reads fast (profiles/r2_zc_write_probe.txt, r2_sweep_pack*.txt)
+    c->pack_blocks = getenv("FRUGAL_PACK_BLOCKS") ? atoi(getenv("FRUGAL_PACK_BLOCKS")) : 8;
+    c->pack_2stage = getenv("FRUGAL_PACK_2STAGE") && atoi(getenv("FRUGAL_PACK_2STAGE"));  // measured slower (r2_sweep_pack_2stage.txt)
     c->pack_rows = getenv("FRUGAL_PACK_ROWS") ? atoi(getenv("FRUGAL_PACK_ROWS")) : 1;
+    c->pack_threads = getenv("FRUGAL_PACK_THREADS") ? atoi(getenv("FRUGAL_PACK_THREADS")) : 256;
     // the deadline-(s+1) part of the drain (the next gate waits for it) may run wider
     c->side_first_blocks = getenv("FRUGAL_SIDE_FIRST_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_FIRST_BLOCKS"))
                                                                : c->side_blocks;
@@ -848,6 +854,11 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
             return FRUGAL_ENOMEM;
         }
         memset(c->hfl_ctl, 0, 4096);
+        if (c->pack_2stage)
+            for (int i = 0; i < 2; i++) {
+                DMALLOC(c->dst_rows[i], (size_t)cap * rowb);
+                DMALLOC(c->dst_keys[i], (size_t)cap * 8);
+            }
         cudaHostGetDevicePointer((void**)&c->dfl_ctl, c->hfl_ctl, 0);
         const long ncpu = sysconf(_SC_NPROCESSORS_ONLN);
         c->n_flushers = getenv("FRUGAL_FLUSH_THREADS") ? atoi(getenv("FRUGAL_FLUSH_THREADS"))
@@ -1186,15 +1197,18 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
         static const bool strict_gate = getenv("FRUGAL_GATE_STRICT") && atoi(getenv("FRUGAL_GATE_STRICT"));
         if (!c->xhost && c->urgent_side && c->L >= 3 && !strict_gate) {
             // world 1 reading its dirty pool (R7'): step s reads from the host only rows outside
-            // the pool window (last update < s-D-1, or never).  The deadline-s part of drain s-1
-            // holds rows updated at s-2 -- inside the window -- and, for L >= 3, no
-            // AdjustPriority'd row (those have deadline s-1+L-1 > s); every host-read row of s was
-            // drained at a step <= s-2 (deferred by AdjustPriority at s-L+1, or aged out, and
-            // an aged row read at s had no read in sight at its age-out).  So the gate of s
-            // needs drain s-2 applied in full, one step of slack more than the general rule.
-            if (s >= 2 && c->side_pending[par]) {
-                if (c->host_flush) launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_ALL, (uint32_t)(s - 1), st);
-                else CK(cudaStreamWaitEvent(st, c->ev_side[par], 0));
+            // the pool window (last update < s-D-1, or never).  Such a row, if it was ever
+            // updated, was flushed by (a) an AdjustPriority'd deferral made at s-L+1 (deadline s),
+            // (b) a deferral with deadline s made at b <= s-D-1 (its update b-1 is outside the
+            // window at s only if s-b > D), or (c) an age-out at a <= s-L (an aged row had no
+            // read in sight, L steps).  So the gate of s needs the drains up to s - lag applied,
+            // lag = min(L-1, D+1) >= 2 -- instead of the deadline-s part of drain s-1 (which
+            // holds rows updated at s-2, inside the window).  The GPU drain waits for drain s-2.
+            const int64_t lag = std::min<int64_t>(c->L - 1, (int64_t)c->D + 1);
+            if (c->host_flush) {
+                if (s - lag >= 0) launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_ALL, (uint32_t)(s - lag + 1), st);
+            } else if (s >= 2 && c->side_pending[par]) {
+                CK(cudaStreamWaitEvent(st, c->ev_side[par], 0));
             }
         } else if (!c->xhost) {  // world 1, or the comparison path: only this rank reads its host rows
             if (s >= 1 && c->side_pending[par ^ 1]) {
