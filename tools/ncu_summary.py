@@ -20,6 +20,7 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 PHASE = {"k_gather_uniq": "gather", "k_flush_rows": "urgent", "k_segreduce": "segred", "k_dot_model": "model",
+         "k_update1": "segred", "k_dot_rg": "model", "k_pack_drain": "side",
          "k_expand": "expand", "k_segred_combine": "segred_combine", "k_segred_chunks": "segred_chunks",
          "k_schedule": "schedule", "k_optimizer": "optimizer", "k_transe_pos": "model_pos",
          "k_transe_pairs_tiled": "model_pairs", "k_transe_grads_tiled": "model_grads"}

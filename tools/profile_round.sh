@@ -15,10 +15,12 @@ ncu --metrics gpu__time_duration.sum --clock-control none --launch-skip 600 -c 6
 if [[ $CFG == fb15k || $CFG == freebase ]]; then
     KS="k_transe_pos k_transe_pairs_tiled k_transe_grads_tiled k_gather_uniq k_segreduce k_flush_rows"
 else
-    KS="k_gather_uniq k_segreduce k_segred_combine k_flush_rows k_dot_model k_schedule k_expand"
+    KS="k_gather_uniq k_update1 k_pack_drain k_dot_rg k_schedule k_radix_scatter k_dedup_emit k_flush_rows"
 fi
 for k in $KS; do
     ncu --set full --import-source on --clock-control none -k regex:$k --launch-skip 30 -c 3 \
         -o $OUT/$k -f $B > $OUT/$k.log 2>&1
     ncu -i $OUT/$k.ncu-rep --page raw --csv --print-units base > $OUT/$k.csv 2>> $OUT/$k.log
+    ncu -i $OUT/$k.ncu-rep --page source --csv --print-units base > $OUT/$k.source.csv 2>> $OUT/$k.log
+    rm -f $OUT/$k.ncu-rep  # gpurun copies back <= 64 MiB: keep the exported pages only
 done
