@@ -643,9 +643,9 @@ def main():
                              "flush_side_d2h": per["side"]["achieved_gbs"],
                              "host_link_peak": link, "hbm_peak": hbm_peak},
         "rows_per_step": {k: v / K for k, v in cnt.items()},
-        "flushing_threads": {"jobs": st1.get("flush_jobs"), "ms_per_job": (st1["flush_ms"] / st1["flush_jobs"])
+        "flushing_threads": {"jobs": st1.get("flush_jobs"), "copy_ms_per_job": (st1["flush_ms"] / st1["flush_jobs"])
                              if st1.get("flush_jobs") else None,
-                             "idle_ms_per_job": (st1["flush_wait_ms"] / st1["flush_jobs"])
+                             "wait_ms_per_job": (st1["flush_wait_ms"] / st1["flush_jobs"])
                              if st1.get("flush_jobs") else None},
         "top_main_stream_phase": top,
         "clocks": clk,

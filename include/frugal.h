@@ -320,8 +320,8 @@ typedef struct {
     int64_t kernel_launches;       /* library kernels launched since init                  */
     int64_t count[FRUGAL_N_COUNTERS];
     int64_t flush_jobs;            /* drain jobs applied by the flushing threads (since the last call) */
-    double flush_ms;               /* their wall time: part-0 flag seen -> job applied, summed       */
-    double flush_wait_ms;          /* time the threads waited for the device between jobs, summed    */
+    double flush_ms;               /* time thread 0 spent copying its share of the rows, summed      */
+    double flush_wait_ms;          /* time thread 0 waited for the device's part flags, summed       */
 } frugal_stats;
 frugal_status frugal_get_stats(frugal_ctx* ctx, frugal_stats* out);
 

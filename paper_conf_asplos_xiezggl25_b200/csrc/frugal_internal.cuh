@@ -118,6 +118,7 @@ struct frugal_ctx {
     int pack_rows = 1;               // rows in flight per lane group in the pack kernel (FRUGAL_PACK_ROWS=4)
     int pack_threads = 256;          // threads per CTA of the pack kernel (FRUGAL_PACK_THREADS)
     bool pack_2stage = false;        // pack via a contiguous HBM run + an 8-CTA sequential copy (FRUGAL_PACK_2STAGE=1)
+    bool pack_tma = false;           // pack chunks staged in smem, written by TMA bulk copies (FRUGAL_PACK_TMA=1)
     float* dst_rows[2] = {nullptr, nullptr};    // HBM staging of the two-stage pack
     int64_t* dst_keys[2] = {nullptr, nullptr};
     int flush_tma = 0;               // flushes by TMA bulk stores: 0 none, 1 side drain, 2 all (FRUGAL_FLUSH_TMA; measured no gain: profiles/r1_sweep21_flush_tma.txt)

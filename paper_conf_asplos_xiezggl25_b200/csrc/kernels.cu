@@ -1053,6 +1053,69 @@ __global__ void k_pack_drain(const int32_t* __restrict__ lists, const int32_t* _
     block_count(ustats + 1, uc);
 }
 
+// TMA variant of the pack (default): each CTA stages a chunk of kPackChunk consecutive rows
+// (and their keys) in shared memory and writes it to the pinned staging queue with two bulk
+// async copies (cp.async.bulk.global.shared::cta) -- a few large writes per chunk instead of a
+// 128-B store per row group, ~50 GB/s from 8 CTAs (profiles/r2_zc_write_probe.txt) with the same
+// short queue of posted writes.  Two smem buffers: the next chunk is gathered while the bulk
+// copy of this one drains.
+template <int GS>
+__global__ void __launch_bounds__(256) k_pack_drain_tma(const int32_t* __restrict__ lists,
+                                                        const int32_t* __restrict__ srcl,
+                                                        const int32_t* __restrict__ cnt, int64_t cap, int world,
+                                                        int g, int d4, const float4* __restrict__ cw,
+                                                        const float4* __restrict__ pw, const int32_t* __restrict__ hs,
+                                                        char* hrows, int64_t* hkeys, unsigned long long* stats,
+                                                        unsigned long long* ustats, int part, int with_urgent,
+                                                        int kPackChunk) {
+    extern __shared__ __align__(128) float4 psm[];  // [2][kPackChunk * d4] rows, then [2][kPackChunk] keys
+    int64_t* ksm = (int64_t*)(psm + 2 * kPackChunk * d4);
+    const int n1 = cnt[1], n2 = cnt[2], n3 = cnt[3], n0 = with_urgent ? cnt[0] : 0;
+    const int lo = part == 0 ? 0 : n1, n = part == 0 ? n1 : n1 + n2 + n3 + n0;
+    const int l = threadIdx.x & (GS - 1), grp = threadIdx.x / GS, ngrp = blockDim.x / GS;
+    unsigned nh = 0, nc = 0, uh = 0, uc = 0;
+    int stage = 0;
+    for (int64_t c0 = lo + (int64_t)blockIdx.x * kPackChunk; c0 < n; c0 += (int64_t)gridDim.x * kPackChunk) {
+        const int rows = (int)min((int64_t)kPackChunk, n - c0);
+        float4* rb = psm + (size_t)stage * kPackChunk * d4;
+        int64_t* kb = ksm + stage * kPackChunk;
+        // this buffer's previous bulk copy has finished reading shared memory
+        if (threadIdx.x == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+        __syncthreads();
+        for (int r = grp; r < rows; r += ngrp) {
+            const int64_t a = c0 + r;
+            const int64_t at = a < n1 ? cap + a : a < n1 + n2 ? 2 * cap + (a - n1)
+                             : a < n1 + n2 + n3 ? 3 * cap + (a - n1 - n2) : (a - n1 - n2 - n3);
+            const int32_t code = srcl[at];
+            const float4* src = code < 0 ? cw + (int64_t)(-1 - code) * d4 : pw + (int64_t)code * d4;
+            for (int v = l; v < d4; v += GS) rb[r * d4 + v] = src[v];
+            if (l == 0) {
+                kb[r] = host_row(hs, (int64_t)lists[at] * world + g);
+                const bool urg = a >= n1 + n2 + n3;
+                if (code < 0) { if (urg) uh++; else nh++; }
+                else { if (urg) uc++; else nc++; }
+            }
+        }
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            const unsigned sr = (unsigned)__cvta_generic_to_shared(rb), sk = (unsigned)__cvta_generic_to_shared(kb);
+            asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(hrows + c0 * d4 * 16),
+                         "r"(sr), "r"(rows * d4 * 16) : "memory");
+            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+            (void)sk;
+        }
+        for (int r = threadIdx.x; r < rows; r += blockDim.x) hkeys[c0 + r] = kb[r];  // coalesced; 8-B aligned only
+        stage ^= 1;
+    }
+    if (threadIdx.x == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // writes complete
+    block_fence_system();
+    block_count(stats, nh);
+    block_count(stats + 1, nc);
+    block_count(ustats, uh);
+    block_count(ustats + 1, uc);
+}
+
 // second stage of the two-stage pack: one part of the job, already contiguous in HBM, copied to
 // the pinned staging queue by a FEW CTAs as one sequential run (8 CTAs reach ~50 GB/s of
 // zero-copy writes, profiles/r2_zc_write_probe.txt) -- few CTAs keep the queue of posted PCIe
@@ -1097,7 +1160,16 @@ void launch_pack_drain(frugal_ctx* c, int par, uint32_t seq, int max_blocks, cud
                         c->sl_rows[par], c->sl_src[par], c->sl_cnt[par], c->sl_cap, c->n, c->g, d4,           \
                         (const float4*)c->cw, (const float4*)c->pw, c->hs, rows_dst, keys_dst,                \
                         c->dstats + FRUGAL_C_SIDE_HOT, c->dstats + FRUGAL_C_URGENT_HOT, part, wu, two ? 0 : 1)))
-        if (c->pack_rows >= 4) {
+        if (c->pack_tma && !two) {
+            // chunk rows: two buffers of chunk * d floats + keys within 48 KB of shared memory
+            const int chunk = std::max(1, std::min(64, (int)(49152 / (2 * (c->d * 4 + 8)))));
+            const size_t smem = 2 * (size_t)chunk * d4 * 16 + 2 * (size_t)chunk * 8;
+            DISPATCH_GS(gs, (k_pack_drain_tma<GS><<<grid, 256, smem, st>>>(
+                                c->sl_rows[par], c->sl_src[par], c->sl_cnt[par], c->sl_cap, c->n, c->g, d4,
+                                (const float4*)c->cw, (const float4*)c->pw, c->hs, (char*)c->dfl_rows[par],
+                                c->dfl_keys[par], c->dstats + FRUGAL_C_SIDE_HOT, c->dstats + FRUGAL_C_URGENT_HOT, part,
+                                wu, chunk)));
+        } else if (c->pack_rows >= 4) {
             PACK(4);
         } else {
             PACK(1);

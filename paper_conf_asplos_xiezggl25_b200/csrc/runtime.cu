@@ -139,7 +139,7 @@ struct frugal::Flushers {
     std::vector<std::thread> th;
     std::atomic<bool> stop{false};
     std::atomic<int> done[2][2];  // [parity][part]: threads finished
-    // instrumentation (thread 0): jobs, ns from its part-0 flag to the job's end, ns waiting
+    // instrumentation (thread 0): jobs, ns copying its share, ns waiting for the device's flags
     std::atomic<int64_t> jobs{0}, busy_ns{0}, wait_ns{0};
 };
 static inline int64_t mono_ns() {
@@ -172,8 +172,8 @@ static void flusher_main(frugal_ctx* c, int t) {
         const uint32_t seq = (uint32_t)(job + 1);
         const float* rows = c->hfl_rows[par];
         const int64_t* keys = c->hfl_keys[par];
-        int64_t t_wait0 = t == 0 ? mono_ns() : 0, t_start = 0;
         for (int part = 0; part < 2; part++) {
+            const int64_t t_wait0 = t == 0 ? mono_ns() : 0;
             // wait for the device to publish the part: spin while jobs keep coming, then poll gently
             const uint32_t* ready = ctl + (part == 0 ? CTL_READY1 : CTL_READY) + par;
             while (!seq_reached(ctl_load(ready), seq)) {
@@ -189,13 +189,15 @@ static void flusher_main(frugal_ctx* c, int t) {
                 }
             }
             idle_since = 0.0;
-            if (t == 0 && part == 0) {
+            int64_t t_start = 0;
+            if (t == 0) {
                 t_start = mono_ns();
                 F->wait_ns.fetch_add(t_start - t_wait0, std::memory_order_relaxed);
             }
             const int64_t n1 = ctl_load(ctl + CTL_N1 + par), nt = ctl_load(ctl + CTL_NTOT + par);
             const int64_t b = part == 0 ? 0 : n1, e = part == 0 ? n1 : nt;
             copy_rows_nt(c->h_w, rows, keys, b + (e - b) * t / T, b + (e - b) * (t + 1) / T, c->d);
+            if (t == 0) F->busy_ns.fetch_add(mono_ns() - t_start, std::memory_order_relaxed);
             if (F->done[par][part].fetch_add(1, std::memory_order_acq_rel) + 1 == T) {
                 F->done[par][part].store(0, std::memory_order_relaxed);
                 ctl_store(ctl + (part == 0 ? CTL_APPLIED_FIRST : CTL_APPLIED_ALL), seq);
@@ -205,10 +207,7 @@ static void flusher_main(frugal_ctx* c, int t) {
                 }
             }
         }
-        if (t == 0) {
-            F->busy_ns.fetch_add(mono_ns() - t_start, std::memory_order_relaxed);
-            F->jobs.fetch_add(1, std::memory_order_relaxed);
-        }
+        if (t == 0) F->jobs.fetch_add(1, std::memory_order_relaxed);
     }
 }
 
@@ -508,6 +507,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->pack_blocks = getenv("FRUGAL_PACK_BLOCKS") ? atoi(getenv("FRUGAL_PACK_BLOCKS")) : 8;
     c->pack_2stage = getenv("FRUGAL_PACK_2STAGE") && atoi(getenv("FRUGAL_PACK_2STAGE"));  // measured slower (r2_sweep_pack_2stage.txt)
     c->pack_rows = getenv("FRUGAL_PACK_ROWS") ? atoi(getenv("FRUGAL_PACK_ROWS")) : 1;
+    c->pack_tma = getenv("FRUGAL_PACK_TMA") && atoi(getenv("FRUGAL_PACK_TMA"));  // measured slower (r2_sweep_pack_tma.txt)
     c->pack_threads = getenv("FRUGAL_PACK_THREADS") ? atoi(getenv("FRUGAL_PACK_THREADS")) : 256;
     // the deadline-(s+1) part of the drain (the next gate waits for it) may run wider
     c->side_first_blocks = getenv("FRUGAL_SIDE_FIRST_BLOCKS") ? atoi(getenv("FRUGAL_SIDE_FIRST_BLOCKS"))
@@ -747,6 +747,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         int prio = lo_prio;
         if (sp && !strcmp(sp, "high")) prio = hi_prio;
         if (sp && !strcmp(sp, "normal")) prio = 0;
+        if (!sp && c->host_flush) prio = hi_prio;  // the flushing-thread pack: 8 small CTAs, scheduled promptly
         CK(cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, prio));
     }
     CK(cudaEventCreateWithFlags(&c->ev_sched, cudaEventDisableTiming));

@@ -325,7 +325,10 @@ def test_host_layout_errors():
                                  {"FRUGAL_FLUSH_TMA": "2", "FRUGAL_HOST_FLUSH": "0"},
                                  {"FRUGAL_EARLY": "1", "FUSED": "1", "FRUGAL_HOST_FLUSH": "0"},
                                  {"FRUGAL_GLUE_CACHE": "0", "FUSED": "1"}, {"FRUGAL_GLUE_CACHE": "1", "FUSED": "1"},
-                                 {"FRUGAL_GLUE_CACHE": "0"}, {"FRUGAL_GLUE_RG": "0", "FUSED": "1"}])
+                                 {"FRUGAL_GLUE_CACHE": "0"}, {"FRUGAL_GLUE_RG": "0", "FUSED": "1"},
+                                 {"FRUGAL_PACK_TMA": "1", "FUSED": "1"}, {"FRUGAL_PACK_2STAGE": "1", "FUSED": "1"},
+                                 {"FRUGAL_PACK_ROWS": "4"}, {"FRUGAL_GRAPHS": "0"}, {"FRUGAL_URGENT_SIDE": "0"},
+                                 {"FRUGAL_GATE_STRICT": "1"}])
 def test_pipeline_modes_parity(env):
     """The optional schedules (early gather of the next step, drain after the gather,
     inline drain) keep every artefact bit-exact (run in a subprocess: the knobs are read
