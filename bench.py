@@ -510,6 +510,11 @@ def main():
     # a10 urgent flush (critical path) / a11 side drain: r per flushed row (w only, R8), D2H
     for nm, h, c_ in [("urgent", "urgent_hot", "urgent_cold"), ("side", "side_hot", "side_cold")]:
         per[nm] = dict(bound="host-link d2h", bytes=(cnt[h] + cnt[c_]) * r / K, ms=ph[nm], peak=link["d2h"])
+    if ph["urgent"] == 0.0 and cnt["urgent_hot"] + cnt["urgent_cold"] > 0:
+        # world 1: the urgent bucket is packed with the step's drain job (reading R7')
+        per["side"]["bytes"] += (cnt["urgent_hot"] + cnt["urgent_cold"]) * r / K
+        per["side"]["note"] = "drain pack incl. the urgent bucket (world 1); side ms include the wait for a free staging buffer"
+        per["urgent"]["bytes"] = 0.0
     # a4 expand: out[i] = rows[inv[i]]: write r + read r + 4 B index per position
     per["expand"] = dict(bound="hbm", bytes=0.0 if fused else (cnt["positions"] * (2 * r + 4)) / K,
                          ms=ph["expand"], peak=hbm_peak)
@@ -525,7 +530,7 @@ def main():
     if world == 1 and ph["optimizer"] == 0.0 and ph["segred"] > 0.0:
         # world 1: the optimizer is fused into the segment-reduce (one pass, no partials buffer):
         # per position r + 4 B (grad row, pos); per touched row w r, G r + r, w out r, 28 B metadata
-        per["segred"] = dict(bound="hbm", kernel="k_segreduce / k_segred_combine (a6 + a8 fused)",
+        per["segred"] = dict(bound="hbm", kernel="k_update1 (a6 + a8 fused, one launch)",
                              bytes=(cnt["positions"] * (r + 4) + touched * (4 * r + 28)) / K,
                              ms=ph["segred"], peak=hbm_peak)
         per["optimizer"]["bytes"] = 0.0

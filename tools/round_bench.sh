@@ -1,15 +1,16 @@
 #!/bin/bash
-# Round bench lines (one B200) -> gpurun_out/r1_bench*.json; then parity tests and smoke.
-set -x
-python -c "import __graft_entry__ as g; g.build(); g.smoke()" > gpurun_out/smoke_final.log 2>&1
-timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/gputests_final.log 2>&1
-python bench.py > gpurun_out/r1_bench.json 2> gpurun_out/rb.err
-python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/r1_bench_reference.json 2>> gpurun_out/rb.err
-python bench.py --no-cpu-baseline --config avazu > gpurun_out/r1_bench_avazu.json 2>> gpurun_out/rb.err
-python bench.py --no-cpu-baseline --mode write_through > gpurun_out/r1_bench_wt.json 2>> gpurun_out/rb.err
-python bench.py --no-cpu-baseline --alpha 0.99 > gpurun_out/r1_bench_a099.json 2>> gpurun_out/rb.err
-python bench.py --no-cpu-baseline --alpha 0 > gpurun_out/r1_bench_a0.json 2>> gpurun_out/rb.err
-python bench.py --no-cpu-baseline --cache-refresh 50 > gpurun_out/r1_bench_dyn.json 2>> gpurun_out/rb.err
-python bench.py --no-cpu-baseline --host-layout freq > gpurun_out/r1_bench_layout_freq.json 2>> gpurun_out/rb.err
-python bench.py --no-cpu-baseline --config fb15k > gpurun_out/r1_bench_fb15k.json 2>> gpurun_out/rb.err
-python bench.py --no-cpu-baseline --config freebase --steps 100 --warmup 10 > gpurun_out/r1_bench_freebase.json 2>> gpurun_out/rb.err
+# Round bench lines on one B200 -> gpurun_out/r2_bench_*.json (the headline first)
+cd "${GRAFT_REPO_ROOT:-.}"
+python -m paper_conf_asplos_xiezggl25_b200.build > /dev/null
+O=gpurun_out
+python bench.py > $O/r2_bench.json 2> $O/r2_rb.err
+python bench.py --impl reference --steps 3 --warmup 3 > $O/r2_bench_reference.json 2>> $O/r2_rb.err
+python bench.py --no-cpu-baseline --drain gpu > $O/r2_bench_gpudrain.json 2>> $O/r2_rb.err
+python bench.py --config avazu > $O/r2_bench_avazu.json 2>> $O/r2_rb.err
+python bench.py --no-cpu-baseline --mode write_through > $O/r2_bench_wt.json 2>> $O/r2_rb.err
+python bench.py --no-cpu-baseline --alpha 0.99 > $O/r2_bench_a099.json 2>> $O/r2_rb.err
+python bench.py --no-cpu-baseline --alpha 0 > $O/r2_bench_a0.json 2>> $O/r2_rb.err
+python bench.py --no-cpu-baseline --cache-refresh 50 > $O/r2_bench_dyn.json 2>> $O/r2_rb.err
+python bench.py --config fb15k > $O/r2_bench_fb15k.json 2>> $O/r2_rb.err
+python bench.py --config freebase --steps 100 --warmup 10 > $O/r2_bench_freebase.json 2>> $O/r2_rb.err
+FRUGAL_BENCH_SAME_DEVICE=1 timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --dist-backend gloo --steps 50 --warmup 5 --no-cpu-baseline > $O/r2_bench_n2_samedev.json 2>> $O/r2_rb.err
