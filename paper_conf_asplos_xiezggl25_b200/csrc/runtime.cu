@@ -1207,7 +1207,12 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
             // holds rows updated at s-2, inside the window).  The GPU drain waits for drain s-2.
             const int64_t lag = std::min<int64_t>(c->L - 1, (int64_t)c->D + 1);
             if (c->host_flush) {
-                if (s - lag >= 0) launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_ALL, (uint32_t)(s - lag + 1), st);
+                // the threads' progress word is host memory: when it already covers the job the
+                // gate needs (nearly always, lag steps back) no device wait is enqueued -- a
+                // device-side read of it would queue behind the pack's posted PCIe writes
+                const uint32_t need = (uint32_t)(s - lag + 1);
+                if (s - lag >= 0 && !seq_reached(ctl_load(c->hfl_ctl + CTL_APPLIED_ALL), need))
+                    launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_ALL, need, st);
             } else if (s >= 2 && c->side_pending[par]) {
                 CK(cudaStreamWaitEvent(st, c->ev_side[par], 0));
             }
