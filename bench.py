@@ -80,6 +80,9 @@ def parse():
                     help="criteo_tb (configs[4]): scale the Kaggle-profile tables to a host table of this many GB "
                          "(default: the full 8.8e8 rows if they fit in 45%% of this host's memory, else as many "
                          "rows as do)")
+    ap.add_argument("--timer-every", type=int, default=int(os.environ.get("FRUGAL_TIMER_EVERY", "1")),
+                    help="phase timers (CUDA events around every phase) on every k-th step only: their "
+                         "records cost the step a few %%; per-phase times are averages over the timed steps")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for barriers / the max-over-ranks timing only")
     return ap.parse_args()
@@ -314,6 +317,7 @@ def main():
                          device=coll_dev)
         dist.broadcast(t, 0)
         nonce = int(t.item())
+    os.environ["FRUGAL_TIMER_EVERY"] = str(max(1, args.timer_every))  # read by frugal_init
     fr = make_context(st, rank=rank, device=local, shm_name=shm, run_nonce=nonce,
                       flags=F.F_TIMERS | (F.F_NO_HOST_STATE if no_host_state else 0) | (F.F_A2A if a2a else 0)
                       | (F.F_PEER if (args.peer and world > 1) else 0)
@@ -487,7 +491,8 @@ def main():
 
     # ---- per-phase rooflines for this rank
     cnt = {k: st1["count"][k] - st0["count"][k] for k in st1["count"]}
-    ph = {k: v / K for k, v in st1["ms"].items()}  # ms per step (per launch of the phase)
+    # ms per step (per launch of the phase), averaged over the steps the timers covered
+    ph = {k: v / max(1, st1["timer_steps"]) for k, v in st1["ms"].items()}
     r = 4 * d
     adag = cfg.opt == "adagrad"
     peaks = measured_peaks()
@@ -641,6 +646,7 @@ def main():
         "gpu_launches": int(launches),
         "roofline": roofline,
         "phases_ms_per_step": {k: round(v, 5) for k, v in ph.items()},
+        "phase_timers": {"every": max(1, args.timer_every), "timed_steps": int(st1["timer_steps"])},
         "rooflines": {k: {kk: (round(vv, 4) if isinstance(vv, float) else vv) for kk, vv in v.items()}
                       for k, v in per.items()},
         "flush_gather_gbs": {"gather_host_h2d": per["gather"]["achieved_gbs"],

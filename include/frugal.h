@@ -322,6 +322,9 @@ typedef struct {
     int64_t flush_jobs;            /* drain jobs applied by the flushing threads (since the last call) */
     double flush_ms;               /* time thread 0 spent copying its share of the rows, summed      */
     double flush_wait_ms;          /* time thread 0 waited for the device's part flags, summed       */
+    int64_t timer_steps;           /* steps whose phases `ms` covers (FRUGAL_F_TIMERS; with the
+                                      environment knob FRUGAL_TIMER_EVERY=k only steps s % k == 0
+                                      are timed, so per-step phase time = ms / timer_steps)        */
 } frugal_stats;
 frugal_status frugal_get_stats(frugal_ctx* ctx, frugal_stats* out);
 

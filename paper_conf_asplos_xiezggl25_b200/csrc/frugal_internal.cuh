@@ -128,6 +128,8 @@ struct frugal_ctx {
     bool update1 = true;         // world 1 fused: one-launch k_update1 (FRUGAL_UPDATE1=0: the 3-kernel path)
     int gather_blocks = 120;     // grid cap of the zero-copy gathers (120 CTAs: +3% over 74 and 148 in the step, profiles/r1_sweep34_gather_grid.txt)
     bool side_inline = false;    // experiment: drain on the caller stream
+    int gather_rows = 1;         // rows in flight per lane group in the gather (FRUGAL_GATHER_ROWS)
+    bool pack_serial = false;    // the gather of s+1 waits for the pack of s (no posted writes beside it)
     bool drain_after_gather = true;  // side drain after the step's gather (FRUGAL_DRAIN_AT=sched: after the scheduler)
     bool urgent_side = false;        // world 1: urgent flush on the side stream (reading R7'), see frugal_step
     int64_t capT;                // max owned rows touched per step
@@ -292,6 +294,9 @@ struct frugal_ctx {
     size_t ev_used = 0;
     double phase_ms[FRUGAL_N_PHASES] = {0};
     int64_t timed_steps = 0;
+    int64_t tstep = -1;            // step of the current frugal_step call (phase-timer sampling)
+    int timer_every = 1;           // FRUGAL_TIMER_EVERY: phase timers on steps s % k == 0 only
+    int64_t timer_steps = 0;       // steps whose phases were timed since the last get_stats
     unsigned long long* dstats = nullptr;  // device counters [FRUGAL_N_COUNTERS]
     // recorded schedule artefacts (FRUGAL_F_RECORD)
     std::vector<int32_t> rec_urgent, rec_deferred, rec_deferred_p, rec_ageout, rec_final;

@@ -1257,6 +1257,104 @@ __global__ void k_gather_uniq(const int32_t* __restrict__ uniq, const int32_t* _
     block_count(stats + FRUGAL_C_GATHER_POOL, np);
     block_count(stats + FRUGAL_C_GATHER_PEER, npeer);
 }
+// a4 gather, R rows in flight per lane group (default R = 4, FRUGAL_GATHER_ROWS): the
+// per-row chain uniq -> {slot, last update, pool index} -> row is latency-bound (one dependent
+// HBM round trip per link, then a host read of ~2 us); here the R rows' uniq loads, then all
+// their metadata loads (independent of each other: last update and pool index are read for
+// every owned row, needed or not), then their row loads are issued together.  Same sources
+// as k_gather_uniq (R7'), same bits.
+template <int GS, int R>
+__global__ void k_gather_uniq_r(const int32_t* __restrict__ uniq, const int32_t* __restrict__ list,
+                                const int32_t* cnt, int world, int g, int d4, const int32_t* __restrict__ slot,
+                                const float4* __restrict__ cw, const float4* hw, float4* __restrict__ rows,
+                                const int32_t* __restrict__ last_upd, const int32_t* __restrict__ pool_idx,
+                                const float4* __restrict__ pw, int P, int64_t capT, int32_t pool_min,
+                                const int32_t* __restrict__ gslot, const PeerTab* __restrict__ pt,
+                                const int32_t* __restrict__ hs, unsigned long long* stats) {
+    int64_t gid, gs;
+    int l;
+    RowGroup<GS>::ids(gid, gs, l);
+    const int n = *cnt;
+    unsigned nh = 0, nc = 0, np = 0, npeer = 0;
+    for (int64_t a0 = gid; a0 < n; a0 += gs * R) {
+        int u[R];
+        int32_t k[R];
+#pragma unroll
+        for (int r = 0; r < R; r++) {
+            const int64_t a = a0 + (int64_t)r * gs;
+            u[r] = a < n ? (list ? list[a] : (int)a) : -1;
+        }
+#pragma unroll
+        for (int r = 0; r < R; r++) k[r] = u[r] >= 0 ? uniq[u[r]] : -1;
+        int32_t sl[R], lu[R], pi[R];
+#pragma unroll
+        for (int r = 0; r < R; r++) {
+            sl[r] = -1;
+            lu[r] = -1;
+            pi[r] = 0;
+            if (k[r] < 0) continue;
+            const int32_t lk = k[r] / world;
+            if (k[r] % world == g) {
+                sl[r] = slot[lk];
+                if (pw) {
+                    lu[r] = last_upd[lk];
+                    pi[r] = pool_idx[lk];
+                }
+            } else if (pt) {
+                const int o = k[r] % world;
+                sl[r] = gslot[k[r]];
+                lu[r] = pt->lu[o][lk];
+                pi[r] = pt->pi[o][lk];
+            }
+        }
+        const float4* src[R];
+#pragma unroll
+        for (int r = 0; r < R; r++) {
+            src[r] = nullptr;
+            if (k[r] < 0) continue;
+            int kind = 0;  // 0 host, 1 cache, 2 pool, 3 peer
+            if (k[r] % world == g) {
+                if (sl[r] >= 0) {
+                    src[r] = cw + (int64_t)sl[r] * d4;
+                    kind = 1;
+                } else if (pw && lu[r] >= 0 && lu[r] >= pool_min) {
+                    src[r] = pw + ((int64_t)(lu[r] % P) * capT + pi[r]) * d4;
+                    kind = 2;
+                }
+            } else if (pt) {  // N4: see k_gather_uniq
+                const int o = k[r] % world;
+                if (sl[r] >= 0) {
+                    src[r] = pt->cw[o] + (int64_t)sl[r] * d4;
+                    kind = 3;
+                } else if (lu[r] >= 0 && lu[r] >= pool_min) {
+                    src[r] = pt->pw[o] + ((int64_t)(lu[r] % P) * pt->capT[o] + pi[r]) * d4;
+                    kind = 3;
+                }
+            }
+            if (kind == 0) src[r] = hw + host_row(hs, k[r]) * d4;
+            if (l == 0) {
+                nh += kind == 0;
+                nc += kind == 1;
+                np += kind == 2;
+                npeer += kind == 3;
+            }
+        }
+        for (int v0 = 0; v0 < d4; v0 += GS) {
+            const int v = v0 + l;
+            float4 x[R];
+#pragma unroll
+            for (int r = 0; r < R; r++)
+                if (src[r] && v < d4) x[r] = src[r][v];
+#pragma unroll
+            for (int r = 0; r < R; r++)
+                if (src[r] && v < d4) rows[(int64_t)u[r] * d4 + v] = x[r];
+        }
+    }
+    block_count(stats + FRUGAL_C_GATHER_HOST, nh);
+    block_count(stats + FRUGAL_C_GATHER_CACHE, nc);
+    block_count(stats + FRUGAL_C_GATHER_POOL, np);
+    block_count(stats + FRUGAL_C_GATHER_PEER, npeer);
+}
 // a4 expand: out[i] = rows[inv[i]]
 template <int GS>
 __global__ void k_expand(const int32_t* __restrict__ inv, const int32_t* d_m, int d4, const float4* __restrict__ rows,
@@ -1293,12 +1391,18 @@ void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32
     // bigger grid only parks stalled warps on SMs other streams need
     int grid = std::min(grid_for((int64_t)c->M * gs, 256, 8), c->gather_blocks);
     const int32_t pool_min = (int32_t)std::max<int64_t>(0, step - c->P + 2);
-    DISPATCH_GS(gs, (k_gather_uniq<GS><<<grid, 256, 0, st>>>(q.uniq, list, cnt, c->n, c->g, d4, c->slot,
-                                                             (const float4*)c->cw, (const float4*)c->dh_w,
-                                                             (float4*)rows, c->last_upd, c->pool_idx,
-                                                             c->pool_hits ? (const float4*)c->pw : nullptr, c->P,
-                                                             c->capT, pool_min, c->gslot, c->peer_tab, c->hs,
-                                                             c->dstats)));
+#define GATHER_ARGS                                                                                          \
+    q.uniq, list, cnt, c->n, c->g, d4, c->slot, (const float4*)c->cw, (const float4*)c->dh_w, (float4*)rows,   \
+        c->last_upd, c->pool_idx, c->pool_hits ? (const float4*)c->pw : nullptr, c->P, c->capT, pool_min, c->gslot, \
+        c->peer_tab, c->hs, c->dstats
+    if (c->gather_rows >= 4) {
+        DISPATCH_GS(gs, (k_gather_uniq_r<GS, 4><<<grid, 256, 0, st>>>(GATHER_ARGS)));
+    } else if (c->gather_rows >= 2) {
+        DISPATCH_GS(gs, (k_gather_uniq_r<GS, 2><<<grid, 256, 0, st>>>(GATHER_ARGS)));
+    } else {
+        DISPATCH_GS(gs, (k_gather_uniq<GS><<<grid, 256, 0, st>>>(GATHER_ARGS)));
+    }
+#undef GATHER_ARGS
     c->launches++;
 }
 // host-link calibration: n pseudo-random rows of the host table (hash of i and seed) read

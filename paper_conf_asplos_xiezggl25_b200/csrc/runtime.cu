@@ -106,6 +106,7 @@ struct Timer {
     cudaEvent_t a = nullptr;
     Timer(frugal_ctx* c_, int ph_, cudaStream_t st_) : c(c_), ph(ph_), st(st_) {
         if (!(c->cfg.flags & FRUGAL_F_TIMERS)) return;
+        if (c->timer_every > 1 && (c->tstep < 0 || c->tstep % c->timer_every != 0)) return;
         if (c->ev_used + 2 > c->ev_pool.size()) {
             for (int i = 0; i < 64; i++) {
                 cudaEvent_t e;
@@ -514,6 +515,9 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
                                                                : c->side_blocks;
     c->gather_blocks = getenv("FRUGAL_GATHER_BLOCKS") ? atoi(getenv("FRUGAL_GATHER_BLOCKS")) : 120;
     c->side_inline = getenv("FRUGAL_SIDE_INLINE") && atoi(getenv("FRUGAL_SIDE_INLINE"));
+    c->gather_rows = getenv("FRUGAL_GATHER_ROWS") ? atoi(getenv("FRUGAL_GATHER_ROWS")) : 1;
+    c->timer_every = getenv("FRUGAL_TIMER_EVERY") ? std::max(1, atoi(getenv("FRUGAL_TIMER_EVERY"))) : 1;
+    c->pack_serial = getenv("FRUGAL_PACK_SERIAL") && atoi(getenv("FRUGAL_PACK_SERIAL"));
     c->drain_after_gather = !(getenv("FRUGAL_DRAIN_AT") && !strcmp(getenv("FRUGAL_DRAIN_AT"), "sched"));
     // world 1 with pool reads (R7'): the urgent bucket is not read from the host at its step
     // (FRUGAL_URGENT_SIDE=0: keep it on the critical path)
@@ -1102,6 +1106,7 @@ extern "C" frugal_status frugal_step(frugal_ctx* c, int64_t s, const int64_t* id
     }
     cudaStream_t st = (cudaStream_t)stream;
     const int par = (int)(s & 1);
+    c->tstep = s;
     // the read bits of steps <= s+L-1 and the adjust list of this step are complete
     {
         const int64_t last = std::min<int64_t>(s + c->L - 1, c->next_prefetch - 1);
@@ -1243,6 +1248,10 @@ extern "C" frugal_status frugal_lookup(frugal_ctx* c, int64_t s, float* d_out, f
     QueueSlot& q = c->q[s % c->QN];
     float* rows = c->rows_buf[s & 1];
     {
+        // the gather's PCIe reads would queue behind the pack's posted writes: with
+        // FRUGAL_PACK_SERIAL the pack of s-1 (run beside the backward of s-1) is complete first
+        if (c->pack_serial && s >= 1 && c->side_pending[(s - 1) & 1])
+            CK(cudaStreamWaitEvent(st, c->ev_side[(s - 1) & 1], 0));
         Timer tm(c, PH_GATHER, st);
         if (c->early) {
             CK(cudaStreamWaitEvent(st, c->ev_early[s & 1], 0));
@@ -1384,6 +1393,7 @@ extern "C" frugal_status frugal_backward_update(frugal_ctx* c, int64_t s, const 
     CKL();
     c->phase_in_step = 0;
     c->timed_steps++;
+    if ((c->cfg.flags & FRUGAL_F_TIMERS) && (c->timer_every <= 1 || (s >= 0 && s % c->timer_every == 0))) c->timer_steps++;
     return check_err_word(c);
 }
 
@@ -1480,6 +1490,7 @@ extern "C" frugal_status frugal_a2a_update(frugal_ctx* c, int64_t s, const float
     CKL();
     c->phase_in_step = 0;
     c->timed_steps++;
+    if ((c->cfg.flags & FRUGAL_F_TIMERS) && (c->timer_every <= 1 || (s >= 0 && s % c->timer_every == 0))) c->timer_steps++;
     return check_err_word(c);
 }
 
@@ -1681,6 +1692,8 @@ extern "C" frugal_status frugal_get_stats(frugal_ctx* c, frugal_stats* out) {
     c->ev_used = 0;
     for (int i = 0; i < FRUGAL_N_PHASES; i++) out->ms[i] = c->phase_ms[i];
     out->steps = c->timed_steps;
+    out->timer_steps = c->timer_steps;
+    c->timer_steps = 0;
     out->kernel_launches = c->launches;
     unsigned long long cnt[FRUGAL_N_COUNTERS];
     CK(cudaMemcpy(cnt, c->dstats, sizeof cnt, cudaMemcpyDeviceToHost));

@@ -328,7 +328,9 @@ def test_host_layout_errors():
                                  {"FRUGAL_GLUE_CACHE": "0"}, {"FRUGAL_GLUE_RG": "0", "FUSED": "1"},
                                  {"FRUGAL_PACK_TMA": "1", "FUSED": "1"}, {"FRUGAL_PACK_2STAGE": "1", "FUSED": "1"},
                                  {"FRUGAL_PACK_ROWS": "4"}, {"FRUGAL_GRAPHS": "0"}, {"FRUGAL_URGENT_SIDE": "0"},
-                                 {"FRUGAL_GATE_STRICT": "1"}])
+                                 {"FRUGAL_GATE_STRICT": "1"}, {"FRUGAL_GATHER_ROWS": "4", "FUSED": "1"},
+                                 {"FRUGAL_GATHER_ROWS": "2"}, {"FRUGAL_PACK_SERIAL": "1", "FUSED": "1"},
+                                 {"FRUGAL_GATHER_ROWS": "1", "FRUGAL_PACK_SERIAL": "0"}])
 def test_pipeline_modes_parity(env):
     """The optional schedules (early gather of the next step, drain after the gather,
     inline drain) keep every artefact bit-exact (run in a subprocess: the knobs are read
@@ -453,7 +455,9 @@ def test_overlapped_pipeline_tiny_100_steps(fused):
     run_overlapped(st, fused=fused, exact=True)
 
 
-@pytest.mark.parametrize("env", [{"FRUGAL_EARLY": "1"}, {"FRUGAL_DRAIN_AT": "sched"}, {"FRUGAL_FUSE_OPT": "0"}])
+@pytest.mark.parametrize("env", [{"FRUGAL_EARLY": "1"}, {"FRUGAL_DRAIN_AT": "sched"}, {"FRUGAL_FUSE_OPT": "0"},
+                                 {"FRUGAL_GATHER_ROWS": "1", "FRUGAL_PACK_SERIAL": "0"},
+                                 {"FRUGAL_GATHER_ROWS": "4", "FRUGAL_PACK_SERIAL": "1"}])
 def test_overlapped_pipeline_knobs(env):
     """The optional schedules of DESIGN.md §10 in the overlapped configuration (subprocess:
     the knobs are read at context creation)."""
