@@ -325,6 +325,9 @@ typedef struct {
     int64_t timer_steps;           /* steps whose phases `ms` covers (FRUGAL_F_TIMERS; with the
                                       environment knob FRUGAL_TIMER_EVERY=k only steps s % k == 0
                                       are timed, so per-step phase time = ms / timer_steps)        */
+    double host_wait_ms;           /* host time the calls spent blocked on the device (the ingest's
+                                      staging-buffer reuse waits): the caller's enqueue cost per
+                                      step is its call time minus this                           */
 } frugal_stats;
 frugal_status frugal_get_stats(frugal_ctx* ctx, frugal_stats* out);
 

@@ -123,6 +123,8 @@ struct frugal_ctx {
     int64_t* dst_keys[2] = {nullptr, nullptr};
     int flush_tma = 0;               // flushes by TMA bulk stores: 0 none, 1 side drain, 2 all (FRUGAL_FLUSH_TMA; measured no gain: profiles/r1_sweep21_flush_tma.txt)
     int glue_cache = -1;         // REC glue keeps a sample's rows in registers (F <= 32): -1 auto, 0 never, 1 always
+    bool update_short8 = true;   // k_update1: rows with <= 8 occurrences load all their gradient rows at once (FRUGAL_UPDATE_SHORT)
+    int glue_unroll = 8;         // REC glue k_dot_rg: rows of a sample in flight (FRUGAL_GLUE_UNROLL; 1 = round-1 order of loads)
     bool glue_rg = true;         // REC glue: row-group kernel k_dot_rg (FRUGAL_GLUE_RG=0: the warp-per-sample k_dot_model)
     bool fuse_opt = true;        // world 1: a8 fused into a6 (k_segreduce / k_segred_combine)
     bool update1 = true;         // world 1 fused: one-launch k_update1 (FRUGAL_UPDATE1=0: the 3-kernel path)
@@ -235,6 +237,7 @@ struct frugal_ctx {
     bool early = false;                                 // pipelined gather enabled (world 1)
     bool pool_hits = true;                              // owner reads its dirty-pool rows from HBM
     int early_blocks = 16;                              // grid of the early gather
+    int early_rows = 4;                                 // rows in flight per lane group in the early gather
     bool early_on_side = false;                         // early gather queued behind the drain
     bool a2a = false;                                   // comparison path (FRUGAL_F_A2A)
     bool peer = false;                                  // NVLink-native variant (FRUGAL_F_PEER)
@@ -296,7 +299,8 @@ struct frugal_ctx {
     int64_t timed_steps = 0;
     int64_t tstep = -1;            // step of the current frugal_step call (phase-timer sampling)
     int timer_every = 1;           // FRUGAL_TIMER_EVERY: phase timers on steps s % k == 0 only
-    int64_t timer_steps = 0;       // steps whose phases were timed since the last get_stats
+    int64_t timer_steps = 0;
+    int64_t host_wait_ns = 0;      // host time blocked in the ingest's buffer-reuse waits since the last get_stats       // steps whose phases were timed since the last get_stats
     unsigned long long* dstats = nullptr;  // device counters [FRUGAL_N_COUNTERS]
     // recorded schedule artefacts (FRUGAL_F_RECORD)
     std::vector<int32_t> rec_urgent, rec_deferred, rec_deferred_p, rec_ageout, rec_final;

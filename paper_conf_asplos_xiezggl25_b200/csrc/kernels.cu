@@ -1592,11 +1592,14 @@ __global__ void __launch_bounds__(256) k_dot_model(const float* __restrict__ emb
 // gradient -- instead of being kept in registers, so ~40 registers and full occupancy.
 // Same arithmetic as k_dot_model: S in fp32, f ascending; z, p, loss in fp64; c rounded to
 // fp32 once; grad = c*((S - e_f) + x) with each op rounded (R16).
-template <int GS, int VPL, bool FUSED>
+template <int GS, int VPL, bool FUSED, int U>
 __global__ void __launch_bounds__(256) k_dot_rg(const float4* __restrict__ emb, const int32_t* __restrict__ inv,
                                                 const float4* __restrict__ x, const float* __restrict__ y,
                                                 float4* __restrict__ grad, double* loss, int count, int F, int d4,
                                                 double nb) {
+    // U rows of the sample in flight (FRUGAL_GLUE_UNROLL): their inverse indices, then their
+    // columns, are loaded together before the adds, which stay in f order (f outer, k inner:
+    // the same order as U = 1) -- one L2 round trip per U rows instead of two per row
     __shared__ double sl[8];
     int64_t gid, gs;
     int l;
@@ -1615,20 +1618,32 @@ __global__ void __launch_bounds__(256) k_dot_rg(const float4* __restrict__ emb, 
             const int v = l + k * GS;
             xv[k] = v < d4 ? x[b * d4 + v] : make_float4(0.f, 0.f, 0.f, 0.f);
         }
-        for (int f = 0; f < F; f++) {
-            const float4* e = row(b, f);
+        for (int f0 = 0; f0 < F; f0 += U) {
+            const float4* e[U];
 #pragma unroll
-            for (int k = 0; k < VPL; k++) {
-                const int v = l + k * GS;
-                if (v < d4) {
-                    const float4 a = e[v];
-                    S[k].x = __fadd_rn(S[k].x, a.x);
-                    S[k].y = __fadd_rn(S[k].y, a.y);
-                    S[k].z = __fadd_rn(S[k].z, a.z);
-                    S[k].w = __fadd_rn(S[k].w, a.w);
-                    ee += (double)a.x * a.x + (double)a.y * a.y + (double)a.z * a.z + (double)a.w * a.w;
+            for (int u = 0; u < U; u++) e[u] = f0 + u < F ? row(b, f0 + u) : nullptr;
+            float4 a[U][VPL];
+#pragma unroll
+            for (int u = 0; u < U; u++)
+#pragma unroll
+                for (int k = 0; k < VPL; k++) {
+                    const int v = l + k * GS;
+                    if (e[u] && v < d4) a[u][k] = e[u][v];
                 }
-            }
+#pragma unroll
+            for (int u = 0; u < U; u++)
+#pragma unroll
+                for (int k = 0; k < VPL; k++) {
+                    const int v = l + k * GS;
+                    if (e[u] && v < d4) {
+                        S[k].x = __fadd_rn(S[k].x, a[u][k].x);
+                        S[k].y = __fadd_rn(S[k].y, a[u][k].y);
+                        S[k].z = __fadd_rn(S[k].z, a[u][k].z);
+                        S[k].w = __fadd_rn(S[k].w, a[u][k].w);
+                        ee += (double)a[u][k].x * a[u][k].x + (double)a[u][k].y * a[u][k].y +
+                              (double)a[u][k].z * a[u][k].z + (double)a[u][k].w * a[u][k].w;
+                    }
+                }
         }
 #pragma unroll
         for (int k = 0; k < VPL; k++) {
@@ -1647,20 +1662,32 @@ __global__ void __launch_bounds__(256) k_dot_rg(const float4* __restrict__ emb, 
         const double yb = (double)y[b];
         if (l == 0) lsum += (z > 0 ? z + log1p(exp(-z)) : log1p(exp(z))) - yb * z;
         const float cc = (float)((p - yb) / nb);  // same rounding as the definition (R16)
-        for (int f = 0; f < F; f++) {
-            const float4* e = row(b, f);
-            float4* g0 = grad + (b * F + f) * d4;
+        for (int f0 = 0; f0 < F; f0 += U) {
+            const float4* e[U];
 #pragma unroll
-            for (int k = 0; k < VPL; k++) {
-                const int v = l + k * GS;
-                if (v < d4) {
-                    const float4 a = e[v];
-                    float4 r;
-                    r.x = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[k].x, a.x), xv[k].x));
-                    r.y = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[k].y, a.y), xv[k].y));
-                    r.z = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[k].z, a.z), xv[k].z));
-                    r.w = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[k].w, a.w), xv[k].w));
-                    g0[v] = r;
+            for (int u = 0; u < U; u++) e[u] = f0 + u < F ? row(b, f0 + u) : nullptr;
+            float4 a[U][VPL];
+#pragma unroll
+            for (int u = 0; u < U; u++)
+#pragma unroll
+                for (int k = 0; k < VPL; k++) {
+                    const int v = l + k * GS;
+                    if (e[u] && v < d4) a[u][k] = e[u][v];
+                }
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+                float4* g0 = grad + (b * F + f0 + u) * d4;
+#pragma unroll
+                for (int k = 0; k < VPL; k++) {
+                    const int v = l + k * GS;
+                    if (e[u] && v < d4) {
+                        float4 r;
+                        r.x = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[k].x, a[u][k].x), xv[k].x));
+                        r.y = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[k].y, a[u][k].y), xv[k].y));
+                        r.z = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[k].z, a[u][k].z), xv[k].z));
+                        r.w = __fmul_rn(cc, __fadd_rn(__fsub_rn(S[k].w, a[u][k].w), xv[k].w));
+                        g0[v] = r;
+                    }
                 }
             }
         }
@@ -1683,21 +1710,32 @@ void launch_dot_model(frugal_ctx* c, QueueSlot& q, const float* emb, const int32
     if (c->glue_rg) {
         const int d4 = c->d / 4, gs = group_size(d4), vpl = (d4 + gs - 1) / gs;
         const double nbd = (double)nb;
-#define RG(V)                                                                                                         \
+        // rows in flight per sample: 8 / VPL (register budget), FRUGAL_GLUE_UNROLL=1: one at a time
+        const int un = c->glue_unroll;
+#define RGU(V, UU)                                                                                                    \
     do {                                                                                                              \
         if (inv) {                                                                                                    \
-            DISPATCH_GS(gs, (k_dot_rg<GS, V, true><<<grid_for((int64_t)count * GS, 256, 8), 256, 0, st>>>(           \
+            DISPATCH_GS(gs, (k_dot_rg<GS, V, true, UU><<<grid_for((int64_t)count * GS, 256, 8), 256, 0, st>>>(       \
                                 (const float4*)emb, inv, (const float4*)x, y, (float4*)grad, loss, count, c->F, d4, nbd))); \
         } else {                                                                                                      \
-            DISPATCH_GS(gs, (k_dot_rg<GS, V, false><<<grid_for((int64_t)count * GS, 256, 8), 256, 0, st>>>(          \
+            DISPATCH_GS(gs, (k_dot_rg<GS, V, false, UU><<<grid_for((int64_t)count * GS, 256, 8), 256, 0, st>>>(      \
                                 (const float4*)emb, inv, (const float4*)x, y, (float4*)grad, loss, count, c->F, d4, nbd))); \
         }                                                                                                             \
     } while (0)
-        if (vpl <= 1) RG(1);
-        else if (vpl <= 2) RG(2);
-        else if (vpl <= 4) RG(4);
-        else RG(8);
-#undef RG
+        if (vpl <= 1) {
+            if (un >= 8) RGU(1, 8);
+            else if (un >= 4) RGU(1, 4);
+            else RGU(1, 1);
+        } else if (vpl <= 2) {
+            if (un >= 4) RGU(2, 4);
+            else RGU(2, 1);
+        } else if (vpl <= 4) {
+            if (un >= 2) RGU(4, 2);
+            else RGU(4, 1);
+        } else {
+            RGU(8, 1);
+        }
+#undef RGU
         c->launches++;
         return;
     }

@@ -93,9 +93,24 @@ __device__ __forceinline__ void fused_update_row(const FusedOpt& fo, int j, int 
 // k_segreduce_long, which computes their chunks in parallel.
 constexpr int kChunk = 64;
 
-template <int GS>
+template <int GS, bool SHORT8 = true>
 __device__ __forceinline__ float4 chunk_sum(const float4* __restrict__ grad, const int32_t* __restrict__ pos, int b,
                                             int e, int d4, int v) {
+    if (SHORT8 && e - b <= 8) {  // short rows (most of them): all positions, then all gradient rows in flight
+        const int n = e - b;
+        int pq[8];
+#pragma unroll
+        for (int q = 0; q < 8; q++) pq[q] = q < n ? pos[b + q] : 0;
+        float4 x[8];
+#pragma unroll
+        for (int q = 0; q < 8; q++)
+            if (q < n) x[q] = grad[(int64_t)pq[q] * d4 + v];
+        float4 acc = x[0];
+#pragma unroll
+        for (int q = 1; q < 8; q++)
+            if (q < n) acc = add4(acc, x[q]);
+        return acc;
+    }
     float4 acc = grad[(int64_t)pos[b] * d4 + v];
     int j = b + 1;
     for (; j + 16 <= e; j += 16) {  // 16 loads in flight, adds in position order
@@ -430,7 +445,7 @@ __device__ __forceinline__ void update_row_pf(const FusedOpt& fo, int j, int d4,
 // [nt, nt + nu) the unique rows, of which the short ones (<= 64 occurrences) are reduced
 // and updated directly.  Same arithmetic, same order as k_segreduce + k_segred_chunks +
 // k_segred_combine (reading R23), without their serialisation.
-template <int GS, int VPL>
+template <int GS, int VPL, bool SHORT8>
 __global__ void __launch_bounds__(256) k_update1(const int32_t* __restrict__ off, const int32_t* __restrict__ pos,
                                                  const int32_t* d_nu, const int4* __restrict__ ltask,
                                                  const int4* __restrict__ linfo, int32_t* lcnt,
@@ -446,7 +461,8 @@ __global__ void __launch_bounds__(256) k_update1(const int32_t* __restrict__ off
     for (int64_t w = gid; w < (int64_t)nt + nu; w += gs) {
         if (w < nt) {
             const int4 tk = ltask[w];
-            for (int v = l; v < d4; v += GS) __stcg(scratch + w * d4 + v, chunk_sum<GS>(grad, pos, tk.x, tk.y, d4, v));
+            for (int v = l; v < d4; v += GS)
+                __stcg(scratch + w * d4 + v, chunk_sum<GS, SHORT8>(grad, pos, tk.x, tk.y, d4, v));
             __threadfence();
             __syncwarp(gmask);
             const int4 li = linfo[tk.z];
@@ -461,7 +477,7 @@ __global__ void __launch_bounds__(256) k_update1(const int32_t* __restrict__ off
             const int u = (int)(w - nt);
             const int b = off[u], e = off[u + 1];
             if (e - b > kChunk) continue;  // a long row: its last chunk task updates it
-            update_row_pf<GS, VPL>(fo, u, d4, l, [&](int v) { return chunk_sum<GS>(grad, pos, b, e, d4, v); },
+            update_row_pf<GS, VPL>(fo, u, d4, l, [&](int v) { return chunk_sum<GS, SHORT8>(grad, pos, b, e, d4, v); },
                                    nhot, ncold);
         }
     }
@@ -493,17 +509,23 @@ void launch_update1(frugal_ctx* c, QueueSlot& q, const float* grad, int64_t s, c
     fo.pkey = c->pkey + (size_t)seg * c->capT;
     fo.pcount = c->pcount + seg;
     const int grid = grid_for((int64_t)c->M * gs, 256, 8);
-#define U1(V)                                                                                                     \
+#define U1S(V, SH)                                                                                                \
     do {                                                                                                          \
-        DISPATCH_GS(gs, (k_update1<GS, V><<<grid, 256, 0, st>>>(q.off, q.pos, q.n_uniq, q.ltask, q.linfo, q.lcnt, \
-                                                                 q.lnum, d4, (const float4*)grad,                  \
-                                                                 (float4*)c->chunk_scratch, c->dstats, fo)));      \
+        DISPATCH_GS(gs, (k_update1<GS, V, SH><<<grid, 256, 0, st>>>(q.off, q.pos, q.n_uniq, q.ltask, q.linfo,     \
+                                                                     q.lcnt, q.lnum, d4, (const float4*)grad,      \
+                                                                     (float4*)c->chunk_scratch, c->dstats, fo)));  \
+    } while (0)
+#define U1(V)                          \
+    do {                               \
+        if (c->update_short8) U1S(V, true); \
+        else U1S(V, false);            \
     } while (0)
     if (vpl <= 1) U1(1);
     else if (vpl <= 2) U1(2);
     else if (vpl <= 4) U1(4);
     else U1(8);
 #undef U1
+#undef U1S
     c->launches++;
 }
 

@@ -197,7 +197,9 @@ static void flusher_main(frugal_ctx* c, int t) {
             }
             const int64_t n1 = ctl_load(ctl + CTL_N1 + par), nt = ctl_load(ctl + CTL_NTOT + par);
             const int64_t b = part == 0 ? 0 : n1, e = part == 0 ? n1 : nt;
-            copy_rows_nt(c->h_w, rows, keys, b + (e - b) * t / T, b + (e - b) * (t + 1) / T, c->d);
+            static const bool diag_no_apply = getenv("FRUGAL_DIAG_NO_APPLY") && atoi(getenv("FRUGAL_DIAG_NO_APPLY"));
+            if (!diag_no_apply)  // (diagnostic only: without the copy the host table is stale)
+                copy_rows_nt(c->h_w, rows, keys, b + (e - b) * t / T, b + (e - b) * (t + 1) / T, c->d);
             if (t == 0) F->busy_ns.fetch_add(mono_ns() - t_start, std::memory_order_relaxed);
             if (F->done[par][part].fetch_add(1, std::memory_order_acq_rel) + 1 == T) {
                 F->done[par][part].store(0, std::memory_order_relaxed);
@@ -482,6 +484,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->early = c->n == 1 && getenv("FRUGAL_EARLY") && atoi(getenv("FRUGAL_EARLY"));
     c->pool_hits = !(getenv("FRUGAL_NO_POOL_HITS") && atoi(getenv("FRUGAL_NO_POOL_HITS")));
     c->early_blocks = getenv("FRUGAL_EARLY_BLOCKS") ? atoi(getenv("FRUGAL_EARLY_BLOCKS")) : 16;
+    c->early_rows = getenv("FRUGAL_EARLY_ROWS") ? atoi(getenv("FRUGAL_EARLY_ROWS")) : 4;
     c->early_on_side = getenv("FRUGAL_EARLY_ON_SIDE") && atoi(getenv("FRUGAL_EARLY_ON_SIDE"));
     c->a2a = (k.flags & FRUGAL_F_A2A) != 0;
     c->peer = (k.flags & FRUGAL_F_PEER) != 0;
@@ -517,11 +520,13 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->side_inline = getenv("FRUGAL_SIDE_INLINE") && atoi(getenv("FRUGAL_SIDE_INLINE"));
     c->gather_rows = getenv("FRUGAL_GATHER_ROWS") ? atoi(getenv("FRUGAL_GATHER_ROWS")) : 1;
     c->timer_every = getenv("FRUGAL_TIMER_EVERY") ? std::max(1, atoi(getenv("FRUGAL_TIMER_EVERY"))) : 1;
+    c->glue_unroll = getenv("FRUGAL_GLUE_UNROLL") ? atoi(getenv("FRUGAL_GLUE_UNROLL")) : 8;
+    c->update_short8 = !(getenv("FRUGAL_UPDATE_SHORT") && !atoi(getenv("FRUGAL_UPDATE_SHORT")));
     c->pack_serial = getenv("FRUGAL_PACK_SERIAL") && atoi(getenv("FRUGAL_PACK_SERIAL"));
     c->drain_after_gather = !(getenv("FRUGAL_DRAIN_AT") && !strcmp(getenv("FRUGAL_DRAIN_AT"), "sched"));
     // world 1 with pool reads (R7'): the urgent bucket is not read from the host at its step
     // (FRUGAL_URGENT_SIDE=0: keep it on the critical path)
-    c->urgent_side = c->n == 1 && c->pool_hits && !c->side_inline && !c->early &&
+    c->urgent_side = c->n == 1 && c->pool_hits && !c->side_inline && (!c->early || c->L >= 3) &&
                      k.mode == FRUGAL_MODE_P2F &&
                      !(getenv("FRUGAL_URGENT_SIDE") && !atoi(getenv("FRUGAL_URGENT_SIDE")));
     c->capT = std::max<int64_t>(1, std::min<int64_t>((int64_t)c->n * c->M, c->No));
@@ -928,10 +933,12 @@ static frugal_status ingest(frugal_ctx* c, int64_t t, const int64_t* ids_all, co
     // previous call has finished once this call returns (host wait, normally long done), so
     // the caller may reuse a buffer after the next frugal_step/frugal_prefetch returns
     static const bool no_copy_wait = getenv("FRUGAL_NO_COPY_WAIT") && atoi(getenv("FRUGAL_NO_COPY_WAIT"));  // diagnostic
+    const int64_t hw0 = mono_ns();
     if (!no_copy_wait) CK(cudaEventSynchronize(c->ev_copied));
     CK(cudaEventRecord(c->ev_call, caller));
     CK(cudaStreamWaitEvent(is, c->ev_call, 0));
     CK(cudaEventSynchronize(c->ev_counts[qi]));  // pinned counts / parameter staging of this slot is free
+    c->host_wait_ns += mono_ns() - hw0;
     int32_t* pin = c->counts_pin + (size_t)qi * c->n;
     memcpy(pin, counts, (size_t)c->n * 4);
     CK(cudaMemcpyAsync(q.counts, pin, (size_t)c->n * 4, cudaMemcpyHostToDevice, is));
@@ -1035,14 +1042,32 @@ static frugal_status launch_early_gather(frugal_ctx* c, int64_t u, cudaEvent_t s
     // next step) that fills the link while the main stream runs the backward
     cudaStream_t ps = c->early_on_side ? c->side : c->pstream;
     CK(cudaStreamWaitEvent(ps, c->ev_ingest[u % c->QN], 0));
-    if (side_first) CK(cudaStreamWaitEvent(ps, side_first, 0));
     if (c->opt_pending[u & 1]) CK(cudaStreamWaitEvent(ps, c->ev_opt[u & 1], 0));
+    Timer tm(c, PH_PREFETCH, ps);
+    if (c->urgent_side) {
+        // world 1 reading its dirty pool (R7'): the early rows of u that come from the host were
+        // last updated before u-D-1, so their host copies are final once the drains up to
+        // u - lag are applied (the gate's rule, frugal_step) -- long before step u-1 runs
+        const int64_t lag = std::min<int64_t>(c->L - 1, (int64_t)c->D + 1);
+        if (u - lag >= 0) {
+            if (c->host_flush) {
+                const uint32_t need = (uint32_t)(u - lag + 1);
+                if (!seq_reached(ctl_load(c->hfl_ctl + CTL_APPLIED_ALL), need))
+                    launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_ALL, need, ps);
+            } else if (u >= 2 && c->side_pending[(u - 2) & 1]) {
+                CK(cudaStreamWaitEvent(ps, c->ev_side[(u - 2) & 1], 0));  // drain u-2 (FIFO: and earlier)
+            }
+        }
+    } else if (side_first) {
+        CK(cudaStreamWaitEvent(ps, side_first, 0));
+    }
     {
-        Timer tm(c, PH_PREFETCH, ps);
-        const int keep = c->gather_blocks;
+        const int keep = c->gather_blocks, keep_rows = c->gather_rows;
         c->gather_blocks = c->early_blocks;  // few SMs: its loads must not crowd the backward
+        c->gather_rows = c->early_rows;
         launch_gather(c, q, q.eidx, q.elcnt, c->rows_buf[u & 1], u, ps);
         c->gather_blocks = keep;
+        c->gather_rows = keep_rows;
     }
     CK(cudaEventRecord(c->ev_early[u & 1], ps));
     c->early_issued = u;
@@ -1265,7 +1290,7 @@ extern "C" frugal_status frugal_lookup(frugal_ctx* c, int64_t s, float* d_out, f
         frugal_status r = launch_drain(c, s, st, c->ev_gathered);
         if (r) return r;
         if (c->early && s + 1 < c->next_prefetch) {
-            r = launch_early_gather(c, s + 1, c->ev_side_first[s & 1]);
+            r = launch_early_gather(c, s + 1, c->urgent_side ? nullptr : c->ev_side_first[s & 1]);
             if (r) return r;
         }
     }
@@ -1693,6 +1718,8 @@ extern "C" frugal_status frugal_get_stats(frugal_ctx* c, frugal_stats* out) {
     for (int i = 0; i < FRUGAL_N_PHASES; i++) out->ms[i] = c->phase_ms[i];
     out->steps = c->timed_steps;
     out->timer_steps = c->timer_steps;
+    out->host_wait_ms = c->host_wait_ns * 1e-6;
+    c->host_wait_ns = 0;
     c->timer_steps = 0;
     out->kernel_launches = c->launches;
     unsigned long long cnt[FRUGAL_N_COUNTERS];

@@ -54,7 +54,8 @@ COUNTERS = ["positions", "unique", "gather_host", "gather_cache", "opt_hot", "op
 class Stats(C.Structure):
     _fields_ = [("ms", C.c_double * 12), ("steps", C.c_int64), ("kernel_launches", C.c_int64),
                 ("count", C.c_int64 * 20), ("flush_jobs", C.c_int64), ("flush_ms", C.c_double),
-                ("flush_wait_ms", C.c_double), ("timer_steps", C.c_int64)]
+                ("flush_wait_ms", C.c_double), ("timer_steps", C.c_int64),
+                ("host_wait_ms", C.c_double)]
 
 
 _lib = None
@@ -308,7 +309,7 @@ class Frugal:
         return dict(ms={p: s.ms[i] for i, p in enumerate(PHASES)}, steps=s.steps,
                     kernel_launches=s.kernel_launches, count={n: s.count[i] for i, n in enumerate(COUNTERS)},
                     flush_jobs=s.flush_jobs, flush_ms=s.flush_ms, flush_wait_ms=s.flush_wait_ms,
-                    timer_steps=s.timer_steps)
+                    timer_steps=s.timer_steps, host_wait_ms=s.host_wait_ms)
 
     def get_timeline(self, cap=4096):
         """[(phase name, start ms, end ms)] of the last `cap` recorded phases (all streams)."""

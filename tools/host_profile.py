@@ -37,6 +37,7 @@ for flags, name in [(F.F_TIMERS, "F_TIMERS"), (0, "no timers")]:
     for s in range(S):
         if s == W0:
             torch.cuda.synchronize()
+            fr.get_stats()  # resets the counters (host wait included)
             e0.record()
             acc[:] = 0
         t0 = time.perf_counter()
@@ -54,6 +55,8 @@ for flags, name in [(F.F_TIMERS, "F_TIMERS"), (0, "no timers")]:
     torch.cuda.synchronize()
     n = S - W0
     us = acc / n * 1e6
+    wait_us = fr.get_stats()["host_wait_ms"] / n * 1e3
     print(f"{name:10s} host us/call: step {us[0]:6.1f} lookup {us[1]:6.1f} dot_model {us[2]:6.1f} "
-          f"backward {us[3]:6.1f}  total {us.sum():6.1f}   GPU ms/step {e0.elapsed_time(e1) / n:.4f}", flush=True)
+          f"backward {us[3]:6.1f}  total {us.sum():6.1f} (of which blocked on the device {wait_us:6.1f}: "
+          f"enqueue cost {us.sum() - wait_us:6.1f})   GPU ms/step {e0.elapsed_time(e1) / n:.4f}", flush=True)
     fr.close()
