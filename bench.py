@@ -512,6 +512,12 @@ def main():
     per["gather"] = dict(bound="host-link h2d", bytes=cnt["gather_host"] * r / K,
                          hbm_bytes=(cnt["gather_cache"] + cnt["gather_pool"] + cnt["unique"]) * r / K,
                          ms=ph["gather"], peak=link["h2d"])
+    if ph.get("prefetch", 0.0) > 0.0:
+        # early gather (world 1, FRUGAL_EARLY): every host row of step s+1 is read by the early
+        # gather on the library's prefetch stream during step s (the lag rule); the main-stream
+        # gather of s+1 reads only the rows updated at s (HBM: pool / cache)
+        per["gather"].update(ms=ph["prefetch"], kernel="k_gather_uniq_r (early part: host rows, prefetch stream)",
+                             main_stream_ms=ph["gather"])
     # a10 urgent flush (critical path) / a11 side drain: r per flushed row (w only, R8), D2H
     for nm, h, c_ in [("urgent", "urgent_hot", "urgent_cold"), ("side", "side_hot", "side_cold")]:
         per[nm] = dict(bound="host-link d2h", bytes=(cnt[h] + cnt[c_]) * r / K, ms=ph[nm], peak=link["d2h"])
@@ -588,7 +594,7 @@ def main():
     except Exception as e:
         tnote = f"null: {e}"
     if D.get("bound") != "alu":
-        roofline = {"bound": "hbm" if D["bound"] == "hbm" else "host-link", "kernel": dom,
+        roofline = {"bound": "hbm" if D["bound"] == "hbm" else "host-link", "kernel": D.get("kernel", dom),
                     "achieved": D["achieved_gbs"], "peak": D["peak"], "unit": "GB/s", "frac": D["frac"],
                     "random_row_ceiling": link["random_rows_h2d"] if D["bound"] != "hbm" else None,
                     "frac_of_random_row_ceiling": (D["achieved_gbs"] / link["random_rows_h2d"])

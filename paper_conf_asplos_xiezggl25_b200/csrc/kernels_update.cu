@@ -96,18 +96,18 @@ constexpr int kChunk = 64;
 template <int GS, bool SHORT8 = true>
 __device__ __forceinline__ float4 chunk_sum(const float4* __restrict__ grad, const int32_t* __restrict__ pos, int b,
                                             int e, int d4, int v) {
-    if (SHORT8 && e - b <= 8) {  // short rows (most of them): all positions, then all gradient rows in flight
+    if (SHORT8 && e - b <= 4) {  // short rows (most of them): all positions, then all gradient rows in flight
         const int n = e - b;
-        int pq[8];
+        int pq[4];
 #pragma unroll
-        for (int q = 0; q < 8; q++) pq[q] = q < n ? pos[b + q] : 0;
-        float4 x[8];
+        for (int q = 0; q < 4; q++) pq[q] = q < n ? pos[b + q] : 0;
+        float4 x[4];
 #pragma unroll
-        for (int q = 0; q < 8; q++)
+        for (int q = 0; q < 4; q++)
             if (q < n) x[q] = grad[(int64_t)pq[q] * d4 + v];
         float4 acc = x[0];
 #pragma unroll
-        for (int q = 1; q < 8; q++)
+        for (int q = 1; q < 4; q++)
             if (q < n) acc = add4(acc, x[q]);
         return acc;
     }

@@ -494,7 +494,6 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     // FRUGAL_HOST_FLUSH=0/1 (experiments) overrides the flag
     c->host_flush = (k.flags & FRUGAL_F_GPU_DRAIN) == 0;
     if (getenv("FRUGAL_HOST_FLUSH")) c->host_flush = atoi(getenv("FRUGAL_HOST_FLUSH")) != 0;
-    if (c->host_flush) c->early = false;  // the early gather synchronises on the GPU drain's events
     c->xhost = c->n > 1 && !c->a2a;
     c->own_ids = (k.flags & FRUGAL_F_OWN_IDS) != 0 && c->n > 1;
     // side-drain flushes by TMA bulk stores (FRUGAL_FLUSH_TMA=0 none, 1 side, 2 all)
@@ -529,6 +528,9 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->urgent_side = c->n == 1 && c->pool_hits && !c->side_inline && (!c->early || c->L >= 3) &&
                      k.mode == FRUGAL_MODE_P2F &&
                      !(getenv("FRUGAL_URGENT_SIDE") && !atoi(getenv("FRUGAL_URGENT_SIDE")));
+    // the early gather waits for the GPU drain's events -- or, world 1 under the lag rule
+    // (urgent_side), for the flushing threads' progress word
+    if (c->host_flush && !c->urgent_side) c->early = false;
     c->capT = std::max<int64_t>(1, std::min<int64_t>((int64_t)c->n * c->M, c->No));
     c->sl_cap = 2 * c->capT;
     c->key_bits = bits_for(c->N - 1);

@@ -1,7 +1,7 @@
 #!/bin/bash
 # session 2, call 4: glue with 8 rows in flight, short-row update ILP, world-1 early host gather (lag rule)
 cd "${GRAFT_REPO_ROOT:-.}"
-python -m paper_conf_asplos_xiezggl25_b200.build > /dev/null
+python -m paper_conf_asplos_xiezggl25_b200.build --force > /dev/null
 timeout 1200 python -m pytest tests/test_gpu_parity.py -m gpu -q -x -k "pipeline_modes or overlapped_pipeline" > gpurun_out/r2_c28_tests.log 2>&1
 echo "rc=$?" >> gpurun_out/r2_c28_tests.log
 O=gpurun_out/r2_c28_sweep.txt
