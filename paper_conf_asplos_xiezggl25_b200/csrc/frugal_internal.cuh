@@ -117,13 +117,15 @@ struct frugal_ctx {
     int pack_blocks = 20;            // grid cap of the drain's pack kernel (flushing-thread drain)
     int pack_rows = 1;               // rows in flight per lane group in the pack kernel (FRUGAL_PACK_ROWS=4)
     int pack_threads = 256;          // threads per CTA of the pack kernel (FRUGAL_PACK_THREADS)
+    bool pack_ce = false;            // pack into HBM, the flushing threads move it D2H with cudaMemcpyAsync (FRUGAL_PACK_CE=1)
+    cudaStream_t ce_stream = nullptr; // their copy stream
     bool pack_2stage = false;        // pack via a contiguous HBM run + an 8-CTA sequential copy (FRUGAL_PACK_2STAGE=1)
     bool pack_tma = false;           // pack chunks staged in smem, written by TMA bulk copies (FRUGAL_PACK_TMA=1)
     float* dst_rows[2] = {nullptr, nullptr};    // HBM staging of the two-stage pack
     int64_t* dst_keys[2] = {nullptr, nullptr};
     int flush_tma = 0;               // flushes by TMA bulk stores: 0 none, 1 side drain, 2 all (FRUGAL_FLUSH_TMA; measured no gain: profiles/r1_sweep21_flush_tma.txt)
     int glue_cache = -1;         // REC glue keeps a sample's rows in registers (F <= 32): -1 auto, 0 never, 1 always
-    bool update_short8 = true;   // k_update1: rows with <= 8 occurrences load all their gradient rows at once (FRUGAL_UPDATE_SHORT)
+    bool update_short8 = false;   // k_update1: rows with <= 8 occurrences load all their gradient rows at once (FRUGAL_UPDATE_SHORT)
     int glue_unroll = 8;         // REC glue k_dot_rg: rows of a sample in flight (FRUGAL_GLUE_UNROLL; 1 = round-1 order of loads)
     bool glue_rg = true;         // REC glue: row-group kernel k_dot_rg (FRUGAL_GLUE_RG=0: the warp-per-sample k_dot_model)
     bool fuse_opt = true;        // world 1: a8 fused into a6 (k_segreduce / k_segred_combine)

@@ -1149,7 +1149,8 @@ void launch_pack_drain(frugal_ctx* c, int par, uint32_t seq, int max_blocks, cud
     // two stages (default): the rows are gathered into a contiguous HBM staging run by a full
     // grid (HBM-bound, a few us), then copied to the host by k_copy_seq with max_blocks CTAs;
     // FRUGAL_PACK_2STAGE=0: one kernel gathers straight to the host with max_blocks CTAs
-    const bool two = c->pack_2stage;
+    const bool ce = c->pack_ce;  // HBM run only: the flushing threads copy it with the copy engine
+    const bool two = c->pack_2stage || ce;
     const int grid = two ? grid_for(3 * c->sl_cap * (int64_t)gs, 256, 2)
                          : std::min(grid_for(3 * c->sl_cap * (int64_t)gs, nthr, 4), max_blocks);
     float4* rows_dst = two ? (float4*)c->dst_rows[par] : (float4*)c->dfl_rows[par];
@@ -1175,7 +1176,7 @@ void launch_pack_drain(frugal_ctx* c, int par, uint32_t seq, int max_blocks, cud
             PACK(1);
         }
 #undef PACK
-        if (two) {
+        if (two && !ce) {
             k_copy_seq<<<max_blocks, 256, 0, st>>>(c->sl_cnt[par], part, wu, d4, (const float4*)c->dst_rows[par],
                                                     c->dst_keys[par], (float4*)c->dfl_rows[par], c->dfl_keys[par]);
             c->launches++;

@@ -140,6 +140,8 @@ struct frugal::Flushers {
     std::vector<std::thread> th;
     std::atomic<bool> stop{false};
     std::atomic<int> done[2][2];  // [parity][part]: threads finished
+    std::atomic<uint32_t> copied[2][2];  // [parity][part]: job seq whose rows thread 0 copied D2H (FRUGAL_PACK_CE)
+    std::atomic<int> ce_error{0};
     // instrumentation (thread 0): jobs, ns copying its share, ns waiting for the device's flags
     std::atomic<int64_t> jobs{0}, busy_ns{0}, wait_ns{0};
 };
@@ -165,6 +167,7 @@ static void copy_rows_nt(float* table, const float* rows, const int64_t* keys, i
 
 static void flusher_main(frugal_ctx* c, int t) {
     frugal::Flushers* F = c->flushers;
+    if (c->pack_ce && t == 0) cudaSetDevice(c->cfg.device);  // thread 0 issues the D2H copies
     const int T = c->n_flushers;
     uint32_t* ctl = c->hfl_ctl;
     double idle_since = 0.0;
@@ -197,6 +200,27 @@ static void flusher_main(frugal_ctx* c, int t) {
             }
             const int64_t n1 = ctl_load(ctl + CTL_N1 + par), nt = ctl_load(ctl + CTL_NTOT + par);
             const int64_t b = part == 0 ? 0 : n1, e = part == 0 ? n1 : nt;
+            if (c->pack_ce) {
+                // the part is packed in HBM: thread 0 moves it into the pinned staging buffer with
+                // the copy engine (one sequential DMA per part), the others wait for it
+                if (t == 0) {
+                    if (e > b) {
+                        const size_t rb = (size_t)c->d * 4;
+                        bool ok = cudaMemcpyAsync((char*)c->hfl_rows[par] + b * rb, (char*)c->dst_rows[par] + b * rb,
+                                                  (size_t)(e - b) * rb, cudaMemcpyDeviceToHost, c->ce_stream) == cudaSuccess;
+                        ok = ok && cudaMemcpyAsync(c->hfl_keys[par] + b, c->dst_keys[par] + b, (size_t)(e - b) * 8,
+                                                   cudaMemcpyDeviceToHost, c->ce_stream) == cudaSuccess;
+                        ok = ok && cudaStreamSynchronize(c->ce_stream) == cudaSuccess;
+                        if (!ok) F->ce_error.store(1);
+                    }
+                    F->copied[par][part].store(seq, std::memory_order_release);
+                } else {
+                    while (F->copied[par][part].load(std::memory_order_acquire) != seq) {
+                        if (F->stop.load(std::memory_order_relaxed)) return;
+                        _mm_pause();
+                    }
+                }
+            }
             static const bool diag_no_apply = getenv("FRUGAL_DIAG_NO_APPLY") && atoi(getenv("FRUGAL_DIAG_NO_APPLY"));
             if (!diag_no_apply)  // (diagnostic only: without the copy the host table is stale)
                 copy_rows_nt(c->h_w, rows, keys, b + (e - b) * t / T, b + (e - b) * (t + 1) / T, c->d);
@@ -247,6 +271,10 @@ static void interleave_numa(void* base, size_t bytes) {
     syscall(SYS_mbind, base, bytes, 3 /* MPOL_INTERLEAVE */, &mask, 65ul, 0u);
 }
 static frugal_status check_err_word(frugal_ctx* c) {
+    if (c->flushers && c->flushers->ce_error.load()) {
+        set_err("flushing threads: a device-to-host copy of the drain staging run failed");
+        return FRUGAL_ECUDA;
+    }
     if (c->herr && *(volatile int32_t*)c->herr) {
         int e = *(volatile int32_t*)c->herr;
         if (e == 2) {
@@ -330,6 +358,7 @@ static void free_ctx(frugal_ctx* c) {
         if (c->ev_opt[i]) cudaEventDestroy(c->ev_opt[i]);
     }
     if (c->pstream) cudaStreamDestroy(c->pstream);
+    if (c->ce_stream) cudaStreamDestroy(c->ce_stream);
     for (auto e : c->ev_pool) cudaEventDestroy(e);
     if (c->ev_hot) cudaEventDestroy(c->ev_hot);
     if (c->shm_base) {
@@ -508,6 +537,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     // few CTAs for the zero-copy writes of the pack: 8 reach the link rate, and a short queue of
     // posted writes keeps concurrent PCIe reads fast (profiles/r2_zc_write_probe.txt, r2_sweep_pack*.txt)
     c->pack_blocks = getenv("FRUGAL_PACK_BLOCKS") ? atoi(getenv("FRUGAL_PACK_BLOCKS")) : 8;
+    c->pack_ce = getenv("FRUGAL_PACK_CE") && atoi(getenv("FRUGAL_PACK_CE"));
     c->pack_2stage = getenv("FRUGAL_PACK_2STAGE") && atoi(getenv("FRUGAL_PACK_2STAGE"));  // measured slower (r2_sweep_pack_2stage.txt)
     c->pack_rows = getenv("FRUGAL_PACK_ROWS") ? atoi(getenv("FRUGAL_PACK_ROWS")) : 1;
     c->pack_tma = getenv("FRUGAL_PACK_TMA") && atoi(getenv("FRUGAL_PACK_TMA"));  // measured slower (r2_sweep_pack_tma.txt)
@@ -520,7 +550,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->gather_rows = getenv("FRUGAL_GATHER_ROWS") ? atoi(getenv("FRUGAL_GATHER_ROWS")) : 1;
     c->timer_every = getenv("FRUGAL_TIMER_EVERY") ? std::max(1, atoi(getenv("FRUGAL_TIMER_EVERY"))) : 1;
     c->glue_unroll = getenv("FRUGAL_GLUE_UNROLL") ? atoi(getenv("FRUGAL_GLUE_UNROLL")) : 8;
-    c->update_short8 = !(getenv("FRUGAL_UPDATE_SHORT") && !atoi(getenv("FRUGAL_UPDATE_SHORT")));
+    c->update_short8 = getenv("FRUGAL_UPDATE_SHORT") && atoi(getenv("FRUGAL_UPDATE_SHORT"));  // measured slower (r2_sweep_glue_update.txt)
     c->pack_serial = getenv("FRUGAL_PACK_SERIAL") && atoi(getenv("FRUGAL_PACK_SERIAL"));
     c->drain_after_gather = !(getenv("FRUGAL_DRAIN_AT") && !strcmp(getenv("FRUGAL_DRAIN_AT"), "sched"));
     // world 1 with pool reads (R7'): the urgent bucket is not read from the host at its step
@@ -866,7 +896,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
             return FRUGAL_ENOMEM;
         }
         memset(c->hfl_ctl, 0, 4096);
-        if (c->pack_2stage)
+        if (c->pack_2stage || c->pack_ce)
             for (int i = 0; i < 2; i++) {
                 DMALLOC(c->dst_rows[i], (size_t)cap * rowb);
                 DMALLOC(c->dst_keys[i], (size_t)cap * 8);
@@ -878,7 +908,11 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
         c->n_flushers = std::max(1, c->n_flushers);
         c->flushers = new frugal::Flushers();
         for (int i = 0; i < 2; i++)
-            for (int j = 0; j < 2; j++) c->flushers->done[i][j].store(0);
+            for (int j = 0; j < 2; j++) {
+                c->flushers->done[i][j].store(0);
+                c->flushers->copied[i][j].store(0);
+            }
+        if (c->pack_ce) CK(cudaStreamCreateWithFlags(&c->ce_stream, cudaStreamNonBlocking));
         for (int t = 0; t < c->n_flushers; t++) c->flushers->th.emplace_back(flusher_main, c, t);
     }
     if (c->peer) {
@@ -1088,9 +1122,13 @@ static frugal_status launch_drain(frugal_ctx* c, int64_t s, cudaStream_t st, cud
     cudaStream_t sd = c->side_inline ? st : c->side;
     if (!c->side_inline) CK(cudaStreamWaitEvent(c->side, after, 0));
     if (c->host_flush) {
-        // host flushing threads: staging buffer `par` was last used by job s-2
+        // host flushing threads: staging buffer `par` was last used by job s-2 (its own timer
+        // instance: the timeline shows the wait and the pack apart)
+        if (s >= 2) {
+            Timer tw(c, PH_SIDE, sd);
+            launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_ALL, (uint32_t)(s - 1), sd);
+        }
         Timer tm(c, PH_SIDE, sd);
-        if (s >= 2) launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_ALL, (uint32_t)(s - 1), sd);
         launch_pack_drain(c, par, (uint32_t)(s + 1), c->pack_blocks, sd);
         CK(cudaEventRecord(c->ev_side_first[par], sd));  // the lists of this parity were read
         CKL();
