@@ -1201,7 +1201,7 @@ __global__ void k_gather_uniq(const int32_t* __restrict__ uniq, const int32_t* _
                               const int32_t* __restrict__ last_upd, const int32_t* __restrict__ pool_idx,
                               const float4* __restrict__ pw, int P, int64_t capT, int32_t pool_min,
                               const int32_t* __restrict__ gslot, const PeerTab* __restrict__ pt,
-                              const int32_t* __restrict__ hs, unsigned long long* stats) {
+                              const int32_t* __restrict__ hs, unsigned long long* stats, int64_t hmask) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
@@ -1244,7 +1244,7 @@ __global__ void k_gather_uniq(const int32_t* __restrict__ uniq, const int32_t* _
                 }
             }
         }
-        if (kind == 0) src = hw + host_row(hs, k) * d4;
+        if (kind == 0) src = hw + (host_row(hs, k) & hmask) * d4;  // hmask: -1 (diagnostic knob aside)
         if (l == 0) {
             nh += kind == 0;
             nc += kind == 1;
@@ -1401,7 +1401,10 @@ void launch_gather(frugal_ctx* c, QueueSlot& q, const int32_t* list, const int32
     } else if (c->gather_rows >= 2) {
         DISPATCH_GS(gs, (k_gather_uniq_r<GS, 2><<<grid, 256, 0, st>>>(GATHER_ARGS)));
     } else {
-        DISPATCH_GS(gs, (k_gather_uniq<GS><<<grid, 256, 0, st>>>(GATHER_ARGS)));
+        // FRUGAL_DIAG_HOST_MASK (diagnostic only, wrong rows): host row index & mask -- is the
+        // gather bound by the translation of its random host reads over the whole table?
+        static const int64_t hmask = getenv("FRUGAL_DIAG_HOST_MASK") ? atoll(getenv("FRUGAL_DIAG_HOST_MASK")) : -1;
+        DISPATCH_GS(gs, (k_gather_uniq<GS><<<grid, 256, 0, st>>>(GATHER_ARGS, hmask)));
     }
 #undef GATHER_ARGS
     c->launches++;

@@ -51,6 +51,7 @@ struct FusedOpt {
     float4* cw;
     float4* Gd;
     float4* pw;  // pool segment s % P
+    int32_t gmask;  // diagnostic only (FRUGAL_DIAG_G_MASK): G row index & gmask (-1: all rows)
     int32_t* pkey;
     int32_t* pcount;
 };
@@ -296,6 +297,7 @@ void launch_segreduce(frugal_ctx* c, QueueSlot& q, const float* grad, int par, f
                       int64_t fused_step) {
     const int d4 = c->d / 4, gs = group_size(d4);
     FusedOpt fo{};
+    fo.gmask = -1;
     if (fused_step >= 0) {  // world 1: a6 + a8 in one pass (launch_optimizer is not called)
         const int seg = (int)(fused_step % c->P);
         fo.on = 1;
@@ -413,7 +415,7 @@ __device__ __forceinline__ void update_row_pf(const FusedOpt& fo, int j, int d4,
         G[k] = make_float4(0.f, 0.f, 0.f, 0.f);
         if (v < d4) {
             w[k] = wsrc[v];
-            if (fo.adagrad) G[k] = fo.Gd[(int64_t)lk * d4 + v];
+            if (fo.adagrad) G[k] = fo.Gd[(int64_t)(lk & fo.gmask) * d4 + v];
         }
     }
 #pragma unroll
@@ -424,7 +426,7 @@ __device__ __forceinline__ void update_row_pf(const FusedOpt& fo, int j, int d4,
             opt4(w[k], G[k], acc, fo.adagrad, fo.lr, fo.eps);
             if (sl >= 0) fo.cw[(int64_t)sl * d4 + v] = w[k];
             else fo.pw[(int64_t)j * d4 + v] = w[k];
-            if (fo.adagrad) fo.Gd[(int64_t)lk * d4 + v] = G[k];
+            if (fo.adagrad) fo.Gd[(int64_t)(lk & fo.gmask) * d4 + v] = G[k];
         }
     }
     if (l == 0) {
@@ -494,6 +496,10 @@ void launch_update1(frugal_ctx* c, QueueSlot& q, const float* grad, int64_t s, c
     fo.on = 1;
     fo.s = (int32_t)s;
     fo.adagrad = c->cfg.opt == FRUGAL_ADAGRAD;
+    // diagnostic only (wrong results): G footprint folded to gmask+1 rows -- is the update
+    // bound by address translation of its random G accesses over the dense [N][d] array?
+    static const int32_t diag_gmask = getenv("FRUGAL_DIAG_G_MASK") ? atoi(getenv("FRUGAL_DIAG_G_MASK")) : -1;
+    fo.gmask = diag_gmask;
     fo.lr = c->cfg.lr;
     fo.eps = c->cfg.eps;
     fo.uniq = q.uniq;
