@@ -125,7 +125,8 @@ struct frugal_ctx {
     int64_t* dst_keys[2] = {nullptr, nullptr};
     int flush_tma = 0;               // flushes by TMA bulk stores: 0 none, 1 side drain, 2 all (FRUGAL_FLUSH_TMA; measured no gain: profiles/r1_sweep21_flush_tma.txt)
     int glue_cache = -1;         // REC glue keeps a sample's rows in registers (F <= 32): -1 auto, 0 never, 1 always
-    bool update_short8 = false;   // k_update1: rows with <= 8 occurrences load all their gradient rows at once (FRUGAL_UPDATE_SHORT)
+    bool update_short8 = false;
+    bool update_dyn = true;      // k_update1: warps fetch batches of work items from a counter (FRUGAL_UPDATE_DYN=0: static grid-stride)   // k_update1: rows with <= 8 occurrences load all their gradient rows at once (FRUGAL_UPDATE_SHORT)
     int glue_unroll = 8;         // REC glue k_dot_rg: rows of a sample in flight (FRUGAL_GLUE_UNROLL; 1 = round-1 order of loads)
     bool glue_rg = true;         // REC glue: row-group kernel k_dot_rg (FRUGAL_GLUE_RG=0: the warp-per-sample k_dot_model)
     bool fuse_opt = true;        // world 1: a8 fused into a6 (k_segreduce / k_segred_combine)
@@ -199,6 +200,7 @@ struct frugal_ctx {
     float* chunk_scratch = nullptr;  // [M][d] chunk sums of long segments
     int32_t* long_q = nullptr;       // [M] long segments of the current step
     int32_t* long_cnt = nullptr;     // [2]: long segments, chunk tasks
+    int32_t* upd_ctr = nullptr;      // [2]: k_update1 work counters by step parity (dynamic fetch)
     int2* long_tasks = nullptr;      // [M/32 + 2] chunk [begin, end) positions
     int32_t* owned_cnt = nullptr;  // scalar
     // schedule lists (double buffered by step parity): 4 lists of sl_cap rows each --

@@ -447,20 +447,24 @@ __device__ __forceinline__ void update_row_pf(const FusedOpt& fo, int j, int d4,
 // [nt, nt + nu) the unique rows, of which the short ones (<= 64 occurrences) are reduced
 // and updated directly.  Same arithmetic, same order as k_segreduce + k_segred_chunks +
 // k_segred_combine (reading R23), without their serialisation.
+constexpr int kUpdBatch = 8;  // work items a warp takes per fetch (dynamic mode)
+
 template <int GS, int VPL, bool SHORT8>
 __global__ void __launch_bounds__(256) k_update1(const int32_t* __restrict__ off, const int32_t* __restrict__ pos,
                                                  const int32_t* d_nu, const int4* __restrict__ ltask,
                                                  const int4* __restrict__ linfo, int32_t* lcnt,
                                                  const int32_t* lnum, int d4, const float4* __restrict__ grad,
-                                                 float4* scratch, unsigned long long* stats, const FusedOpt fo) {
+                                                 float4* scratch, unsigned long long* stats, const FusedOpt fo,
+                                                 int32_t* ctr, int par) {
     int64_t gid, gs;
     int l;
     RowGroup<GS>::ids(gid, gs, l);
     const unsigned gmask = GS == 32 ? 0xffffffffu : (((1u << GS) - 1u) << ((threadIdx.x & 31) & ~(GS - 1)));
     const int leader = (threadIdx.x & 31) & ~(GS - 1);
     const int nt = lnum[1], nu = *d_nu;
+    const int64_t total = (int64_t)nt + nu;
     unsigned nhot = 0, ncold = 0;
-    for (int64_t w = gid; w < (int64_t)nt + nu; w += gs) {
+    auto item = [&](int64_t w) {
         if (w < nt) {
             const int4 tk = ltask[w];
             for (int v = l; v < d4; v += GS)
@@ -471,16 +475,33 @@ __global__ void __launch_bounds__(256) k_update1(const int32_t* __restrict__ off
             int last = 0;
             if (l == 0) last = atomicAdd(&lcnt[tk.z], 1) == li.z - 1;
             last = __shfl_sync(gmask, last, leader);
-            if (!last) continue;
+            if (!last) return;
             __threadfence();  // every chunk of the row is in scratch
             update_row_pf<GS, VPL>(fo, li.x, d4, l, [&](int v) {
                 return ordered_rows_cg(scratch + (int64_t)li.y * d4 + v, d4, li.z); }, nhot, ncold);
         } else {
             const int u = (int)(w - nt);
             const int b = off[u], e = off[u + 1];
-            if (e - b > kChunk) continue;  // a long row: its last chunk task updates it
+            if (e - b > kChunk) return;  // a long row: its last chunk task updates it
             update_row_pf<GS, VPL>(fo, u, d4, l, [&](int v) { return chunk_sum<GS, SHORT8>(grad, pos, b, e, d4, v); },
                                    nhot, ncold);
+        }
+    };
+    if (!ctr) {
+        for (int64_t w = gid; w < total; w += gs) item(w);
+    } else {
+        // dynamic: each warp takes the next kUpdBatch items (the long rows' chunks come first) --
+        // no block waits for a slow neighbour's static share; the counter of the next step's
+        // launch (other parity) is reset here, before that launch can start
+        if (blockIdx.x == 0 && threadIdx.x == 0) ctr[par ^ 1] = 0;
+        const int lane = threadIdx.x & 31, gpw = 32 / GS, grp = lane / GS;
+        for (;;) {
+            int base = 0;
+            if (lane == 0) base = atomicAdd(&ctr[par], kUpdBatch);
+            base = __shfl_sync(0xffffffffu, base, 0);
+            if (base >= total) break;
+            for (int k = grp; k < kUpdBatch; k += gpw)
+                if (base + k < total) item((int64_t)base + k);
         }
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) *fo.pcount = nu;
@@ -515,11 +536,14 @@ void launch_update1(frugal_ctx* c, QueueSlot& q, const float* grad, int64_t s, c
     fo.pkey = c->pkey + (size_t)seg * c->capT;
     fo.pcount = c->pcount + seg;
     const int grid = grid_for((int64_t)c->M * gs, 256, 8);
+    int32_t* ctr = c->update_dyn ? c->upd_ctr : nullptr;
+    const int par = (int)(s & 1);
 #define U1S(V, SH)                                                                                                \
     do {                                                                                                          \
         DISPATCH_GS(gs, (k_update1<GS, V, SH><<<grid, 256, 0, st>>>(q.off, q.pos, q.n_uniq, q.ltask, q.linfo,     \
                                                                      q.lcnt, q.lnum, d4, (const float4*)grad,      \
-                                                                     (float4*)c->chunk_scratch, c->dstats, fo)));  \
+                                                                     (float4*)c->chunk_scratch, c->dstats, fo,     \
+                                                                     ctr, par)));                                  \
     } while (0)
 #define U1(V)                          \
     do {                               \

@@ -332,7 +332,7 @@ static void free_ctx(frugal_ctx* c) {
         F(q.linfo); F(q.ltask); F(q.lcnt); F(q.lnum);
         if (c->n > 1) { F(q.T); F(q.Tmask); F(q.Tidx); F(q.nT); F(q.gl); F(q.goff); }
     }
-    F(c->hs); F(c->rows_buf[0]); F(c->rows_buf[1]); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->long_tasks); F(c->owned_cnt);
+    F(c->hs); F(c->rows_buf[0]); F(c->rows_buf[1]); F(c->Pp); F(c->chunk_scratch); F(c->long_q); F(c->long_cnt); F(c->upd_ctr); F(c->long_tasks); F(c->owned_cnt);
     for (int i = 0; i < 2; i++) { F(c->adj_rows[i]); F(c->adj_p[i]); F(c->adj_cnt[i]); }
     for (int i = 0; i < 2; i++) { F(c->sl_rows[i]); F(c->sl_p[i]); F(c->sl_src[i]); F(c->sl_cnt[i]); }
     F(c->dstats); F(c->kg_W); F(c->kg_A); F(c->a2a_roff); F(c->peer_tab); F(c->gslot);
@@ -551,6 +551,7 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     c->timer_every = getenv("FRUGAL_TIMER_EVERY") ? std::max(1, atoi(getenv("FRUGAL_TIMER_EVERY"))) : 1;
     c->glue_unroll = getenv("FRUGAL_GLUE_UNROLL") ? atoi(getenv("FRUGAL_GLUE_UNROLL")) : 8;
     c->update_short8 = getenv("FRUGAL_UPDATE_SHORT") && atoi(getenv("FRUGAL_UPDATE_SHORT"));  // measured slower (r2_sweep_glue_update.txt)
+    c->update_dyn = !(getenv("FRUGAL_UPDATE_DYN") && !atoi(getenv("FRUGAL_UPDATE_DYN")));
     c->pack_serial = getenv("FRUGAL_PACK_SERIAL") && atoi(getenv("FRUGAL_PACK_SERIAL"));
     c->drain_after_gather = !(getenv("FRUGAL_DRAIN_AT") && !strcmp(getenv("FRUGAL_DRAIN_AT"), "sched"));
     // world 1 with pool reads (R7'): the urgent bucket is not read from the host at its step
@@ -749,6 +750,8 @@ extern "C" frugal_status frugal_init(const frugal_config* cfg, frugal_ctx** out)
     DMALLOC(c->chunk_scratch, (size_t)c->M * rowb);
     DMALLOC(c->long_q, (size_t)c->M * 4);
     DMALLOC(c->long_cnt, 8);
+    DMALLOC(c->upd_ctr, 8);
+    CK(cudaMemset(c->upd_ctr, 0, 8));
     DMALLOC(c->long_tasks, ((size_t)c->M / 32 + 2) * sizeof(int2));
     DMALLOC(c->owned_cnt, 4);
 
