@@ -126,7 +126,7 @@ struct frugal_ctx {
     int flush_tma = 0;               // flushes by TMA bulk stores: 0 none, 1 side drain, 2 all (FRUGAL_FLUSH_TMA; measured no gain: profiles/r1_sweep21_flush_tma.txt)
     int glue_cache = -1;         // REC glue keeps a sample's rows in registers (F <= 32): -1 auto, 0 never, 1 always
     bool update_short8 = false;
-    bool update_dyn = true;      // k_update1: warps fetch batches of work items from a counter (FRUGAL_UPDATE_DYN=0: static grid-stride)   // k_update1: rows with <= 8 occurrences load all their gradient rows at once (FRUGAL_UPDATE_SHORT)
+    bool update_dyn = false;     // k_update1: warps fetch batches of work items from a counter (FRUGAL_UPDATE_DYN=1; measured slower)   // k_update1: rows with <= 8 occurrences load all their gradient rows at once (FRUGAL_UPDATE_SHORT)
     int glue_unroll = 8;         // REC glue k_dot_rg: rows of a sample in flight (FRUGAL_GLUE_UNROLL; 1 = round-1 order of loads)
     bool glue_rg = true;         // REC glue: row-group kernel k_dot_rg (FRUGAL_GLUE_RG=0: the warp-per-sample k_dot_model)
     bool fuse_opt = true;        // world 1: a8 fused into a6 (k_segreduce / k_segred_combine)

@@ -335,7 +335,7 @@ def test_host_layout_errors():
                                  {"FRUGAL_GLUE_UNROLL": "1", "FUSED": "1"}, {"FRUGAL_GLUE_UNROLL": "4"},
                                  {"FRUGAL_UPDATE_SHORT": "1", "FUSED": "1"}, {"FRUGAL_PACK_CE": "1"},
                                  {"FRUGAL_PACK_CE": "1", "FUSED": "1", "FRUGAL_FLUSH_THREADS": "3"},
-                                 {"FRUGAL_UPDATE_DYN": "0", "FUSED": "1"}])
+                                 {"FRUGAL_UPDATE_DYN": "1", "FUSED": "1"}])
 def test_pipeline_modes_parity(env):
     """The optional schedules (early gather of the next step, drain after the gather,
     inline drain) keep every artefact bit-exact (run in a subprocess: the knobs are read
@@ -464,7 +464,7 @@ def test_overlapped_pipeline_tiny_100_steps(fused):
                                  {"FRUGAL_GATHER_ROWS": "1", "FRUGAL_PACK_SERIAL": "0"},
                                  {"FRUGAL_GATHER_ROWS": "4", "FRUGAL_PACK_SERIAL": "1"},
                                  {"FRUGAL_EARLY": "1", "FRUGAL_EARLY_BLOCKS": "64"}, {"FRUGAL_GLUE_UNROLL": "1"},
-                                 {"FRUGAL_UPDATE_SHORT": "1"}, {"FRUGAL_PACK_CE": "1"}, {"FRUGAL_UPDATE_DYN": "0"}])
+                                 {"FRUGAL_UPDATE_SHORT": "1"}, {"FRUGAL_PACK_CE": "1"}, {"FRUGAL_UPDATE_DYN": "1"}])
 def test_overlapped_pipeline_knobs(env):
     """The optional schedules of DESIGN.md §10 in the overlapped configuration (subprocess:
     the knobs are read at context creation)."""
