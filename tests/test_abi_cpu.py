@@ -129,3 +129,27 @@ def test_workload_host_order():
     assert len(set(o.tolist())) == len(o) == int((freq > 0).sum())
     key = [(-int(freq[k]), int(k)) for k in o]
     assert key == sorted(key)
+
+
+@pytest.mark.parametrize("cname,pyname", [("frugal_config", "Config"), ("frugal_schedule_info", "ScheduleInfo"),
+                                          ("frugal_stats", "Stats")])
+def test_struct_layouts_match_header(cname, pyname, tmp_path):
+    """The ctypes mirrors of the ABI structs have the C compiler's size and field offsets
+    (a field appended to frugal.h but not to frugal.py -- or vice versa -- would make the
+    library write past, or read garbage from, the binding's buffer)."""
+    import subprocess
+    F = _lib()
+    py = getattr(F, pyname)
+    fields = [f[0] for f in py._fields_]
+    prog = ["#include <stdio.h>", "#include <stddef.h>", '#include "frugal.h"', "int main(void) {",
+            f'  printf("%zu\\n", sizeof({cname}));']
+    prog += [f'  printf("%zu\\n", offsetof({cname}, {f}));' for f in fields]
+    prog += ["  return 0;", "}"]
+    src = tmp_path / "layout.c"
+    src.write_text("\n".join(prog) + "\n")
+    exe = tmp_path / "layout"
+    subprocess.check_call(["gcc", "-std=c11", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)])
+    got = [int(x) for x in subprocess.check_output([str(exe)]).split()]
+    assert got[0] == C.sizeof(py), (cname, got[0], C.sizeof(py))
+    for f, off in zip(fields, got[1:]):
+        assert getattr(py, f).offset == off, (cname, f, off, getattr(py, f).offset)
