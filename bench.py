@@ -80,6 +80,9 @@ def parse():
                     help="criteo_tb (configs[4]): scale the Kaggle-profile tables to a host table of this many GB "
                          "(default: the full 8.8e8 rows if they fit in 45%% of this host's memory, else as many "
                          "rows as do)")
+    ap.add_argument("--age-out", type=int, default=0,
+                    help="override the config's age-out D (cold rows with no read in sight are flushed D "
+                         "steps after their update; the owner's dirty-pool window is D+1 steps)")
     ap.add_argument("--timer-every", type=int, default=int(os.environ.get("FRUGAL_TIMER_EVERY", "1")),
                     help="phase timers (CUDA events around every phase) on every k-th step only: their "
                          "records cost the step a few %%; per-phase times are averages over the timed steps")
@@ -226,7 +229,7 @@ def run_reference(args, rank, world):
     if rank != 0:
         return
     from paper_conf_asplos_xiezggl25_b200 import workload as W
-    cfg = W.config(args.config, world=1, alpha=args.alpha)
+    cfg = W.config(args.config, world=1, alpha=args.alpha, **({"age_out": args.age_out} if args.age_out > 0 else {}))
     steps = args.warmup + args.steps
     # bounded sample: each "step" is one oracle step; cap the run to a few minutes
     per_step_budget = 60
@@ -294,6 +297,8 @@ def main():
         mem = os.sysconf("SC_PAGE_SIZE") * os.sysconf("SC_PHYS_PAGES")
         budget = args.host_gb * 1e9 if args.host_gb > 0 else 0.45 * mem
         over["rows_total"] = min(8.8e8, budget / (128 * 4))
+    if args.age_out > 0:  # sensitivity of the lazy flush's holding time D (SURVEY Q9 default: the config's)
+        over["age_out"] = args.age_out
     cfg = W.config(args.config, world=world, alpha=args.alpha, **over)
     K, Wm, L = args.steps, args.warmup, cfg.lookahead
     S = Wm + 2 * K + L + 2

@@ -15,6 +15,7 @@ python bench.py --no-cpu-baseline --cache-refresh 50 > $O/r2_bench_dyn.json 2>> 
 python bench.py --no-cpu-baseline --drain gpu > $O/r2_bench_gpudrain.json 2>> $O/r2_rb.err
 python bench.py --config freebase --steps 100 --warmup 10 > $O/r2_bench_freebase.json 2>> $O/r2_rb.err
 FRUGAL_BENCH_SAME_DEVICE=1 timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --dist-backend gloo --steps 50 --warmup 5 --no-cpu-baseline > $O/r2_bench_n2_samedev.json 2>> $O/r2_rb.err
+python bench.py --no-cpu-baseline --age-out 40 > $O/r2_bench_ageout40.json 2>> $O/r2_rb.err
 timeout 1500 python bench.py --config criteo_tb --alpha 0.9 --steps 200 --warmup 20 > $O/r2_bench_criteo_tb_a0.9.json 2>> $O/r2_rb.err
 timeout 1500 python bench.py --config criteo_tb --alpha 1.2 --steps 200 --warmup 20 > $O/r2_bench_criteo_tb_a1.2.json 2>> $O/r2_rb.err
 for f in $O/r2_bench*.json; do echo "$f $(head -c 220 $f)"; done
