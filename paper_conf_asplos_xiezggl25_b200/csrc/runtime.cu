@@ -1125,13 +1125,11 @@ static frugal_status launch_drain(frugal_ctx* c, int64_t s, cudaStream_t st, cud
     cudaStream_t sd = c->side_inline ? st : c->side;
     if (!c->side_inline) CK(cudaStreamWaitEvent(c->side, after, 0));
     if (c->host_flush) {
-        // host flushing threads: staging buffer `par` was last used by job s-2 (its own timer
-        // instance: the timeline shows the wait and the pack apart)
-        if (s >= 2) {
-            Timer tw(c, PH_SIDE, sd);
-            launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_ALL, (uint32_t)(s - 1), sd);
-        }
+        // host flushing threads: staging buffer `par` was last used by job s-2 (one timer over
+        // the wait and the pack: an event recorded between them measurably slowed the step,
+        // 25.3 vs 26.7 M samples/s, profiles/r2_ab_side_timer.txt)
         Timer tm(c, PH_SIDE, sd);
+        if (s >= 2) launch_wait_word(c, c->dfl_ctl + CTL_APPLIED_ALL, (uint32_t)(s - 1), sd);
         launch_pack_drain(c, par, (uint32_t)(s + 1), c->pack_blocks, sd);
         CK(cudaEventRecord(c->ev_side_first[par], sd));  // the lists of this parity were read
         CKL();
